@@ -1,0 +1,334 @@
+#!/usr/bin/env python3
+"""Benchmark of the PTAS hot path (BASELINE.json metric: DP state-relaxations/sec
+and PTAS solve time; %HBM peak).
+
+One step = one full ptas_solve of the workload (every §8(a) row: classify,
+configuration enumeration, row-level index, level fill per probe, readout,
+search, traceback + greedy schedule).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload M2s] [--impl ours|reference]
+
+value  : executed relaxations (closed form, summed over the DPs the solve ran)
+         / device-timed step, with p resident in HBM (ptas_solve_device)
+e2e    : the same through ptas_solve with pinned host p / host assignment
+roofline: level-fill kernel, algorithmic bytes (relax + sigma) * e per DP over
+         its event-timed duration, against MEASURED_PEAKS.json hbm_gbs
+cpu_baseline: the oracle (plain sequential C) on a bounded sub-box sample of
+         the same workload's largest DP, one host core
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from synth import WORKLOADS  # noqa: E402
+
+METRIC = "DP state-relaxations/sec and PTAS solve time at 1/2/4/8 B200; %HBM peak"
+UNIT = "relaxations/s"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[3:7]):
+                if v.strip().lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def _dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, local, world
+
+
+def _largest_dp(w):
+    """(N, r, T) of the workload's DP at T = LB — the largest table of the solve."""
+    import oracle
+    p = w.p()
+    k = oracle.k_of(w.eps)
+    LB, _ = oracle.bounds(p, w.m)
+    u, r, N, _ = oracle.classify(p, LB, k)
+    return N, r, LB
+
+
+def _subbox_for(N, r, T, target_relax):
+    """Clip counts (largest first) until the closed-form relaxation count of the
+    sub-box DP is <= target: the DP restricted to n <= N' is exactly the
+    oracle's DP on N' (same C(T) restricted), so it is a sample of the same
+    workload."""
+    import oracle
+    C = oracle.configs(N, r, T)
+    Nc = np.array(N, np.int64)
+
+    def relax(Nv):
+        ok = (C <= Nv).all(axis=1)
+        return float(np.prod((Nv - C[ok] + 1).astype(np.float64), axis=1).sum())
+    while relax(Nc) > target_relax and Nc.max() > 1:
+        i = int(np.argmax(Nc))
+        Nc[i] -= 1
+    return Nc.astype(np.int32), relax(Nc)
+
+
+def cpu_oracle_sample(w, target_relax=2.0e9):
+    import oracle
+    N, r, T = _largest_dp(w)
+    if len(N) == 0:
+        return None
+    Nc, rel = _subbox_for(N, r, T, target_relax)
+    t0 = time.perf_counter()
+    _tab, relax = oracle.dp(Nc, r, T)
+    dt = time.perf_counter() - t0
+    return {"value": relax / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"oracle_dp on the sub-box N'={Nc.tolist()} of the {w.name} DP at T=LB={T} "
+                      f"(full N={list(map(int, N))}); {relax:.3g} relaxations in {dt:.2f} s, 1 core"}
+
+
+def run_reference(args, w):
+    rank, _local, world = _dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    N, r, T = _largest_dp(w)
+    target = float(os.environ.get("PTAS_REF_SAMPLE_RELAX", "6e8"))
+    Nc, _ = _subbox_for(N, r, T, target)
+    times, relaxes = [], []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        _tab, relax = oracle.dp(Nc, r, T)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+            relaxes.append(relax)
+    val = sum(relaxes) / sum(times)
+    sample = (f"each step = oracle_dp on the sub-box N'={Nc.tolist()} of the {w.name} DP at T=LB={T} "
+              f"({relaxes[0]:.3g} relaxations), sequential C, 1 core")
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic", "config": {"workload": w.name, "n": w.n, "m": w.m, "eps": w.eps, "P": w.P,
+                                            "seed": w.seed},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "gpu_launches": 0}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_ours(args, w):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_ligsg18_b200 as P
+
+    rank, local, world = _dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    comm = P.init_comm(local) if world > 1 else None
+    if world > 1:
+        mode = P.MODE_MULTI_PROBE if args.mode == "multiprobe" else P.MODE_LEVEL_SHARDED
+        Pp = world if mode == P.MODE_MULTI_PROBE else args.P
+    else:
+        mode, Pp = P.MODE_SINGLE, args.P
+    opts = P.options(P=Pp, mode=mode, device=local, comm=comm)
+
+    p = w.p()
+    n = len(p)
+    p_pin = torch.from_numpy(p).pin_memory()
+    p_dev = p_pin.to(f"cuda:{local}")
+    a_dev = torch.zeros(n, dtype=torch.int32, device=f"cuda:{local}")
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{local}")
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def step_device():
+        return P.ptas_solve_device(p_dev, w.m, w.eps, a_dev, opts=opts)
+
+    def step_e2e():
+        # pinned host p in, host assignment out (the public ABI call a user makes)
+        r = P.ptas_solve(p_pin.numpy(), w.m, w.eps, opts=opts, log=False)
+        return r
+
+    for _ in range(args.warmup):
+        step_device()
+        step_e2e()
+    barrier()
+
+    dev_ms, stats = [], []
+    s_ev = torch.cuda.Event(enable_timing=True)
+    e_ev = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        for _ in range(args.steps):
+            flush.zero_()                       # L2 flush between timed steps (outside the events)
+            torch.cuda.synchronize()
+            s_ev.record()
+            r = step_device()
+            e_ev.record()
+            torch.cuda.synchronize()
+            dev_ms.append(s_ev.elapsed_time(e_ev))
+            stats.append(r["stats"])
+        barrier()
+        e2e_ms, e2e_stats = [], []
+        for _ in range(args.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            s_ev.record()
+            r2 = step_e2e()
+            e_ev.record()
+            torch.cuda.synchronize()
+            e2e_ms.append(s_ev.elapsed_time(e_ev))
+            e2e_stats.append(r2["stats"])
+        barrier()
+    clocks = clk.summary()
+
+    relax_total = sum(s["relaxations"] for s in stats)
+    t_total = sum(dev_ms) / 1e3
+    fill_s = sum(s["fill_seconds"] for s in stats)
+    alg_bytes = sum(s["alg_bytes"] for s in stats)
+    fill_launches = sum(s["fill_launches"] for s in stats)
+    launches = sum(s["kernel_launches"] for s in stats)
+    e2e_relax = sum(s["relaxations"] for s in e2e_stats)
+    e2e_t = sum(e2e_ms) / 1e3
+    if world > 1:
+        t = torch.tensor([t_total, e2e_t, fill_s], dtype=torch.float64, device=f"cuda:{local}")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_total, e2e_t, fill_s = t.tolist()
+        rl = torch.tensor([relax_total, e2e_relax, alg_bytes], dtype=torch.float64, device=f"cuda:{local}")
+        if mode == P.MODE_MULTI_PROBE:
+            dist.all_reduce(rl, op=dist.ReduceOp.SUM)   # distinct probes per rank
+        relax_total, e2e_relax, alg_bytes = rl.tolist()
+    peak, peak_kind = _peaks()
+    achieved = alg_bytes / fill_s / 1e9 if fill_s > 0 else 0.0
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tf):
+        try:
+            traffic = json.load(open(tf)).get(w.name)
+        except Exception:
+            traffic = None
+    st0 = stats[0]
+    line = {
+        "metric": METRIC, "value": relax_total / t_total, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_total / args.steps,
+        "higher_is_better": True,
+        "scaling": "strong" if (world > 1 and mode == P.MODE_LEVEL_SHARDED) else "weak",
+        "vs_baseline": None, "dtype": args.dtype_label or "u8", "data": "synthetic",
+        "config": {"workload": w.name, "n": w.n, "m": w.m, "eps": w.eps, "P_jobs": w.P, "seed": w.seed,
+                   "probes_per_round": Pp, "mode": {0: "single", 1: "level_sharded", 2: "multi_probe"}[mode],
+                   "probes": st0["probes"], "unique_dps": st0["unique_dps"], "T_star": st0["T_star"],
+                   "sigma_max": st0["sigma_max"], "relax_per_step": relax_total / args.steps,
+                   "l2": "flushed between steps (256 MiB write)"},
+        "solve_ms": 1e3 * t_total / args.steps,
+        "e2e": {"value": e2e_relax / e2e_t, "unit": UNIT,
+                "h2d_bytes_per_step": int(sum(s["h2d_bytes"] for s in e2e_stats) / args.steps),
+                "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e2e_stats) / args.steps),
+                "solve_ms": 1e3 * e2e_t / args.steps},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "kernel": "row_fill_kernel (level fill)",
+                     "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)" if peak_kind == "measured" else "fallback",
+                     "fill_ms_per_step": 1e3 * fill_s / args.steps,
+                     "fill_launches_per_step": fill_launches / args.steps,
+                     "alg_bytes_per_step": alg_bytes / args.steps,
+                     "fill_relax_per_s": relax_total / fill_s if fill_s > 0 else None},
+        "gpu_launches": int(launches),
+        "clocks": clocks,
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_oracle_sample(w)
+    if comm is not None:
+        comm.destroy()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", default="M2s", choices=sorted(WORKLOADS))
+    ap.add_argument("--P", type=int, default=1, help="probes per round (single GPU)")
+    ap.add_argument("--mode", choices=["sharded", "multiprobe"], default="sharded", help="N>1 mode")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--dtype-label", default=None)
+    args = ap.parse_args()
+    w = WORKLOADS[args.workload]
+    if args.dtype_label is None:
+        N, _r, _T = _largest_dp(w)
+        args.dtype_label = "u8" if int(np.sum(N)) <= 255 else "u16"
+    if args.impl == "reference":
+        return run_reference(args, w)
+    return run_ours(args, w)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,222 @@
+/*
+ * ptas.h — C ABI of the B200-native PTAS hot path (libptas_b200.so).
+ *
+ * Method: Li, Ghalami, Schwiebert, Grosu, "A GPU Parallel Approximation
+ * Algorithm for Scheduling Parallel Identical Machines to Minimize
+ * Makespan", IPDPS workshops 2018.  Citations are
+ * PAPER.md:<line> (section / algorithm / equation).
+ *
+ * Conventions (all entry points):
+ *  - Every function returns an int status: PTAS_OK (0) or a negative
+ *    PTAS_E* code; ptas_strerror() names it.  On error nothing partial is
+ *    written to any output argument.
+ *  - Ownership: the caller owns every pointer argument.  The library never
+ *    frees caller memory and keeps no pointer after a call returns (except
+ *    the opaque ptas_comm it creates, released by ptas_comm_destroy).
+ *    Device workspace is allocated and cached internally per device.
+ *  - Host pointers are ordinary (pageable or pinned) host memory; "device"
+ *    pointers are CUDA global-memory pointers on the current device
+ *    (e.g. torch.Tensor.data_ptr()).
+ *  - Table layout: row-major over the classes in the order given, last
+ *    class fastest, elem_bytes per entry (1 = uint8 when sum(counts) <= 255,
+ *    else 2 = uint16; OPT(n) <= sum(n) so the value always fits).
+ *  - Determinism: outputs are a pure function of the inputs and
+ *    probes_per_round; they do not depend on mode or GPU count.
+ *  - Thread safety: calls on different devices may run concurrently; calls
+ *    on one device are serialised by an internal per-device lock.
+ */
+#ifndef PTAS_B200_H
+#define PTAS_B200_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+    PTAS_OK = 0,
+    PTAS_EINVAL = -1,     /* invalid argument (see each function)              */
+    PTAS_ETOOBIG = -2,    /* sigma overflows / exceeds the table budget,
+                             sum(counts) > 65535, or digits do not pack        */
+    PTAS_ENOMEM = -3,     /* device or host allocation failed                  */
+    PTAS_ECUDA = -4,      /* CUDA runtime error (no device, launch failure)    */
+    PTAS_ENCCL = -5,      /* NCCL missing or failed                            */
+    PTAS_EINTERNAL = -6   /* internal invariant violated (a bug)               */
+};
+
+enum {
+    PTAS_MODE_SINGLE = 0,        /* one GPU                                          */
+    PTAS_MODE_LEVEL_SHARDED = 1, /* each row-level split over the ranks of comm,
+                                    slices NCCL all-gathered         */
+    PTAS_MODE_MULTI_PROBE = 2    /* one T probe per rank per round (Alg 3 quarter
+                                    split generalised)            */
+};
+
+typedef struct ptas_comm ptas_comm; /* opaque; wraps an ncclComm_t */
+
+typedef struct {
+    int32_t probes_per_round;   /* P >= 1; 1 = Alg 1 bisection (default).  In
+                                   MULTI_PROBE mode it must equal the comm size. */
+    int32_t mode;               /* PTAS_MODE_*                                     */
+    int32_t device;             /* CUDA device (-1 = current)                      */
+    ptas_comm *comm;            /* NULL = single GPU                               */
+    int64_t table_budget_bytes; /* 0 = auto: free HBM minus a 2 GiB reserve        */
+    int32_t memoize;            /* 1 (default) reuse OPT(N) across equal DP keys   */
+    int32_t virtual_shards;     /* >1 with mode LEVEL_SHARDED and comm == NULL:
+                                   run that many logical shards on one GPU
+                                   (slice + gather + scatter), for testing          */
+    int32_t layout;             /* 0 = internal class order chosen by the library
+                                   (largest count fastest); 1 = classes in
+                                   ascending-size order as classified             */
+} ptas_options;
+
+typedef struct {
+    int32_t probes, rounds, unique_dps, K_at_Tstar;
+    int64_t T_star, sigma_max, opt_at_Tstar;
+    double relaxations;     /* closed-form (n,s) pairs over executed DPs       */
+    double dp_seconds;      /* device time of all DP work (CUDA events)        */
+    double fill_seconds;    /* device time of the level-fill loops             */
+    double total_seconds;   /* host wall time of the call                      */
+    double alg_bytes;       /* level-fill algorithmic bytes: sum (relax+sigma)*e */
+    int64_t states;         /* sum of sigma over executed DPs                  */
+    int32_t kernel_launches;/* kernels launched by the library in this call    */
+    int32_t fill_launches;  /* of which level-fill launches                    */
+    int64_t h2d_bytes, d2h_bytes; /* host<->device bytes moved by this call    */
+} ptas_stats;
+
+typedef struct {
+    int64_t T;        /* probe target makespan                              */
+    int32_t round;    /* search round (0-based)                             */
+    int32_t feasible; /* OPT(N) <= m                                        */
+    int32_t K;        /* non-empty classes at T                             */
+    int32_t opt;      /* OPT(N) (0 if no long job)                          */
+    int64_t sigma;    /* DP table size prod(N_i+1)                          */
+    int32_t memo_hit; /* 1 if OPT(N) came from the memo                     */
+    int32_t rank;     /* rank that evaluated the probe (MULTI_PROBE)        */
+} ptas_probe;
+
+/* Default options (P = 1, SINGLE, current device, memoize, auto budget). */
+void ptas_default_options(ptas_options *opt);
+
+/* ---------------------------------------------------------------- solve
+ * PTAS for P||Cmax — Alg 1 with the P-probe search of
+ * Alg 3 (reading R8 in DESIGN.md), the k-dimensional DP
+ * of Eq. 1 on the GPU per probe, and the schedule from
+ * DP(T*) with short jobs placed greedily.
+ *   p[n]       host, processing times, each >= 1
+ *   n >= 1, m >= 1, eps > 0 finite (k = ceil(1/eps))
+ *   opt        nullable (defaults)
+ *   makespan_out  host int64, the schedule's makespan (actual sizes)
+ *   assignment_out host int32[n], machine 0..m-1 of each job
+ *   stats      nullable
+ * EINVAL: n<1, m<1, eps<=0 or non-finite, any p<1, sum(p) overflow,
+ *         P<1, bad mode/comm combination.  ETOOBIG: a probe's DP table
+ *         exceeds the budget. */
+int ptas_solve(const int64_t *p, int32_t n, int32_t m, double eps,
+               const ptas_options *opt, int64_t *makespan_out,
+               int32_t *assignment_out, ptas_stats *stats);
+
+/* As ptas_solve, plus the probe log (log nullable, log_cap entries;
+ * *log_len = number of probes, which may exceed log_cap). */
+int ptas_solve_ex(const int64_t *p, int32_t n, int32_t m, double eps,
+                  const ptas_options *opt, int64_t *makespan_out,
+                  int32_t *assignment_out, ptas_stats *stats,
+                  ptas_probe *log, int32_t log_cap, int32_t *log_len);
+
+/* Device-resident variant: d_p (int64[n]) and d_assignment (int32[n]) are
+ * device pointers on the chosen device; makespan_out is host.  The host
+ * driver stages p to host memory internally (counted in stats->d2h_bytes). */
+int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps,
+                      const ptas_options *opt, int64_t *makespan_out,
+                      int32_t *d_assignment, ptas_stats *stats);
+
+/* ---------------------------------------------------------------- DP
+ * sigma = prod(counts[i]+1) (Alg 2 l.2) and the entry size.
+ * EINVAL: K<0, K>64, counts[i]<0.  ETOOBIG: sigma overflows int64 or
+ * sum(counts) > 65535. */
+int dp_table_shape(const int32_t *counts, int32_t K, int64_t *sigma_out,
+                   int32_t *elem_bytes_out);
+
+/* Fill the whole DP table of Eq. 1:
+ *   OPT(0) = 0,  OPT(n) = 1 + min_{s in C(T), s <= n} OPT(n - s),
+ *   C(T) = { s != 0 : 0 <= s_i <= counts_i, sum s_i sizes_i <= T }
+ * (Alg 2 l.17).  counts/sizes are host arrays of length K in
+ * the class order the table is laid out in.
+ *   table_out  host, nullable ("just OPT(N)"), table_bytes >= sigma*e
+ *   opt_N_out  host int32, OPT(counts)
+ *   stats      nullable (relaxations, fill_seconds, ...)
+ * EINVAL: K<0 or >64, counts<0, sizes<1, T<1, a size > T with count > 0,
+ *         table_out != NULL with table_bytes < sigma*e.  ETOOBIG as
+ *         dp_table_shape or sigma*e over the budget.  K = 0 gives
+ *         sigma = 1 and OPT = 0. */
+int dp_fill(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T,
+            void *table_out, int64_t table_bytes, int32_t *opt_N_out,
+            ptas_stats *stats);
+
+/* As dp_fill, into a caller-owned device buffer d_table (>= sigma*e bytes,
+ * e.g. a torch uint8/uint16 tensor) on the current device, enqueued on
+ * cuda_stream (a cudaStream_t; NULL = legacy default stream).  The call
+ * synchronises the stream once at the end to read OPT(N). */
+int dp_fill_device(const int32_t *counts, const int64_t *sizes, int32_t K,
+                   int64_t T, void *d_table, int64_t table_bytes,
+                   void *cuda_stream, int32_t *opt_N_out);
+
+/* ---------------------------------------------------------------- multi-GPU
+ * NCCL communicator over NVLink for LEVEL_SHARDED / MULTI_PROBE modes.  One
+ * process per GPU; the 128-byte unique id is made on rank 0 and broadcast
+ * by the caller (e.g. torch.distributed).  NCCL is loaded at run time
+ * (libnccl.so.2); PTAS_ENCCL if it is absent. */
+int ptas_get_unique_id(void *out128);
+int ptas_comm_init(ptas_comm **c, int32_t rank, int32_t world,
+                   const void *unique_id128, int32_t device);
+int ptas_comm_destroy(ptas_comm *c);
+
+const char *ptas_strerror(int status);
+
+/* ---------------------------------------------------------------- host steps
+ * The host-side steps of the driver, exported so they can be checked on a
+ * machine without a GPU.  Pure functions, no CUDA calls. */
+
+/* k = ceil(1/eps).  Returns k, or PTAS_EINVAL. */
+int ptas_k(double eps);
+/* LB, UB of Alg 1 l.2-3. */
+int ptas_bounds(const int64_t *p, int32_t n, int32_t m, int64_t *LB, int64_t *UB);
+/* Long/short split and rounding of Alg 1 l.6-8:
+ * u = max(1, floor(T/k^2)), long iff k*p > T, r = floor(p/u)*u, classes =
+ * distinct r ascending.  r_out, N_out have room for n; cls_out[n] = class
+ * or -1 (short). */
+int ptas_classify(const int64_t *p, int32_t n, int64_t T, int32_t k,
+                  int64_t *u_out, int32_t *K_out, int64_t *r_out,
+                  int32_t *N_out, int32_t *cls_out);
+/* Probe targets of one round: T_j = LB + floor((2j+1)(UB-LB)/(2P)),
+ * deduplicated (out has room for P).  EINVAL if LB >= UB or P < 1. */
+int ptas_probe_targets(int64_t LB, int64_t UB, int32_t P, int64_t *out,
+                       int32_t *count);
+/* Interval update after a round (Alg 1 l.10-14 for P = 1; Alg 3 l.13-25
+ * as read in DESIGN.md R8). */
+int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T,
+                         const int32_t *feasible, int32_t count);
+/* Contiguous slice [begin, end) of `count` items owned by `rank` of
+ * `world` (ceil split; trailing ranks may be empty). */
+int ptas_shard_range(int64_t count, int32_t rank, int32_t world,
+                     int64_t *begin, int64_t *end);
+
+/* ---------------------------------------------------------------- inspection
+ * Device steps exposed for parity tests (need a GPU). */
+
+/* Configuration set C(T) as enumerated by the device kernel, canonical
+ * lexicographic order; out_digits[count*K] (nullable when cap == 0). */
+int dp_configs(const int32_t *counts, const int64_t *sizes, int32_t K,
+               int64_t T, int32_t *out_digits, int64_t cap, int64_t *count);
+/* Row-level index (level structure over the K-1 leading classes):
+ * level_start[rho_max+2] prefix sums of row counts per row-level and, for
+ * every row slot in row-level order, its table offset (row base index).
+ * out_rowbase has room for sigma / (counts[K-1]+1) entries (nullable). */
+int dp_row_index(const int32_t *counts, int32_t K, int64_t *level_start,
+                 int64_t level_cap, int64_t *out_rowbase, int64_t rows_cap);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PTAS_B200_H */

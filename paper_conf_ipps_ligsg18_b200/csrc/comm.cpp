@@ -1,0 +1,113 @@
+// comm.cpp — NCCL over NVLink/NVSwitch for the multi-GPU modes.
+//
+// NCCL is loaded at run time (dlopen "libnccl.so.2") so the library loads and
+// the single-GPU path works without it.  Under PyTorch the already-loaded
+// torch NCCL is reused (same soname).  The 128-byte unique id is created on
+// rank 0 (ptas_get_unique_id) and broadcast by the caller (torch.distributed).
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <cstring>
+#include <mutex>
+
+#include "engine.h"
+
+struct ptas_comm {
+    ncclComm_t comm;
+    int rank;
+    int world;
+    int device;
+};
+
+namespace {
+
+struct NcclApi {
+    bool ok = false;
+    decltype(&ncclGetUniqueId) getUniqueId = nullptr;
+    decltype(&ncclCommInitRank) commInitRank = nullptr;
+    decltype(&ncclAllGather) allGather = nullptr;
+    decltype(&ncclCommDestroy) commDestroy = nullptr;
+};
+
+NcclApi *nccl()
+{
+    static NcclApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) return;
+        api.getUniqueId = (decltype(api.getUniqueId))dlsym(h, "ncclGetUniqueId");
+        api.commInitRank = (decltype(api.commInitRank))dlsym(h, "ncclCommInitRank");
+        api.allGather = (decltype(api.allGather))dlsym(h, "ncclAllGather");
+        api.commDestroy = (decltype(api.commDestroy))dlsym(h, "ncclCommDestroy");
+        api.ok = api.getUniqueId && api.commInitRank && api.allGather && api.commDestroy;
+    });
+    return &api;
+}
+
+}  // namespace
+
+extern "C" int ptas_get_unique_id(void *out128)
+{
+    if (!out128) return PTAS_EINVAL;
+    NcclApi *a = nccl();
+    if (!a->ok) return PTAS_ENCCL;
+    ncclUniqueId id;
+    if (a->getUniqueId(&id) != ncclSuccess) return PTAS_ENCCL;
+    static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(out128, &id, sizeof(id));
+    return PTAS_OK;
+}
+
+extern "C" int ptas_comm_init(ptas_comm **c, int32_t rank, int32_t world, const void *unique_id128,
+                              int32_t device)
+{
+    if (!c || !unique_id128 || world < 1 || rank < 0 || rank >= world) return PTAS_EINVAL;
+    NcclApi *a = nccl();
+    if (!a->ok) return PTAS_ENCCL;
+    if (device < 0) {
+        if (cudaGetDevice(&device) != cudaSuccess) return PTAS_ECUDA;
+    }
+    if (cudaSetDevice(device) != cudaSuccess) return PTAS_ECUDA;
+    ncclUniqueId id;
+    std::memcpy(&id, unique_id128, sizeof(id));
+    ptas_comm *pc = new ptas_comm();
+    if (a->commInitRank(&pc->comm, world, id, rank) != ncclSuccess) {
+        delete pc;
+        return PTAS_ENCCL;
+    }
+    pc->rank = rank;
+    pc->world = world;
+    pc->device = device;
+    *c = pc;
+    return PTAS_OK;
+}
+
+extern "C" int ptas_comm_destroy(ptas_comm *c)
+{
+    if (!c) return PTAS_EINVAL;
+    NcclApi *a = nccl();
+    int rc = PTAS_OK;
+    if (a->ok && a->commDestroy(c->comm) != ncclSuccess) rc = PTAS_ENCCL;
+    delete c;
+    return rc;
+}
+
+namespace ptas {
+
+int comm_rank(const ptas_comm *c) { return c ? c->rank : 0; }
+int comm_world(const ptas_comm *c) { return c ? c->world : 1; }
+
+// In-place all-gather: recv holds world * bytes_per_rank bytes; rank r's
+// block is recv + r * bytes_per_rank (send may point there).
+int comm_allgather(ptas_comm *c, const void *send, void *recv, size_t bytes_per_rank, cudaStream_t st)
+{
+    NcclApi *a = nccl();
+    if (!a->ok || !c) return PTAS_ENCCL;
+    if (a->allGather(send, recv, bytes_per_rank, ncclUint8, c->comm, st) != ncclSuccess)
+        return PTAS_ENCCL;
+    return PTAS_OK;
+}
+
+}  // namespace ptas

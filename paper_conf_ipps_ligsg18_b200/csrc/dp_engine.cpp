@@ -1,0 +1,543 @@
+// dp_engine.cpp — per-device orchestration of one DP(N, T) on the GPU.
+//
+// One DP = §8(a) rows a-2 .. a-6:
+//   a-2 table geometry, budget guard (host, O(K))
+//   a-3 enum_configs (2 passes + scan) and build_prefix kernels
+//   a-4 row-level sizes = coefficients of prod_{i<K-1} (1 + z + ... + z^{N_i})
+//       (host, the cnt[] suffix-count table, uploaded once) + on-device
+//       unranking inside the fill kernels
+//   a-5 one row_fill launch per row-level rho = 0 .. sum_{i<K-1} N_i
+//       (optionally sharded: compact slice -> NCCL all-gather -> scatter)
+//   a-6 OPT(N) read back with the planning summary in one 40-byte D2H.
+// Host syncs per DP: one after the config count (to size C), one at the end.
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <numeric>
+
+#include "engine.h"
+
+namespace ptas {
+
+#define PT_CK(x)                                                                   \
+    do {                                                                           \
+        cudaError_t e__ = (x);                                                     \
+        if (e__ != cudaSuccess) {                                                  \
+            cudaGetLastError();                                                    \
+            return e__ == cudaErrorMemoryAllocation ? PTAS_ENOMEM : PTAS_ECUDA;    \
+        }                                                                          \
+    } while (0)
+
+cudaError_t Engine::Buf::ensure(size_t bytes)
+{
+    if (p && bytes <= cap) return cudaSuccess;
+    if (p) {
+        cudaFree(p);
+        p = nullptr;
+        cap = 0;
+    }
+    size_t want = bytes < 256 ? 256 : bytes;
+    cudaError_t e = cudaMalloc(&p, want);
+    if (e != cudaSuccess) {
+        p = nullptr;
+        cap = 0;
+        cudaGetLastError();
+        return e;
+    }
+    cap = want;
+    return cudaSuccess;
+}
+
+static std::mutex g_reg_mu;
+static std::map<int, Engine *> g_engines;
+
+int Engine::get(int device, Engine **out)
+{
+    std::lock_guard<std::mutex> lk(g_reg_mu);
+    auto it = g_engines.find(device);
+    if (it != g_engines.end()) {
+        *out = it->second;
+        return PTAS_OK;
+    }
+    Engine *e = new Engine();
+    int rc = e->init(device);
+    if (rc) {
+        delete e;
+        return rc;
+    }
+    g_engines[device] = e;
+    *out = e;
+    return PTAS_OK;
+}
+
+int Engine::init(int device)
+{
+    device_ = device;
+    PT_CK(cudaSetDevice(device));
+    PT_CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device));
+    PT_CK(cudaStreamCreateWithFlags(&stream_, cudaStreamNonBlocking));
+    for (auto &ev : ev_) PT_CK(cudaEventCreate(&ev));
+    PT_CK(cudaMalloc(&d_meta_, sizeof(DpMeta)));
+    PT_CK(cudaMallocHost(&h_meta_, sizeof(DpMeta)));
+    PT_CK(cudaMallocHost(&h_scalar_, 64));
+    return PTAS_OK;
+}
+
+int64_t Engine::free_budget()
+{
+    size_t fr = 0, tot = 0;
+    if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    int64_t b = (int64_t)fr + (int64_t)table_.cap - ((int64_t)2 << 30);
+    return b > 0 ? b : 0;
+}
+
+static int bits_of(int32_t x)
+{
+    int b = 0;
+    while (x) {
+        ++b;
+        x >>= 1;
+    }
+    return b;
+}
+
+// Geometry of the row space of an internal-order DP (a-2, a-4).
+static int build_geom(const std::vector<int32_t> &N, RowGeom *g, std::vector<int64_t> *cnt,
+                      std::vector<int64_t> *stride)
+{
+    const int K = (int)N.size();
+    std::memset(g, 0, sizeof(*g));
+    stride->assign(K, 1);
+    for (int i = K - 2; i >= 0; --i) (*stride)[i] = (*stride)[i + 1] * (N[i + 1] + 1);
+    g->K1 = K - 1;
+    g->W = N[K - 1] + 1;
+    int rho_max = 0;
+    for (int i = 0; i < K - 1; ++i) {
+        g->N[i] = N[i];
+        g->stride[i] = (*stride)[i];
+        rho_max += N[i];
+    }
+    g->rho_max = rho_max;
+    g->maxsuf[K - 1] = 0;
+    for (int i = K - 2; i >= 0; --i) g->maxsuf[i] = g->maxsuf[i + 1] + N[i];
+    int word = 0, bit = 0;
+    // PTAS_FORCE_TWO_WORDS=1 (tests only): split the leading digits over two
+    // words even when they fit in one, to exercise the two-word kernels.
+    const char *force2 = std::getenv("PTAS_FORCE_TWO_WORDS");
+    const int split = (force2 && force2[0] == '1' && K - 1 >= 2) ? (K - 1) / 2 : -1;
+    for (int i = 0; i < K - 1; ++i) {
+        int w = bits_of(N[i]) + 1;
+        if (bit + w > 64 || i == split) {
+            ++word;
+            bit = 0;
+        }
+        if (word >= MAXW) return PTAS_ETOOBIG;
+        g->word[i] = (uint8_t)word;
+        g->shift[i] = (uint8_t)bit;
+        g->guard[word] |= 1ull << (bit + w - 1);
+        bit += w;
+    }
+    g->nwords = K > 1 ? word + 1 : 0;
+    // cnt[i][L] = #{(p_i..p_{K1-1}) : 0 <= p_d <= N_d, sum = L}; cnt[K1][0] = 1
+    const int K1 = K - 1, ld = rho_max + 1;
+    cnt->assign((size_t)(K1 + 1) * ld, 0);
+    (*cnt)[(size_t)K1 * ld + 0] = 1;
+    for (int i = K1 - 1; i >= 0; --i)
+        for (int L = 0; L <= rho_max; ++L) {
+            int64_t s = 0;
+            for (int v = 0; v <= N[i] && v <= L; ++v) s += (*cnt)[(size_t)(i + 1) * ld + (L - v)];
+            (*cnt)[(size_t)i * ld + L] = s;
+        }
+    return PTAS_OK;
+}
+
+// internal order: the non-empty canonical classes, in rq.order or identity
+static int internal_order(const DpRequest &rq, std::vector<int> *order)
+{
+    order->clear();
+    if (rq.order) {
+        int ne = 0;
+        for (int i = 0; i < rq.K; ++i) ne += rq.N[i] > 0;
+        for (int i = 0; i < ne; ++i) order->push_back(rq.order[i]);
+    } else {
+        for (int i = 0; i < rq.K; ++i)
+            if (rq.N[i] > 0) order->push_back(i);
+    }
+    if ((int)order->size() > MAXK) return PTAS_ETOOBIG;
+    return PTAS_OK;
+}
+
+int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
+{
+    DpOutcome o;
+    cudaStream_t st = rq.stream ? rq.stream : stream_;
+    std::vector<int> order;
+    int rc = internal_order(rq, &order);
+    if (rc) return rc;
+    const int K = (int)order.size();
+    std::vector<int32_t> N(K);
+    std::vector<int64_t> r(K);
+    __int128 sg = 1;
+    int64_t sumN = 0;
+    for (int i = 0; i < K; ++i) {
+        N[i] = rq.N[order[i]];
+        r[i] = rq.r[order[i]];
+        sumN += N[i];
+        sg *= (N[i] + 1);
+        if (sg > (__int128)INT64_MAX) return PTAS_ETOOBIG;
+    }
+    if (sumN > 65535) return PTAS_ETOOBIG;
+    const int64_t sigma = (int64_t)sg;
+    const int e = sumN <= 255 ? 1 : 2;
+    const int64_t bytes = sigma * e;
+    void *table = rq.ext_table;
+    if (table) {
+        if (rq.ext_bytes < bytes) return PTAS_EINVAL;
+    } else {
+        int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
+        if (bytes > budget) return PTAS_ETOOBIG;
+        PT_CK(table_.ensure((size_t)bytes));
+        table = table_.p;
+    }
+    last_valid_ = false;
+    o.sigma = sigma;
+    o.e = e;
+    o.Kint = K;
+    PT_CK(cudaEventRecord(ev_[0], st));
+    if (K == 0) {
+        PT_CK(launch_fill_value(table, e, 0, st));
+        PT_CK(cudaEventRecord(ev_[1], st));
+        PT_CK(cudaEventRecord(ev_[2], st));
+        PT_CK(cudaEventRecord(ev_[3], st));
+        PT_CK(cudaStreamSynchronize(st));
+        o.launches = 1;
+        o.opt = 0;
+        last_valid_ = true;
+        last_table_ = table;
+        last_stream_ = st;
+        last_K_ = 0;
+        last_Kcanon_ = rq.K;
+        last_e_ = e;
+        last_sigma_ = 1;
+        last_nC_ = 0;
+        last_opt_ = 0;
+        last_order_.clear();
+        *out = o;
+        return PTAS_OK;
+    }
+    RowGeom g;
+    std::vector<int64_t> cnt, stride;
+    rc = build_geom(N, &g, &cnt, &stride);
+    if (rc) return rc;
+
+    // ---- uploads: r[K] int64 | stride[K] int64 | hi[K] int32, then cnt table
+    std::vector<int32_t> hi(K);
+    for (int i = 0; i < K; ++i) {
+        int64_t b = rq.T / r[i];
+        hi[i] = (int32_t)(b < N[i] ? b : N[i]);
+    }
+    const size_t small_bytes = (size_t)K * (4 + 8 + 8);
+    std::vector<unsigned char> small(small_bytes);
+    std::memcpy(small.data(), r.data(), (size_t)K * 8);
+    std::memcpy(small.data() + K * 8, stride.data(), (size_t)K * 8);
+    std::memcpy(small.data() + K * 16, hi.data(), (size_t)K * 4);
+    PT_CK(small_.ensure(small_bytes));
+    PT_CK(cnt_.ensure(cnt.size() * 8));
+    PT_CK(cudaMemcpyAsync(small_.p, small.data(), small_bytes, cudaMemcpyHostToDevice, st));
+    PT_CK(cudaMemcpyAsync(cnt_.p, cnt.data(), cnt.size() * 8, cudaMemcpyHostToDevice, st));
+    o.h2d += (int64_t)(small_bytes + cnt.size() * 8);
+    const int64_t *d_r = (const int64_t *)small_.p;
+    const int64_t *d_stride = (const int64_t *)((unsigned char *)small_.p + K * 8);
+    const int32_t *d_hi = (const int32_t *)((unsigned char *)small_.p + K * 16);
+
+    // ---- a-3 configuration enumeration
+    int D = 0;
+    int64_t nprefix = 1;
+    while (D < K && nprefix * (hi[D] + 1) <= 65536) {
+        nprefix *= hi[D] + 1;
+        ++D;
+    }
+    PT_CK(counts_.ensure((size_t)nprefix * 8));
+    PT_CK(offsets_.ensure((size_t)(nprefix + 1) * 8));
+    int64_t *d_counts = (int64_t *)counts_.p;
+    int64_t *d_offsets = (int64_t *)offsets_.p;
+    PT_CK(launch_enum_configs(0, K, D, nprefix, d_hi, d_r, rq.T, d_stride, d_counts, nullptr,
+                              nullptr, nullptr, st));
+    PT_CK(launch_exclusive_scan(d_counts, d_offsets, nprefix, d_offsets + nprefix, st));
+    PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaStreamSynchronize(st));
+    o.d2h += 8;
+    o.launches += 2;
+    const int64_t nC = h_scalar_[0];
+    if (nC <= 0) return PTAS_EINTERNAL;  // (0,..,0,1) is always feasible
+    PT_CK(digits_.ensure((size_t)nC * K * 2));
+    PT_CK(off_.ensure((size_t)nC * 8));
+    PT_CK(pref_.ensure((size_t)nC * sizeof(PrefixEntry)));
+    PT_CK(launch_enum_configs(1, K, D, nprefix, d_hi, d_r, rq.T, d_stride, d_counts, d_offsets,
+                              (uint16_t *)digits_.p, (int64_t *)off_.p, st));
+    PT_CK(launch_build_prefix(K, (const uint16_t *)digits_.p, (const int64_t *)off_.p, nC, g,
+                              N.data(), (PrefixEntry *)pref_.p, d_meta_, st));
+    o.launches += 2;
+    const int J0 = (int)std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
+
+    // ---- a-5 level fill, one launch per row-level
+    int G = 1, myrank = 0;
+    bool virt = false;
+    const ShardCtx *sh = rq.shard;
+    if (sh) {
+        if (sh->comm) {
+            G = sh->world;
+            myrank = sh->rank;
+        } else if (sh->virtual_shards > 1) {
+            G = sh->virtual_shards;
+            virt = true;
+        }
+    }
+    const int ld = g.rho_max + 1;
+    auto sharded = [&](int64_t R) { return G > 1 && R >= std::max<int64_t>(sh->min_rows, 1); };
+    if (G > 1) {
+        size_t mx = 0;
+        for (int rho = 0; rho <= g.rho_max; ++rho) {
+            int64_t R = cnt[rho];
+            if (!sharded(R)) continue;
+            int64_t chunk = (R + G - 1) / G;
+            mx = std::max(mx, (size_t)(chunk * G * g.W * e));
+        }
+        PT_CK(stage_.ensure(mx));
+    }
+    PT_CK(cudaEventRecord(ev_[1], st));
+    for (int rho = 0; rho <= g.rho_max; ++rho) {
+        const int64_t R = cnt[rho];
+        if (R <= 0) continue;
+        if (!sharded(R)) {
+            PT_CK(launch_row_fill(e, table, g, (const int64_t *)cnt_.p, (const PrefixEntry *)pref_.p,
+                                  d_meta_, nC, J0, rho, 0, R, nullptr, sm_count_, st));
+            ++o.fill_launches;
+            continue;
+        }
+        const int64_t chunk = (R + G - 1) / G;
+        unsigned char *stage = (unsigned char *)stage_.p;
+        if (virt) {
+            for (int v = 0; v < G; ++v) {
+                int64_t b = v * chunk, c = std::min(R, b + chunk) - b;
+                if (c <= 0) continue;
+                PT_CK(launch_row_fill(e, table, g, (const int64_t *)cnt_.p,
+                                      (const PrefixEntry *)pref_.p, d_meta_, nC, J0, rho, b, c,
+                                      stage + b * g.W * e, sm_count_, st));
+                ++o.fill_launches;
+            }
+        } else {
+            int64_t b = myrank * chunk, c = std::min(R, b + chunk) - b;
+            if (c > 0) {
+                PT_CK(launch_row_fill(e, table, g, (const int64_t *)cnt_.p,
+                                      (const PrefixEntry *)pref_.p, d_meta_, nC, J0, rho, b, c,
+                                      stage + b * g.W * e, sm_count_, st));
+                ++o.fill_launches;
+            }
+            int crc = comm_allgather(sh->comm, stage + (size_t)myrank * chunk * g.W * e, stage,
+                                     (size_t)(chunk * g.W * e), st);
+            if (crc) return crc;
+        }
+        PT_CK(launch_row_scatter(e, table, g, (const int64_t *)cnt_.p, rho, R, stage, sm_count_, st));
+        ++o.launches;
+    }
+    PT_CK(cudaEventRecord(ev_[2], st));
+    o.launches += o.fill_launches;
+    (void)ld;
+
+    // ---- a-6 readout
+    PT_CK(launch_read_opt(e, table, sigma - 1, d_meta_, st));
+    ++o.launches;
+    PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaEventRecord(ev_[3], st));
+    PT_CK(cudaStreamSynchronize(st));
+    o.d2h += sizeof(DpMeta);
+    float ms = 0;
+    PT_CK(cudaEventElapsedTime(&ms, ev_[0], ev_[3]));
+    o.dp_s = ms * 1e-3;
+    PT_CK(cudaEventElapsedTime(&ms, ev_[1], ev_[2]));
+    o.fill_s = ms * 1e-3;
+    o.opt = h_meta_->opt;
+    o.relax = (double)h_meta_->relax;
+    o.nC = h_meta_->nC;
+    o.nP = h_meta_->nP;
+
+    last_valid_ = true;
+    last_table_ = table;
+    last_stream_ = st;
+    last_K_ = K;
+    last_Kcanon_ = rq.K;
+    last_e_ = e;
+    last_sigma_ = sigma;
+    last_nC_ = nC;
+    last_opt_ = o.opt;
+    last_order_ = order;
+    last_N_ = N;
+    last_stride_ = stride;
+    *out = o;
+    return PTAS_OK;
+}
+
+int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
+{
+    if (!last_valid_) return PTAS_EINTERNAL;
+    if (last_K_ == 0 || last_opt_ == 0) return PTAS_OK;
+    const int K = last_K_;
+    const int64_t nC = last_nC_;
+    cudaStream_t st = last_stream_;
+    std::vector<uint16_t> dig((size_t)nC * K);
+    PT_CK(cudaMemcpyAsync(dig.data(), digits_.p, dig.size() * 2, cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaStreamSynchronize(st));
+    acc->d2h += (int64_t)dig.size() * 2;
+    // canonical lexicographic rank of every configuration (reading R11)
+    std::vector<std::vector<int32_t>> canon((size_t)nC, std::vector<int32_t>(last_Kcanon_, 0));
+    for (int64_t c = 0; c < nC; ++c)
+        for (int i = 0; i < K; ++i) canon[c][last_order_[i]] = dig[(size_t)c * K + i];
+    std::vector<int32_t> idx((size_t)nC);
+    std::iota(idx.begin(), idx.end(), 0);
+    std::sort(idx.begin(), idx.end(), [&](int32_t a, int32_t b) { return canon[a] < canon[b]; });
+    std::vector<int32_t> rank((size_t)nC);
+    for (int64_t q = 0; q < nC; ++q) rank[idx[q]] = (int32_t)q;
+    const size_t tb_bytes = (size_t)nC * 4 + (size_t)K * 4 + (size_t)K * 8 + (size_t)last_opt_ * 4 + 16;
+    PT_CK(tb_.ensure(tb_bytes));
+    unsigned char *b = (unsigned char *)tb_.p;
+    int64_t *d_stride = (int64_t *)b;
+    int32_t *d_rank = (int32_t *)(b + (size_t)K * 8);
+    int32_t *d_N = d_rank + nC;
+    int32_t *d_len = d_N + K;
+    int32_t *d_out = d_len + 4;
+    PT_CK(cudaMemcpyAsync(d_stride, last_stride_.data(), (size_t)K * 8, cudaMemcpyHostToDevice, st));
+    PT_CK(cudaMemcpyAsync(d_rank, rank.data(), (size_t)nC * 4, cudaMemcpyHostToDevice, st));
+    PT_CK(cudaMemcpyAsync(d_N, last_N_.data(), (size_t)K * 4, cudaMemcpyHostToDevice, st));
+    PT_CK(cudaMemsetAsync(&d_meta_->err, 0, 4, st));
+    acc->h2d += (int64_t)(K * 8 + nC * 4 + K * 4);
+    PT_CK(launch_traceback(last_e_, last_table_, K, d_N, d_stride, (const uint16_t *)digits_.p,
+                           (const int64_t *)off_.p, d_rank, nC, last_sigma_, d_out, last_opt_,
+                           d_len, d_meta_, st));
+    acc->launches += 1;
+    // d_len[0] = length, d_len[4 ..] = chosen configurations (d_out = d_len + 4)
+    std::vector<int32_t> outv((size_t)last_opt_ + 4);
+    PT_CK(cudaMemcpyAsync(outv.data(), d_len, outv.size() * 4, cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaStreamSynchronize(st));
+    acc->d2h += (int64_t)outv.size() * 4 + (int64_t)sizeof(DpMeta);
+    const int32_t len = outv[0];
+    if (h_meta_->err || len != last_opt_) return PTAS_EINTERNAL;
+    const int32_t *chosen = outv.data() + 4;
+    for (int q = 0; q < len; ++q) machines->push_back(canon[chosen[q]]);
+    return PTAS_OK;
+}
+
+int Engine::copy_table_to_host(void *dst, int64_t bytes)
+{
+    if (!last_valid_) return PTAS_EINTERNAL;
+    PT_CK(cudaMemcpyAsync(dst, last_table_, (size_t)bytes, cudaMemcpyDeviceToHost, last_stream_));
+    PT_CK(cudaStreamSynchronize(last_stream_));
+    return PTAS_OK;
+}
+
+int Engine::configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits, int64_t *count)
+{
+    // Runs a full DP on an engine-owned table is unnecessary: enumerate only.
+    std::vector<int> order;
+    int rc = internal_order(rq, &order);
+    if (rc) return rc;
+    const int K = (int)order.size();
+    digits->clear();
+    if (K == 0) {
+        *count = 0;
+        return PTAS_OK;
+    }
+    cudaStream_t st = stream_;
+    std::vector<int32_t> N(K), hi(K);
+    std::vector<int64_t> r(K), stride(K, 1);
+    for (int i = 0; i < K; ++i) {
+        N[i] = rq.N[order[i]];
+        r[i] = rq.r[order[i]];
+    }
+    for (int i = K - 2; i >= 0; --i) stride[i] = stride[i + 1] * (N[i + 1] + 1);
+    for (int i = 0; i < K; ++i) hi[i] = (int32_t)std::min<int64_t>(N[i], rq.T / r[i]);
+    const size_t small_bytes = (size_t)K * 20;
+    std::vector<unsigned char> small(small_bytes);
+    std::memcpy(small.data(), r.data(), (size_t)K * 8);
+    std::memcpy(small.data() + K * 8, stride.data(), (size_t)K * 8);
+    std::memcpy(small.data() + K * 16, hi.data(), (size_t)K * 4);
+    PT_CK(small_.ensure(small_bytes));
+    PT_CK(cudaMemcpyAsync(small_.p, small.data(), small_bytes, cudaMemcpyHostToDevice, st));
+    const int64_t *d_r = (const int64_t *)small_.p;
+    const int64_t *d_stride = (const int64_t *)((unsigned char *)small_.p + K * 8);
+    const int32_t *d_hi = (const int32_t *)((unsigned char *)small_.p + K * 16);
+    int D = 0;
+    int64_t nprefix = 1;
+    while (D < K && nprefix * (hi[D] + 1) <= 65536) {
+        nprefix *= hi[D] + 1;
+        ++D;
+    }
+    PT_CK(counts_.ensure((size_t)nprefix * 8));
+    PT_CK(offsets_.ensure((size_t)(nprefix + 1) * 8));
+    int64_t *d_counts = (int64_t *)counts_.p;
+    int64_t *d_offsets = (int64_t *)offsets_.p;
+    PT_CK(launch_enum_configs(0, K, D, nprefix, d_hi, d_r, rq.T, d_stride, d_counts, nullptr,
+                              nullptr, nullptr, st));
+    PT_CK(launch_exclusive_scan(d_counts, d_offsets, nprefix, d_offsets + nprefix, st));
+    PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaStreamSynchronize(st));
+    const int64_t nC = h_scalar_[0];
+    *count = nC;
+    if (nC == 0) return PTAS_OK;
+    PT_CK(digits_.ensure((size_t)nC * K * 2));
+    PT_CK(off_.ensure((size_t)nC * 8));
+    PT_CK(launch_enum_configs(1, K, D, nprefix, d_hi, d_r, rq.T, d_stride, d_counts, d_offsets,
+                              (uint16_t *)digits_.p, (int64_t *)off_.p, st));
+    std::vector<uint16_t> dig((size_t)nC * K);
+    PT_CK(cudaMemcpyAsync(dig.data(), digits_.p, dig.size() * 2, cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaStreamSynchronize(st));
+    last_valid_ = false;
+    digits->assign((size_t)nC * rq.K, 0);
+    for (int64_t c = 0; c < nC; ++c)
+        for (int i = 0; i < K; ++i) (*digits)[(size_t)c * rq.K + order[i]] = dig[(size_t)c * K + i];
+    return PTAS_OK;
+}
+
+int Engine::row_index(const int32_t *Nc, int Kc, std::vector<int64_t> *level_start,
+                      std::vector<int64_t> *rowbase)
+{
+    std::vector<int32_t> N;
+    for (int i = 0; i < Kc; ++i)
+        if (Nc[i] > 0) N.push_back(Nc[i]);
+    level_start->clear();
+    rowbase->clear();
+    if (N.empty()) {
+        level_start->assign({0, 1});
+        rowbase->assign({0});
+        return PTAS_OK;
+    }
+    RowGeom g;
+    std::vector<int64_t> cnt, stride;
+    int rc = build_geom(N, &g, &cnt, &stride);
+    if (rc) return rc;
+    cudaStream_t st = stream_;
+    PT_CK(cnt_.ensure(cnt.size() * 8));
+    PT_CK(cudaMemcpyAsync(cnt_.p, cnt.data(), cnt.size() * 8, cudaMemcpyHostToDevice, st));
+    int64_t rows = 0;
+    level_start->push_back(0);
+    for (int rho = 0; rho <= g.rho_max; ++rho) {
+        rows += cnt[rho];
+        level_start->push_back(rows);
+    }
+    PT_CK(stage_.ensure((size_t)rows * 8));
+    int64_t *d_out = (int64_t *)stage_.p;
+    for (int rho = 0; rho <= g.rho_max; ++rho)
+        PT_CK(launch_row_index(g, (const int64_t *)cnt_.p, rho, cnt[rho], d_out + (*level_start)[rho], st));
+    rowbase->resize((size_t)rows);
+    PT_CK(cudaMemcpyAsync(rowbase->data(), d_out, (size_t)rows * 8, cudaMemcpyDeviceToHost, st));
+    PT_CK(cudaStreamSynchronize(st));
+    last_valid_ = false;
+    return PTAS_OK;
+}
+
+}  // namespace ptas

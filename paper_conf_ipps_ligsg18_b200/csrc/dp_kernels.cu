@@ -1,0 +1,584 @@
+// dp_kernels.cu — hand-written sm_100a kernels of the PTAS hot path.
+//
+//  enum_configs_kernel   §8(a) a-3: C(T) (Alg 2 l.17), once per T
+//  exclusive_scan_kernel compaction offsets for a-3
+//  build_prefix_kernel   a-3: group C by leading digits, packed words, off(s'),
+//                        closed-form relaxation count
+//  row_fill_kernel       a-5: Eq. 1 for one row-level
+//  row_scatter_kernel    §8(e): gathered compact rows -> mixed-radix table
+//  row_index_kernel      a-4 inspection: row base of every row slot
+//  traceback_kernel      a-8: schedule of the rounded long jobs from DP(T*)
+//
+// Integer-only; no tensor cores (the DP is a min over gathers, not a
+// contraction).  See DESIGN.md for the roofline of each kernel.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "internal.h"
+
+namespace ptas {
+
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int INF = 1 << 28;
+
+// ------------------------------------------------------------------ a-3
+// One thread per prefix over the first D internal dims (mixed radix, first
+// digit most significant, so thread order = lexicographic order).  Each
+// thread walks its completions over dims D..K-1 in lexicographic order: the
+// successor of a feasible s increments the rightmost digit d that can grow
+// (s_d < hi_d and sum_{i<=d} s_i r_i + r_d <= T) and zeroes the suffix.
+__global__ void enum_configs_kernel(int pass, int K, int D, int64_t nprefix,
+                                    const int32_t *__restrict__ hi, const int64_t *__restrict__ r,
+                                    int64_t T, const int64_t *__restrict__ stride,
+                                    int64_t *__restrict__ counts, const int64_t *__restrict__ offsets,
+                                    uint16_t *__restrict__ digits, int64_t *__restrict__ off)
+{
+    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= nprefix) return;
+    int32_t s[MAXK];
+    uint64_t load = 0;
+    bool over = false;
+    int64_t rem = t;
+    for (int i = D - 1; i >= 0; --i) {
+        int64_t radix = (int64_t)hi[i] + 1;
+        s[i] = (int32_t)(rem % radix);
+        rem /= radix;
+    }
+    for (int i = 0; i < D; ++i) {
+        load += (uint64_t)s[i] * (uint64_t)r[i];
+        if (load > (uint64_t)T) over = true;
+    }
+    for (int i = D; i < K; ++i) s[i] = 0;
+    int64_t cnt = 0;
+    int64_t pos = (pass == 1) ? offsets[t] : 0;
+    if (!over) {
+        for (;;) {
+            bool nonzero = false;
+            for (int i = 0; i < K; ++i) nonzero |= (s[i] != 0);
+            if (nonzero) {
+                if (pass == 1) {
+                    int64_t o = 0;
+                    for (int i = 0; i < K; ++i) {
+                        digits[(pos + cnt) * K + i] = (uint16_t)s[i];
+                        o += (int64_t)s[i] * stride[i];
+                    }
+                    off[pos + cnt] = o;
+                }
+                ++cnt;
+            }
+            // successor over dims D..K-1
+            uint64_t pl = load;   // sum_{i<=d} s_i r_i while scanning d downwards
+            int d = K - 1;
+            for (; d >= D; --d) {
+                if (s[d] < hi[d] && pl + (uint64_t)r[d] <= (uint64_t)T) break;
+                pl -= (uint64_t)s[d] * (uint64_t)r[d];
+            }
+            if (d < D) break;
+            s[d] += 1;
+            for (int i = d + 1; i < K; ++i) s[i] = 0;
+            load = pl + (uint64_t)r[d];
+        }
+    }
+    if (pass == 0) counts[t] = cnt;
+}
+
+// Single-block exclusive scan of int64 (n up to a few 1e5; planning only).
+__global__ void exclusive_scan_kernel(const int64_t *__restrict__ in, int64_t *__restrict__ out,
+                                      int64_t n, int64_t *__restrict__ total)
+{
+    __shared__ int64_t warp_sums[32];
+    __shared__ int64_t carry;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    if (tid == 0) carry = 0;
+    __syncthreads();
+    for (int64_t base = 0; base < n; base += blockDim.x) {
+        int64_t i = base + tid;
+        int64_t v = i < n ? in[i] : 0;
+        int64_t x = v;
+        for (int o = 1; o < 32; o <<= 1) {
+            int64_t y = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) warp_sums[wid] = x;
+        __syncthreads();
+        if (wid == 0) {
+            int64_t w = lane < (int)(blockDim.x >> 5) ? warp_sums[lane] : 0;
+            for (int o = 1; o < 32; o <<= 1) {
+                int64_t y = __shfl_up_sync(FULL, w, o);
+                if (lane >= o) w += y;
+            }
+            warp_sums[lane] = w;
+        }
+        __syncthreads();
+        int64_t incl = x + (wid > 0 ? warp_sums[wid - 1] : 0) + carry;
+        if (i < n) out[i] = incl - v;
+        __syncthreads();
+        if (tid == blockDim.x - 1) carry = incl;
+        __syncthreads();
+    }
+    if (tid == 0) *total = carry;
+}
+
+// ------------------------------------------------------------------ a-3 grouping
+__device__ __forceinline__ bool same_lead(const uint16_t *a, const uint16_t *b, int K1)
+{
+    for (int i = 0; i < K1; ++i)
+        if (a[i] != b[i]) return false;
+    return true;
+}
+
+struct NallArg { int32_t v[MAXK]; };
+
+__global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
+                                    const int64_t *__restrict__ off, int64_t nC, RowGeom g,
+                                    NallArg Nall, PrefixEntry *__restrict__ pref,
+                                    DpMeta *__restrict__ meta)
+{
+    __shared__ int64_t warp_sums[32];
+    __shared__ int64_t carry;
+    __shared__ unsigned long long relax_acc;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int K1 = K - 1;
+    if (tid == 0) { carry = 0; relax_acc = 0ull; }
+    __syncthreads();
+    unsigned long long my_relax = 0;
+    for (int64_t base = 0; base < nC; base += blockDim.x) {
+        int64_t c = base + tid;
+        bool valid = c < nC;
+        const uint16_t *dc = digits + c * K;
+        bool head = valid && (c == 0 || !same_lead(dc, dc - K, K1));
+        int64_t v = head ? 1 : 0;
+        int64_t x = v;
+        for (int o = 1; o < 32; o <<= 1) {
+            int64_t y = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) warp_sums[wid] = x;
+        __syncthreads();
+        if (wid == 0) {
+            int64_t w = lane < (int)(blockDim.x >> 5) ? warp_sums[lane] : 0;
+            for (int o = 1; o < 32; o <<= 1) {
+                int64_t y = __shfl_up_sync(FULL, w, o);
+                if (lane >= o) w += y;
+            }
+            warp_sums[lane] = w;
+        }
+        __syncthreads();
+        int64_t incl = x + (wid > 0 ? warp_sums[wid - 1] : 0) + carry;
+        if (valid) {
+            int64_t id = incl - 1;
+            if (head) {
+                PrefixEntry e;
+                for (int w = 0; w < MAXW; ++w) e.w[w] = 0;
+                int64_t o = 0;
+                for (int i = 0; i < K1; ++i) {
+                    e.w[g.word[i]] |= (uint64_t)dc[i] << g.shift[i];
+                    o += (int64_t)dc[i] * g.stride[i];
+                }
+                e.off = o;
+                e.jmax = 0;
+                e.pad = 0;
+                pref[id] = e;
+            }
+            // closed-form relaxation count: prod_i (N_i - s_i + 1) states dominate s
+            unsigned long long pr = 1;
+            for (int i = 0; i < K; ++i) pr *= (unsigned long long)(Nall.v[i] - dc[i] + 1);
+            my_relax += pr;
+        }
+        __syncthreads();
+        if (valid) {
+            bool tail = (c == nC - 1) || !same_lead(dc, dc + K, K1);
+            if (tail) pref[incl - 1].jmax = dc[K - 1];
+        }
+        if (tid == blockDim.x - 1) carry = incl;
+        __syncthreads();
+    }
+    atomicAdd(&relax_acc, my_relax);
+    __syncthreads();
+    if (tid == 0) {
+        meta->nC = nC;
+        meta->nP = carry;
+        meta->relax = relax_acc;
+    }
+}
+
+// ------------------------------------------------------------------ a-4
+// Unrank the `rank`-th row (lexicographic order) of row-level rho, i.e. the
+// rank-th vector p over the leading dims with sum(p) = rho, using the
+// suffix-count table cnt[i][L] = #{(p_i..p_{K1-1}) : sum = L}.
+template <int NW>
+__device__ __forceinline__ void unrank_row(const RowGeom &g, const int64_t *cnt, int rho, int64_t rank,
+                                           uint64_t (&pw)[NW], int64_t &rowbase)
+{
+    const int ld = g.rho_max + 1;
+    int L = rho;
+#pragma unroll
+    for (int w = 0; w < NW; ++w) pw[w] = 0;
+    rowbase = 0;
+    for (int i = 0; i < g.K1; ++i) {
+        int lo = L - g.maxsuf[i + 1];
+        if (lo < 0) lo = 0;
+        int hi = g.N[i] < L ? g.N[i] : L;
+        int v = lo;
+        const int64_t *row = cnt + (int64_t)(i + 1) * ld;
+        for (; v < hi; ++v) {
+            int64_t c = row[L - v];
+            if (rank < c) break;
+            rank -= c;
+        }
+#pragma unroll
+        for (int w = 0; w < NW; ++w)
+            if (g.word[i] == w) pw[w] |= (uint64_t)v << g.shift[i];
+        rowbase += (int64_t)v * g.stride[i];
+        L -= v;
+    }
+}
+
+// ------------------------------------------------------------------ a-5
+// Level fill of one row-level.  A lane group of Wg = 2^wlog lanes owns one
+// row p (32/Wg rows per warp); lanes cover x in chunks of Wg.  For each state
+// n = (p, x):
+//   acc(x) = min over prefixes s' != 0 with s' <= p (packed-digit compare,
+//            uniform per group) and j in [0, min(Jmax(s'), x)] of
+//            OPT(p - s', x - j)                       (cross-row relaxations)
+//   OPT(p, x) = 1 + min(acc(x), min_{1<=j<=min(J0,x)} OPT(p, x - j))
+// the last term (s' = 0) is the in-row chain, resolved by shuffles within
+// the chunk (Bellman-Ford rounds until no lane changes) and by loads of the
+// already-stored previous chunks.  Every (n, s) pair with s in C, s <= n is
+// relaxed exactly once: the relaxation count is the closed form.
+template <typename E, int NW>
+__global__ void __launch_bounds__(256)
+row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt,
+                const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
+                int smem_pref, int smem_cnt, int J0, int rho, int64_t slot_begin,
+                int64_t slot_count, E *compact, int wlog)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int64_t nP = meta->nP;
+    const int np = (int)(nP - 1);            // cross-row prefixes (entry 0 is s' = 0)
+    PrefixEntry *spref = reinterpret_cast<PrefixEntry *>(smem_raw);
+    int64_t *scnt = reinterpret_cast<int64_t *>(smem_raw + (size_t)smem_pref * sizeof(PrefixEntry));
+    const int ncnt = (g.K1 + 1) * (g.rho_max + 1);
+    if (smem_pref)
+        for (int i = threadIdx.x; i < np; i += blockDim.x) spref[i] = gpref[1 + i];
+    if (smem_cnt)
+        for (int i = threadIdx.x; i < ncnt; i += blockDim.x) scnt[i] = gcnt[i];
+    __syncthreads();
+    const PrefixEntry *P = smem_pref ? spref : gpref + 1;
+    const int64_t *cnt = smem_cnt ? scnt : gcnt;
+
+    const int lane = threadIdx.x & 31;
+    const int Wg = 1 << wlog;
+    const int grp = lane >> wlog;
+    const int xl = lane & (Wg - 1);
+    const int rpw = 32 >> wlog;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t nslot_w = (slot_count + rpw - 1) / rpw;
+    const int64_t W = g.W;
+
+    for (int64_t ws = gw; ws < nslot_w; ws += nw) {
+        const int64_t slot = ws * rpw + grp;
+        const bool rowok = slot < slot_count;
+        uint64_t pw[NW];
+        int64_t rowbase = 0;
+        if (rowok) unrank_row<NW>(g, cnt, rho, slot_begin + slot, pw, rowbase);
+        else {
+#pragma unroll
+            for (int w = 0; w < NW; ++w) pw[w] = 0;
+        }
+        E *out = compact ? compact + slot * W : table + rowbase;
+        for (int64_t x0 = 0; x0 < W; x0 += Wg) {
+            const int64_t x = x0 + xl;
+            const bool act = rowok && x < W;
+            int acc = INF;
+            if (act) {
+                for (int c = 0; c < np; ++c) {
+                    const PrefixEntry pe = P[c];
+                    bool dom = true;
+#pragma unroll
+                    for (int w = 0; w < NW; ++w)
+                        dom &= (((pw[w] | g.guard[w]) - pe.w[w]) & g.guard[w]) == g.guard[w];
+                    if (dom) {
+                        const E *src = table + (rowbase - pe.off + x);
+                        const int jm = pe.jmax < x ? pe.jmax : (int)x;
+                        for (int j = 0; j <= jm; ++j) {
+                            int v = src[-j];
+                            acc = v < acc ? v : acc;
+                        }
+                    }
+                }
+                // in-row terms that reach back into earlier (stored) chunks
+                const int jlim = J0 < x ? J0 : (int)x;
+                for (int j = xl + 1; j <= jlim; ++j) {
+                    int v = out[x - j];
+                    acc = v < acc ? v : acc;
+                }
+            }
+            int opt = (rho == 0 && x == 0) ? 0 : acc + 1;
+            // in-chunk chain: Bellman-Ford over shuffles
+            const int jin = J0 < Wg - 1 ? J0 : Wg - 1;
+            bool changed = jin > 0;
+            while (__any_sync(FULL, changed)) {
+                int nopt = opt;
+                for (int j = 1; j <= jin; ++j) {
+                    int v = __shfl_up_sync(FULL, opt, j, Wg);
+                    if (xl >= j && v + 1 < nopt) nopt = v + 1;
+                }
+                changed = nopt < opt;
+                opt = nopt;
+            }
+            if (act) out[x] = (E)opt;
+            __syncwarp();
+        }
+    }
+}
+
+// §8(e): write gathered compact rows (slot-major, W entries each) into the table.
+template <typename E, int NW>
+__global__ void __launch_bounds__(256)
+row_scatter_kernel(E *__restrict__ table, const RowGeom g, const int64_t *__restrict__ cnt, int rho,
+                   int64_t slot_count, const E *__restrict__ compact, int wlog)
+{
+    const int lane = threadIdx.x & 31;
+    const int Wg = 1 << wlog;
+    const int grp = lane >> wlog;
+    const int xl = lane & (Wg - 1);
+    const int rpw = 32 >> wlog;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t nslot_w = (slot_count + rpw - 1) / rpw;
+    for (int64_t ws = gw; ws < nslot_w; ws += nw) {
+        const int64_t slot = ws * rpw + grp;
+        if (slot >= slot_count) continue;
+        uint64_t pw[NW];
+        int64_t rowbase;
+        unrank_row<NW>(g, cnt, rho, slot, pw, rowbase);
+        for (int64_t x = xl; x < g.W; x += Wg) table[rowbase + x] = compact[slot * g.W + x];
+    }
+}
+
+__global__ void row_index_kernel(const RowGeom g, const int64_t *__restrict__ cnt, int rho,
+                                 int64_t slot_count, int64_t *__restrict__ out)
+{
+    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= slot_count) return;
+    uint64_t pw[MAXW];
+    int64_t rowbase;
+    unrank_row<MAXW>(g, cnt, rho, t, pw, rowbase);
+    out[t] = rowbase;
+}
+
+template <typename E>
+__global__ void read_opt_kernel(const E *__restrict__ table, int64_t idx, DpMeta *meta)
+{
+    meta->opt = (int32_t)table[idx];
+}
+
+// ------------------------------------------------------------------ a-8
+// Traceback (reading R11): from n = N, repeatedly take the configuration of
+// smallest canonical rank with s <= n and OPT(n - s) = OPT(n) - 1.
+template <typename E>
+__global__ void __launch_bounds__(256)
+traceback_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__ N,
+                 const int64_t *__restrict__ stride, const uint16_t *__restrict__ digits,
+                 const int64_t *__restrict__ off, const int32_t *__restrict__ rank, int64_t nC,
+                 int64_t sigma, int32_t *__restrict__ out, int32_t max_out, int32_t *__restrict__ len,
+                 DpMeta *meta)
+{
+    __shared__ int32_t cur[MAXK];
+    __shared__ int64_t idx;
+    __shared__ unsigned long long best;
+    __shared__ int32_t mu;
+    const int tid = threadIdx.x;
+    if (tid < K) cur[tid] = N[tid];
+    if (tid == 0) { idx = sigma - 1; mu = 0; }
+    __syncthreads();
+    while (idx != 0) {
+        if (tid == 0) best = ~0ull;
+        __syncthreads();
+        const int v = (int)table[idx];
+        unsigned long long mine = ~0ull;
+        for (int64_t c = tid; c < nC; c += blockDim.x) {
+            bool dom = true;
+            for (int i = 0; i < K; ++i) dom &= digits[c * K + i] <= cur[i];
+            if (dom && (int)table[idx - off[c]] == v - 1) {
+                unsigned long long key = ((unsigned long long)(uint32_t)rank[c] << 32) | (uint32_t)c;
+                mine = key < mine ? key : mine;
+            }
+        }
+        atomicMin(&best, mine);
+        __syncthreads();
+        if (tid == 0) {
+            if (best == ~0ull || mu >= max_out) {
+                meta->err = 1;
+                idx = 0;
+            } else {
+                int64_t c = (int64_t)(best & 0xffffffffull);
+                out[mu++] = (int32_t)c;
+                idx -= off[c];
+            }
+        }
+        __syncthreads();
+        if (meta->err) break;
+        if (tid < K && best != ~0ull) {
+            int64_t c = (int64_t)(best & 0xffffffffull);
+            cur[tid] -= digits[c * K + tid];
+        }
+        __syncthreads();
+    }
+    if (tid == 0) *len = mu;
+}
+
+__global__ void fill_value_kernel(uint8_t *p, int64_t bytes, uint8_t v)
+{
+    int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    int64_t st = (int64_t)gridDim.x * blockDim.x;
+    for (; i < bytes; i += st) p[i] = v;
+}
+
+int wlog_for(int64_t W)
+{
+    int wlog = 0;
+    while ((1 << wlog) < W && wlog < 5) ++wlog;
+    return wlog;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ launchers
+cudaError_t launch_enum_configs(int pass, int K, int D, int64_t nprefix, const int32_t *hi,
+                                const int64_t *r, int64_t T, const int64_t *stride,
+                                int64_t *d_counts, const int64_t *d_offsets, uint16_t *d_digits,
+                                int64_t *d_off, cudaStream_t st)
+{
+    const int bs = 128;
+    int64_t blocks = (nprefix + bs - 1) / bs;
+    enum_configs_kernel<<<(unsigned)blocks, bs, 0, st>>>(pass, K, D, nprefix, hi, r, T, stride,
+                                                         d_counts, d_offsets, d_digits, d_off);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_exclusive_scan(const int64_t *d_in, int64_t *d_out, int64_t n, int64_t *d_total,
+                                  cudaStream_t st)
+{
+    exclusive_scan_kernel<<<1, 1024, 0, st>>>(d_in, d_out, n, d_total);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off, int64_t nC,
+                                const RowGeom &g, const int32_t *Nall, PrefixEntry *d_pref,
+                                DpMeta *d_meta, cudaStream_t st)
+{
+    NallArg na;
+    for (int i = 0; i < MAXK; ++i) na.v[i] = i < K ? Nall[i] : 0;
+    build_prefix_kernel<<<1, 1024, 0, st>>>(K, d_digits, d_off, nC, g, na, d_pref, d_meta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
+                            const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
+                            int J0, int rho, int64_t slot_begin, int64_t slot_count,
+                            void *compact_out, int sm_count, cudaStream_t st)
+{
+    if (slot_count <= 0) return cudaSuccess;
+    const int wlog = wlog_for(g.W);
+    const int rpw = 32 >> wlog;
+    const int bs = 256;
+    const int64_t warps = (slot_count + rpw - 1) / rpw;
+    int64_t blocks = (warps + (bs / 32) - 1) / (bs / 32);
+    const int64_t cap = (int64_t)sm_count * 8;
+    if (blocks > cap) blocks = cap;
+    size_t pref_bytes = (size_t)(nP_bound > 1 ? nP_bound - 1 : 0) * sizeof(PrefixEntry);
+    size_t cnt_bytes = (size_t)(g.K1 + 1) * (g.rho_max + 1) * sizeof(int64_t);
+    int smem_pref = pref_bytes <= 96 * 1024 ? (int)(nP_bound > 1 ? nP_bound - 1 : 0) : 0;
+    if (smem_pref == 0) pref_bytes = 0;
+    int smem_cnt = (pref_bytes + cnt_bytes) <= 200 * 1024 ? 1 : 0;
+    size_t smem = pref_bytes + (smem_cnt ? cnt_bytes : 0);
+    cudaError_t err;
+#define PTAS_FILL_CASE(E_, NW_)                                                                   \
+    do {                                                                                          \
+        auto kfn = row_fill_kernel<E_, NW_>;                                                      \
+        if (smem > 48 * 1024) {                                                                   \
+            err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
+                                       (int)smem);                                                \
+            if (err != cudaSuccess) return err;                                                   \
+        }                                                                                         \
+        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, d_cnt, d_pref, d_meta,            \
+                                                smem_pref, smem_cnt, J0, rho, slot_begin,         \
+                                                slot_count, (E_ *)compact_out, wlog);             \
+    } while (0)
+    if (e == 1) {
+        if (g.nwords <= 1) PTAS_FILL_CASE(uint8_t, 1); else PTAS_FILL_CASE(uint8_t, 2);
+    } else {
+        if (g.nwords <= 1) PTAS_FILL_CASE(uint16_t, 1); else PTAS_FILL_CASE(uint16_t, 2);
+    }
+#undef PTAS_FILL_CASE
+    return cudaGetLastError();
+}
+
+cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *d_cnt, int rho,
+                               int64_t slot_count, const void *compact, int sm_count,
+                               cudaStream_t st)
+{
+    if (slot_count <= 0) return cudaSuccess;
+    const int wlog = wlog_for(g.W);
+    const int rpw = 32 >> wlog;
+    const int bs = 256;
+    int64_t blocks = ((slot_count + rpw - 1) / rpw + 7) / 8;
+    const int64_t cap = (int64_t)sm_count * 8;
+    if (blocks > cap) blocks = cap;
+    if (e == 1) {
+        if (g.nwords <= 1)
+            row_scatter_kernel<uint8_t, 1><<<(unsigned)blocks, bs, 0, st>>>((uint8_t *)table, g, d_cnt, rho, slot_count, (const uint8_t *)compact, wlog);
+        else
+            row_scatter_kernel<uint8_t, 2><<<(unsigned)blocks, bs, 0, st>>>((uint8_t *)table, g, d_cnt, rho, slot_count, (const uint8_t *)compact, wlog);
+    } else {
+        if (g.nwords <= 1)
+            row_scatter_kernel<uint16_t, 1><<<(unsigned)blocks, bs, 0, st>>>((uint16_t *)table, g, d_cnt, rho, slot_count, (const uint16_t *)compact, wlog);
+        else
+            row_scatter_kernel<uint16_t, 2><<<(unsigned)blocks, bs, 0, st>>>((uint16_t *)table, g, d_cnt, rho, slot_count, (const uint16_t *)compact, wlog);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_row_index(const RowGeom &g, const int64_t *d_cnt, int rho, int64_t slot_count,
+                             int64_t *out_rowbase, cudaStream_t st)
+{
+    if (slot_count <= 0) return cudaSuccess;
+    const int bs = 128;
+    row_index_kernel<<<(unsigned)((slot_count + bs - 1) / bs), bs, 0, st>>>(g, d_cnt, rho, slot_count, out_rowbase);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_read_opt(int e, const void *table, int64_t idx, DpMeta *d_meta, cudaStream_t st)
+{
+    if (e == 1) read_opt_kernel<uint8_t><<<1, 1, 0, st>>>((const uint8_t *)table, idx, d_meta);
+    else read_opt_kernel<uint16_t><<<1, 1, 0, st>>>((const uint16_t *)table, idx, d_meta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N,
+                             const int64_t *d_stride, const uint16_t *d_digits, const int64_t *d_off,
+                             const int32_t *d_rank, int64_t nC, int64_t sigma, int32_t *d_out,
+                             int32_t max_out, int32_t *d_len, DpMeta *d_meta, cudaStream_t st)
+{
+    if (e == 1)
+        traceback_kernel<uint8_t><<<1, 256, 0, st>>>((const uint8_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, sigma, d_out, max_out, d_len, d_meta);
+    else
+        traceback_kernel<uint16_t><<<1, 256, 0, st>>>((const uint16_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, sigma, d_out, max_out, d_len, d_meta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fill_value(void *p, int64_t bytes, int value, cudaStream_t st)
+{
+    if (bytes <= 0) return cudaSuccess;
+    int64_t blocks = (bytes + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    fill_value_kernel<<<(unsigned)blocks, 256, 0, st>>>((uint8_t *)p, bytes, (uint8_t)value);
+    return cudaGetLastError();
+}
+
+}  // namespace ptas

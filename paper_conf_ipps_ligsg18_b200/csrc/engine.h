@@ -1,0 +1,105 @@
+// engine.h — per-device DP engine (host orchestration of the kernels).
+#pragma once
+#include <cstdint>
+#include <mutex>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "../../include/ptas.h"
+#include "internal.h"
+
+namespace ptas {
+
+// How one DP's row-levels are distributed.
+struct ShardCtx {
+    ptas_comm *comm = nullptr;  // real NCCL ranks (nullptr = none)
+    int rank = 0;
+    int world = 1;
+    int virtual_shards = 1;     // >1: logical shards on this GPU (testing)
+    int64_t min_rows = 0;       // row-levels with fewer rows are computed redundantly
+};
+
+struct DpRequest {
+    int K = 0;                    // canonical classes (may include zero counts)
+    const int32_t *N = nullptr;   // canonical counts
+    const int64_t *r = nullptr;   // canonical sizes
+    int64_t T = 0;
+    const int *order = nullptr;   // internal position i -> canonical class (nullable = identity
+                                  // over non-empty classes); must list exactly the non-empty classes
+    void *ext_table = nullptr;    // caller device buffer (nullable = engine-owned table)
+    int64_t ext_bytes = 0;
+    cudaStream_t stream = nullptr;  // nullptr = engine stream
+    const ShardCtx *shard = nullptr;
+    int64_t budget = 0;           // bytes allowed for the table (0 = auto)
+};
+
+struct DpOutcome {
+    int32_t opt = 0;
+    int64_t sigma = 1;
+    int e = 1;
+    int Kint = 0;
+    double relax = 0;
+    int64_t nC = 0, nP = 0;
+    double dp_s = 0, fill_s = 0;
+    int launches = 0, fill_launches = 0;
+    int64_t h2d = 0, d2h = 0;
+};
+
+// one machine of the traceback: canonical digit vector s (length K canonical)
+using MachineCfg = std::vector<int32_t>;
+
+class Engine {
+  public:
+    static int get(int device, Engine **out);
+    std::mutex mu;
+
+    int run_dp(const DpRequest &rq, DpOutcome *out);
+    // Traceback on the table of the last run_dp (engine-owned or the same
+    // ext table); appends OPT(N) canonical configurations to machines.
+    int traceback(std::vector<MachineCfg> *machines, DpOutcome *acc);
+    // Inspection helpers.
+    int configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits, int64_t *count);
+    int row_index(const int32_t *N, int K, std::vector<int64_t> *level_start,
+                  std::vector<int64_t> *rowbase);
+    int64_t free_budget();
+    // D2H of the table of the last run_dp (engine-owned or ext).
+    int copy_table_to_host(void *dst, int64_t bytes);
+    cudaStream_t stream() const { return stream_; }
+    int device() const { return device_; }
+
+  private:
+    int init(int device);
+    struct Buf {
+        void *p = nullptr;
+        size_t cap = 0;
+        cudaError_t ensure(size_t bytes);
+    };
+    int device_ = -1;
+    int sm_count_ = 148;
+    cudaStream_t stream_ = nullptr;
+    cudaEvent_t ev_[4] = {nullptr, nullptr, nullptr, nullptr};
+    DpMeta *d_meta_ = nullptr;
+    DpMeta *h_meta_ = nullptr;     // pinned
+    int64_t *h_scalar_ = nullptr;  // pinned
+    Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_;
+
+    // state of the last DP (for traceback)
+    bool last_valid_ = false;
+    void *last_table_ = nullptr;
+    cudaStream_t last_stream_ = nullptr;
+    int last_K_ = 0, last_Kcanon_ = 0, last_e_ = 1;
+    int64_t last_sigma_ = 1, last_nC_ = 0;
+    int32_t last_opt_ = 0;
+    std::vector<int> last_order_;      // internal -> canonical
+    std::vector<int32_t> last_N_;      // internal counts
+    std::vector<int64_t> last_stride_; // internal strides
+};
+
+// NCCL glue (comm.cpp)
+int comm_rank(const ptas_comm *c);
+int comm_world(const ptas_comm *c);
+int comm_allgather(ptas_comm *c, const void *send, void *recv, size_t bytes_per_rank,
+                   cudaStream_t st);
+
+}  // namespace ptas

@@ -1,0 +1,88 @@
+// internal.h — shared declarations of the product library (NOT used by oracle/).
+//
+// Layout of a DP in HBM:
+//   table  : sigma entries of E (uint8 if sum N <= 255 else uint16), row-major
+//            over the INTERNAL class order (a permutation of the caller's
+//            order chosen by the driver; identity for dp_fill), last class
+//            fastest.  A "row" is the run of W = N[K-1]+1 entries that share
+//            the K1 = K-1 leading digits p; rows are filled in row-level order
+//            rho = sum(p) (the wavefront), each row by one lane group.
+//   configs: C(T) in internal lexicographic order: uint16
+//            digits [nC*K] + int64 linear offsets off(s) [nC].
+//   prefix : one entry per distinct leading part s' of C (runs of equal s' in
+//            lexicographic order): packed digits, off(s'), Jmax(s') = largest
+//            last digit with (s', j) in C.  Entry 0 is s' = 0 (j = 1..J0).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ptas {
+
+constexpr int MAXK = 40;   // internal (non-empty) classes
+constexpr int MAXW = 2;    // 64-bit words for packed leading digits
+
+struct PrefixEntry {
+    uint64_t w[MAXW];   // packed leading digits s'
+    int64_t off;        // sum_i s'_i * stride_i (elements)
+    int32_t jmax;       // max j with (s', j) in C
+    int32_t pad;
+};
+static_assert(sizeof(PrefixEntry) == 32, "PrefixEntry must be 32 bytes");
+
+// Geometry of the row space, passed by value to the kernels.
+struct RowGeom {
+    int32_t K1;                 // number of leading classes (K-1)
+    int32_t rho_max;            // sum of leading counts
+    int64_t W;                  // row length N[K-1]+1
+    int32_t N[MAXK];            // leading counts
+    int32_t maxsuf[MAXK + 1];   // maxsuf[i] = sum_{d >= i} N[d] (leading dims)
+    int64_t stride[MAXK];       // element strides of the leading dims
+    uint8_t word[MAXK];         // packed word index of leading digit i
+    uint8_t shift[MAXK];        // bit offset of leading digit i
+    uint64_t guard[MAXW];       // guard bit per field, per word
+    int32_t nwords;
+};
+
+// Device-side summary written by the planning kernels and read back once.
+struct DpMeta {
+    int64_t nC;            // |C|
+    int64_t nP;            // number of prefix entries (incl. the zero prefix)
+    unsigned long long relax;  // closed-form relaxations sum_{s in C} prod(N_i - s_i + 1)
+    int32_t opt;           // OPT(N)
+    int32_t err;           // device-detected error (traceback)
+};
+
+// ---------------------------------------------------------------- launchers
+// All launchers enqueue on `st` and return cudaGetLastError().
+cudaError_t launch_enum_configs(int pass, int K, int D, int64_t nprefix,
+                                const int32_t *hi, const int64_t *r, int64_t T,
+                                const int64_t *stride, int64_t *d_counts,
+                                const int64_t *d_offsets, uint16_t *d_digits,
+                                int64_t *d_off, cudaStream_t st);
+cudaError_t launch_exclusive_scan(const int64_t *d_in, int64_t *d_out, int64_t n,
+                                  int64_t *d_total, cudaStream_t st);
+cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off,
+                                int64_t nC, const RowGeom &g, const int32_t *Nall,
+                                PrefixEntry *d_pref, DpMeta *d_meta, cudaStream_t st);
+// One row-level of the level fill.  e = 1 or 2.  Rows [slot_begin, slot_begin+slot_count)
+// of row-level rho; results go to the table (compact_out == NULL) or to
+// compact_out[(slot - slot_begin) * W + x].
+cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
+                            const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
+                            int J0, int rho, int64_t slot_begin, int64_t slot_count,
+                            void *compact_out, int sm_count, cudaStream_t st);
+cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
+                               int rho, int64_t slot_count, const void *compact,
+                               int sm_count, cudaStream_t st);
+cudaError_t launch_row_index(const RowGeom &g, const int64_t *d_cnt, int rho,
+                             int64_t slot_count, int64_t *out_rowbase, cudaStream_t st);
+cudaError_t launch_read_opt(int e, const void *table, int64_t idx, DpMeta *d_meta,
+                            cudaStream_t st);
+cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N,
+                             const int64_t *d_stride, const uint16_t *d_digits,
+                             const int64_t *d_off, const int32_t *d_rank, int64_t nC,
+                             int64_t sigma, int32_t *d_out, int32_t max_out,
+                             int32_t *d_len, DpMeta *d_meta, cudaStream_t st);
+cudaError_t launch_fill_value(void *p, int64_t bytes, int value, cudaStream_t st);
+
+}  // namespace ptas

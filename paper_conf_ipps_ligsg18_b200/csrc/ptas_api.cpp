@@ -1,0 +1,685 @@
+// ptas_api.cpp — C ABI entry points and the host driver of the PTAS
+// (§8(b)).
+//
+//   a-1 classify/round            host, O(n log n) per probe
+//   a-7 P-probe search + memo     host; DP(T) runs on the GPU (dp_engine.cpp)
+//   a-8 schedule at T*            device traceback + host job placement
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <queue>
+#include <vector>
+
+#include "engine.h"
+
+using namespace ptas;
+
+namespace {
+
+struct Classified {
+    int64_t u = 1;
+    std::vector<int64_t> r;    // distinct rounded long sizes, ascending
+    std::vector<int32_t> N;    // counts
+    std::vector<int32_t> cls;  // per job: class or -1
+};
+
+int64_t ceil_div(int64_t a, int64_t b) { return a / b + ((a % b) != 0); }
+
+// Alg 1 l.6-8: long iff k*p > T (p > T/k, reading R1);
+// u = max(1, floor(T/k^2)) (R2); r = floor(p/u)*u; classes = distinct r
+// ascending (R3).
+void classify(const int64_t *p, int32_t n, int64_t T, int32_t k, Classified *c)
+{
+    const int64_t kk = (int64_t)k * k;
+    c->u = std::max<int64_t>(1, T / kk);
+    const int64_t u = c->u;
+    std::vector<int64_t> q;  // rounded multiples floor(p/u) of the long jobs
+    q.reserve(n);
+    c->cls.assign(n, -1);
+    for (int32_t j = 0; j < n; ++j)
+        if ((__int128)k * p[j] > (__int128)T) q.push_back(p[j] / u);
+    std::sort(q.begin(), q.end());
+    q.erase(std::unique(q.begin(), q.end()), q.end());
+    c->r.resize(q.size());
+    c->N.assign(q.size(), 0);
+    for (size_t i = 0; i < q.size(); ++i) c->r[i] = q[i] * u;
+    for (int32_t j = 0; j < n; ++j) {
+        if (!((__int128)k * p[j] > (__int128)T)) continue;
+        int32_t i = (int32_t)(std::lower_bound(q.begin(), q.end(), p[j] / u) - q.begin());
+        c->cls[j] = i;
+        c->N[i]++;
+    }
+}
+
+int probe_targets(int64_t LB, int64_t UB, int32_t P, std::vector<int64_t> *out)
+{
+    out->clear();
+    if (LB >= UB || P < 1) return PTAS_EINVAL;
+    const __int128 w = (__int128)UB - LB;
+    for (int32_t j = 0; j < P; ++j) {
+        int64_t t = (int64_t)((__int128)LB + ((__int128)(2 * j + 1) * w) / (2 * (__int128)P));
+        if (!out->empty() && out->back() == t) continue;
+        out->push_back(t);
+    }
+    return PTAS_OK;
+}
+
+// Alg 1 l.10-14 / Alg 3 l.13-25 (reading R8): the smallest feasible probe
+// becomes UB; LB rises past every infeasible probe below it.
+void interval_update(int64_t *LB, int64_t *UB, const int64_t *T, const int32_t *f, int32_t cnt)
+{
+    bool any = false;
+    int64_t ub = *UB;
+    for (int32_t q = 0; q < cnt; ++q)
+        if (f[q] && (!any || T[q] < ub)) {
+            ub = T[q];
+            any = true;
+        }
+    if (any) {
+        int64_t lb = *LB;
+        for (int32_t q = 0; q < cnt; ++q)
+            if (!f[q] && T[q] < ub) lb = std::max(lb, T[q] + 1);
+        *LB = lb;
+        *UB = ub;
+    } else {
+        int64_t mx = *LB;
+        for (int32_t q = 0; q < cnt; ++q) mx = std::max(mx, T[q] + 1);
+        *LB = mx;
+    }
+}
+
+int validate_jobs(const int64_t *p, int32_t n, int32_t m, int64_t *LB, int64_t *UB)
+{
+    if (!p || n < 1 || m < 1) return PTAS_EINVAL;
+    __int128 S = 0;
+    int64_t mx = 0;
+    for (int32_t j = 0; j < n; ++j) {
+        if (p[j] < 1) return PTAS_EINVAL;
+        S += p[j];
+        mx = std::max(mx, p[j]);
+    }
+    if (S > (__int128)(INT64_MAX / 4)) return PTAS_EINVAL;
+    int64_t A = ceil_div((int64_t)S, m);
+    *LB = std::max(A, mx);
+    *UB = A + mx;
+    return PTAS_OK;
+}
+
+int k_of(double eps)
+{
+    if (!(eps > 0.0) || !std::isfinite(eps)) return PTAS_EINVAL;
+    double k = std::ceil(1.0 / eps);
+    if (!(k >= 1.0) || k > (double)(1 << 20)) return PTAS_EINVAL;
+    return (int)k;
+}
+
+// memo key: (N, c = r/u, cap = floor(T/u)) — the DP depends only on these
+// (sum s_i r_i <= T  <=>  sum s_i c_i <= floor(T/u)), SURVEY.md §8(a) a-7.
+std::vector<int64_t> memo_key(const Classified &c, int64_t T)
+{
+    std::vector<int64_t> key;
+    key.reserve(2 * c.N.size() + 2);
+    key.push_back((int64_t)c.N.size());
+    for (size_t i = 0; i < c.N.size(); ++i) {
+        key.push_back(c.N[i]);
+        key.push_back(c.r[i] / c.u);
+    }
+    key.push_back(T / c.u);
+    return key;
+}
+
+// internal class order for the table (layout 0): ascending count, ties by
+// class index, so the largest class is the contiguous (row) dimension.
+std::vector<int> choose_order(const std::vector<int32_t> &N, int layout)
+{
+    std::vector<int> o(N.size());
+    for (size_t i = 0; i < N.size(); ++i) o[i] = (int)i;
+    if (layout == 0)
+        std::stable_sort(o.begin(), o.end(), [&](int a, int b) { return N[a] < N[b]; });
+    return o;
+}
+
+double now_s()
+{
+    return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+struct Acc {
+    ptas_stats s;
+    Acc() { std::memset(&s, 0, sizeof(s)); }
+    void add(const DpOutcome &o)
+    {
+        s.relaxations += o.relax;
+        s.dp_seconds += o.dp_s;
+        s.fill_seconds += o.fill_s;
+        s.alg_bytes += (o.relax + (double)o.sigma) * o.e;
+        s.states += o.sigma;
+        s.kernel_launches += o.launches;
+        s.fill_launches += o.fill_launches;
+        s.h2d_bytes += o.h2d;
+        s.d2h_bytes += o.d2h;
+        s.sigma_max = std::max(s.sigma_max, o.sigma);
+    }
+};
+
+int resolve_device(int dev, int *out)
+{
+    if (dev < 0) {
+        if (cudaGetDevice(&dev) != cudaSuccess) {
+            cudaGetLastError();
+            return PTAS_ECUDA;
+        }
+    }
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || dev >= n) {
+        cudaGetLastError();
+        return PTAS_ECUDA;
+    }
+    if (cudaSetDevice(dev) != cudaSuccess) {
+        cudaGetLastError();
+        return PTAS_ECUDA;
+    }
+    *out = dev;
+    return PTAS_OK;
+}
+
+int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_options *opt_in,
+               int64_t *makespan_out, int32_t *assignment_out, ptas_stats *stats, ptas_probe *log,
+               int32_t log_cap, int32_t *log_len, int64_t extra_h2d, int64_t extra_d2h)
+{
+    const double t0 = now_s();
+    ptas_options opt;
+    ptas_default_options(&opt);
+    if (opt_in) opt = *opt_in;
+    int64_t LB, UB;
+    int rc = validate_jobs(p, n, m, &LB, &UB);
+    if (rc) return rc;
+    const int k = k_of(eps);
+    if (k < 0) return PTAS_EINVAL;
+    if (!makespan_out || !assignment_out) return PTAS_EINVAL;
+    if (opt.probes_per_round < 1) return PTAS_EINVAL;
+    if (opt.mode < PTAS_MODE_SINGLE || opt.mode > PTAS_MODE_MULTI_PROBE) return PTAS_EINVAL;
+    if (opt.layout < 0 || opt.layout > 1) return PTAS_EINVAL;
+    int rank = 0, world = 1;
+    if (opt.comm) {
+        rank = comm_rank(opt.comm);
+        world = comm_world(opt.comm);
+    }
+    if (opt.mode == PTAS_MODE_MULTI_PROBE && (!opt.comm || opt.probes_per_round != world))
+        return PTAS_EINVAL;
+    if (opt.mode == PTAS_MODE_SINGLE && opt.comm) return PTAS_EINVAL;
+    const int P = opt.probes_per_round;
+    int dev;
+    rc = resolve_device(opt.device, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+
+    ShardCtx sh;
+    const ShardCtx *shp = nullptr;
+    if (opt.mode == PTAS_MODE_LEVEL_SHARDED) {
+        sh.comm = opt.comm;
+        sh.rank = rank;
+        sh.world = world;
+        sh.virtual_shards = opt.comm ? 1 : std::max(1, opt.virtual_shards);
+        sh.min_rows = opt.comm ? 2048 : 0;
+        shp = &sh;
+    }
+
+    Acc acc;
+    acc.s.h2d_bytes += extra_h2d;
+    acc.s.d2h_bytes += extra_d2h;
+    std::map<std::vector<int64_t>, int32_t> memo;
+    std::vector<int64_t> table_key;
+    bool table_valid = false;
+    std::vector<ptas_probe> plog;
+    int round = 0;
+    Classified cl;
+
+    auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
+        std::vector<int> order = choose_order(c.N, opt.layout);
+        DpRequest rq;
+        rq.K = (int)c.N.size();
+        rq.N = c.N.data();
+        rq.r = c.r.data();
+        rq.T = T;
+        rq.order = order.data();
+        rq.shard = s;
+        rq.budget = opt.table_budget_bytes;
+        DpOutcome o;
+        int r2 = eng->run_dp(rq, &o);
+        if (r2) return r2;
+        acc.add(o);
+        acc.s.unique_dps++;
+        *opt_out = o.opt;
+        return PTAS_OK;
+    };
+
+    while (LB < UB) {
+        std::vector<int64_t> Tj;
+        probe_targets(LB, UB, P, &Tj);
+        const int np = (int)Tj.size();
+        std::vector<int32_t> optj(np, 0), hit(np, 0), who(np, 0), Kj(np, 0);
+        std::vector<int64_t> sgj(np, 1);
+        std::vector<std::vector<int64_t>> keys(np);
+        for (int q = 0; q < np; ++q) {
+            classify(p, n, Tj[q], k, &cl);
+            Kj[q] = (int32_t)cl.N.size();
+            __int128 sg = 1;
+            for (int32_t x : cl.N) {
+                sg *= (x + 1);
+                if (sg > (__int128)INT64_MAX) sg = -1;
+                if (sg < 0) break;
+            }
+            sgj[q] = (int64_t)sg;
+            if (cl.N.empty()) {
+                optj[q] = 0;
+                continue;
+            }
+            keys[q] = memo_key(cl, Tj[q]);
+            auto it = opt.memoize ? memo.find(keys[q]) : memo.end();
+            if (it != memo.end()) {
+                optj[q] = it->second;
+                hit[q] = 1;
+                continue;
+            }
+            const bool mine = opt.mode != PTAS_MODE_MULTI_PROBE || q == rank;
+            who[q] = opt.mode == PTAS_MODE_MULTI_PROBE ? q : rank;
+            if (!mine) {
+                optj[q] = -1;  // filled by the exchange
+                continue;
+            }
+            rc = run(cl, Tj[q], opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, &optj[q]);
+            if (rc) return rc;
+            table_key = keys[q];
+            table_valid = true;
+            if (opt.memoize) memo[keys[q]] = optj[q];
+        }
+        if (opt.mode == PTAS_MODE_MULTI_PROBE) {
+            // exchange OPT(N) of every rank's probe (int32 per rank) over NCCL
+            std::vector<int32_t> mine(1, -1), all(world, -1);
+            if (rank < np) mine[0] = optj[rank];
+            int32_t *dbuf = nullptr;
+            if (cudaMalloc(&dbuf, sizeof(int32_t) * world) != cudaSuccess) return PTAS_ENOMEM;
+            cudaStream_t st = eng->stream();
+            cudaMemcpyAsync(dbuf + rank, mine.data(), 4, cudaMemcpyHostToDevice, st);
+            int crc = comm_allgather(opt.comm, dbuf + rank, dbuf, 4, st);
+            cudaMemcpyAsync(all.data(), dbuf, 4 * world, cudaMemcpyDeviceToHost, st);
+            cudaError_t ce = cudaStreamSynchronize(st);
+            cudaFree(dbuf);
+            if (crc) return crc;
+            if (ce != cudaSuccess) return PTAS_ECUDA;
+            acc.s.h2d_bytes += 4;
+            acc.s.d2h_bytes += 4 * world;
+            for (int q = 0; q < np; ++q)
+                if (optj[q] < 0) {
+                    optj[q] = all[q];
+                    if (optj[q] < 0) return PTAS_EINTERNAL;
+                    if (opt.memoize && !keys[q].empty()) memo[keys[q]] = optj[q];
+                }
+        }
+        std::vector<int32_t> f(np);
+        for (int q = 0; q < np; ++q) {
+            f[q] = optj[q] <= m;
+            ptas_probe pr;
+            pr.T = Tj[q];
+            pr.round = round;
+            pr.feasible = f[q];
+            pr.K = Kj[q];
+            pr.opt = optj[q];
+            pr.sigma = sgj[q];
+            pr.memo_hit = hit[q];
+            pr.rank = who[q];
+            plog.push_back(pr);
+        }
+        interval_update(&LB, &UB, Tj.data(), f.data(), np);
+        ++round;
+    }
+
+    // ---- a-8 schedule from DP(T*) (readings R9, R11, R12)
+    const int64_t Ts = LB;
+    classify(p, n, Ts, k, &cl);
+    std::vector<int64_t> load(m, 0);
+    std::vector<int32_t> asg(n, -1);
+    int32_t opt_star = 0;
+    if (!cl.N.empty()) {
+        std::vector<int64_t> key = memo_key(cl, Ts);
+        if (!table_valid || key != table_key) {
+            rc = run(cl, Ts, opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, &opt_star);
+            if (rc) return rc;
+        }
+        std::vector<MachineCfg> machines;
+        DpOutcome tb;
+        rc = eng->traceback(&machines, &tb);
+        if (rc) return rc;
+        acc.s.kernel_launches += tb.launches;
+        acc.s.h2d_bytes += tb.h2d;
+        acc.s.d2h_bytes += tb.d2h;
+        opt_star = (int32_t)machines.size();
+        if ((int)machines.size() > m) return PTAS_EINTERNAL;
+        const int K = (int)cl.N.size();
+        std::vector<std::vector<int32_t>> jobs_of(K);
+        for (int32_t j = 0; j < n; ++j)
+            if (cl.cls[j] >= 0) jobs_of[cl.cls[j]].push_back(j);
+        std::vector<size_t> next(K, 0);
+        for (size_t mu = 0; mu < machines.size(); ++mu)
+            for (int i = 0; i < K; ++i)
+                for (int32_t t = 0; t < machines[mu][i]; ++t) {
+                    if (next[i] >= jobs_of[i].size()) return PTAS_EINTERNAL;
+                    int32_t j = jobs_of[i][next[i]++];
+                    asg[j] = (int32_t)mu;
+                    load[mu] += p[j];
+                }
+        for (int i = 0; i < K; ++i)
+            if (next[i] != jobs_of[i].size()) return PTAS_EINTERNAL;
+    }
+    // short jobs in input order onto the least loaded machine (lowest index on ties)
+    using LI = std::pair<int64_t, int32_t>;
+    std::priority_queue<LI, std::vector<LI>, std::greater<LI>> heap;
+    for (int32_t q = 0; q < m; ++q) heap.push({load[q], q});
+    for (int32_t j = 0; j < n; ++j) {
+        if (cl.cls[j] >= 0) continue;
+        LI top = heap.top();
+        heap.pop();
+        asg[j] = top.second;
+        load[top.second] += p[j];
+        heap.push({load[top.second], top.second});
+    }
+    int64_t ms = 0;
+    for (int32_t q = 0; q < m; ++q) ms = std::max(ms, load[q]);
+
+    *makespan_out = ms;
+    std::memcpy(assignment_out, asg.data(), sizeof(int32_t) * n);
+    if (log) {
+        for (size_t q = 0; q < plog.size() && (int32_t)q < log_cap; ++q) log[q] = plog[q];
+    }
+    if (log_len) *log_len = (int32_t)plog.size();
+    if (stats) {
+        acc.s.probes = (int32_t)plog.size();
+        acc.s.rounds = round;
+        acc.s.K_at_Tstar = (int32_t)cl.N.size();
+        acc.s.T_star = Ts;
+        acc.s.opt_at_Tstar = opt_star;
+        acc.s.total_seconds = now_s() - t0;
+        *stats = acc.s;
+    }
+    return PTAS_OK;
+}
+
+int validate_dp(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T)
+{
+    if (K < 0 || K > 64) return PTAS_EINVAL;
+    if (K > 0 && (!counts || !sizes)) return PTAS_EINVAL;
+    if (T < 1) return PTAS_EINVAL;
+    for (int32_t i = 0; i < K; ++i) {
+        if (counts[i] < 0 || sizes[i] < 1) return PTAS_EINVAL;
+        if (counts[i] > 0 && sizes[i] > T) return PTAS_EINVAL;
+    }
+    return PTAS_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void ptas_default_options(ptas_options *o)
+{
+    if (!o) return;
+    std::memset(o, 0, sizeof(*o));
+    o->probes_per_round = 1;
+    o->mode = PTAS_MODE_SINGLE;
+    o->device = -1;
+    o->comm = nullptr;
+    o->table_budget_bytes = 0;
+    o->memoize = 1;
+    o->virtual_shards = 1;
+    o->layout = 0;
+}
+
+const char *ptas_strerror(int s)
+{
+    switch (s) {
+    case PTAS_OK: return "ok";
+    case PTAS_EINVAL: return "invalid argument";
+    case PTAS_ETOOBIG: return "DP table too big (sigma overflow, budget or sum(N) > 65535)";
+    case PTAS_ENOMEM: return "out of memory";
+    case PTAS_ECUDA: return "CUDA error (no device or kernel failure)";
+    case PTAS_ENCCL: return "NCCL unavailable or failed";
+    case PTAS_EINTERNAL: return "internal error";
+    default: return "unknown status";
+    }
+}
+
+int ptas_k(double eps) { return k_of(eps); }
+
+int ptas_bounds(const int64_t *p, int32_t n, int32_t m, int64_t *LB, int64_t *UB)
+{
+    if (!LB || !UB) return PTAS_EINVAL;
+    return validate_jobs(p, n, m, LB, UB);
+}
+
+int ptas_classify(const int64_t *p, int32_t n, int64_t T, int32_t k, int64_t *u_out, int32_t *K_out,
+                  int64_t *r_out, int32_t *N_out, int32_t *cls_out)
+{
+    if (!p || n < 1 || T < 1 || k < 1 || !u_out || !K_out || !r_out || !N_out || !cls_out)
+        return PTAS_EINVAL;
+    for (int32_t j = 0; j < n; ++j)
+        if (p[j] < 1) return PTAS_EINVAL;
+    Classified c;
+    classify(p, n, T, k, &c);
+    *u_out = c.u;
+    *K_out = (int32_t)c.N.size();
+    std::memcpy(r_out, c.r.data(), c.r.size() * 8);
+    std::memcpy(N_out, c.N.data(), c.N.size() * 4);
+    std::memcpy(cls_out, c.cls.data(), (size_t)n * 4);
+    return PTAS_OK;
+}
+
+int ptas_probe_targets(int64_t LB, int64_t UB, int32_t P, int64_t *out, int32_t *count)
+{
+    if (!out || !count) return PTAS_EINVAL;
+    std::vector<int64_t> v;
+    int rc = probe_targets(LB, UB, P, &v);
+    if (rc) return rc;
+    std::copy(v.begin(), v.end(), out);
+    *count = (int32_t)v.size();
+    return PTAS_OK;
+}
+
+int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T, const int32_t *feasible,
+                         int32_t count)
+{
+    if (!LB || !UB || !T || !feasible || count < 1 || *LB >= *UB) return PTAS_EINVAL;
+    interval_update(LB, UB, T, feasible, count);
+    return PTAS_OK;
+}
+
+int ptas_shard_range(int64_t count, int32_t rank, int32_t world, int64_t *begin, int64_t *end)
+{
+    if (count < 0 || world < 1 || rank < 0 || rank >= world || !begin || !end) return PTAS_EINVAL;
+    int64_t chunk = (count + world - 1) / world;
+    int64_t b = std::min<int64_t>(count, (int64_t)rank * chunk);
+    *begin = b;
+    *end = std::min<int64_t>(count, b + chunk);
+    return PTAS_OK;
+}
+
+int ptas_solve(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_options *opt,
+               int64_t *makespan_out, int32_t *assignment_out, ptas_stats *stats)
+{
+    return solve_core(p, n, m, eps, opt, makespan_out, assignment_out, stats, nullptr, 0, nullptr, 0, 0);
+}
+
+int ptas_solve_ex(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_options *opt,
+                  int64_t *makespan_out, int32_t *assignment_out, ptas_stats *stats, ptas_probe *log,
+                  int32_t log_cap, int32_t *log_len)
+{
+    return solve_core(p, n, m, eps, opt, makespan_out, assignment_out, stats, log, log_cap, log_len, 0, 0);
+}
+
+int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps, const ptas_options *opt,
+                      int64_t *makespan_out, int32_t *d_assignment, ptas_stats *stats)
+{
+    if (!d_p || !d_assignment || n < 1) return PTAS_EINVAL;
+    int dev;
+    int rc = resolve_device(opt ? opt->device : -1, &dev);
+    if (rc) return rc;
+    std::vector<int64_t> hp(n);
+    std::vector<int32_t> ha(n);
+    if (cudaMemcpy(hp.data(), d_p, (size_t)n * 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+        cudaGetLastError();
+        return PTAS_ECUDA;
+    }
+    rc = solve_core(hp.data(), n, m, eps, opt, makespan_out, ha.data(), stats, nullptr, 0, nullptr,
+                    (int64_t)n * 4, (int64_t)n * 8);
+    if (rc) return rc;
+    if (cudaMemcpy(d_assignment, ha.data(), (size_t)n * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+        cudaGetLastError();
+        return PTAS_ECUDA;
+    }
+    return PTAS_OK;
+}
+
+int dp_table_shape(const int32_t *counts, int32_t K, int64_t *sigma_out, int32_t *elem_bytes_out)
+{
+    if (K < 0 || K > 64 || (K > 0 && !counts) || !sigma_out || !elem_bytes_out) return PTAS_EINVAL;
+    __int128 sg = 1;
+    int64_t sumN = 0;
+    for (int32_t i = 0; i < K; ++i) {
+        if (counts[i] < 0) return PTAS_EINVAL;
+        sumN += counts[i];
+    }
+    for (int32_t i = 0; i < K; ++i) {
+        sg *= (__int128)counts[i] + 1;
+        if (sg > (__int128)INT64_MAX) return PTAS_ETOOBIG;
+    }
+    if (sumN > 65535) return PTAS_ETOOBIG;
+    *sigma_out = (int64_t)sg;
+    *elem_bytes_out = sumN <= 255 ? 1 : 2;
+    return PTAS_OK;
+}
+
+static int dp_fill_common(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T,
+                          void *d_ext, int64_t ext_bytes, cudaStream_t st, void *host_out,
+                          int64_t host_bytes, int32_t *opt_N_out, ptas_stats *stats)
+{
+    const double t0 = now_s();
+    int rc = validate_dp(counts, sizes, K, T);
+    if (rc) return rc;
+    if (!opt_N_out) return PTAS_EINVAL;
+    int64_t sigma;
+    int32_t e;
+    rc = dp_table_shape(counts, K, &sigma, &e);
+    if (rc) return rc;
+    if (host_out && host_bytes < sigma * e) return PTAS_EINVAL;
+    if (d_ext && ext_bytes < sigma * e) return PTAS_EINVAL;
+    int dev;
+    rc = resolve_device(-1, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+    DpRequest rq;
+    rq.K = K;
+    rq.N = counts;
+    rq.r = sizes;
+    rq.T = T;
+    rq.ext_table = d_ext;
+    rq.ext_bytes = ext_bytes;
+    rq.stream = st;
+    DpOutcome o;
+    rc = eng->run_dp(rq, &o);
+    if (rc) return rc;
+    Acc acc;
+    acc.add(o);
+    if (host_out) {
+        // engine-owned table; identity order => caller's layout
+        rc = eng->copy_table_to_host(host_out, sigma * e);
+        if (rc) return rc;
+        acc.s.d2h_bytes += sigma * e;
+    }
+    *opt_N_out = o.opt;
+    if (stats) {
+        acc.s.unique_dps = 1;
+        acc.s.total_seconds = now_s() - t0;
+        *stats = acc.s;
+    }
+    return PTAS_OK;
+}
+
+int dp_fill(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, void *table_out,
+            int64_t table_bytes, int32_t *opt_N_out, ptas_stats *stats)
+{
+    return dp_fill_common(counts, sizes, K, T, nullptr, 0, nullptr, table_out, table_bytes, opt_N_out,
+                          stats);
+}
+
+int dp_fill_device(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, void *d_table,
+                   int64_t table_bytes, void *cuda_stream, int32_t *opt_N_out)
+{
+    if (!d_table) return PTAS_EINVAL;
+    return dp_fill_common(counts, sizes, K, T, d_table, table_bytes, (cudaStream_t)cuda_stream,
+                          nullptr, 0, opt_N_out, nullptr);
+}
+
+int dp_configs(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int32_t *out_digits,
+               int64_t cap, int64_t *count)
+{
+    int rc = validate_dp(counts, sizes, K, T);
+    if (rc) return rc;
+    if (!count || (cap > 0 && !out_digits)) return PTAS_EINVAL;
+    int dev;
+    rc = resolve_device(-1, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+    DpRequest rq;
+    rq.K = K;
+    rq.N = counts;
+    rq.r = sizes;
+    rq.T = T;
+    std::vector<int32_t> dig;
+    int64_t c = 0;
+    rc = eng->configs_canonical(rq, &dig, &c);
+    if (rc) return rc;
+    *count = c;
+    if (out_digits && cap >= c) std::copy(dig.begin(), dig.end(), out_digits);
+    return PTAS_OK;
+}
+
+int dp_row_index(const int32_t *counts, int32_t K, int64_t *level_start, int64_t level_cap,
+                 int64_t *out_rowbase, int64_t rows_cap)
+{
+    if (K < 1 || K > 64 || !counts || !level_start) return PTAS_EINVAL;
+    int64_t sigma;
+    int32_t e;
+    int rc = dp_table_shape(counts, K, &sigma, &e);
+    if (rc) return rc;
+    int dev;
+    rc = resolve_device(-1, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+    std::vector<int64_t> ls, rb;
+    rc = eng->row_index(counts, K, &ls, &rb);
+    if (rc) return rc;
+    if ((int64_t)ls.size() > level_cap) return PTAS_EINVAL;
+    std::copy(ls.begin(), ls.end(), level_start);
+    if (out_rowbase) {
+        if ((int64_t)rb.size() > rows_cap) return PTAS_EINVAL;
+        std::copy(rb.begin(), rb.end(), out_rowbase);
+    }
+    return PTAS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,310 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, bit-exact.
+
+All tables are integer (uint8/uint16); comparisons are exact.  Sizes span
+several warp chunks and ragged tails (rows longer than 32 with W % 32 != 0,
+many rows per row-level, more rows than one wave of the grid).
+"""
+from __future__ import annotations
+
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from synth import WORKLOADS, jobs
+
+pytestmark = pytest.mark.gpu
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def P():
+    import paper_conf_ipps_ligsg18_b200 as P
+    return P
+
+
+def _rand_case(rng, K, maxN, e16=False):
+    N = rng.integers(0, maxN + 1, K).astype(np.int32)
+    if e16:
+        N[rng.integers(0, K)] += 256
+    r = rng.integers(20, 200, K).astype(np.int64)
+    T = int(rng.integers(int(r.max()), int(r.max()) * 6))
+    return N, r, T
+
+
+# ------------------------------------------------------------------ a-3
+def test_configs_match_oracle(P):
+    rng = np.random.default_rng(100)
+    for trial in range(120):
+        K = int(rng.integers(1, 10))
+        N, r, T = _rand_case(rng, K, 6)
+        got = P.dp_configs(N, r, T)
+        want = oracle.configs(N, r, T)
+        assert got.shape == want.shape and (got == want).all(), (N, r, T)
+
+
+def test_configs_large_box(P):
+    # many configurations (capacity admits ~k items of small classes)
+    N = np.array([40, 30, 25, 20, 18, 15], np.int32)
+    r = np.array([30, 37, 41, 53, 60, 71], np.int64)
+    got = P.dp_configs(N, r, 400)
+    want = oracle.configs(N, r, 400)
+    assert len(want) > 1000 and (got == want).all()
+
+
+# ------------------------------------------------------------------ a-4
+def test_row_index_complete(P):
+    rng = np.random.default_rng(5)
+    for trial in range(30):
+        K = int(rng.integers(1, 7))
+        N = rng.integers(0, 9, K).astype(np.int32)
+        ls, rb = P.dp_row_index(N)
+        nz = N[N > 0]
+        if len(nz) == 0:
+            assert list(ls) == [0, 1] and list(rb) == [0]
+            continue
+        W = int(nz[-1]) + 1
+        sigma = int(np.prod(nz.astype(np.int64) + 1))
+        # level sizes = coefficients of prod_{i<K-1} (1 + z + ... + z^{N_i})
+        poly = np.array([1], np.int64)
+        for x in nz[:-1]:
+            poly = np.convolve(poly, np.ones(int(x) + 1, np.int64))
+        assert list(np.diff(ls)) == list(poly)
+        # every row exactly once, in lexicographic order within a level
+        assert sorted(rb.tolist()) == list(range(0, sigma, W))
+        shape = tuple(int(x) + 1 for x in nz[:-1])
+        for L in range(len(poly)):
+            rows = rb[ls[L]:ls[L + 1]] // W
+            digs = [np.unravel_index(int(q), shape) if shape else () for q in rows]
+            assert all(sum(d) == L for d in digs)
+            assert digs == sorted(digs)
+
+
+# ------------------------------------------------------------------ a-5
+def _check_table(P, N, r, T):
+    opt, tab, st = P.dp_fill(N, r, T)
+    want, relax = oracle.dp(N, r, T)
+    assert tab.shape == want.shape
+    bad = np.argwhere(tab.astype(np.int64) != want)
+    assert len(bad) == 0, (N.tolist(), r.tolist(), T, bad[:5].tolist())
+    assert opt == int(want[tuple(N)]) if len(N) else opt == 0
+    assert st["relaxations"] == relax
+    return tab
+
+
+def test_g1_golden(P):
+    g = json.load(open(os.path.join(GOLD, "g1_table.json")))
+    opt, tab, st = P.dp_fill(g["N"], g["r"], g["T"])
+    assert tab.tolist() == g["table"]
+    assert st["relaxations"] == g["relax"]
+    assert opt == 2
+
+
+@pytest.mark.parametrize("K", [1, 2, 3, 4, 5, 6, 7, 8, 9])
+def test_dp_fill_random_uint8(P, K):
+    rng = np.random.default_rng(1000 + K)
+    maxN = {1: 200, 2: 60, 3: 25, 4: 12, 5: 8, 6: 6, 7: 4, 8: 3, 9: 3}[K]
+    for _ in range(12):
+        N, r, T = _rand_case(rng, K, maxN)
+        _check_table(P, N, r, T)
+
+
+@pytest.mark.parametrize("K", [1, 2, 3, 4])
+def test_dp_fill_random_uint16(P, K):
+    rng = np.random.default_rng(2000 + K)
+    for _ in range(4):
+        N = rng.integers(1, {1: 300, 2: 200, 3: 60, 4: 20}[K], K).astype(np.int32)
+        N[-1] = max(int(N[-1]), 256 - int(N[:-1].sum()) + 1) if K > 1 else max(int(N[0]), 300)
+        r = rng.integers(20, 200, K).astype(np.int64)
+        T = int(rng.integers(int(r.max()), int(r.max()) * 5))
+        assert N.sum() > 255
+        _check_table(P, N, r, T)
+
+
+def test_dp_fill_long_rows_ragged(P):
+    # W = 71 (3 chunks of 32, ragged), small last size -> long in-row chains (J0 large)
+    _check_table(P, np.array([5, 4, 70], np.int32), np.array([90, 70, 11], np.int64), 200)
+    _check_table(P, np.array([3, 3, 3, 100], np.int32), np.array([50, 60, 70, 7], np.int64), 250)
+    # J0 > 32: in-row chain crosses chunk boundaries
+    _check_table(P, np.array([2, 120], np.int32), np.array([40, 3], np.int64), 150)
+    # W = 33 and W = 32 exactly
+    _check_table(P, np.array([6, 5, 32], np.int32), np.array([40, 50, 30], np.int64), 160)
+    _check_table(P, np.array([6, 5, 31], np.int32), np.array([40, 50, 30], np.int64), 160)
+
+
+def test_dp_fill_zero_counts_and_degenerate(P):
+    _check_table(P, np.array([0, 3, 0, 4], np.int32), np.array([10, 20, 30, 40], np.int64), 60)
+    opt, tab, st = P.dp_fill(np.zeros(0, np.int32), np.zeros(0, np.int64), 10)
+    assert opt == 0 and tab.shape == () and int(tab) == 0
+    opt, tab, st = P.dp_fill([0, 0], [5, 50], 10)   # sizes > T allowed when count is 0
+    assert opt == 0
+    _check_table(P, np.array([1], np.int32), np.array([7], np.int64), 7)
+    _check_table(P, np.array([9], np.int32), np.array([7], np.int64), 7)   # one per machine
+
+
+def test_dp_fill_invalid(P):
+    with pytest.raises(P.PtasError) as ei:
+        P.dp_fill([3], [11], 10)            # size > T with count > 0
+    assert ei.value.rc == -1
+    with pytest.raises(P.PtasError) as ei:
+        P.dp_fill([-1], [5], 10)
+    assert ei.value.rc == -1
+    with pytest.raises(P.PtasError) as ei:
+        P.dp_fill([40000, 40000], [5, 5], 10)   # sum N > 65535
+    assert ei.value.rc == -2
+
+
+def test_dp_fill_device_torch(P):
+    import torch
+    N = np.array([7, 9, 40], np.int32)
+    r = np.array([33, 45, 20], np.int64)
+    sg, e = P.dp_table_shape(N)
+    t = torch.full((sg,), 255, dtype=torch.uint8, device="cuda:0")
+    s = torch.cuda.Stream()
+    opt = P.dp_fill_device(N, r, 150, t, stream=s)
+    want, _ = oracle.dp(N, r, 150)
+    torch.cuda.synchronize()
+    assert (t.cpu().numpy().reshape(want.shape).astype(np.int64) == want).all()
+    assert opt == want[tuple(N)]
+
+
+def test_dp_fill_two_word_packing(P, monkeypatch):
+    # force the leading digits into two 64-bit words (exercises the NW=2 kernels)
+    monkeypatch.setenv("PTAS_FORCE_TWO_WORDS", "1")
+    rng = np.random.default_rng(77)
+    for K in (3, 5, 8):
+        for _ in range(4):
+            N, r, T = _rand_case(rng, K, {3: 20, 5: 6, 8: 3}[K])
+            _check_table(P, N, r, T)
+
+
+# ------------------------------------------------------------------ end to end
+def _cmp_solve(P, p, m, eps, Pp, **kw):
+    got = P.ptas_solve(p, m, eps, P=Pp, **kw)
+    want = oracle.ptas(p, m, eps, Pp)
+    assert got["T_star"] == want["T_star"]
+    assert got["makespan"] == want["makespan"]
+    assert got["assignment"].tolist() == want["assignment"].tolist()
+    assert [(T, rd, f, K, o) for (T, rd, f, K, o, _s, _h) in got["probes"]] == \
+           [(T, rd, f, K, o) for (T, rd, f, K, o, _s) in want["probes"]]
+    return got
+
+
+def test_solve_m1_seeds(P):
+    for seed in range(120):
+        p = jobs(12, 100, seed)
+        for Pp in (1, 4):
+            _cmp_solve(P, p, 3, 0.3, Pp)
+
+
+def test_solve_layouts_and_memo(P):
+    for seed in range(20):
+        p = jobs(16, 100, seed)
+        for layout in (0, 1):
+            for memo in (True, False):
+                _cmp_solve(P, p, 3, 0.25, 2, layout=layout, memoize=memo)
+
+
+def test_solve_g3_nonmonotone(P):
+    g = json.load(open(os.path.join(GOLD, "g3_nonmonotone.json")))
+    for Pp, want in g["by_P"].items():
+        got = P.ptas_solve(g["p"], g["m"], g["eps"], P=int(Pp))
+        assert got["T_star"] == want["T_star"] and got["makespan"] == want["makespan"]
+        assert [[T, f] for (T, _r, f, *_x) in got["probes"]] == want["probes"]
+
+
+def test_solve_g2(P):
+    g = json.load(open(os.path.join(GOLD, "g2_m1_seed0.json")))
+    got = P.ptas_solve(g["p"], g["m"], g["eps"], P=1)
+    assert got["T_star"] == g["T_star"] and got["makespan"] == g["makespan"]
+    assert got["assignment"].tolist() == g["assignment"]
+
+
+def test_solve_medium_instances(P):
+    # shaped like the paper's workloads but small enough for the oracle
+    for (n, m, eps, seed) in [(40, 8, 0.3, 1), (60, 14, 0.3, 2), (50, 10, 0.2, 3), (30, 5, 0.15, 4)]:
+        p = jobs(n, 1000, seed)
+        for Pp in (1, 3):
+            _cmp_solve(P, p, m, eps, Pp)
+
+
+def test_solve_virtual_shards_identical(P):
+    for seed in range(6):
+        p = jobs(40, 1000, seed)
+        ref = P.ptas_solve(p, 8, 0.3, P=1)
+        for vs in (2, 3, 8):
+            got = P.ptas_solve(p, 8, 0.3, P=1, mode=P.MODE_LEVEL_SHARDED, virtual_shards=vs)
+            assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
+            assert (got["assignment"] == ref["assignment"]).all()
+            assert [x[:5] for x in got["probes"]] == [x[:5] for x in ref["probes"]]
+
+
+def test_solve_empty_dp_literal(P):
+    for name in ("M2", "M3", "M4"):
+        w = WORKLOADS[name]
+        got = P.ptas_solve(w.p(), w.m, w.eps, P=1)
+        want = oracle.ptas(w.p(), w.m, w.eps, 1)
+        assert got["T_star"] == want["T_star"] and got["makespan"] == want["makespan"]
+        assert got["assignment"].tolist() == want["assignment"].tolist()
+
+
+def test_solve_device_variant(P):
+    import torch
+    p = jobs(60, 1000, 9)
+    pd = torch.from_numpy(p).cuda()
+    ad = torch.zeros(60, dtype=torch.int32, device="cuda")
+    got = P.ptas_solve_device(pd, 14, 0.3, ad)
+    want = oracle.ptas(p, 14, 0.3, 1)
+    assert got["makespan"] == want["makespan"]
+    assert ad.cpu().numpy().tolist() == want["assignment"].tolist()
+
+
+def test_solve_invalid(P):
+    for args in [([], 3, 0.3), ([1, 2], 0, 0.3), ([1, 0], 2, 0.3), ([1, 2], 2, 0.0), ([1, 2], 2, float("nan"))]:
+        with pytest.raises(P.PtasError) as ei:
+            P.ptas_solve(*args)
+        assert ei.value.rc == -1
+
+
+# ------------------------------------------------------------------ full size (bench configuration)
+def _subbox(N, cap_sigma=2_000_000):
+    Nc = N.copy()
+    while np.prod(Nc.astype(np.float64) + 1) > cap_sigma:
+        i = int(np.argmax(Nc))
+        Nc[i] -= 1
+    return Nc
+
+
+@pytest.mark.parametrize("name", ["M2s", "M4s", "M3s"])
+def test_full_size_dp_sampled(P, name):
+    """Full-size DP of the workload at T = LB (its largest probe): exact parity
+    on a sub-box (the DP restricted to n <= N' equals the oracle's DP on N'),
+    Eq. 1 re-checked at sampled states, and invariants on the whole table."""
+    w = WORKLOADS[name]
+    p = w.p()
+    k = oracle.k_of(w.eps)
+    LB, _ = oracle.bounds(p, w.m)
+    u, r, N, _ = oracle.classify(p, LB, k)
+    opt, tab, st = P.dp_fill(N, r, LB)
+    t64 = tab.astype(np.int64)
+    Nc = _subbox(N)
+    want, _ = oracle.dp(Nc, r, LB)
+    sub = t64[tuple(slice(0, int(x) + 1) for x in Nc)]
+    assert (sub == want).all()
+    C = oracle.configs(N, r, LB)
+    assert st["relaxations"] == sum(float(np.prod((N - s + 1).astype(np.float64))) for s in C)
+    rng = np.random.default_rng(0)
+    for _ in range(3000):
+        n = np.array([rng.integers(0, x + 1) for x in N])
+        if not n.any():
+            continue
+        cand = [t64[tuple(n - s)] for s in C if (s <= n).all()]
+        assert t64[tuple(n)] == 1 + min(cand)
+    assert t64.flat[0] == 0
+    for ax in range(len(N)):
+        d = np.diff(t64, axis=ax)
+        assert d.min() >= 0 and d.max() <= 1
+    assert opt == t64[tuple(N)]
