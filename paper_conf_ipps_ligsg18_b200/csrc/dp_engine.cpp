@@ -11,6 +11,7 @@
 //   a-6 OPT(N) read back with the planning summary in one 40-byte D2H.
 // Host syncs per DP: one after the config count (to size C), one at the end.
 #include <algorithm>
+#include <cstdint>
 #include <cstdlib>
 #include <cstring>
 #include <map>
@@ -106,15 +107,19 @@ static int bits_of(int32_t x)
 }
 
 // Geometry of the row space of an internal-order DP (a-2, a-4).
-static int build_geom(const std::vector<int32_t> &N, RowGeom *g, std::vector<int64_t> *cnt,
-                      std::vector<int64_t> *stride)
+// pad: rows stored with pitch Wp = W*e rounded up to 4 bytes (the packed-word
+// kernel's layout); without padding the layout is the caller's (pitch W).
+static int build_geom(const std::vector<int32_t> &N, int e, bool pad, RowGeom *g,
+                      std::vector<int64_t> *cnt, std::vector<int64_t> *stride)
 {
     const int K = (int)N.size();
     std::memset(g, 0, sizeof(*g));
-    stride->assign(K, 1);
-    for (int i = K - 2; i >= 0; --i) (*stride)[i] = (*stride)[i + 1] * (N[i + 1] + 1);
     g->K1 = K - 1;
     g->W = N[K - 1] + 1;
+    g->Wp = pad ? ((g->W * e + 3) / 4 * 4) / e : g->W;
+    stride->assign(K, 1);
+    if (K >= 2) (*stride)[K - 2] = g->Wp;
+    for (int i = K - 3; i >= 0; --i) (*stride)[i] = (*stride)[i + 1] * (N[i + 1] + 1);
     int rho_max = 0;
     for (int i = 0; i < K - 1; ++i) {
         g->N[i] = N[i];
@@ -194,21 +199,18 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     const int64_t sigma = (int64_t)sg;
     const int e = sumN <= 255 ? 1 : 2;
     const int64_t bytes = sigma * e;
-    void *table = rq.ext_table;
-    if (table) {
-        if (rq.ext_bytes < bytes) return PTAS_EINVAL;
-    } else {
-        int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
-        if (bytes > budget) return PTAS_ETOOBIG;
-        PT_CK(table_.ensure((size_t)bytes));
-        table = table_.p;
-    }
+    if (rq.ext_table && rq.ext_bytes < bytes) return PTAS_EINVAL;
     last_valid_ = false;
     o.sigma = sigma;
     o.e = e;
     o.Kint = K;
-    PT_CK(cudaEventRecord(ev_[0], st));
     if (K == 0) {
+        void *table = rq.ext_table;
+        if (!table) {
+            PT_CK(table_.ensure(16));
+            table = table_.p;
+        }
+        PT_CK(cudaEventRecord(ev_[0], st));
         PT_CK(launch_fill_value(table, e, 0, st));
         PT_CK(cudaEventRecord(ev_[1], st));
         PT_CK(cudaEventRecord(ev_[2], st));
@@ -225,14 +227,32 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
         last_sigma_ = 1;
         last_nC_ = 0;
         last_opt_ = 0;
+        last_W_ = last_Wp_ = 1;
+        last_rows_ = 1;
         last_order_.clear();
         *out = o;
         return PTAS_OK;
     }
     RowGeom g;
     std::vector<int64_t> cnt, stride;
-    rc = build_geom(N, &g, &cnt, &stride);
+    rc = build_geom(N, e, true, &g, &cnt, &stride);
     if (rc) return rc;
+    const int64_t rows = sigma / g.W;
+    const int64_t ibytes = rows * g.Wp * e;  // padded internal table
+    // compute in the caller's buffer when its layout is the padded one
+    void *table = nullptr;
+    const bool in_place = rq.ext_table && g.Wp == g.W && ((uintptr_t)rq.ext_table & 3) == 0;
+    if (in_place) {
+        table = rq.ext_table;
+    } else {
+        int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
+        if (ibytes > budget) return PTAS_ETOOBIG;
+        PT_CK(table_.ensure((size_t)ibytes));
+        table = table_.p;
+    }
+    PT_CK(cudaEventRecord(ev_[0], st));
+    int64_t idxN = N[K - 1];
+    for (int i = 0; i < K - 1; ++i) idxN += (int64_t)N[i] * stride[i];
 
     // ---- uploads: r[K] int64 | stride[K] int64 | hi[K] int32, then cnt table
     std::vector<int32_t> hi(K);
@@ -283,6 +303,20 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
                               N.data(), (PrefixEntry *)pref_.p, d_meta_, st));
     o.launches += 2;
     const int J0 = (int)std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
+    const char *fs = std::getenv("PTAS_FORCE_SCALAR");
+    const bool force_scalar = fs && fs[0] == '1';
+    // one row-level (or slice of it): packed-word kernel, scalar kernel as fallback
+    auto fill = [&](void *tab, const RowGeom &gg, int j0, int rho_, int64_t b, int64_t c,
+                    void *compact) -> cudaError_t {
+        cudaError_t err = cudaErrorNotSupported;
+        if (!force_scalar)
+            err = launch_row_fill_swar(e, tab, gg, (const int64_t *)cnt_.p, (const PrefixEntry *)pref_.p,
+                                       d_meta_, nC, j0, rho_, b, c, compact, sm_count_, st);
+        if (err == cudaErrorNotSupported)
+            err = launch_row_fill(e, tab, gg, (const int64_t *)cnt_.p, (const PrefixEntry *)pref_.p,
+                                  d_meta_, nC, j0, rho_, b, c, compact, sm_count_, st);
+        return err;
+    };
 
     // ---- a-5 level fill, one launch per row-level
     int G = 1, myrank = 0;
@@ -305,7 +339,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
             int64_t R = cnt[rho];
             if (!sharded(R)) continue;
             int64_t chunk = (R + G - 1) / G;
-            mx = std::max(mx, (size_t)(chunk * G * g.W * e));
+            mx = std::max(mx, (size_t)(chunk * G * g.Wp * e));
         }
         PT_CK(stage_.ensure(mx));
     }
@@ -314,8 +348,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
         const int64_t R = cnt[rho];
         if (R <= 0) continue;
         if (!sharded(R)) {
-            PT_CK(launch_row_fill(e, table, g, (const int64_t *)cnt_.p, (const PrefixEntry *)pref_.p,
-                                  d_meta_, nC, J0, rho, 0, R, nullptr, sm_count_, st));
+            PT_CK(fill(table, g, J0, rho, 0, R, nullptr));
             ++o.fill_launches;
             continue;
         }
@@ -325,21 +358,17 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
             for (int v = 0; v < G; ++v) {
                 int64_t b = v * chunk, c = std::min(R, b + chunk) - b;
                 if (c <= 0) continue;
-                PT_CK(launch_row_fill(e, table, g, (const int64_t *)cnt_.p,
-                                      (const PrefixEntry *)pref_.p, d_meta_, nC, J0, rho, b, c,
-                                      stage + b * g.W * e, sm_count_, st));
+                PT_CK(fill(table, g, J0, rho, b, c, stage + b * g.Wp * e));
                 ++o.fill_launches;
             }
         } else {
             int64_t b = myrank * chunk, c = std::min(R, b + chunk) - b;
             if (c > 0) {
-                PT_CK(launch_row_fill(e, table, g, (const int64_t *)cnt_.p,
-                                      (const PrefixEntry *)pref_.p, d_meta_, nC, J0, rho, b, c,
-                                      stage + b * g.W * e, sm_count_, st));
+                PT_CK(fill(table, g, J0, rho, b, c, stage + b * g.Wp * e));
                 ++o.fill_launches;
             }
-            int crc = comm_allgather(sh->comm, stage + (size_t)myrank * chunk * g.W * e, stage,
-                                     (size_t)(chunk * g.W * e), st);
+            int crc = comm_allgather(sh->comm, stage + (size_t)myrank * chunk * g.Wp * e, stage,
+                                     (size_t)(chunk * g.Wp * e), st);
             if (crc) return crc;
         }
         PT_CK(launch_row_scatter(e, table, g, (const int64_t *)cnt_.p, rho, R, stage, sm_count_, st));
@@ -350,8 +379,12 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     (void)ld;
 
     // ---- a-6 readout
-    PT_CK(launch_read_opt(e, table, sigma - 1, d_meta_, st));
+    PT_CK(launch_read_opt(e, table, idxN, d_meta_, st));
     ++o.launches;
+    if (rq.ext_table && !in_place) {
+        PT_CK(launch_compact_rows(e, table, rq.ext_table, rows, g.W, g.Wp, st));
+        ++o.launches;
+    }
     PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
     PT_CK(cudaEventRecord(ev_[3], st));
     PT_CK(cudaStreamSynchronize(st));
@@ -378,6 +411,10 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     last_order_ = order;
     last_N_ = N;
     last_stride_ = stride;
+    last_W_ = g.W;
+    last_Wp_ = g.Wp;
+    last_rows_ = rows;
+    last_idxN_ = idxN;
     *out = o;
     return PTAS_OK;
 }
@@ -416,7 +453,7 @@ int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
     PT_CK(cudaMemsetAsync(&d_meta_->err, 0, 4, st));
     acc->h2d += (int64_t)(K * 8 + nC * 4 + K * 4);
     PT_CK(launch_traceback(last_e_, last_table_, K, d_N, d_stride, (const uint16_t *)digits_.p,
-                           (const int64_t *)off_.p, d_rank, nC, last_sigma_, d_out, last_opt_,
+                           (const int64_t *)off_.p, d_rank, nC, last_idxN_, d_out, last_opt_,
                            d_len, d_meta_, st));
     acc->launches += 1;
     // d_len[0] = length, d_len[4 ..] = chosen configurations (d_out = d_len + 4)
@@ -435,7 +472,14 @@ int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
 int Engine::copy_table_to_host(void *dst, int64_t bytes)
 {
     if (!last_valid_) return PTAS_EINTERNAL;
-    PT_CK(cudaMemcpyAsync(dst, last_table_, (size_t)bytes, cudaMemcpyDeviceToHost, last_stream_));
+    const void *src = last_table_;
+    if (last_Wp_ != last_W_) {
+        PT_CK(stage_.ensure((size_t)bytes));
+        PT_CK(launch_compact_rows(last_e_, last_table_, stage_.p, last_rows_, last_W_, last_Wp_,
+                                  last_stream_));
+        src = stage_.p;
+    }
+    PT_CK(cudaMemcpyAsync(dst, src, (size_t)bytes, cudaMemcpyDeviceToHost, last_stream_));
     PT_CK(cudaStreamSynchronize(last_stream_));
     return PTAS_OK;
 }
@@ -518,7 +562,7 @@ int Engine::row_index(const int32_t *Nc, int Kc, std::vector<int64_t> *level_sta
     }
     RowGeom g;
     std::vector<int64_t> cnt, stride;
-    int rc = build_geom(N, &g, &cnt, &stride);
+    int rc = build_geom(N, 1, false, &g, &cnt, &stride);
     if (rc) return rc;
     cudaStream_t st = stream_;
     PT_CK(cnt_.ensure(cnt.size() * 8));

@@ -15,13 +15,11 @@
 #include <cuda_runtime.h>
 
 #include "internal.h"
+#include "device_common.cuh"
 
 namespace ptas {
 
 namespace {
-
-constexpr unsigned FULL = 0xffffffffu;
-constexpr int INF = 1 << 28;
 
 // ------------------------------------------------------------------ a-3
 // One thread per prefix over the first D internal dims (mixed radix, first
@@ -237,101 +235,165 @@ __device__ __forceinline__ void unrank_row(const RowGeom &g, const int64_t *cnt,
 }
 
 // ------------------------------------------------------------------ a-5
-// Level fill of one row-level.  A lane group of Wg = 2^wlog lanes owns one
-// row p (32/Wg rows per warp); lanes cover x in chunks of Wg.  For each state
-// n = (p, x):
-//   acc(x) = min over prefixes s' != 0 with s' <= p (packed-digit compare,
-//            uniform per group) and j in [0, min(Jmax(s'), x)] of
-//            OPT(p - s', x - j)                       (cross-row relaxations)
+// Level fill of one row-level (Eq. 1).  A lane group of
+// Wg = 2^wlog lanes owns one row p (32/Wg rows per warp) and walks a chunk of
+// `crows` consecutive rows of the level (unrank once, then step with
+// next_in_level); lanes cover x in chunks of Wg.  For each state n = (p, x):
+//   acc(x) = min over prefixes s' != 0 with s' <= p and j in
+//            [0, min(Jmax(s'), x)] of OPT(p - s', x - j)   (cross-row relaxations)
 //   OPT(p, x) = 1 + min(acc(x), min_{1<=j<=min(J0,x)} OPT(p, x - j))
-// the last term (s' = 0) is the in-row chain, resolved by shuffles within
-// the chunk (Bellman-Ford rounds until no lane changes) and by loads of the
+// Dominance s' <= p is a packed-digit compare ((P|G) - S') & G == G done
+// cooperatively: lane xl tests prefix base+xl and a ballot yields the group's
+// dominated set, which every lane of the group then walks (ffs loop).  The
+// prefix table (off, Jmax, packed words) and the row-count table are staged
+// in shared memory.  The in-row term (s' = 0) is resolved by shuffles within
+// the chunk (Bellman-Ford rounds until no lane changes) and loads of the
 // already-stored previous chunks.  Every (n, s) pair with s in C, s <= n is
 // relaxed exactly once: the relaxation count is the closed form.
-template <typename E, int NW>
+template <typename E, int NW, bool MULTI>
 __global__ void __launch_bounds__(256)
 row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt,
-                const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
-                int smem_pref, int smem_cnt, int J0, int rho, int64_t slot_begin,
-                int64_t slot_count, E *compact, int wlog)
+                const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
+                int rho, int64_t slot_begin, int64_t slot_count, E *compact, int wlog, int crows)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int64_t nP = meta->nP;
-    const int np = (int)(nP - 1);            // cross-row prefixes (entry 0 is s' = 0)
-    PrefixEntry *spref = reinterpret_cast<PrefixEntry *>(smem_raw);
-    int64_t *scnt = reinterpret_cast<int64_t *>(smem_raw + (size_t)smem_pref * sizeof(PrefixEntry));
+    const int np = (int)(meta->nP - 1);      // cross-row prefixes (entry 0 is s' = 0)
     const int ncnt = (g.K1 + 1) * (g.rho_max + 1);
-    if (smem_pref)
-        for (int i = threadIdx.x; i < np; i += blockDim.x) spref[i] = gpref[1 + i];
-    if (smem_cnt)
-        for (int i = threadIdx.x; i < ncnt; i += blockDim.x) scnt[i] = gcnt[i];
+    // s_oj[c] = (Jmax << 48) | off(s')   (off < 2^48 since sigma < 2^48)
+    uint64_t *s_oj = reinterpret_cast<uint64_t *>(smem_raw);
+    uint64_t *s_w = s_oj + np;
+    int64_t *s_cnt = reinterpret_cast<int64_t *>(s_w + (size_t)NW * np);
+    for (int i = threadIdx.x; i < np; i += blockDim.x) {
+        const PrefixEntry pe = gpref[1 + i];
+        s_oj[i] = ((uint64_t)(uint32_t)pe.jmax << 48) | (uint64_t)pe.off;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
+    }
+    for (int i = threadIdx.x; i < ncnt; i += blockDim.x) s_cnt[i] = gcnt[i];
     __syncthreads();
-    const PrefixEntry *P = smem_pref ? spref : gpref + 1;
-    const int64_t *cnt = smem_cnt ? scnt : gcnt;
 
     const int lane = threadIdx.x & 31;
     const int Wg = 1 << wlog;
     const int grp = lane >> wlog;
     const int xl = lane & (Wg - 1);
     const int rpw = 32 >> wlog;
+    const unsigned gmask = Wg == 32 ? 0xffffffffu : ((1u << Wg) - 1u);
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t nslot_w = (slot_count + rpw - 1) / rpw;
     const int64_t W = g.W;
-
-    for (int64_t ws = gw; ws < nslot_w; ws += nw) {
-        const int64_t slot = ws * rpw + grp;
-        const bool rowok = slot < slot_count;
-        uint64_t pw[NW];
-        int64_t rowbase = 0;
-        if (rowok) unrank_row<NW>(g, cnt, rho, slot_begin + slot, pw, rowbase);
-        else {
+    const int64_t nchunks = (slot_count + crows - 1) / crows;
+    uint64_t guard[NW];
 #pragma unroll
-            for (int w = 0; w < NW; ++w) pw[w] = 0;
-        }
-        E *out = compact ? compact + slot * W : table + rowbase;
-        for (int64_t x0 = 0; x0 < W; x0 += Wg) {
-            const int64_t x = x0 + xl;
-            const bool act = rowok && x < W;
-            int acc = INF;
-            if (act) {
-                for (int c = 0; c < np; ++c) {
-                    const PrefixEntry pe = P[c];
-                    bool dom = true;
+    for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
+    int32_t d[MAXK];
+
+    for (int64_t cb = gw * rpw; cb < nchunks; cb += nw * rpw) {
+        const int64_t ch = cb + grp;
+        const int64_t r0 = ch * crows;
+        const int64_t r1 = r0 + crows < slot_count ? r0 + crows : slot_count;
+        int64_t rowbase = 0;
+        uint64_t pw[NW];
+#pragma unroll
+        for (int w = 0; w < NW; ++w) pw[w] = 0;
+        for (int rr = 0; rr < crows; ++rr) {
+            const int64_t slot = r0 + rr;
+            const bool rowok = slot < r1;
+            if (!__any_sync(FULL, rowok)) break;
+            if (rowok) {
+                if (rr == 0) unrank_digits(g, s_cnt, rho, slot_begin + slot, d);
+                else next_in_level(g, d);
+                rowbase = 0;
+#pragma unroll
+                for (int w = 0; w < NW; ++w) pw[w] = 0;
+                for (int i = 0; i < g.K1; ++i) {
+                    rowbase += (int64_t)d[i] * g.stride[i];
 #pragma unroll
                     for (int w = 0; w < NW; ++w)
-                        dom &= (((pw[w] | g.guard[w]) - pe.w[w]) & g.guard[w]) == g.guard[w];
-                    if (dom) {
-                        const E *src = table + (rowbase - pe.off + x);
-                        const int jm = pe.jmax < x ? pe.jmax : (int)x;
-                        for (int j = 0; j <= jm; ++j) {
-                            int v = src[-j];
-                            acc = v < acc ? v : acc;
+                        if (g.word[i] == w) pw[w] |= (uint64_t)d[i] << g.shift[i];
+                }
+            }
+            E *out = compact ? compact + slot * g.Wp : table + rowbase;
+            for (int64_t x0 = 0; x0 < W; x0 += Wg) {
+                const int64_t x = x0 + xl;
+                const bool act = rowok && x < W;
+                const E *rowp = table + (rowbase + x);
+                const int xi = x < (1 << 20) ? (int)x : (1 << 20);
+                int acc = INF;
+                for (int base = 0; base < np; base += Wg) {
+                    const int c = base + xl;
+                    bool dom = false;
+                    if (rowok && c < np) {
+                        dom = true;
+#pragma unroll
+                        for (int w = 0; w < NW; ++w)
+                            dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
+                    }
+                    unsigned m = (__ballot_sync(FULL, dom) >> (grp << wlog)) & gmask;
+                    // Walk the group's dominated prefixes, 4 at a time so that 4 (or 8)
+                    // coalesced gathers are in flight.  Lane xl loads OPT(p - s', x) (and,
+                    // for rows longer than a chunk, OPT(p - s', x - Wg)); the values at
+                    // x - j for j = 1..Jmax(s') arrive by shuffle from lane xl - j: source
+                    // lane t sends v0 if t + j < Wg (same chunk) else vprev (previous chunk).
+                    while (__any_sync(FULL, m != 0)) {
+                        int v0[4], vp[4], jm[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            v0[q] = INF;
+                            vp[q] = INF;
+                            jm[q] = -1;
+                            if (m) {
+                                const int b = __ffs(m) - 1;
+                                m &= m - 1;
+                                const uint64_t oj = s_oj[base + b];
+                                const E *src = rowp - (int64_t)(oj & 0xffffffffffffull);
+                                jm[q] = (int)(oj >> 48);
+                                if (act) v0[q] = src[0];
+                                if (MULTI && x0 > 0 && xl + jm[q] >= Wg) vp[q] = src[-Wg];
+                            }
+                        }
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            acc = v0[q] < acc ? v0[q] : acc;
+                            int jmq = jm[q];
+                            // jm is uniform within a group; the shuffle loop runs to the
+                            // max over the warp's groups
+                            int jmax_w = jmq;
+                            for (int o = 16; o >= Wg; o >>= 1) {
+                                int t = __shfl_xor_sync(FULL, jmax_w, o);
+                                jmax_w = t > jmax_w ? t : jmax_w;
+                            }
+                            for (int j = 1; j <= jmax_w; ++j) {
+                                const int send = (xl + j < Wg) ? v0[q] : vp[q];
+                                const int t = __shfl_sync(FULL, send, (xl - j) & (Wg - 1), Wg);
+                                if (j <= jmq && t < acc) acc = t;
+                            }
                         }
                     }
                 }
-                // in-row terms that reach back into earlier (stored) chunks
-                const int jlim = J0 < x ? J0 : (int)x;
-                for (int j = xl + 1; j <= jlim; ++j) {
-                    int v = out[x - j];
-                    acc = v < acc ? v : acc;
+                if (act) {
+                    // in-row terms that reach back into earlier (stored) chunks
+                    const int jlim = J0 < x ? J0 : (int)x;
+                    for (int j = xl + 1; j <= jlim; ++j) {
+                        int v = out[x - j];
+                        acc = v < acc ? v : acc;
+                    }
                 }
-            }
-            int opt = (rho == 0 && x == 0) ? 0 : acc + 1;
-            // in-chunk chain: Bellman-Ford over shuffles
-            const int jin = J0 < Wg - 1 ? J0 : Wg - 1;
-            bool changed = jin > 0;
-            while (__any_sync(FULL, changed)) {
-                int nopt = opt;
-                for (int j = 1; j <= jin; ++j) {
-                    int v = __shfl_up_sync(FULL, opt, j, Wg);
-                    if (xl >= j && v + 1 < nopt) nopt = v + 1;
+                int opt = (rho == 0 && x == 0) ? 0 : acc + 1;
+                // in-chunk chain: Bellman-Ford over shuffles
+                const int jin = J0 < Wg - 1 ? J0 : Wg - 1;
+                bool changed = jin > 0;
+                while (__any_sync(FULL, changed)) {
+                    int nopt = opt;
+                    for (int j = 1; j <= jin; ++j) {
+                        int v = __shfl_up_sync(FULL, opt, j, Wg);
+                        if (xl >= j && v + 1 < nopt) nopt = v + 1;
+                    }
+                    changed = nopt < opt;
+                    opt = nopt;
                 }
-                changed = nopt < opt;
-                opt = nopt;
+                if (act) out[x] = (E)opt;
+                __syncwarp();
             }
-            if (act) out[x] = (E)opt;
-            __syncwarp();
         }
     }
 }
@@ -356,7 +418,7 @@ row_scatter_kernel(E *__restrict__ table, const RowGeom g, const int64_t *__rest
         uint64_t pw[NW];
         int64_t rowbase;
         unrank_row<NW>(g, cnt, rho, slot, pw, rowbase);
-        for (int64_t x = xl; x < g.W; x += Wg) table[rowbase + x] = compact[slot * g.W + x];
+        for (int64_t x = xl; x < g.Wp; x += Wg) table[rowbase + x] = compact[slot * g.Wp + x];
     }
 }
 
@@ -385,7 +447,7 @@ __global__ void __launch_bounds__(256)
 traceback_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__ N,
                  const int64_t *__restrict__ stride, const uint16_t *__restrict__ digits,
                  const int64_t *__restrict__ off, const int32_t *__restrict__ rank, int64_t nC,
-                 int64_t sigma, int32_t *__restrict__ out, int32_t max_out, int32_t *__restrict__ len,
+                 int64_t idx_start, int32_t *__restrict__ out, int32_t max_out, int32_t *__restrict__ len,
                  DpMeta *meta)
 {
     __shared__ int32_t cur[MAXK];
@@ -394,7 +456,7 @@ traceback_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__
     __shared__ int32_t mu;
     const int tid = threadIdx.x;
     if (tid < K) cur[tid] = N[tid];
-    if (tid == 0) { idx = sigma - 1; mu = 0; }
+    if (tid == 0) { idx = idx_start; mu = 0; }
     __syncthreads();
     while (idx != 0) {
         if (tid == 0) best = ~0ull;
@@ -430,6 +492,17 @@ traceback_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__
         __syncthreads();
     }
     if (tid == 0) *len = mu;
+}
+
+template <typename E>
+__global__ void compact_rows_kernel(const E *__restrict__ src, E *__restrict__ dst, int64_t rows, int64_t W,
+                                    int64_t Wp)
+{
+    const int lane = threadIdx.x & 31;
+    int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (; r < rows; r += nw)
+        for (int64_t x = lane; x < W; x += 32) dst[r * W + x] = src[r * Wp + x];
 }
 
 __global__ void fill_value_kernel(uint8_t *p, int64_t bytes, uint8_t v)
@@ -487,34 +560,43 @@ cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t 
     const int wlog = wlog_for(g.W);
     const int rpw = 32 >> wlog;
     const int bs = 256;
-    const int64_t warps = (slot_count + rpw - 1) / rpw;
-    int64_t blocks = (warps + (bs / 32) - 1) / (bs / 32);
+    const int64_t groups_full = (int64_t)sm_count * 8 * (bs / 32) * rpw;
+    int64_t crows = slot_count / (groups_full * 2);
+    if (crows < 1) crows = 1;
+    if (crows > 16) crows = 16;
+    const int64_t nchunks = (slot_count + crows - 1) / crows;
+    int64_t blocks = (nchunks + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
     const int64_t cap = (int64_t)sm_count * 8;
     if (blocks > cap) blocks = cap;
-    size_t pref_bytes = (size_t)(nP_bound > 1 ? nP_bound - 1 : 0) * sizeof(PrefixEntry);
-    size_t cnt_bytes = (size_t)(g.K1 + 1) * (g.rho_max + 1) * sizeof(int64_t);
-    int smem_pref = pref_bytes <= 96 * 1024 ? (int)(nP_bound > 1 ? nP_bound - 1 : 0) : 0;
-    if (smem_pref == 0) pref_bytes = 0;
-    int smem_cnt = (pref_bytes + cnt_bytes) <= 200 * 1024 ? 1 : 0;
-    size_t smem = pref_bytes + (smem_cnt ? cnt_bytes : 0);
+    const int NWk = g.nwords <= 1 ? 1 : 2;
+    const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
+    const size_t smem = (size_t)np * (8 + 8 * NWk) + (size_t)(g.K1 + 1) * (g.rho_max + 1) * 8 + 16;
+    if (smem > 220 * 1024) return cudaErrorInvalidValue;
+    const bool MULTI = g.W > 32;
     cudaError_t err;
-#define PTAS_FILL_CASE(E_, NW_)                                                                   \
+#define PTAS_FILL_CASE(E_, NW_, MU_)                                                              \
     do {                                                                                          \
-        auto kfn = row_fill_kernel<E_, NW_>;                                                      \
+        auto kfn = row_fill_kernel<E_, NW_, MU_>;                                                 \
         if (smem > 48 * 1024) {                                                                   \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
                                        (int)smem);                                                \
             if (err != cudaSuccess) return err;                                                   \
         }                                                                                         \
-        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, d_cnt, d_pref, d_meta,            \
-                                                smem_pref, smem_cnt, J0, rho, slot_begin,         \
-                                                slot_count, (E_ *)compact_out, wlog);             \
+        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, d_cnt, d_pref, d_meta, J0, rho,   \
+                                                slot_begin, slot_count, (E_ *)compact_out, wlog,  \
+                                                (int)crows);                                      \
+    } while (0)
+#define PTAS_FILL_JU(E_, NW_)                                                                     \
+    do {                                                                                          \
+        if (MULTI) PTAS_FILL_CASE(E_, NW_, true);                                                 \
+        else PTAS_FILL_CASE(E_, NW_, false);                                                      \
     } while (0)
     if (e == 1) {
-        if (g.nwords <= 1) PTAS_FILL_CASE(uint8_t, 1); else PTAS_FILL_CASE(uint8_t, 2);
+        if (NWk == 1) PTAS_FILL_JU(uint8_t, 1); else PTAS_FILL_JU(uint8_t, 2);
     } else {
-        if (g.nwords <= 1) PTAS_FILL_CASE(uint16_t, 1); else PTAS_FILL_CASE(uint16_t, 2);
+        if (NWk == 1) PTAS_FILL_JU(uint16_t, 1); else PTAS_FILL_JU(uint16_t, 2);
     }
+#undef PTAS_FILL_JU
 #undef PTAS_FILL_CASE
     return cudaGetLastError();
 }
@@ -562,13 +644,24 @@ cudaError_t launch_read_opt(int e, const void *table, int64_t idx, DpMeta *d_met
 
 cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N,
                              const int64_t *d_stride, const uint16_t *d_digits, const int64_t *d_off,
-                             const int32_t *d_rank, int64_t nC, int64_t sigma, int32_t *d_out,
+                             const int32_t *d_rank, int64_t nC, int64_t idx_start, int32_t *d_out,
                              int32_t max_out, int32_t *d_len, DpMeta *d_meta, cudaStream_t st)
 {
     if (e == 1)
-        traceback_kernel<uint8_t><<<1, 256, 0, st>>>((const uint8_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, sigma, d_out, max_out, d_len, d_meta);
+        traceback_kernel<uint8_t><<<1, 256, 0, st>>>((const uint8_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, idx_start, d_out, max_out, d_len, d_meta);
     else
-        traceback_kernel<uint16_t><<<1, 256, 0, st>>>((const uint16_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, sigma, d_out, max_out, d_len, d_meta);
+        traceback_kernel<uint16_t><<<1, 256, 0, st>>>((const uint16_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, idx_start, d_out, max_out, d_len, d_meta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows, int64_t W, int64_t Wp,
+                                cudaStream_t st)
+{
+    if (rows <= 0) return cudaSuccess;
+    int64_t blocks = (rows + 7) / 8;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (e == 1) compact_rows_kernel<uint8_t><<<(unsigned)blocks, 256, 0, st>>>((const uint8_t *)src, (uint8_t *)dst, rows, W, Wp);
+    else compact_rows_kernel<uint16_t><<<(unsigned)blocks, 256, 0, st>>>((const uint16_t *)src, (uint16_t *)dst, rows, W, Wp);
     return cudaGetLastError();
 }
 

@@ -91,6 +91,7 @@ class Engine {
     int last_K_ = 0, last_Kcanon_ = 0, last_e_ = 1;
     int64_t last_sigma_ = 1, last_nC_ = 0;
     int32_t last_opt_ = 0;
+    int64_t last_W_ = 1, last_Wp_ = 1, last_rows_ = 1, last_idxN_ = 0;
     std::vector<int> last_order_;      // internal -> canonical
     std::vector<int32_t> last_N_;      // internal counts
     std::vector<int64_t> last_stride_; // internal strides

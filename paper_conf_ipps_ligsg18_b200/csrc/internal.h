@@ -1,12 +1,15 @@
 // internal.h — shared declarations of the product library (NOT used by oracle/).
 //
 // Layout of a DP in HBM:
-//   table  : sigma entries of E (uint8 if sum N <= 255 else uint16), row-major
-//            over the INTERNAL class order (a permutation of the caller's
-//            order chosen by the driver; identity for dp_fill), last class
-//            fastest.  A "row" is the run of W = N[K-1]+1 entries that share
-//            the K1 = K-1 leading digits p; rows are filled in row-level order
-//            rho = sum(p) (the wavefront), each row by one lane group.
+//   table  : entries of E (uint8 if sum N <= 255 else uint16), row-major over
+//            the INTERNAL class order (a permutation of the caller's order
+//            chosen by the driver; identity for dp_fill), last class fastest.
+//            A "row" is the run of W = N[K-1]+1 entries that share the K1 = K-1
+//            leading digits p; rows are stored with pitch Wp (W*e rounded up
+//            to a multiple of 4 bytes) so every row and every off(s') is word
+//            aligned.  Rows are filled in row-level order rho = sum(p) (the
+//            wavefront).  The caller's layout (pitch W) is produced by a
+//            compaction copy when Wp != W.
 //   configs: C(T) in internal lexicographic order: uint16
 //            digits [nC*K] + int64 linear offsets off(s) [nC].
 //   prefix : one entry per distinct leading part s' of C (runs of equal s' in
@@ -34,6 +37,7 @@ struct RowGeom {
     int32_t K1;                 // number of leading classes (K-1)
     int32_t rho_max;            // sum of leading counts
     int64_t W;                  // row length N[K-1]+1
+    int64_t Wp;                 // padded row pitch (entries): W*e rounded up to 4 bytes
     int32_t N[MAXK];            // leading counts
     int32_t maxsuf[MAXK + 1];   // maxsuf[i] = sum_{d >= i} N[d] (leading dims)
     int64_t stride[MAXK];       // element strides of the leading dims
@@ -66,11 +70,19 @@ cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *
                                 PrefixEntry *d_pref, DpMeta *d_meta, cudaStream_t st);
 // One row-level of the level fill.  e = 1 or 2.  Rows [slot_begin, slot_begin+slot_count)
 // of row-level rho; results go to the table (compact_out == NULL) or to
-// compact_out[(slot - slot_begin) * W + x].
+// compact_out[(slot - slot_begin) * Wp + x].
 cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
                             const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
                             int J0, int rho, int64_t slot_begin, int64_t slot_count,
                             void *compact_out, int sm_count, cudaStream_t st);
+// Packed-word fill (row_fill_swar.cu); cudaErrorNotSupported -> use launch_row_fill.
+cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
+                                 const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
+                                 int J0, int rho, int64_t slot_begin, int64_t slot_count,
+                                 void *compact_out, int sm_count, cudaStream_t st);
+// Copy rows of pitch Wp (src) to pitch W (dst), `rows` rows of e-byte entries.
+cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows, int64_t W,
+                                int64_t Wp, cudaStream_t st);
 cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
                                int rho, int64_t slot_count, const void *compact,
                                int sm_count, cudaStream_t st);
@@ -81,7 +93,7 @@ cudaError_t launch_read_opt(int e, const void *table, int64_t idx, DpMeta *d_met
 cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N,
                              const int64_t *d_stride, const uint16_t *d_digits,
                              const int64_t *d_off, const int32_t *d_rank, int64_t nC,
-                             int64_t sigma, int32_t *d_out, int32_t max_out,
+                             int64_t idx_start, int32_t *d_out, int32_t max_out,
                              int32_t *d_len, DpMeta *d_meta, cudaStream_t st);
 cudaError_t launch_fill_value(void *p, int64_t bytes, int value, cudaStream_t st);
 

@@ -157,6 +157,32 @@ def test_dp_fill_invalid(P):
     assert ei.value.rc == -2
 
 
+def test_dp_fill_scalar_kernel(P, monkeypatch):
+    # the scalar fill kernel (fallback for rows > 1 KiB) on the same random cases
+    monkeypatch.setenv("PTAS_FORCE_SCALAR", "1")
+    rng = np.random.default_rng(31)
+    for K in (1, 2, 3, 5, 7):
+        for _ in range(4):
+            N, r, T = _rand_case(rng, K, {1: 200, 2: 60, 3: 25, 5: 8, 7: 4}[K])
+            _check_table(P, N, r, T)
+    _check_table(P, np.array([5, 4, 70], np.int32), np.array([90, 70, 11], np.int64), 200)
+
+
+def test_dp_fill_very_long_rows(P):
+    # rows longer than 1 KiB (uint16, W = 701) use the scalar kernel; W*e = 1024 B exactly uses 8 chunks
+    _check_table(P, np.array([2, 700], np.int32), np.array([60, 13], np.int64), 120)
+    _check_table(P, np.array([3, 511], np.int32), np.array([60, 13], np.int64), 120)
+    _check_table(P, np.array([1, 1, 300], np.int32), np.array([50, 40, 7], np.int64), 120)
+
+
+def test_dp_fill_padding_pitches(P):
+    # row byte lengths 1..9 (u8) and odd u16 lengths: every padding case of the packed kernel
+    for W in range(1, 10):
+        _check_table(P, np.array([4, 3, W - 1], np.int32), np.array([35, 50, 21], np.int64), 110)
+    for W in (1, 2, 3, 5, 33, 65):
+        _check_table(P, np.array([100, 150, W - 1], np.int32), np.array([35, 50, 21], np.int64), 110)
+
+
 def test_dp_fill_device_torch(P):
     import torch
     N = np.array([7, 9, 40], np.int32)
