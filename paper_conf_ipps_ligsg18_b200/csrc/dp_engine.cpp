@@ -72,6 +72,18 @@ int Engine::get(int device, Engine **out)
     return PTAS_OK;
 }
 
+// The host driver waits for small readbacks many times per solve; a spin on
+// an event query avoids the scheduler wake-up latency of a blocking sync.
+cudaError_t Engine::sync_spin(cudaStream_t st)
+{
+    cudaError_t e = cudaEventRecord(ev_sync_, st);
+    if (e != cudaSuccess) return e;
+    for (;;) {
+        e = cudaEventQuery(ev_sync_);
+        if (e != cudaErrorNotReady) return e;
+    }
+}
+
 int Engine::init(int device)
 {
     device_ = device;
@@ -79,6 +91,7 @@ int Engine::init(int device)
     PT_CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device));
     PT_CK(cudaStreamCreateWithFlags(&stream_, cudaStreamNonBlocking));
     for (auto &ev : ev_) PT_CK(cudaEventCreate(&ev));
+    PT_CK(cudaEventCreateWithFlags(&ev_sync_, cudaEventDisableTiming));
     PT_CK(cudaMalloc(&d_meta_, sizeof(DpMeta)));
     PT_CK(cudaMallocHost(&h_meta_, sizeof(DpMeta)));
     PT_CK(cudaMallocHost(&h_scalar_, 64));
@@ -215,7 +228,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
         PT_CK(cudaEventRecord(ev_[1], st));
         PT_CK(cudaEventRecord(ev_[2], st));
         PT_CK(cudaEventRecord(ev_[3], st));
-        PT_CK(cudaStreamSynchronize(st));
+        PT_CK(sync_spin(st));
         o.launches = 1;
         o.opt = 0;
         last_valid_ = true;
@@ -289,7 +302,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
                               nullptr, nullptr, st));
     PT_CK(launch_exclusive_scan(d_counts, d_offsets, nprefix, d_offsets + nprefix, st));
     PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     o.d2h += 8;
     o.launches += 2;
     const int64_t nC = h_scalar_[0];
@@ -387,7 +400,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     }
     PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
     PT_CK(cudaEventRecord(ev_[3], st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     o.d2h += sizeof(DpMeta);
     float ms = 0;
     PT_CK(cudaEventElapsedTime(&ms, ev_[0], ev_[3]));
@@ -428,7 +441,7 @@ int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
     cudaStream_t st = last_stream_;
     std::vector<uint16_t> dig((size_t)nC * K);
     PT_CK(cudaMemcpyAsync(dig.data(), digits_.p, dig.size() * 2, cudaMemcpyDeviceToHost, st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     acc->d2h += (int64_t)dig.size() * 2;
     // canonical lexicographic rank of every configuration (reading R11)
     std::vector<std::vector<int32_t>> canon((size_t)nC, std::vector<int32_t>(last_Kcanon_, 0));
@@ -460,7 +473,7 @@ int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
     std::vector<int32_t> outv((size_t)last_opt_ + 4);
     PT_CK(cudaMemcpyAsync(outv.data(), d_len, outv.size() * 4, cudaMemcpyDeviceToHost, st));
     PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     acc->d2h += (int64_t)outv.size() * 4 + (int64_t)sizeof(DpMeta);
     const int32_t len = outv[0];
     if (h_meta_->err || len != last_opt_) return PTAS_EINTERNAL;
@@ -480,7 +493,7 @@ int Engine::copy_table_to_host(void *dst, int64_t bytes)
         src = stage_.p;
     }
     PT_CK(cudaMemcpyAsync(dst, src, (size_t)bytes, cudaMemcpyDeviceToHost, last_stream_));
-    PT_CK(cudaStreamSynchronize(last_stream_));
+    PT_CK(sync_spin(last_stream_));
     return PTAS_OK;
 }
 
@@ -529,7 +542,7 @@ int Engine::configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits,
                               nullptr, nullptr, st));
     PT_CK(launch_exclusive_scan(d_counts, d_offsets, nprefix, d_offsets + nprefix, st));
     PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     const int64_t nC = h_scalar_[0];
     *count = nC;
     if (nC == 0) return PTAS_OK;
@@ -539,7 +552,7 @@ int Engine::configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits,
                               (uint16_t *)digits_.p, (int64_t *)off_.p, st));
     std::vector<uint16_t> dig((size_t)nC * K);
     PT_CK(cudaMemcpyAsync(dig.data(), digits_.p, dig.size() * 2, cudaMemcpyDeviceToHost, st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     last_valid_ = false;
     digits->assign((size_t)nC * rq.K, 0);
     for (int64_t c = 0; c < nC; ++c)
@@ -579,7 +592,7 @@ int Engine::row_index(const int32_t *Nc, int Kc, std::vector<int64_t> *level_sta
         PT_CK(launch_row_index(g, (const int64_t *)cnt_.p, rho, cnt[rho], d_out + (*level_start)[rho], st));
     rowbase->resize((size_t)rows);
     PT_CK(cudaMemcpyAsync(rowbase->data(), d_out, (size_t)rows * 8, cudaMemcpyDeviceToHost, st));
-    PT_CK(cudaStreamSynchronize(st));
+    PT_CK(sync_spin(st));
     last_valid_ = false;
     return PTAS_OK;
 }

@@ -68,6 +68,8 @@ class Engine {
     cudaStream_t stream() const { return stream_; }
     int device() const { return device_; }
 
+    cudaError_t sync_spin(cudaStream_t st);
+
   private:
     int init(int device);
     struct Buf {
@@ -79,6 +81,7 @@ class Engine {
     int sm_count_ = 148;
     cudaStream_t stream_ = nullptr;
     cudaEvent_t ev_[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev_sync_ = nullptr;
     DpMeta *d_meta_ = nullptr;
     DpMeta *h_meta_ = nullptr;     // pinned
     int64_t *h_scalar_ = nullptr;  // pinned

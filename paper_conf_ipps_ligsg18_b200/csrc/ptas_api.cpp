@@ -310,7 +310,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             cudaMemcpyAsync(dbuf + rank, mine.data(), 4, cudaMemcpyHostToDevice, st);
             int crc = comm_allgather(opt.comm, dbuf + rank, dbuf, 4, st);
             cudaMemcpyAsync(all.data(), dbuf, 4 * world, cudaMemcpyDeviceToHost, st);
-            cudaError_t ce = cudaStreamSynchronize(st);
+            cudaError_t ce = eng->sync_spin(st);
             cudaFree(dbuf);
             if (crc) return crc;
             if (ce != cudaSuccess) return PTAS_ECUDA;
@@ -529,16 +529,27 @@ int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps, cons
     int dev;
     int rc = resolve_device(opt ? opt->device : -1, &dev);
     if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
     std::vector<int64_t> hp(n);
     std::vector<int32_t> ha(n);
-    if (cudaMemcpy(hp.data(), d_p, (size_t)n * 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
-        cudaGetLastError();
-        return PTAS_ECUDA;
+    {
+        std::lock_guard<std::mutex> lk(eng->mu);
+        cudaStream_t st = eng->stream();
+        if (cudaMemcpyAsync(hp.data(), d_p, (size_t)n * 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+            eng->sync_spin(st) != cudaSuccess) {
+            cudaGetLastError();
+            return PTAS_ECUDA;
+        }
     }
     rc = solve_core(hp.data(), n, m, eps, opt, makespan_out, ha.data(), stats, nullptr, 0, nullptr,
                     (int64_t)n * 4, (int64_t)n * 8);
     if (rc) return rc;
-    if (cudaMemcpy(d_assignment, ha.data(), (size_t)n * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+    std::lock_guard<std::mutex> lk(eng->mu);
+    cudaStream_t st = eng->stream();
+    if (cudaMemcpyAsync(d_assignment, ha.data(), (size_t)n * 4, cudaMemcpyHostToDevice, st) != cudaSuccess ||
+        eng->sync_spin(st) != cudaSuccess) {
         cudaGetLastError();
         return PTAS_ECUDA;
     }

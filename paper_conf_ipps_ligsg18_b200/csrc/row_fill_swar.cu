@@ -144,65 +144,78 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                 }
                 const unsigned m = (__ballot_sync(FULL, dom) >> (grp << lglog)) & gmask;
                 const int cend = np - base < Lg ? np - base : Lg;
-                for (int q = 0; q < cend; ++q) {
-                    const bool pd = (m >> q) & 1u;
-                    const uint64_t oj = s_oj[base + q];
-                    const int64_t offw = (int64_t)(oj & 0xffffffffffffull);
-                    const int jm = (int)(oj >> 48);
-                    const uint32_t *src = row32 - offw;
-                    Words<CH> cur;
+                // 4 prefixes per step: their gathers are issued before any is consumed
+                for (int q0 = 0; q0 < cend; q0 += 4) {
+                    Words<CH> curq[4];
+                    int jmq[4];
 #pragma unroll
-                    for (int t = 0; t < CH; ++t) cur.v[t] = (pd && wok[t]) ? src[32 * t] : 0xffffffffu;
-                    // j = 0: the aligned word itself
+                    for (int u = 0; u < 4; ++u) {
+                        const int q = q0 + u;
+                        const bool live = q < cend;
+                        const bool pd = live && ((m >> q) & 1u);
+                        const uint64_t oj = live ? s_oj[base + q] : 0ull;
+                        const uint32_t *src = row32 - (int64_t)(oj & 0xffffffffffffull);
+                        jmq[u] = live ? (int)(oj >> 48) : -1;
 #pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        if constexpr (EB == 1) {
-                            ae.v[t] = vmin2(ae.v[t], prmt(cur.v[t], cur.v[t], 0xA280u));
-                            ao.v[t] = vmin2(ao.v[t], prmt(cur.v[t], cur.v[t], 0xB391u));
-                        } else {
-                            ae.v[t] = vmin2(ae.v[t], cur.v[t]);
+                        for (int t = 0; t < CH; ++t)
+                            curq[u].v[t] = (pd && wok[t]) ? src[32 * t] : 0xffffffffu;
+                    }
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const int jm = jmq[u];
+                        if (jm < 0) break;
+                        const Words<CH> &cur = curq[u];
+                        // j = 0: the aligned word itself
+#pragma unroll
+                        for (int t = 0; t < CH; ++t) {
+                            if constexpr (EB == 1) {
+                                ae.v[t] = vmin2(ae.v[t], prmt(cur.v[t], cur.v[t], 0xA280u));
+                                ao.v[t] = vmin2(ao.v[t], prmt(cur.v[t], cur.v[t], 0xB391u));
+                            } else {
+                                ae.v[t] = vmin2(ae.v[t], cur.v[t]);
+                            }
                         }
-                    }
-                    if (jm == 0) continue;
-                    Words<CH> w1, w2;
-#pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                        w1.v[t] = word_left(cur.v[t], prev, xl, 1, Lg);
-                    }
-                    if (jm * EB > 4) {
+                        if (jm == 0) continue;
+                        Words<CH> w1, w2;
 #pragma unroll
                         for (int t = 0; t < CH; ++t) {
                             const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                            w2.v[t] = word_left(cur.v[t], prev, xl, 2, Lg);
+                            w1.v[t] = word_left(cur.v[t], prev, xl, 1, Lg);
                         }
-                    }
-                    for (int j = 1; j <= jm; ++j) {
-                        const int db = j * EB;  // byte shift
+                        if (jm * EB > 4) {
 #pragma unroll
-                        for (int t = 0; t < CH; ++t) {
-                            uint32_t lo, hi;
-                            int o;
-                            if (db <= 4) {
-                                lo = w1.v[t];
-                                hi = cur.v[t];
-                                o = 4 - db;
-                            } else if (db <= 8) {
-                                lo = w2.v[t];
-                                hi = w1.v[t];
-                                o = 8 - db;
-                            } else {
-                                const int k = (db + 3) >> 2;
+                            for (int t = 0; t < CH; ++t) {
                                 const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                                lo = word_left(cur.v[t], prev, xl, k, Lg);
-                                hi = word_left(cur.v[t], prev, xl, k - 1, Lg);
-                                o = 4 * k - db;
+                                w2.v[t] = word_left(cur.v[t], prev, xl, 2, Lg);
                             }
-                            if constexpr (EB == 1) {
-                                ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, 0xA280u + 0x1111u * o));
-                                ao.v[t] = vmin2(ao.v[t], prmt(lo, hi, 0xB391u + 0x1111u * o));
-                            } else {
-                                ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, 0x3210u + 0x1111u * o));
+                        }
+                        for (int j = 1; j <= jm; ++j) {
+                            const int db = j * EB;  // byte shift
+#pragma unroll
+                            for (int t = 0; t < CH; ++t) {
+                                uint32_t lo, hi;
+                                int o;
+                                if (db <= 4) {
+                                    lo = w1.v[t];
+                                    hi = cur.v[t];
+                                    o = 4 - db;
+                                } else if (db <= 8) {
+                                    lo = w2.v[t];
+                                    hi = w1.v[t];
+                                    o = 8 - db;
+                                } else {
+                                    const int k = (db + 3) >> 2;
+                                    const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
+                                    lo = word_left(cur.v[t], prev, xl, k, Lg);
+                                    hi = word_left(cur.v[t], prev, xl, k - 1, Lg);
+                                    o = 4 * k - db;
+                                }
+                                if constexpr (EB == 1) {
+                                    ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, 0xA280u + 0x1111u * o));
+                                    ao.v[t] = vmin2(ao.v[t], prmt(lo, hi, 0xB391u + 0x1111u * o));
+                                } else {
+                                    ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, 0x3210u + 0x1111u * o));
+                                }
                             }
                         }
                     }
@@ -343,9 +356,9 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
     const int rpw = 32 >> lglog;
     const int bs = 256;
     const int64_t groups_full = (int64_t)sm_count * 8 * (bs / 32) * rpw;
-    int64_t crows = slot_count / (groups_full * 2);
+    int64_t crows = (slot_count + groups_full - 1) / groups_full;  // one unrank per group, then successors
     if (crows < 1) crows = 1;
-    if (crows > 16) crows = 16;
+    if (crows > 32) crows = 32;
     const int64_t nchunks = (slot_count + crows - 1) / crows;
     int64_t blocks = (nchunks + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
     const int64_t cap = (int64_t)sm_count * 8;
