@@ -50,7 +50,7 @@ class ClockSampler:
     """SM clock and throttle reasons sampled in-process through NVML during the
     timed region (no nvidia-smi subprocesses, which stall the driver)."""
 
-    def __init__(self, index: int, period: float = 0.1):
+    def __init__(self, index: int, period: float = float(os.environ.get("BENCH_CLOCK_PERIOD", "0.25"))):
         self.index = index
         self.period = period
         self.rows = []
@@ -74,12 +74,14 @@ class ClockSampler:
             self.err = repr(e)
 
     def __enter__(self):
-        self._t.start()
+        if os.environ.get("BENCH_NO_CLOCKS") != "1":
+            self._t.start()
         return self
 
     def __exit__(self, *a):
         self._stop.set()
-        self._t.join(timeout=10)
+        if self._t.is_alive():
+            self._t.join(timeout=10)
 
     def summary(self):
         if not self.rows:
@@ -296,6 +298,8 @@ def run_ours(args, w):
                      "fill_launches_per_step": fill_launches / args.steps,
                      "alg_bytes_per_step": alg_bytes / args.steps,
                      "fill_relax_per_s": relax_total / fill_s if fill_s > 0 else None},
+        "step_ms": [round(x, 3) for x in dev_ms],
+        "e2e_step_ms": [round(x, 3) for x in e2e_ms],
         "gpu_launches": int(launches),
         "clocks": clocks,
     }

@@ -54,9 +54,83 @@ struct Words {
     uint32_t v[CH];
 };
 
+// acc <- min(acc, window of `lo:hi` at byte offset o) for one word position.
+template <int EB>
+__device__ __forceinline__ void acc_window(uint32_t lo, uint32_t hi, int o, uint32_t &ae, uint32_t &ao)
+{
+    if constexpr (EB == 1) {
+        ae = vmin2(ae, prmt(lo, hi, 0xA280u + 0x1111u * o));
+        ao = vmin2(ao, prmt(lo, hi, 0xB391u + 0x1111u * o));
+    } else {
+        ae = vmin2(ae, prmt(lo, hi, 0x3210u + 0x1111u * o));
+    }
+}
+
+// All relaxations (s', j), j = 0..jm, of one prefix on the lane's words.
+// JB > 0: shifts up to JB bytes, fully unrolled (jm * EB <= JB guaranteed by
+// the host); JB == 0: any shift (runtime loop, generic word fetch).
+template <int EB, int CH, int JB>
+__device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int xl, int Lg, Words<CH> &ae,
+                                             Words<CH> &ao)
+{
+#pragma unroll
+    for (int t = 0; t < CH; ++t) acc_window<EB>(cur.v[t], cur.v[t], 0, ae.v[t], ao.v[t]);
+    if (jm <= 0) return;
+    Words<CH> w1, w2;
+#pragma unroll
+    for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur.v[t], t ? cur.v[t - 1] : 0xffffffffu, xl, 1, Lg);
+    if (JB == 0 || JB > 4) {
+        if (jm * EB > 4) {
+#pragma unroll
+            for (int t = 0; t < CH; ++t) w2.v[t] = word_left(cur.v[t], t ? cur.v[t - 1] : 0xffffffffu, xl, 2, Lg);
+        }
+    }
+    if constexpr (JB > 0) {
+#pragma unroll
+        for (int j = 1; j <= JB / EB; ++j) {
+            if (j <= jm) {
+                constexpr int dummy = 0;
+                (void)dummy;
+                const int db = j * EB;
+#pragma unroll
+                for (int t = 0; t < CH; ++t) {
+                    if (db <= 4) acc_window<EB>(w1.v[t], cur.v[t], 4 - db, ae.v[t], ao.v[t]);
+                    else acc_window<EB>(w2.v[t], w1.v[t], 8 - db, ae.v[t], ao.v[t]);
+                }
+            }
+        }
+    } else {
+        for (int j = 1; j <= jm; ++j) {
+            const int db = j * EB;
+#pragma unroll
+            for (int t = 0; t < CH; ++t) {
+                if (db <= 4) acc_window<EB>(w1.v[t], cur.v[t], 4 - db, ae.v[t], ao.v[t]);
+                else if (db <= 8) acc_window<EB>(w2.v[t], w1.v[t], 8 - db, ae.v[t], ao.v[t]);
+                else {
+                    const int k = (db + 3) >> 2;
+                    const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
+                    acc_window<EB>(word_left(cur.v[t], prev, xl, k, Lg), word_left(cur.v[t], prev, xl, k - 1, Lg),
+                                   4 * k - db, ae.v[t], ao.v[t]);
+                }
+            }
+        }
+    }
+}
+
+// u16-lane window of a packed array shifted right by s u16 positions
+// (byte shift db = 2s) given the words 1 and 2 to the left.
+__device__ __forceinline__ uint32_t lane_shift(const uint32_t w0, const uint32_t w1, const uint32_t w2, int db,
+                                               uint32_t prevk_lo, uint32_t prevk_hi, int ok)
+{
+    if (db == 0) return w0;
+    if (db <= 4) return prmt(w1, w0, 0x3210u + 0x1111u * (4 - db));
+    if (db <= 8) return prmt(w2, w1, 0x3210u + 0x1111u * (8 - db));
+    return prmt(prevk_lo, prevk_hi, 0x3210u + 0x1111u * ok);
+}
+
 }  // namespace
 
-template <typename E, int NW, int CH>
+template <typename E, int NW, int CH, int JB>
 __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
@@ -161,64 +235,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                             curq[u].v[t] = (pd && wok[t]) ? src[32 * t] : 0xffffffffu;
                     }
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const int jm = jmq[u];
-                        if (jm < 0) break;
-                        const Words<CH> &cur = curq[u];
-                        // j = 0: the aligned word itself
-#pragma unroll
-                        for (int t = 0; t < CH; ++t) {
-                            if constexpr (EB == 1) {
-                                ae.v[t] = vmin2(ae.v[t], prmt(cur.v[t], cur.v[t], 0xA280u));
-                                ao.v[t] = vmin2(ao.v[t], prmt(cur.v[t], cur.v[t], 0xB391u));
-                            } else {
-                                ae.v[t] = vmin2(ae.v[t], cur.v[t]);
-                            }
-                        }
-                        if (jm == 0) continue;
-                        Words<CH> w1, w2;
-#pragma unroll
-                        for (int t = 0; t < CH; ++t) {
-                            const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                            w1.v[t] = word_left(cur.v[t], prev, xl, 1, Lg);
-                        }
-                        if (jm * EB > 4) {
-#pragma unroll
-                            for (int t = 0; t < CH; ++t) {
-                                const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                                w2.v[t] = word_left(cur.v[t], prev, xl, 2, Lg);
-                            }
-                        }
-                        for (int j = 1; j <= jm; ++j) {
-                            const int db = j * EB;  // byte shift
-#pragma unroll
-                            for (int t = 0; t < CH; ++t) {
-                                uint32_t lo, hi;
-                                int o;
-                                if (db <= 4) {
-                                    lo = w1.v[t];
-                                    hi = cur.v[t];
-                                    o = 4 - db;
-                                } else if (db <= 8) {
-                                    lo = w2.v[t];
-                                    hi = w1.v[t];
-                                    o = 8 - db;
-                                } else {
-                                    const int k = (db + 3) >> 2;
-                                    const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                                    lo = word_left(cur.v[t], prev, xl, k, Lg);
-                                    hi = word_left(cur.v[t], prev, xl, k - 1, Lg);
-                                    o = 4 * k - db;
-                                }
-                                if constexpr (EB == 1) {
-                                    ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, 0xA280u + 0x1111u * o));
-                                    ao.v[t] = vmin2(ao.v[t], prmt(lo, hi, 0xB391u + 0x1111u * o));
-                                } else {
-                                    ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, 0x3210u + 0x1111u * o));
-                                }
-                            }
-                        }
-                    }
+                    for (int u = 0; u < 4; ++u)
+                        if (jmq[u] >= 0) relax_prefix<EB, CH, JB>(curq[u], jmq[u], xl, Lg, ae, ao);
                 }
             }
 
@@ -237,81 +255,83 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                 }
             }
             if (rho == 0 && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
+            // one Bellman-Ford step for shift j: ne/no <- min(ne/no, opt(x - j) + 1)
+            auto chain_step = [&](int j, const Words<CH> &e1, const Words<CH> &o1, const Words<CH> &e2,
+                                  const Words<CH> &o2, Words<CH> &ne, Words<CH> &no) {
+#pragma unroll
+                for (int t = 0; t < CH; ++t) {
+                    if constexpr (EB == 1) {
+                        // even dest x = 2i: j even -> E shifted j/2; j odd -> O shifted (j+1)/2
+                        // odd dest  x = 2i+1: j even -> O shifted j/2; j odd -> E shifted (j-1)/2
+                        const bool odd = j & 1;
+                        const int sa = odd ? (j + 1) >> 1 : j >> 1;
+                        const int sb = odd ? (j - 1) >> 1 : j >> 1;
+                        const uint32_t A0 = odd ? oo.v[t] : oe.v[t], A1 = odd ? o1.v[t] : e1.v[t],
+                                       A2 = odd ? o2.v[t] : e2.v[t];
+                        const uint32_t B0 = odd ? oe.v[t] : oo.v[t], B1 = odd ? e1.v[t] : o1.v[t],
+                                       B2 = odd ? e2.v[t] : o2.v[t];
+                        uint32_t plo = 0, phi = 0, qlo = 0, qhi = 0;
+                        int po = 0, qo = 0;
+                        if (JB == 0 && 2 * sa > 8) {
+                            const int k = (2 * sa + 3) >> 2;
+                            const uint32_t pv = t ? (odd ? oo.v[t - 1] : oe.v[t - 1]) : CFILL;
+                            plo = word_left(A0, pv, xl, k, Lg);
+                            phi = word_left(A0, pv, xl, k - 1, Lg);
+                            po = 4 * k - 2 * sa;
+                        }
+                        if (JB == 0 && 2 * sb > 8) {
+                            const int k = (2 * sb + 3) >> 2;
+                            const uint32_t pv = t ? (odd ? oe.v[t - 1] : oo.v[t - 1]) : CFILL;
+                            qlo = word_left(B0, pv, xl, k, Lg);
+                            qhi = word_left(B0, pv, xl, k - 1, Lg);
+                            qo = 4 * k - 2 * sb;
+                        }
+                        const uint32_t va = lane_shift(A0, A1, A2, 2 * sa, plo, phi, po);
+                        const uint32_t vb = lane_shift(B0, B1, B2, 2 * sb, qlo, qhi, qo);
+                        ne.v[t] = vmin2(ne.v[t], va + ONES);
+                        no.v[t] = vmin2(no.v[t], vb + ONES);
+                    } else {
+                        uint32_t plo = 0, phi = 0;
+                        int po = 0;
+                        if (JB == 0 && 2 * j > 8) {
+                            const int k = (2 * j + 3) >> 2;
+                            const uint32_t pv = t ? oe.v[t - 1] : CFILL;
+                            plo = word_left(oe.v[t], pv, xl, k, Lg);
+                            phi = word_left(oe.v[t], pv, xl, k - 1, Lg);
+                            po = 4 * k - 2 * j;
+                        }
+                        const uint32_t va = lane_shift(oe.v[t], e1.v[t], e2.v[t], 2 * j, plo, phi, po);
+                        ne.v[t] = vmin2(ne.v[t], vmin2(va, 0xfffefffeu) + ONES);
+                    }
+                }
+            };
+            // largest u16-lane shift the chain needs: u8 (J0+1)/2, u16 J0 -> bytes
+            const int chain_db = EB == 1 ? 2 * ((J0 + 1) >> 1) : 2 * J0;
             bool changed = true;
             while (__any_sync(FULL, changed)) {
                 changed = false;
-                // left neighbour words (1 and 2 back) of both arrays
                 Words<CH> e1, o1, e2, o2;
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
                     e1.v[t] = word_left(oe.v[t], t ? oe.v[t - 1] : CFILL, xl, 1, Lg);
-                    if constexpr (EB == 1) o1.v[t] = word_left(oo.v[t], t ? oo.v[t - 1] : CFILL, xl, 1, Lg);
+                    o1.v[t] = EB == 1 ? word_left(oo.v[t], t ? oo.v[t - 1] : CFILL, xl, 1, Lg) : 0u;
+                    e2.v[t] = e1.v[t];
+                    o2.v[t] = o1.v[t];
                 }
-                const int jl = J0;
-                // lanes are shifted by s u16 positions = 2s bytes within (word_left, word)
-                if ((EB == 1 && jl > 4) || (EB == 2 && jl > 2)) {
+                if (chain_db > 4) {
 #pragma unroll
                     for (int t = 0; t < CH; ++t) {
                         e2.v[t] = word_left(oe.v[t], t ? oe.v[t - 1] : CFILL, xl, 2, Lg);
-                        if constexpr (EB == 1) o2.v[t] = word_left(oo.v[t], t ? oo.v[t - 1] : CFILL, xl, 2, Lg);
+                        o2.v[t] = EB == 1 ? word_left(oo.v[t], t ? oo.v[t - 1] : CFILL, xl, 2, Lg) : 0u;
                     }
                 }
                 Words<CH> ne = oe, no = oo;
-                for (int j = 1; j <= jl; ++j) {
+                if constexpr (JB > 0) {
 #pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        if constexpr (EB == 1) {
-                            // even dest x = 2i: j even -> E shifted h = j/2; j odd -> O shifted (j+1)/2
-                            // odd dest  x = 2i+1: j even -> O shifted j/2;  j odd -> E shifted (j-1)/2
-                            const int sa = (j & 1) ? (j + 1) >> 1 : j >> 1;  // shift for even dest
-                            const int sb = (j & 1) ? (j - 1) >> 1 : j >> 1;  // shift for odd dest
-                            const Words<CH> &A = (j & 1) ? oo : oe;          // source of even dest
-                            const Words<CH> &A1 = (j & 1) ? o1 : e1;
-                            const Words<CH> &A2 = (j & 1) ? o2 : e2;
-                            const Words<CH> &B = (j & 1) ? oe : oo;          // source of odd dest
-                            const Words<CH> &B1 = (j & 1) ? e1 : o1;
-                            const Words<CH> &B2 = (j & 1) ? e2 : o2;
-                            uint32_t va, vb;
-                            {
-                                const int db = 2 * sa;
-                                if (db == 0) va = A.v[t];
-                                else if (db <= 4) va = prmt(A1.v[t], A.v[t], 0x3210u + 0x1111u * (4 - db));
-                                else if (db <= 8) va = prmt(A2.v[t], A1.v[t], 0x3210u + 0x1111u * (8 - db));
-                                else {
-                                    const int k = (db + 3) >> 2;
-                                    const uint32_t pv = t ? A.v[t - 1] : CFILL;
-                                    va = prmt(word_left(A.v[t], pv, xl, k, Lg), word_left(A.v[t], pv, xl, k - 1, Lg),
-                                              0x3210u + 0x1111u * (4 * k - db));
-                                }
-                            }
-                            {
-                                const int db = 2 * sb;
-                                if (db == 0) vb = B.v[t];
-                                else if (db <= 4) vb = prmt(B1.v[t], B.v[t], 0x3210u + 0x1111u * (4 - db));
-                                else if (db <= 8) vb = prmt(B2.v[t], B1.v[t], 0x3210u + 0x1111u * (8 - db));
-                                else {
-                                    const int k = (db + 3) >> 2;
-                                    const uint32_t pv = t ? B.v[t - 1] : CFILL;
-                                    vb = prmt(word_left(B.v[t], pv, xl, k, Lg), word_left(B.v[t], pv, xl, k - 1, Lg),
-                                              0x3210u + 0x1111u * (4 * k - db));
-                                }
-                            }
-                            ne.v[t] = vmin2(ne.v[t], va + ONES);
-                            no.v[t] = vmin2(no.v[t], vb + ONES);
-                        } else {
-                            const int db = 2 * j;
-                            uint32_t va;
-                            if (db <= 4) va = prmt(e1.v[t], oe.v[t], 0x3210u + 0x1111u * (4 - db));
-                            else if (db <= 8) va = prmt(e2.v[t], e1.v[t], 0x3210u + 0x1111u * (8 - db));
-                            else {
-                                const int k = (db + 3) >> 2;
-                                const uint32_t pv = t ? oe.v[t - 1] : CFILL;
-                                va = prmt(word_left(oe.v[t], pv, xl, k, Lg), word_left(oe.v[t], pv, xl, k - 1, Lg),
-                                          0x3210u + 0x1111u * (4 * k - db));
-                            }
-                            ne.v[t] = vmin2(ne.v[t], vmin2(va, 0xfffefffeu) + ONES);
-                        }
-                    }
+                    for (int j = 1; j <= JB / EB; ++j)
+                        if (j <= J0) chain_step(j, e1, o1, e2, o2, ne, no);
+                } else {
+                    for (int j = 1; j <= J0; ++j) chain_step(j, e1, o1, e2, o2, ne, no);
                 }
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
@@ -368,9 +388,12 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
     const size_t smem = (size_t)np * (8 + 8 * NWk) + (size_t)(g.K1 + 1) * (g.rho_max + 1) * 8 + 16;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     cudaError_t err;
-#define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
+    // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
+    const int need = e == 1 ? ((J0 + 1) / 2 * 2 > J0 ? (J0 + 1) / 2 * 2 : J0) : 2 * J0;
+    const int JBsel = need <= 4 ? 4 : (need <= 8 ? 8 : 0);
+#define PTAS_SWAR_JB(E_, NW_, CH_, JB_)                                                           \
     do {                                                                                          \
-        auto kfn = row_fill_swar_kernel<E_, NW_, CH_>;                                            \
+        auto kfn = row_fill_swar_kernel<E_, NW_, CH_, JB_>;                                            \
         if (smem > 48 * 1024) {                                                                   \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
                                        (int)smem);                                                \
@@ -379,6 +402,12 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
         kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, d_cnt, d_pref, d_meta, J0, rho,   \
                                                 slot_begin, slot_count, (E_ *)compact_out, lglog, \
                                                 (int)crows);                                      \
+    } while (0)
+#define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
+    do {                                                                                          \
+        if (JBsel == 4) PTAS_SWAR_JB(E_, NW_, CH_, 4);                                            \
+        else if (JBsel == 8) PTAS_SWAR_JB(E_, NW_, CH_, 8);                                       \
+        else PTAS_SWAR_JB(E_, NW_, CH_, 0);                                                       \
     } while (0)
 #define PTAS_SWAR_CH(E_, NW_)                                                                     \
     do {                                                                                          \
@@ -394,6 +423,7 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
     }
 #undef PTAS_SWAR_CH
 #undef PTAS_SWAR_CASE
+#undef PTAS_SWAR_JB
     return cudaGetLastError();
 }
 
