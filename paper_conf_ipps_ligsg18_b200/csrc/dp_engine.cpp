@@ -279,10 +279,24 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     std::memcpy(small.data() + K * 8, stride.data(), (size_t)K * 8);
     std::memcpy(small.data() + K * 16, hi.data(), (size_t)K * 4);
     PT_CK(small_.ensure(small_bytes));
-    PT_CK(cnt_.ensure(cnt.size() * 8));
+    // cnt table followed by level_start[rho_max + 2] (prefix sums of the row counts)
+    std::vector<int64_t> lstart((size_t)g.rho_max + 2, 0);
+    for (int rho = 0; rho <= g.rho_max; ++rho) lstart[rho + 1] = lstart[rho] + cnt[rho];
+    const size_t cnt_words = cnt.size() + lstart.size();
+    PT_CK(cnt_.ensure(cnt_words * 8));
     PT_CK(cudaMemcpyAsync(small_.p, small.data(), small_bytes, cudaMemcpyHostToDevice, st));
     PT_CK(cudaMemcpyAsync(cnt_.p, cnt.data(), cnt.size() * 8, cudaMemcpyHostToDevice, st));
-    o.h2d += (int64_t)(small_bytes + cnt.size() * 8);
+    PT_CK(cudaMemcpyAsync((int64_t *)cnt_.p + cnt.size(), lstart.data(), lstart.size() * 8,
+                          cudaMemcpyHostToDevice, st));
+    o.h2d += (int64_t)(small_bytes + cnt_words * 8);
+    // ---- a-4 level-ordered row index (row base + packed leading digits per row)
+    const int NWk = g.nwords <= 1 ? 1 : 2;
+    PT_CK(rowidx_.ensure((size_t)rows * 8 * (1 + NWk)));
+    int64_t *d_rb = (int64_t *)rowidx_.p;
+    uint64_t *d_pw = (uint64_t *)(d_rb + rows);
+    PT_CK(launch_build_row_index(g, (const int64_t *)cnt_.p, (const int64_t *)cnt_.p + cnt.size(), rows, d_rb,
+                                 d_pw, st));
+    ++o.launches;
     const int64_t *d_r = (const int64_t *)small_.p;
     const int64_t *d_stride = (const int64_t *)((unsigned char *)small_.p + K * 8);
     const int32_t *d_hi = (const int32_t *)((unsigned char *)small_.p + K * 16);
@@ -321,13 +335,15 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     // one row-level (or slice of it): packed-word kernel, scalar kernel as fallback
     auto fill = [&](void *tab, const RowGeom &gg, int j0, int rho_, int64_t b, int64_t c,
                     void *compact) -> cudaError_t {
+        const int64_t *rbl = d_rb + lstart[rho_];
+        const uint64_t *pwl = d_pw + lstart[rho_];
         cudaError_t err = cudaErrorNotSupported;
         if (!force_scalar)
-            err = launch_row_fill_swar(e, tab, gg, (const int64_t *)cnt_.p, (const PrefixEntry *)pref_.p,
-                                       d_meta_, nC, j0, rho_, b, c, compact, sm_count_, st);
+            err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC,
+                                       j0, rho_, b, c, compact, sm_count_, st);
         if (err == cudaErrorNotSupported)
-            err = launch_row_fill(e, tab, gg, (const int64_t *)cnt_.p, (const PrefixEntry *)pref_.p,
-                                  d_meta_, nC, j0, rho_, b, c, compact, sm_count_, st);
+            err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC, j0,
+                                  rho_, b, c, compact, sm_count_, st);
         return err;
     };
 
@@ -384,7 +400,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
                                      (size_t)(chunk * g.Wp * e), st);
             if (crc) return crc;
         }
-        PT_CK(launch_row_scatter(e, table, g, (const int64_t *)cnt_.p, rho, R, stage, sm_count_, st));
+        PT_CK(launch_row_scatter(e, table, g, d_rb + lstart[rho], R, stage, sm_count_, st));
         ++o.launches;
     }
     PT_CK(cudaEventRecord(ev_[2], st));
@@ -578,18 +594,21 @@ int Engine::row_index(const int32_t *Nc, int Kc, std::vector<int64_t> *level_sta
     int rc = build_geom(N, 1, false, &g, &cnt, &stride);
     if (rc) return rc;
     cudaStream_t st = stream_;
-    PT_CK(cnt_.ensure(cnt.size() * 8));
-    PT_CK(cudaMemcpyAsync(cnt_.p, cnt.data(), cnt.size() * 8, cudaMemcpyHostToDevice, st));
     int64_t rows = 0;
     level_start->push_back(0);
     for (int rho = 0; rho <= g.rho_max; ++rho) {
         rows += cnt[rho];
         level_start->push_back(rows);
     }
-    PT_CK(stage_.ensure((size_t)rows * 8));
-    int64_t *d_out = (int64_t *)stage_.p;
-    for (int rho = 0; rho <= g.rho_max; ++rho)
-        PT_CK(launch_row_index(g, (const int64_t *)cnt_.p, rho, cnt[rho], d_out + (*level_start)[rho], st));
+    PT_CK(cnt_.ensure((cnt.size() + level_start->size()) * 8));
+    PT_CK(cudaMemcpyAsync(cnt_.p, cnt.data(), cnt.size() * 8, cudaMemcpyHostToDevice, st));
+    PT_CK(cudaMemcpyAsync((int64_t *)cnt_.p + cnt.size(), level_start->data(), level_start->size() * 8,
+                          cudaMemcpyHostToDevice, st));
+    const int NWk = g.nwords <= 1 ? 1 : 2;
+    PT_CK(rowidx_.ensure((size_t)rows * 8 * (1 + NWk)));
+    int64_t *d_out = (int64_t *)rowidx_.p;
+    PT_CK(launch_build_row_index(g, (const int64_t *)cnt_.p, (const int64_t *)cnt_.p + cnt.size(), rows, d_out,
+                                 (uint64_t *)(d_out + rows), st));
     rowbase->resize((size_t)rows);
     PT_CK(cudaMemcpyAsync(rowbase->data(), d_out, (size_t)rows * 8, cudaMemcpyDeviceToHost, st));
     PT_CK(sync_spin(st));

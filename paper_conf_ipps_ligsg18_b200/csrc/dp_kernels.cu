@@ -6,7 +6,7 @@
 //                        closed-form relaxation count
 //  row_fill_kernel       a-5: Eq. 1 for one row-level
 //  row_scatter_kernel    §8(e): gathered compact rows -> mixed-radix table
-//  row_index_kernel      a-4 inspection: row base of every row slot
+//  build_row_index_kernel a-4: level-ordered row index (row base + packed digits)
 //  traceback_kernel      a-8: schedule of the rounded long jobs from DP(T*)
 //
 // Integer-only; no tensor cores (the DP is a min over gathers, not a
@@ -203,73 +203,69 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
 }
 
 // ------------------------------------------------------------------ a-4
-// Unrank the `rank`-th row (lexicographic order) of row-level rho, i.e. the
-// rank-th vector p over the leading dims with sum(p) = rho, using the
-// suffix-count table cnt[i][L] = #{(p_i..p_{K1-1}) : sum = L}.
+// Level-ordered row index (the materialised order[] of SURVEY.md §8(a) a-4):
+// thread t finds its row-level rho by binary search in level_start (prefix
+// sums of the row counts = coefficients of prod_{i<K-1} (1+z+...+z^{N_i})),
+// unranks slot t - level_start[rho] within the level (lexicographic order)
+// with the suffix-count table, and stores the row base index and the packed
+// leading digits used by the dominance test.
 template <int NW>
-__device__ __forceinline__ void unrank_row(const RowGeom &g, const int64_t *cnt, int rho, int64_t rank,
-                                           uint64_t (&pw)[NW], int64_t &rowbase)
+__global__ void build_row_index_kernel(const RowGeom g, const int64_t *__restrict__ cnt,
+                                       const int64_t *__restrict__ level_start, int64_t rows,
+                                       int64_t *__restrict__ rb, uint64_t *__restrict__ pw)
 {
-    const int ld = g.rho_max + 1;
-    int L = rho;
-#pragma unroll
-    for (int w = 0; w < NW; ++w) pw[w] = 0;
-    rowbase = 0;
-    for (int i = 0; i < g.K1; ++i) {
-        int lo = L - g.maxsuf[i + 1];
-        if (lo < 0) lo = 0;
-        int hi = g.N[i] < L ? g.N[i] : L;
-        int v = lo;
-        const int64_t *row = cnt + (int64_t)(i + 1) * ld;
-        for (; v < hi; ++v) {
-            int64_t c = row[L - v];
-            if (rank < c) break;
-            rank -= c;
-        }
-#pragma unroll
-        for (int w = 0; w < NW; ++w)
-            if (g.word[i] == w) pw[w] |= (uint64_t)v << g.shift[i];
-        rowbase += (int64_t)v * g.stride[i];
-        L -= v;
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= rows) return;
+    int lo = 0, hi = g.rho_max;  // largest rho with level_start[rho] <= t
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (level_start[mid] <= t) lo = mid;
+        else hi = mid - 1;
     }
+    int32_t d[MAXK];
+    unrank_digits(g, cnt, lo, t - level_start[lo], d);
+    int64_t base = 0;
+    uint64_t w[NW];
+#pragma unroll
+    for (int q = 0; q < NW; ++q) w[q] = 0;
+    for (int i = 0; i < g.K1; ++i) {
+        base += (int64_t)d[i] * g.stride[i];
+#pragma unroll
+        for (int q = 0; q < NW; ++q)
+            if (g.word[i] == q) w[q] |= (uint64_t)d[i] << g.shift[i];
+    }
+    rb[t] = base;
+#pragma unroll
+    for (int q = 0; q < NW; ++q) pw[(int64_t)q * rows + t] = w[q];
 }
 
 // ------------------------------------------------------------------ a-5
-// Level fill of one row-level (Eq. 1).  A lane group of
-// Wg = 2^wlog lanes owns one row p (32/Wg rows per warp) and walks a chunk of
-// `crows` consecutive rows of the level (unrank once, then step with
-// next_in_level); lanes cover x in chunks of Wg.  For each state n = (p, x):
+// Scalar level fill of one row-level (Eq. 1); the fallback of
+// the packed-word kernel (rows longer than 1 KiB, very large shifts).  A lane
+// group of Wg = 2^wlog lanes owns one row p (32/Wg rows per warp); lanes
+// cover x in chunks of Wg.  For each state n = (p, x):
 //   acc(x) = min over prefixes s' != 0 with s' <= p and j in
 //            [0, min(Jmax(s'), x)] of OPT(p - s', x - j)   (cross-row relaxations)
 //   OPT(p, x) = 1 + min(acc(x), min_{1<=j<=min(J0,x)} OPT(p, x - j))
 // Dominance s' <= p is a packed-digit compare ((P|G) - S') & G == G done
 // cooperatively: lane xl tests prefix base+xl and a ballot yields the group's
-// dominated set, which every lane of the group then walks (ffs loop).  The
-// prefix table (off, Jmax, packed words) and the row-count table are staged
-// in shared memory.  The in-row term (s' = 0) is resolved by shuffles within
-// the chunk (Bellman-Ford rounds until no lane changes) and loads of the
-// already-stored previous chunks.  Every (n, s) pair with s in C, s <= n is
-// relaxed exactly once: the relaxation count is the closed form.
+// dominated set.  The row base and packed digits come from the row index.
 template <typename E, int NW, bool MULTI>
 __global__ void __launch_bounds__(256)
-row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt,
-                const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
-                int rho, int64_t slot_begin, int64_t slot_count, E *compact, int wlog, int crows)
+row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const uint64_t *__restrict__ pwa,
+                int64_t pw_stride, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
+                int J0, int rho, int64_t slot_begin, int64_t slot_count, E *compact, int wlog)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int np = (int)(meta->nP - 1);      // cross-row prefixes (entry 0 is s' = 0)
-    const int ncnt = (g.K1 + 1) * (g.rho_max + 1);
-    // s_oj[c] = (Jmax << 48) | off(s')   (off < 2^48 since sigma < 2^48)
     uint64_t *s_oj = reinterpret_cast<uint64_t *>(smem_raw);
     uint64_t *s_w = s_oj + np;
-    int64_t *s_cnt = reinterpret_cast<int64_t *>(s_w + (size_t)NW * np);
     for (int i = threadIdx.x; i < np; i += blockDim.x) {
         const PrefixEntry pe = gpref[1 + i];
         s_oj[i] = ((uint64_t)(uint32_t)pe.jmax << 48) | (uint64_t)pe.off;
 #pragma unroll
         for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
     }
-    for (int i = threadIdx.x; i < ncnt; i += blockDim.x) s_cnt[i] = gcnt[i];
     __syncthreads();
 
     const int lane = threadIdx.x & 31;
@@ -281,156 +277,111 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt,
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int64_t W = g.W;
-    const int64_t nchunks = (slot_count + crows - 1) / crows;
     uint64_t guard[NW];
 #pragma unroll
     for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
-    int32_t d[MAXK];
 
-    for (int64_t cb = gw * rpw; cb < nchunks; cb += nw * rpw) {
-        const int64_t ch = cb + grp;
-        const int64_t r0 = ch * crows;
-        const int64_t r1 = r0 + crows < slot_count ? r0 + crows : slot_count;
+    for (int64_t sb = gw * rpw; sb < slot_count; sb += nw * rpw) {
+        const int64_t slot = sb + grp;
+        const bool rowok = slot < slot_count;
         int64_t rowbase = 0;
         uint64_t pw[NW];
 #pragma unroll
-        for (int w = 0; w < NW; ++w) pw[w] = 0;
-        for (int rr = 0; rr < crows; ++rr) {
-            const int64_t slot = r0 + rr;
-            const bool rowok = slot < r1;
-            if (!__any_sync(FULL, rowok)) break;
-            if (rowok) {
-                if (rr == 0) unrank_digits(g, s_cnt, rho, slot_begin + slot, d);
-                else next_in_level(g, d);
-                rowbase = 0;
-#pragma unroll
-                for (int w = 0; w < NW; ++w) pw[w] = 0;
-                for (int i = 0; i < g.K1; ++i) {
-                    rowbase += (int64_t)d[i] * g.stride[i];
+        for (int w = 0; w < NW; ++w) pw[w] = rowok ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
+        if (rowok) rowbase = rb[slot_begin + slot];
+        E *out = compact ? compact + slot * g.Wp : table + rowbase;
+        for (int64_t x0 = 0; x0 < W; x0 += Wg) {
+            const int64_t x = x0 + xl;
+            const bool act = rowok && x < W;
+            const E *rowp = table + (rowbase + x);
+            int acc = INF;
+            for (int base = 0; base < np; base += Wg) {
+                const int c = base + xl;
+                bool dom = false;
+                if (rowok && c < np) {
+                    dom = true;
 #pragma unroll
                     for (int w = 0; w < NW; ++w)
-                        if (g.word[i] == w) pw[w] |= (uint64_t)d[i] << g.shift[i];
+                        dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
                 }
-            }
-            E *out = compact ? compact + slot * g.Wp : table + rowbase;
-            for (int64_t x0 = 0; x0 < W; x0 += Wg) {
-                const int64_t x = x0 + xl;
-                const bool act = rowok && x < W;
-                const E *rowp = table + (rowbase + x);
-                const int xi = x < (1 << 20) ? (int)x : (1 << 20);
-                int acc = INF;
-                for (int base = 0; base < np; base += Wg) {
-                    const int c = base + xl;
-                    bool dom = false;
-                    if (rowok && c < np) {
-                        dom = true;
+                unsigned m = (__ballot_sync(FULL, dom) >> (grp << wlog)) & gmask;
+                // 4 dominated prefixes at a time; lane xl loads OPT(p - s', x) (and, for
+                // rows longer than a chunk, OPT(p - s', x - Wg)); x - j arrives by
+                // shuffle from lane xl - j (source lane t sends v0 if t + j < Wg, else vprev)
+                while (__any_sync(FULL, m != 0)) {
+                    int v0[4], vp[4], jm[4];
 #pragma unroll
-                        for (int w = 0; w < NW; ++w)
-                            dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
-                    }
-                    unsigned m = (__ballot_sync(FULL, dom) >> (grp << wlog)) & gmask;
-                    // Walk the group's dominated prefixes, 4 at a time so that 4 (or 8)
-                    // coalesced gathers are in flight.  Lane xl loads OPT(p - s', x) (and,
-                    // for rows longer than a chunk, OPT(p - s', x - Wg)); the values at
-                    // x - j for j = 1..Jmax(s') arrive by shuffle from lane xl - j: source
-                    // lane t sends v0 if t + j < Wg (same chunk) else vprev (previous chunk).
-                    while (__any_sync(FULL, m != 0)) {
-                        int v0[4], vp[4], jm[4];
-#pragma unroll
-                        for (int q = 0; q < 4; ++q) {
-                            v0[q] = INF;
-                            vp[q] = INF;
-                            jm[q] = -1;
-                            if (m) {
-                                const int b = __ffs(m) - 1;
-                                m &= m - 1;
-                                const uint64_t oj = s_oj[base + b];
-                                const E *src = rowp - (int64_t)(oj & 0xffffffffffffull);
-                                jm[q] = (int)(oj >> 48);
-                                if (act) v0[q] = src[0];
-                                if (MULTI && x0 > 0 && xl + jm[q] >= Wg) vp[q] = src[-Wg];
-                            }
+                    for (int q = 0; q < 4; ++q) {
+                        v0[q] = INF;
+                        vp[q] = INF;
+                        jm[q] = -1;
+                        if (m) {
+                            const int b = __ffs(m) - 1;
+                            m &= m - 1;
+                            const uint64_t oj = s_oj[base + b];
+                            const E *src = rowp - (int64_t)(oj & 0xffffffffffffull);
+                            jm[q] = (int)(oj >> 48);
+                            if (act) v0[q] = src[0];
+                            if (MULTI && x0 > 0 && xl + jm[q] >= Wg) vp[q] = src[-Wg];
                         }
+                    }
 #pragma unroll
-                        for (int q = 0; q < 4; ++q) {
-                            acc = v0[q] < acc ? v0[q] : acc;
-                            int jmq = jm[q];
-                            // jm is uniform within a group; the shuffle loop runs to the
-                            // max over the warp's groups
-                            int jmax_w = jmq;
-                            for (int o = 16; o >= Wg; o >>= 1) {
-                                int t = __shfl_xor_sync(FULL, jmax_w, o);
-                                jmax_w = t > jmax_w ? t : jmax_w;
-                            }
-                            for (int j = 1; j <= jmax_w; ++j) {
-                                const int send = (xl + j < Wg) ? v0[q] : vp[q];
-                                const int t = __shfl_sync(FULL, send, (xl - j) & (Wg - 1), Wg);
-                                if (j <= jmq && t < acc) acc = t;
-                            }
+                    for (int q = 0; q < 4; ++q) {
+                        acc = v0[q] < acc ? v0[q] : acc;
+                        const int jmq = jm[q];
+                        int jmax_w = jmq;
+                        for (int o = 16; o >= Wg; o >>= 1) {
+                            int t = __shfl_xor_sync(FULL, jmax_w, o);
+                            jmax_w = t > jmax_w ? t : jmax_w;
+                        }
+                        for (int j = 1; j <= jmax_w; ++j) {
+                            const int send = (xl + j < Wg) ? v0[q] : vp[q];
+                            const int t = __shfl_sync(FULL, send, (xl - j) & (Wg - 1), Wg);
+                            if (j <= jmq && t < acc) acc = t;
                         }
                     }
                 }
-                if (act) {
-                    // in-row terms that reach back into earlier (stored) chunks
-                    const int jlim = J0 < x ? J0 : (int)x;
-                    for (int j = xl + 1; j <= jlim; ++j) {
-                        int v = out[x - j];
-                        acc = v < acc ? v : acc;
-                    }
-                }
-                int opt = (rho == 0 && x == 0) ? 0 : acc + 1;
-                // in-chunk chain: Bellman-Ford over shuffles
-                const int jin = J0 < Wg - 1 ? J0 : Wg - 1;
-                bool changed = jin > 0;
-                while (__any_sync(FULL, changed)) {
-                    int nopt = opt;
-                    for (int j = 1; j <= jin; ++j) {
-                        int v = __shfl_up_sync(FULL, opt, j, Wg);
-                        if (xl >= j && v + 1 < nopt) nopt = v + 1;
-                    }
-                    changed = nopt < opt;
-                    opt = nopt;
-                }
-                if (act) out[x] = (E)opt;
-                __syncwarp();
             }
+            if (act) {
+                // in-row terms that reach back into earlier (stored) chunks
+                const int jlim = J0 < x ? J0 : (int)x;
+                for (int j = xl + 1; j <= jlim; ++j) {
+                    int v = out[x - j];
+                    acc = v < acc ? v : acc;
+                }
+            }
+            int opt = (rho == 0 && x == 0) ? 0 : acc + 1;
+            // in-chunk chain: Bellman-Ford over shuffles
+            const int jin = J0 < Wg - 1 ? J0 : Wg - 1;
+            bool changed = jin > 0;
+            while (__any_sync(FULL, changed)) {
+                int nopt = opt;
+                for (int j = 1; j <= jin; ++j) {
+                    int v = __shfl_up_sync(FULL, opt, j, Wg);
+                    if (xl >= j && v + 1 < nopt) nopt = v + 1;
+                }
+                changed = nopt < opt;
+                opt = nopt;
+            }
+            if (act) out[x] = (E)opt;
+            __syncwarp();
         }
     }
 }
 
-// §8(e): write gathered compact rows (slot-major, W entries each) into the table.
-template <typename E, int NW>
+// §8(e): write gathered compact rows (slot-major, pitch Wp) into the table.
+template <typename E>
 __global__ void __launch_bounds__(256)
-row_scatter_kernel(E *__restrict__ table, const RowGeom g, const int64_t *__restrict__ cnt, int rho,
-                   int64_t slot_count, const E *__restrict__ compact, int wlog)
+row_scatter_kernel(E *__restrict__ table, const RowGeom g, const int64_t *__restrict__ rb, int64_t slot_count,
+                   const E *__restrict__ compact)
 {
     const int lane = threadIdx.x & 31;
-    const int Wg = 1 << wlog;
-    const int grp = lane >> wlog;
-    const int xl = lane & (Wg - 1);
-    const int rpw = 32 >> wlog;
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t nslot_w = (slot_count + rpw - 1) / rpw;
-    for (int64_t ws = gw; ws < nslot_w; ws += nw) {
-        const int64_t slot = ws * rpw + grp;
-        if (slot >= slot_count) continue;
-        uint64_t pw[NW];
-        int64_t rowbase;
-        unrank_row<NW>(g, cnt, rho, slot, pw, rowbase);
-        for (int64_t x = xl; x < g.Wp; x += Wg) table[rowbase + x] = compact[slot * g.Wp + x];
+    for (int64_t slot = gw; slot < slot_count; slot += nw) {
+        const int64_t rowbase = rb[slot];
+        for (int64_t x = lane; x < g.Wp; x += 32) table[rowbase + x] = compact[slot * g.Wp + x];
     }
-}
-
-__global__ void row_index_kernel(const RowGeom g, const int64_t *__restrict__ cnt, int rho,
-                                 int64_t slot_count, int64_t *__restrict__ out)
-{
-    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= slot_count) return;
-    uint64_t pw[MAXW];
-    int64_t rowbase;
-    unrank_row<MAXW>(g, cnt, rho, t, pw, rowbase);
-    out[t] = rowbase;
 }
 
 template <typename E>
@@ -551,28 +502,37 @@ cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *
     return cudaGetLastError();
 }
 
-cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
-                            const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
-                            int J0, int rho, int64_t slot_begin, int64_t slot_count,
+cudaError_t launch_build_row_index(const RowGeom &g, const int64_t *d_cnt, const int64_t *d_level_start,
+                                   int64_t rows, int64_t *d_rb, uint64_t *d_pw, cudaStream_t st)
+{
+    if (rows <= 0) return cudaSuccess;
+    const int bs = 128;
+    const int64_t blocks = (rows + bs - 1) / bs;
+    if (g.nwords <= 1)
+        build_row_index_kernel<1><<<(unsigned)blocks, bs, 0, st>>>(g, d_cnt, d_level_start, rows, d_rb, d_pw);
+    else
+        build_row_index_kernel<2><<<(unsigned)blocks, bs, 0, st>>>(g, d_cnt, d_level_start, rows, d_rb, d_pw);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
+                            int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                            int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
                             void *compact_out, int sm_count, cudaStream_t st)
 {
     if (slot_count <= 0) return cudaSuccess;
     const int wlog = wlog_for(g.W);
     const int rpw = 32 >> wlog;
     const int bs = 256;
-    const int64_t groups_full = (int64_t)sm_count * 8 * (bs / 32) * rpw;
-    int64_t crows = slot_count / (groups_full * 2);
-    if (crows < 1) crows = 1;
-    if (crows > 16) crows = 16;
-    const int64_t nchunks = (slot_count + crows - 1) / crows;
-    int64_t blocks = (nchunks + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
+    const int64_t warps = (slot_count + rpw - 1) / rpw;
+    int64_t blocks = (warps + (bs / 32) - 1) / (bs / 32);
     const int64_t cap = (int64_t)sm_count * 8;
     if (blocks > cap) blocks = cap;
+    const bool MULTI = g.W > 32;
     const int NWk = g.nwords <= 1 ? 1 : 2;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (size_t)np * (8 + 8 * NWk) + (size_t)(g.K1 + 1) * (g.rho_max + 1) * 8 + 16;
+    const size_t smem = (size_t)np * (8 + 8 * NWk) + 16;
     if (smem > 220 * 1024) return cudaErrorInvalidValue;
-    const bool MULTI = g.W > 32;
     cudaError_t err;
 #define PTAS_FILL_CASE(E_, NW_, MU_)                                                              \
     do {                                                                                          \
@@ -582,9 +542,9 @@ cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t 
                                        (int)smem);                                                \
             if (err != cudaSuccess) return err;                                                   \
         }                                                                                         \
-        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, d_cnt, d_pref, d_meta, J0, rho,   \
-                                                slot_begin, slot_count, (E_ *)compact_out, wlog,  \
-                                                (int)crows);                                      \
+        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta, \
+                                                J0, rho, slot_begin, slot_count, (E_ *)compact_out, \
+                                                wlog);                                            \
     } while (0)
 #define PTAS_FILL_JU(E_, NW_)                                                                     \
     do {                                                                                          \
@@ -601,37 +561,17 @@ cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t 
     return cudaGetLastError();
 }
 
-cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *d_cnt, int rho,
-                               int64_t slot_count, const void *compact, int sm_count,
-                               cudaStream_t st)
+cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *rb, int64_t slot_count,
+                               const void *compact, int sm_count, cudaStream_t st)
 {
     if (slot_count <= 0) return cudaSuccess;
-    const int wlog = wlog_for(g.W);
-    const int rpw = 32 >> wlog;
-    const int bs = 256;
-    int64_t blocks = ((slot_count + rpw - 1) / rpw + 7) / 8;
+    int64_t blocks = (slot_count + 7) / 8;
     const int64_t cap = (int64_t)sm_count * 8;
     if (blocks > cap) blocks = cap;
-    if (e == 1) {
-        if (g.nwords <= 1)
-            row_scatter_kernel<uint8_t, 1><<<(unsigned)blocks, bs, 0, st>>>((uint8_t *)table, g, d_cnt, rho, slot_count, (const uint8_t *)compact, wlog);
-        else
-            row_scatter_kernel<uint8_t, 2><<<(unsigned)blocks, bs, 0, st>>>((uint8_t *)table, g, d_cnt, rho, slot_count, (const uint8_t *)compact, wlog);
-    } else {
-        if (g.nwords <= 1)
-            row_scatter_kernel<uint16_t, 1><<<(unsigned)blocks, bs, 0, st>>>((uint16_t *)table, g, d_cnt, rho, slot_count, (const uint16_t *)compact, wlog);
-        else
-            row_scatter_kernel<uint16_t, 2><<<(unsigned)blocks, bs, 0, st>>>((uint16_t *)table, g, d_cnt, rho, slot_count, (const uint16_t *)compact, wlog);
-    }
-    return cudaGetLastError();
-}
-
-cudaError_t launch_row_index(const RowGeom &g, const int64_t *d_cnt, int rho, int64_t slot_count,
-                             int64_t *out_rowbase, cudaStream_t st)
-{
-    if (slot_count <= 0) return cudaSuccess;
-    const int bs = 128;
-    row_index_kernel<<<(unsigned)((slot_count + bs - 1) / bs), bs, 0, st>>>(g, d_cnt, rho, slot_count, out_rowbase);
+    if (e == 1)
+        row_scatter_kernel<uint8_t><<<(unsigned)blocks, 256, 0, st>>>((uint8_t *)table, g, rb, slot_count, (const uint8_t *)compact);
+    else
+        row_scatter_kernel<uint16_t><<<(unsigned)blocks, 256, 0, st>>>((uint16_t *)table, g, rb, slot_count, (const uint16_t *)compact);
     return cudaGetLastError();
 }
 

@@ -85,7 +85,7 @@ class Engine {
     DpMeta *d_meta_ = nullptr;
     DpMeta *h_meta_ = nullptr;     // pinned
     int64_t *h_scalar_ = nullptr;  // pinned
-    Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_;
+    Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_, rowidx_;
 
     // state of the last DP (for traceback)
     bool last_valid_ = false;

@@ -71,23 +71,29 @@ cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *
 // One row-level of the level fill.  e = 1 or 2.  Rows [slot_begin, slot_begin+slot_count)
 // of row-level rho; results go to the table (compact_out == NULL) or to
 // compact_out[(slot - slot_begin) * Wp + x].
-cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
+// rb/pw point at the row-level's first slot (rb + level_start[rho]); pw_stride
+// is the distance between the packed words of one row (= total rows).
+cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t *rb,
+                            const uint64_t *pw, int64_t pw_stride,
                             const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
                             int J0, int rho, int64_t slot_begin, int64_t slot_count,
                             void *compact_out, int sm_count, cudaStream_t st);
+// a-4 level-ordered row index: for every row slot t (row-levels concatenated,
+// lexicographic within a level) its row base index rb[t] and packed leading
+// digits pw[w * rows + t].
+cudaError_t launch_build_row_index(const RowGeom &g, const int64_t *d_cnt, const int64_t *d_level_start,
+                                   int64_t rows, int64_t *d_rb, uint64_t *d_pw, cudaStream_t st);
 // Packed-word fill (row_fill_swar.cu); cudaErrorNotSupported -> use launch_row_fill.
-cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
+cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *rb,
+                                 const uint64_t *pw, int64_t pw_stride,
                                  const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
                                  int J0, int rho, int64_t slot_begin, int64_t slot_count,
                                  void *compact_out, int sm_count, cudaStream_t st);
 // Copy rows of pitch Wp (src) to pitch W (dst), `rows` rows of e-byte entries.
 cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows, int64_t W,
                                 int64_t Wp, cudaStream_t st);
-cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
-                               int rho, int64_t slot_count, const void *compact,
-                               int sm_count, cudaStream_t st);
-cudaError_t launch_row_index(const RowGeom &g, const int64_t *d_cnt, int rho,
-                             int64_t slot_count, int64_t *out_rowbase, cudaStream_t st);
+cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *rb,
+                               int64_t slot_count, const void *compact, int sm_count, cudaStream_t st);
 cudaError_t launch_read_opt(int e, const void *table, int64_t idx, DpMeta *d_meta,
                             cudaStream_t st);
 cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N,

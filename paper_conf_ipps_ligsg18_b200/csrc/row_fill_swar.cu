@@ -21,6 +21,7 @@
 // form relaxation count still holds.  Entries in the row padding and in
 // lanes past the row end are computed but never read as sources.
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "device_common.cuh"
@@ -39,20 +40,32 @@ __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel)
 
 __device__ __forceinline__ uint32_t vmin2(uint32_t a, uint32_t b) { return __vminu2(a, b); }
 
-// Word k words to the left of word position (lane xl, chunk t) within a row
-// of lane group width Lg (k >= 1).  Source lane (xl - k) mod Lg; lanes that
-// wrap supply the previous chunk's word (`prev`, `fill` before chunk 0).
-__device__ __forceinline__ uint32_t word_left(uint32_t cur, uint32_t prev, int xl, int k, int Lg)
-{
-    if (k >= Lg) return prev;  // only reachable for Lg == 32 with k == 32 (caller bounds k)
-    const uint32_t send = (xl >= Lg - k) ? prev : cur;
-    return __shfl_sync(FULL, send, (xl - k) & (Lg - 1), Lg);
-}
-
 template <int CH>
 struct Words {
     uint32_t v[CH];
 };
+
+// Word k positions to the left of the lane's word of chunk t.  A row's words
+// are laid out as w = xl + Lg * t (lane xl of a group of Lg lanes, chunk t);
+// with k = qk * Lg + rk, word w - k lives in lane (xl - rk) mod Lg, chunk
+// t - qk (or t - qk - 1 when the lane index wraps).  Chunks before 0 are
+// outside the row and read as `fill`.
+template <int CH>
+__device__ __forceinline__ uint32_t word_left(const Words<CH> &a, int t, int k, int xl, int Lg, int lglog,
+                                              uint32_t fill)
+{
+    const int qk = k >> lglog, rk = k & (Lg - 1);
+    const int c1 = t - qk, c2 = c1 - 1;
+    uint32_t v1 = fill, v2 = fill;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) {
+        if (c == c1) v1 = a.v[c];
+        if (c == c2) v2 = a.v[c];
+    }
+    if (rk == 0) return v1;
+    const uint32_t send = (xl >= Lg - rk) ? v2 : v1;
+    return __shfl_sync(FULL, send, (xl - rk) & (Lg - 1), Lg);
+}
 
 // acc <- min(acc, window of `lo:hi` at byte offset o) for one word position.
 template <int EB>
@@ -70,19 +83,19 @@ __device__ __forceinline__ void acc_window(uint32_t lo, uint32_t hi, int o, uint
 // JB > 0: shifts up to JB bytes, fully unrolled (jm * EB <= JB guaranteed by
 // the host); JB == 0: any shift (runtime loop, generic word fetch).
 template <int EB, int CH, int JB>
-__device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int xl, int Lg, Words<CH> &ae,
-                                             Words<CH> &ao)
+__device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int xl, int Lg, int lglog,
+                                             Words<CH> &ae, Words<CH> &ao)
 {
 #pragma unroll
     for (int t = 0; t < CH; ++t) acc_window<EB>(cur.v[t], cur.v[t], 0, ae.v[t], ao.v[t]);
-    if (jm <= 0) return;
+    if (JB == 0 && jm <= 0) return;
     Words<CH> w1, w2;
 #pragma unroll
-    for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur.v[t], t ? cur.v[t - 1] : 0xffffffffu, xl, 1, Lg);
+    for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur, t, 1, xl, Lg, lglog, 0xffffffffu);
     if (JB == 0 || JB > 4) {
         if (jm * EB > 4) {
 #pragma unroll
-            for (int t = 0; t < CH; ++t) w2.v[t] = word_left(cur.v[t], t ? cur.v[t - 1] : 0xffffffffu, xl, 2, Lg);
+            for (int t = 0; t < CH; ++t) w2.v[t] = word_left(cur, t, 2, xl, Lg, lglog, 0xffffffffu);
         }
     }
     if constexpr (JB > 0) {
@@ -108,9 +121,8 @@ __device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int x
                 else if (db <= 8) acc_window<EB>(w2.v[t], w1.v[t], 8 - db, ae.v[t], ao.v[t]);
                 else {
                     const int k = (db + 3) >> 2;
-                    const uint32_t prev = t ? cur.v[t - 1] : 0xffffffffu;
-                    acc_window<EB>(word_left(cur.v[t], prev, xl, k, Lg), word_left(cur.v[t], prev, xl, k - 1, Lg),
-                                   4 * k - db, ae.v[t], ao.v[t]);
+                    acc_window<EB>(word_left(cur, t, k, xl, Lg, lglog, 0xffffffffu),
+                                   word_left(cur, t, k - 1, xl, Lg, lglog, 0xffffffffu), 4 * k - db, ae.v[t], ao.v[t]);
                 }
             }
         }
@@ -132,27 +144,27 @@ __device__ __forceinline__ uint32_t lane_shift(const uint32_t w0, const uint32_t
 
 template <typename E, int NW, int CH, int JB>
 __global__ void __launch_bounds__(256)
-row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt,
+row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
+                     const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
-                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int lglog, int crows)
+                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int lglog)
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int np = (int)(meta->nP - 1);
-    const int ncnt = (g.K1 + 1) * (g.rho_max + 1);
-    uint64_t *s_oj = reinterpret_cast<uint64_t *>(smem_raw);
-    uint64_t *s_w = s_oj + np;
-    int64_t *s_cnt = reinterpret_cast<int64_t *>(s_w + (size_t)NW * np);
+    // s_oj[c] = {-off(s') in words, Jmax(s')}: int32 offsets (the host routes
+    // tables of 2^31 words or more to the scalar kernel)
+    int2 *s_oj = reinterpret_cast<int2 *>(smem_raw);
+    uint64_t *s_w = reinterpret_cast<uint64_t *>(s_oj + ((np + 1) & ~1));
     for (int i = threadIdx.x; i < np; i += blockDim.x) {
         const PrefixEntry pe = gpref[1 + i];
         // off(s') in words (a multiple of the padded row, hence of 4 bytes)
         const uint64_t offw = (uint64_t)pe.off * EB / 4;
-        s_oj[i] = ((uint64_t)(uint32_t)pe.jmax << 48) | offw;
+        s_oj[i] = make_int2(-(int)offw, pe.jmax);
 #pragma unroll
         for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
     }
-    for (int i = threadIdx.x; i < ncnt; i += blockDim.x) s_cnt[i] = gcnt[i];
     __syncthreads();
 
     const int lane = threadIdx.x & 31;
@@ -164,41 +176,23 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int Lw = (int)(g.Wp * EB / 4);  // words per (padded) row
-    const int64_t nchunks = (slot_count + crows - 1) / crows;
     uint64_t guard[NW];
 #pragma unroll
     for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
-    int32_t d[MAXK];
 
-    for (int64_t cb = gw * rpw; cb < nchunks; cb += nw * rpw) {
-        const int64_t ch = cb + grp;
-        const int64_t r0 = ch * crows;
-        const int64_t r1 = r0 + crows < slot_count ? r0 + crows : slot_count;
-        int64_t rowbase = 0;
-        uint64_t pw[NW];
+    for (int64_t sb = gw * rpw; sb < slot_count; sb += nw * rpw) {
+        {
+            const int64_t slot = sb + grp;
+            const bool rowok = slot < slot_count;
+            int64_t rowbase = 0;
+            uint64_t pw[NW];
 #pragma unroll
-        for (int w = 0; w < NW; ++w) pw[w] = 0;
-        for (int rr = 0; rr < crows; ++rr) {
-            const int64_t slot = r0 + rr;
-            const bool rowok = slot < r1;
-            if (!__any_sync(FULL, rowok)) break;
-            if (rowok) {
-                if (rr == 0) unrank_digits(g, s_cnt, rho, slot_begin + slot, d);
-                else next_in_level(g, d);
-                rowbase = 0;
-#pragma unroll
-                for (int w = 0; w < NW; ++w) pw[w] = 0;
-                for (int i = 0; i < g.K1; ++i) {
-                    rowbase += (int64_t)d[i] * g.stride[i];
-#pragma unroll
-                    for (int w = 0; w < NW; ++w)
-                        if (g.word[i] == w) pw[w] |= (uint64_t)d[i] << g.shift[i];
-                }
-            }
+            for (int w = 0; w < NW; ++w) pw[w] = rowok ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
+            if (rowok) rowbase = rb[slot_begin + slot];
             const uint32_t *row32 = reinterpret_cast<const uint32_t *>(table + rowbase) + xl;
             bool wok[CH];
 #pragma unroll
-            for (int t = 0; t < CH; ++t) wok[t] = rowok && (xl + 32 * t) < Lw;
+            for (int t = 0; t < CH; ++t) wok[t] = rowok && (xl + Lg * t) < Lw;
 
             // ---- cross-row relaxations
             Words<CH> ae, ao;
@@ -227,16 +221,15 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                         const int q = q0 + u;
                         const bool live = q < cend;
                         const bool pd = live && ((m >> q) & 1u);
-                        const uint64_t oj = live ? s_oj[base + q] : 0ull;
-                        const uint32_t *src = row32 - (int64_t)(oj & 0xffffffffffffull);
-                        jmq[u] = live ? (int)(oj >> 48) : -1;
+                        const int2 oj = s_oj[live ? base + q : 0];
+                        const uint32_t *src = row32 + oj.x;
+                        jmq[u] = live ? oj.y : -1;
 #pragma unroll
                         for (int t = 0; t < CH; ++t)
-                            curq[u].v[t] = (pd && wok[t]) ? src[32 * t] : 0xffffffffu;
+                            curq[u].v[t] = (pd && wok[t]) ? src[Lg * t] : 0xffffffffu;
                     }
 #pragma unroll
-                    for (int u = 0; u < 4; ++u)
-                        if (jmq[u] >= 0) relax_prefix<EB, CH, JB>(curq[u], jmq[u], xl, Lg, ae, ao);
+                    for (int u = 0; u < 4; ++u) relax_prefix<EB, CH, JB>(curq[u], jmq[u], xl, Lg, lglog, ae, ao);
                 }
             }
 
@@ -274,16 +267,16 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                         int po = 0, qo = 0;
                         if (JB == 0 && 2 * sa > 8) {
                             const int k = (2 * sa + 3) >> 2;
-                            const uint32_t pv = t ? (odd ? oo.v[t - 1] : oe.v[t - 1]) : CFILL;
-                            plo = word_left(A0, pv, xl, k, Lg);
-                            phi = word_left(A0, pv, xl, k - 1, Lg);
+                            const Words<CH> &AA = odd ? oo : oe;
+                            plo = word_left(AA, t, k, xl, Lg, lglog, CFILL);
+                            phi = word_left(AA, t, k - 1, xl, Lg, lglog, CFILL);
                             po = 4 * k - 2 * sa;
                         }
                         if (JB == 0 && 2 * sb > 8) {
                             const int k = (2 * sb + 3) >> 2;
-                            const uint32_t pv = t ? (odd ? oe.v[t - 1] : oo.v[t - 1]) : CFILL;
-                            qlo = word_left(B0, pv, xl, k, Lg);
-                            qhi = word_left(B0, pv, xl, k - 1, Lg);
+                            const Words<CH> &BB = odd ? oe : oo;
+                            qlo = word_left(BB, t, k, xl, Lg, lglog, CFILL);
+                            qhi = word_left(BB, t, k - 1, xl, Lg, lglog, CFILL);
                             qo = 4 * k - 2 * sb;
                         }
                         const uint32_t va = lane_shift(A0, A1, A2, 2 * sa, plo, phi, po);
@@ -295,9 +288,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                         int po = 0;
                         if (JB == 0 && 2 * j > 8) {
                             const int k = (2 * j + 3) >> 2;
-                            const uint32_t pv = t ? oe.v[t - 1] : CFILL;
-                            plo = word_left(oe.v[t], pv, xl, k, Lg);
-                            phi = word_left(oe.v[t], pv, xl, k - 1, Lg);
+                            plo = word_left(oe, t, k, xl, Lg, lglog, CFILL);
+                            phi = word_left(oe, t, k - 1, xl, Lg, lglog, CFILL);
                             po = 4 * k - 2 * j;
                         }
                         const uint32_t va = lane_shift(oe.v[t], e1.v[t], e2.v[t], 2 * j, plo, phi, po);
@@ -313,16 +305,16 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                 Words<CH> e1, o1, e2, o2;
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
-                    e1.v[t] = word_left(oe.v[t], t ? oe.v[t - 1] : CFILL, xl, 1, Lg);
-                    o1.v[t] = EB == 1 ? word_left(oo.v[t], t ? oo.v[t - 1] : CFILL, xl, 1, Lg) : 0u;
+                    e1.v[t] = word_left(oe, t, 1, xl, Lg, lglog, CFILL);
+                    o1.v[t] = EB == 1 ? word_left(oo, t, 1, xl, Lg, lglog, CFILL) : 0u;
                     e2.v[t] = e1.v[t];
                     o2.v[t] = o1.v[t];
                 }
                 if (chain_db > 4) {
 #pragma unroll
                     for (int t = 0; t < CH; ++t) {
-                        e2.v[t] = word_left(oe.v[t], t ? oe.v[t - 1] : CFILL, xl, 2, Lg);
-                        o2.v[t] = EB == 1 ? word_left(oo.v[t], t ? oo.v[t - 1] : CFILL, xl, 2, Lg) : 0u;
+                        e2.v[t] = word_left(oe, t, 2, xl, Lg, lglog, CFILL);
+                        o2.v[t] = EB == 1 ? word_left(oo, t, 2, xl, Lg, lglog, CFILL) : 0u;
                     }
                 }
                 Words<CH> ne = oe, no = oo;
@@ -349,7 +341,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
                 uint32_t wv;
                 if constexpr (EB == 1) wv = prmt(oe.v[t], oo.v[t], 0x6240u);
                 else wv = oe.v[t];
-                out32[xl + 32 * t] = wv;
+                out32[xl + Lg * t] = wv;
             }
             __syncwarp();
         }
@@ -358,34 +350,40 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ gcnt
 
 // Host launcher: returns cudaErrorNotSupported when the geometry needs the
 // scalar kernel (row longer than 1 KiB, or shifts beyond one chunk).
-cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *d_cnt,
-                                 const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
-                                 int J0, int rho, int64_t slot_begin, int64_t slot_count,
-                                 void *compact_out, int sm_count, cudaStream_t st)
+cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *rb,
+                                 const uint64_t *pw, int64_t pw_stride, const PrefixEntry *d_pref,
+                                 const DpMeta *d_meta, int64_t nP_bound, int J0, int rho,
+                                 int64_t slot_begin, int64_t slot_count, void *compact_out, int sm_count,
+                                 cudaStream_t st)
 {
     if (slot_count <= 0) return cudaSuccess;
     const int Lw = (int)(g.Wp * e / 4);
     if ((g.Wp * e) % 4 != 0 || Lw > 256 || J0 * e > 124) return cudaErrorNotSupported;
-    int lglog = 0;
-    while ((1 << lglog) < Lw && lglog < 5) ++lglog;
-    const int Lg = 1 << lglog;
-    if (Lw <= 32 && J0 * e > 4 * Lg) {
-        // all shifts beyond the row: still correct (INF fill), but keep k < Lg
+    // int32 word offsets: the table (incl. padding) must stay below 2^31 words
+    {
+        int64_t rows_all = 1;
+        for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
+        if (rows_all * (int64_t)Lw >= ((int64_t)1 << 31)) return cudaErrorNotSupported;
     }
-    const int CH = Lw <= 32 ? 1 : (Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8));
+    // words per lane (chunks, stride Lg): amortise the per-prefix cost over
+    // CH words; rows of <= 32 words use Lg = next_pow2(ceil(Lw / CH)).
+    int CH;
+    const char *chs = std::getenv("PTAS_SWAR_CH");
+    if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
+    else if (chs && chs[0]) CH = std::atoi(chs);
+    else CH = Lw >= 8 ? 2 : 1;
+    if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
+    int lglog = 0;
+    while ((1 << lglog) * CH < Lw && lglog < 5) ++lglog;
+    if ((1 << lglog) * CH < Lw) return cudaErrorNotSupported;
     const int rpw = 32 >> lglog;
     const int bs = 256;
-    const int64_t groups_full = (int64_t)sm_count * 8 * (bs / 32) * rpw;
-    int64_t crows = (slot_count + groups_full - 1) / groups_full;  // one unrank per group, then successors
-    if (crows < 1) crows = 1;
-    if (crows > 32) crows = 32;
-    const int64_t nchunks = (slot_count + crows - 1) / crows;
-    int64_t blocks = (nchunks + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
+    int64_t blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
     const int64_t cap = (int64_t)sm_count * 8;
     if (blocks > cap) blocks = cap;
     const int NWk = g.nwords <= 1 ? 1 : 2;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (size_t)np * (8 + 8 * NWk) + (size_t)(g.K1 + 1) * (g.rho_max + 1) * 8 + 16;
+    const size_t smem = (size_t)np * (8 + 8 * NWk) + 16;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     cudaError_t err;
     // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
@@ -399,9 +397,9 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
                                        (int)smem);                                                \
             if (err != cudaSuccess) return err;                                                   \
         }                                                                                         \
-        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, d_cnt, d_pref, d_meta, J0, rho,   \
-                                                slot_begin, slot_count, (E_ *)compact_out, lglog, \
-                                                (int)crows);                                      \
+        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta, \
+                                                J0, rho, slot_begin, slot_count, (E_ *)compact_out, \
+                                                lglog);                                           \
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
     do {                                                                                          \
