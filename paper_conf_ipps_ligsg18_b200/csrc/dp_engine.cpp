@@ -332,18 +332,25 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     const int J0 = (int)std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
     const char *fs = std::getenv("PTAS_FORCE_SCALAR");
     const bool force_scalar = fs && fs[0] == '1';
+    const char *pdls = std::getenv("PTAS_PDL");
+    const bool use_pdl = !(pdls && pdls[0] == '0');
+    bool prev_fill = false;  // the previous launch on st was a packed fill (PDL-safe)
     // one row-level (or slice of it): packed-word kernel, scalar kernel as fallback
     auto fill = [&](void *tab, const RowGeom &gg, int j0, int rho_, int64_t b, int64_t c,
                     void *compact) -> cudaError_t {
         const int64_t *rbl = d_rb + lstart[rho_];
         const uint64_t *pwl = d_pw + lstart[rho_];
         cudaError_t err = cudaErrorNotSupported;
-        if (!force_scalar)
+        if (!force_scalar) {
             err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC,
-                                       j0, rho_, b, c, compact, sm_count_, st);
-        if (err == cudaErrorNotSupported)
+                                       j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0);
+            if (err == cudaSuccess) prev_fill = true;
+        }
+        if (err == cudaErrorNotSupported) {
             err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC, j0,
                                   rho_, b, c, compact, sm_count_, st);
+            prev_fill = false;
+        }
         return err;
     };
 
@@ -401,6 +408,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
             if (crc) return crc;
         }
         PT_CK(launch_row_scatter(e, table, g, d_rb + lstart[rho], R, stage, sm_count_, st));
+        prev_fill = false;
         ++o.launches;
     }
     PT_CK(cudaEventRecord(ev_[2], st));

@@ -84,11 +84,13 @@ cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t 
 cudaError_t launch_build_row_index(const RowGeom &g, const int64_t *d_cnt, const int64_t *d_level_start,
                                    int64_t rows, int64_t *d_rb, uint64_t *d_pw, cudaStream_t st);
 // Packed-word fill (row_fill_swar.cu); cudaErrorNotSupported -> use launch_row_fill.
+// pdl = 1: programmatic dependent launch after the previous fill launch (the
+// first fill launch of a DP must use pdl = 0).
 cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *rb,
                                  const uint64_t *pw, int64_t pw_stride,
                                  const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
                                  int J0, int rho, int64_t slot_begin, int64_t slot_count,
-                                 void *compact_out, int sm_count, cudaStream_t st);
+                                 void *compact_out, int sm_count, cudaStream_t st, int pdl);
 // Copy rows of pitch Wp (src) to pitch W (dst), `rows` rows of e-byte entries.
 cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows, int64_t W,
                                 int64_t Wp, cudaStream_t st);

@@ -147,11 +147,15 @@ __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
-                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int lglog)
+                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int lglog, int nsplit)
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    // Programmatic dependent launch: let the next row-level's grid start its
+    // prologue now; everything before griddepcontrol.wait below reads only data
+    // produced before the first fill launch of the DP (prefix table, row index).
+    asm volatile("griddepcontrol.launch_dependents;");
     const int np = (int)(meta->nP - 1);
     // s_oj[c] = {-off(s') in words, Jmax(s')}: int32 offsets (the host routes
     // tables of 2^31 words or more to the scalar kernel)
@@ -173,22 +177,45 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     const int xl = lane & (Lg - 1);
     const int rpw = 32 >> lglog;
     const unsigned gmask = Lg == 32 ? 0xffffffffu : ((1u << Lg) - 1u);
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    // nsplit == 1: every warp owns its own rows.  nsplit > 1 (small row-levels):
+    // the nsplit warps of a block share one set of rows, each walks every
+    // nsplit-th prefix batch, and warp 0 combines the partial minima (shared
+    // memory) before the chain -- the per-row latency drops by ~nsplit.
+    const int wid = threadIdx.x >> 5;
+    const int64_t gw = nsplit > 1 ? (int64_t)blockIdx.x : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = nsplit > 1 ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int pbase0 = nsplit > 1 ? wid * Lg : 0;
+    const int pstep = nsplit > 1 ? nsplit * Lg : Lg;
+    uint32_t *s_red = reinterpret_cast<uint32_t *>(s_w + (size_t)NW * np);  // [warp][2][CH][32]
     const int Lw = (int)(g.Wp * EB / 4);  // words per (padded) row
     uint64_t guard[NW];
 #pragma unroll
     for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
+    // first row set's index entries, loaded before waiting on the previous level
+    int64_t nrb = 0;
+    uint64_t npw[NW];
+    {
+        const int64_t slot = gw * rpw + grp;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) npw[w] = slot < slot_count ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
+        if (slot < slot_count) nrb = rb[slot_begin + slot];
+    }
+    asm volatile("griddepcontrol.wait;" ::: "memory");
 
     for (int64_t sb = gw * rpw; sb < slot_count; sb += nw * rpw) {
         {
             const int64_t slot = sb + grp;
             const bool rowok = slot < slot_count;
-            int64_t rowbase = 0;
+            int64_t rowbase = nrb;
             uint64_t pw[NW];
 #pragma unroll
-            for (int w = 0; w < NW; ++w) pw[w] = rowok ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
-            if (rowok) rowbase = rb[slot_begin + slot];
+            for (int w = 0; w < NW; ++w) pw[w] = npw[w];
+            {   // prefetch the next row set's index entries
+                const int64_t ns = sb + nw * rpw + grp;
+#pragma unroll
+                for (int w = 0; w < NW; ++w) npw[w] = ns < slot_count ? pwa[(int64_t)w * pw_stride + slot_begin + ns] : 0;
+                nrb = ns < slot_count ? rb[slot_begin + ns] : 0;
+            }
             const uint32_t *row32 = reinterpret_cast<const uint32_t *>(table + rowbase) + xl;
             bool wok[CH];
 #pragma unroll
@@ -201,7 +228,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 ae.v[t] = 0xffffffffu;
                 ao.v[t] = 0xffffffffu;
             }
-            for (int base = 0; base < np; base += Lg) {
+            for (int base = pbase0; base < np; base += pstep) {
                 const int c = base + xl;
                 bool dom = false;
                 if (rowok && c < np) {
@@ -233,6 +260,24 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 }
             }
 
+            if (nsplit > 1) {
+#pragma unroll
+                for (int t = 0; t < CH; ++t) {
+                    s_red[((wid * 2 + 0) * CH + t) * 32 + lane] = ae.v[t];
+                    s_red[((wid * 2 + 1) * CH + t) * 32 + lane] = ao.v[t];
+                }
+                __syncthreads();
+                if (wid == 0) {
+                    for (int w2 = 1; w2 < nsplit; ++w2) {
+#pragma unroll
+                        for (int t = 0; t < CH; ++t) {
+                            ae.v[t] = vmin2(ae.v[t], s_red[((w2 * 2 + 0) * CH + t) * 32 + lane]);
+                            ao.v[t] = vmin2(ao.v[t], s_red[((w2 * 2 + 1) * CH + t) * 32 + lane]);
+                        }
+                    }
+                }
+            }
+            if (nsplit == 1 || wid == 0) {
             // ---- in-row chain on plain uint16 lanes: opt = 1 + min(acc, opt(x - j))
             // uint8: E holds x = 4w, 4w+2; O holds x = 4w+1, 4w+3.  uint16: E holds 2w, 2w+1.
             Words<CH> oe, oo;
@@ -344,6 +389,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 out32[xl + Lg * t] = wv;
             }
             __syncwarp();
+            }  // chain + store (warp 0 in split mode)
+            if (nsplit > 1) __syncthreads();  // s_red reused by the next row set
         }
     }
 }
@@ -354,7 +401,7 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
                                  const uint64_t *pw, int64_t pw_stride, const PrefixEntry *d_pref,
                                  const DpMeta *d_meta, int64_t nP_bound, int J0, int rho,
                                  int64_t slot_begin, int64_t slot_count, void *compact_out, int sm_count,
-                                 cudaStream_t st)
+                                 cudaStream_t st, int pdl)
 {
     if (slot_count <= 0) return cudaSuccess;
     const int Lw = (int)(g.Wp * e / 4);
@@ -381,9 +428,17 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
     int64_t blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
     const int64_t cap = (int64_t)sm_count * 8;
     if (blocks > cap) blocks = cap;
+    // small row-levels: split each row set's prefixes over the 8 warps of a block
+    const char *sp = std::getenv("PTAS_SPLIT_ROWS");
+    const int64_t split_rows = sp ? std::atoll(sp) : (int64_t)sm_count * rpw * 2;
+    int nsplit = 1;
+    if (slot_count <= split_rows) {
+        nsplit = bs / 32;
+        blocks = (slot_count + rpw - 1) / rpw;
+    }
     const int NWk = g.nwords <= 1 ? 1 : 2;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (size_t)np * (8 + 8 * NWk) + 16;
+    const size_t smem = (size_t)np * (8 + 8 * NWk) + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     cudaError_t err;
     // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
@@ -397,9 +452,20 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
                                        (int)smem);                                                \
             if (err != cudaSuccess) return err;                                                   \
         }                                                                                         \
-        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta, \
-                                                J0, rho, slot_begin, slot_count, (E_ *)compact_out, \
-                                                lglog);                                           \
+        cudaLaunchConfig_t cfg = {};                                                              \
+        cudaLaunchAttribute attr[1];                                                              \
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;                          \
+        attr[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;                         \
+        cfg.gridDim = dim3((unsigned)blocks);                                                     \
+        cfg.blockDim = dim3(bs);                                                                  \
+        cfg.dynamicSmemBytes = smem;                                                              \
+        cfg.stream = st;                                                                          \
+        cfg.attrs = attr;                                                                         \
+        cfg.numAttrs = 1;                                                                         \
+        err = cudaLaunchKernelEx(&cfg, kfn, (E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta,    \
+                                 J0, rho, slot_begin, slot_count, (E_ *)compact_out, lglog,       \
+                                 nsplit);                                                         \
+        if (err != cudaSuccess) return err;                                                       \
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
     do {                                                                                          \

@@ -168,6 +168,19 @@ def test_dp_fill_scalar_kernel(P, monkeypatch):
     _check_table(P, np.array([5, 4, 70], np.int32), np.array([90, 70, 11], np.int64), 200)
 
 
+@pytest.mark.parametrize("split", ["0", "1000000000"])
+def test_dp_fill_row_split_modes(P, monkeypatch, split):
+    # small-level mode (8 warps share a row set) forced on / off for every level
+    monkeypatch.setenv("PTAS_SPLIT_ROWS", split)
+    rng = np.random.default_rng(57)
+    for K in (2, 3, 5, 7):
+        for _ in range(3):
+            N, r, T = _rand_case(rng, K, {2: 60, 3: 25, 5: 8, 7: 4}[K])
+            _check_table(P, N, r, T)
+    _check_table(P, np.array([5, 4, 70], np.int32), np.array([90, 70, 11], np.int64), 200)
+    _check_table(P, np.array([30, 40, 300], np.int32), np.array([90, 70, 11], np.int64), 200)
+
+
 def test_dp_fill_very_long_rows(P):
     # rows longer than 1 KiB (uint16, W = 701) use the scalar kernel; W*e = 1024 B exactly uses 8 chunks
     _check_table(P, np.array([2, 700], np.int32), np.array([60, 13], np.int64), 120)
