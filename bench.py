@@ -266,11 +266,15 @@ def run_ours(args, w):
         relax_total, e2e_relax, alg_bytes = rl.tolist()
     peak, peak_kind = _peaks()
     achieved = alg_bytes / fill_s / 1e9 if fill_s > 0 else 0.0
-    traffic = None
+    traffic, traffic_note = None, None
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(w.name)
+            t = json.load(open(tf)).get(w.name)
+            if t:
+                traffic = t["dram_bytes_per_launch"]
+                traffic_note = {"alg_bytes_per_launch": t["alg_bytes_per_launch"],
+                                "traffic_over_alg": t["traffic_over_alg"], "source": t["source"]}
         except Exception:
             traffic = None
     st0 = stats[0]
@@ -291,7 +295,7 @@ def run_ours(args, w):
                 "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e2e_stats) / args.steps),
                 "solve_ms": 1e3 * e2e_t / args.steps},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic,
+                     "frac": achieved / peak, "traffic": traffic, "traffic_note": traffic_note,
                      "kernel": "row_fill_kernel (level fill)",
                      "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)" if peak_kind == "measured" else "fallback",
                      "fill_ms_per_step": 1e3 * fill_s / args.steps,
