@@ -88,7 +88,7 @@ __device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int x
 {
 #pragma unroll
     for (int t = 0; t < CH; ++t) acc_window<EB>(cur.v[t], cur.v[t], 0, ae.v[t], ao.v[t]);
-    if (JB == 0 && jm <= 0) return;
+    if (jm <= 0) return;
     Words<CH> w1, w2;
 #pragma unroll
     for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur, t, 1, xl, Lg, lglog, 0xffffffffu);
@@ -99,11 +99,13 @@ __device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int x
         }
     }
     if constexpr (JB > 0) {
+        // jm is warp-uniform (all groups walk the same prefix): leave the
+        // unrolled sequence with a uniform branch instead of predicating the
+        // remaining steps
 #pragma unroll
         for (int j = 1; j <= JB / EB; ++j) {
-            if (j <= jm) {
-                constexpr int dummy = 0;
-                (void)dummy;
+            if (j > jm) break;
+            {
                 const int db = j * EB;
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
