@@ -161,15 +161,20 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     const int np = (int)(meta->nP - 1);
     // s_oj[c] = {-off(s') in words, Jmax(s')}: int32 offsets (the host routes
     // tables of 2^31 words or more to the scalar kernel)
+    const int npad = (np + 31) & ~31;  // zero-padded: dummy slots never load and have Jmax 0
     int2 *s_oj = reinterpret_cast<int2 *>(smem_raw);
-    uint64_t *s_w = reinterpret_cast<uint64_t *>(s_oj + ((np + 1) & ~1));
-    for (int i = threadIdx.x; i < np; i += blockDim.x) {
-        const PrefixEntry pe = gpref[1 + i];
-        // off(s') in words (a multiple of the padded row, hence of 4 bytes)
-        const uint64_t offw = (uint64_t)pe.off * EB / 4;
-        s_oj[i] = make_int2(-(int)offw, pe.jmax);
+    uint64_t *s_w = reinterpret_cast<uint64_t *>(s_oj + npad);
+    for (int i = threadIdx.x; i < npad; i += blockDim.x) {
+        if (i < np) {
+            const PrefixEntry pe = gpref[1 + i];
+            // off(s') in words (a multiple of the padded row, hence of 4 bytes)
+            const uint64_t offw = (uint64_t)pe.off * EB / 4;
+            s_oj[i] = make_int2(-(int)offw, pe.jmax);
 #pragma unroll
-        for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
+            for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
+        } else {
+            s_oj[i] = make_int2(0, 0);
+        }
     }
     __syncthreads();
 
@@ -188,7 +193,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     const int64_t nw = nsplit > 1 ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int pbase0 = nsplit > 1 ? wid * Lg : 0;
     const int pstep = nsplit > 1 ? nsplit * Lg : Lg;
-    uint32_t *s_red = reinterpret_cast<uint32_t *>(s_w + (size_t)NW * np);  // [warp][2][CH][32]
+    uint32_t *s_red = reinterpret_cast<uint32_t *>(s_w + (size_t)NW * np + 1);  // [warp][2][CH][32]
     const int Lw = (int)(g.Wp * EB / 4);  // words per (padded) row
     uint64_t guard[NW];
 #pragma unroll
@@ -218,7 +223,9 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 for (int w = 0; w < NW; ++w) npw[w] = ns < slot_count ? pwa[(int64_t)w * pw_stride + slot_begin + ns] : 0;
                 nrb = ns < slot_count ? rb[slot_begin + ns] : 0;
             }
-            const uint32_t *row32 = reinterpret_cast<const uint32_t *>(table + rowbase) + xl;
+            // int32 word index of this lane's first word (the launcher guarantees < 2^31 words)
+            const int rw = (int)(rowbase * EB / 4) + xl;
+            const uint32_t *tab32 = reinterpret_cast<const uint32_t *>(table);
             bool wok[CH];
 #pragma unroll
             for (int t = 0; t < CH; ++t) wok[t] = rowok && (xl + Lg * t) < Lw;
@@ -240,7 +247,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
                 }
                 const unsigned m = (__ballot_sync(FULL, dom) >> (grp << lglog)) & gmask;
-                const int cend = np - base < Lg ? np - base : Lg;
+                const int cend = Lg < 4 ? Lg : ((np - base < Lg ? np - base : Lg) + 3) & ~3;
                 // 4 prefixes per step: their gathers are issued before any is consumed
                 for (int q0 = 0; q0 < cend; q0 += 4) {
                     Words<CH> curq[4];
@@ -248,14 +255,13 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #pragma unroll
                     for (int u = 0; u < 4; ++u) {
                         const int q = q0 + u;
-                        const bool live = q < cend;
-                        const bool pd = live && ((m >> q) & 1u);
-                        const int2 oj = s_oj[live ? base + q : 0];
-                        const uint32_t *src = row32 + oj.x;
-                        jmq[u] = live ? oj.y : -1;
+                        const int2 oj = s_oj[base + q];
+                        const bool pd = (m >> q) & 1u;
+                        jmq[u] = (Lg < 4 && q >= Lg) ? -1 : oj.y;
+                        const int wi = rw + oj.x;
 #pragma unroll
                         for (int t = 0; t < CH; ++t)
-                            curq[u].v[t] = (pd && wok[t]) ? src[Lg * t] : 0xffffffffu;
+                            curq[u].v[t] = (pd && wok[t]) ? __ldg(tab32 + (wi + Lg * t)) : 0xffffffffu;
                     }
 #pragma unroll
                     for (int u = 0; u < 4; ++u) relax_prefix<EB, CH, JB>(curq[u], jmq[u], xl, Lg, lglog, ae, ao);
@@ -440,7 +446,7 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
     }
     const int NWk = g.nwords <= 1 ? 1 : 2;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (size_t)np * (8 + 8 * NWk) + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
+    const size_t smem = (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NWk + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     cudaError_t err;
     // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
