@@ -11,6 +11,8 @@
 //   a-6 OPT(N) read back with the planning summary in one 40-byte D2H.
 // Host syncs per DP: one after the config count (to size C), one at the end.
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -189,8 +191,19 @@ static int internal_order(const DpRequest &rq, std::vector<int> *order)
     return PTAS_OK;
 }
 
+static double trace_now()
+{
+    return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
 int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
 {
+    static const bool trace = [] {
+        const char *t = std::getenv("PTAS_TRACE");
+        return t && t[0] == '1';
+    }();
+    const double tr0 = trace ? trace_now() : 0;
+    double tr_enum = 0, tr_fillq = 0;
     DpOutcome o;
     cudaStream_t st = rq.stream ? rq.stream : stream_;
     std::vector<int> order;
@@ -320,6 +333,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     o.d2h += 8;
     o.launches += 2;
     const int64_t nC = h_scalar_[0];
+    if (trace) tr_enum = trace_now();
     if (nC <= 0) return PTAS_EINTERNAL;  // (0,..,0,1) is always feasible
     PT_CK(digits_.ensure((size_t)nC * K * 2));
     PT_CK(off_.ensure((size_t)nC * 8));
@@ -412,6 +426,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
         ++o.launches;
     }
     PT_CK(cudaEventRecord(ev_[2], st));
+    if (trace) tr_fillq = trace_now();
     o.launches += o.fill_launches;
     (void)ld;
 
@@ -431,6 +446,13 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     o.dp_s = ms * 1e-3;
     PT_CK(cudaEventElapsedTime(&ms, ev_[1], ev_[2]));
     o.fill_s = ms * 1e-3;
+    if (trace) {
+        const double t3 = trace_now();
+        std::fprintf(stderr, "[ptas] dp sigma=%lld K=%d levels=%d host: setup+enum-sync %.3f ms, fill enqueue %.3f ms, "
+                             "wait %.3f ms | device: dp %.3f ms fill %.3f ms\n",
+                     (long long)sigma, K, g.rho_max + 1, 1e3 * (tr_enum - tr0), 1e3 * (tr_fillq - tr_enum),
+                     1e3 * (t3 - tr_fillq), 1e3 * o.dp_s, 1e3 * o.fill_s);
+    }
     o.opt = h_meta_->opt;
     o.relax = (double)h_meta_->relax;
     o.nC = h_meta_->nC;
