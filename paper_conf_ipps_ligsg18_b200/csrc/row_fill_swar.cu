@@ -45,16 +45,25 @@ struct Words {
     uint32_t v[CH];
 };
 
-// Word k positions to the left of the lane's word of chunk t.  A row's words
-// are laid out as w = xl + Lg * t (lane xl of a group of Lg lanes, chunk t);
-// with k = qk * Lg + rk, word w - k lives in lane (xl - rk) mod Lg, chunk
-// t - qk (or t - qk - 1 when the lane index wraps).  Chunks before 0 are
-// outside the row and read as `fill`.
+// Lane geometry: a row is owned by a group of Lg lanes (any 1 <= Lg <= 32,
+// rows per warp = 32 / Lg, trailing lanes idle); lane xl of group grp holds
+// the row's words w = xl + Lg * t, t < CH.
+struct LaneMap {
+    int lane, Lg, grp, xl;
+};
+
+// Word k positions to the left of the lane's word of chunk t.  With
+// k = qk * Lg + rk, word w - k lives in lane (xl - rk) mod Lg of the same
+// group, chunk t - qk (or t - qk - 1 when the lane index wraps).  Chunks
+// before 0 are outside the row and read as `fill`.
 template <int CH>
-__device__ __forceinline__ uint32_t word_left(const Words<CH> &a, int t, int k, int xl, int Lg, int lglog,
-                                              uint32_t fill)
+__device__ __forceinline__ uint32_t word_left(const Words<CH> &a, int t, int k, const LaneMap &lm, uint32_t fill)
 {
-    const int qk = k >> lglog, rk = k & (Lg - 1);
+    int qk = 0, rk = k;
+    if (k >= lm.Lg) {
+        qk = k / lm.Lg;
+        rk = k - qk * lm.Lg;
+    }
     const int c1 = t - qk, c2 = c1 - 1;
     uint32_t v1 = fill, v2 = fill;
 #pragma unroll
@@ -63,8 +72,9 @@ __device__ __forceinline__ uint32_t word_left(const Words<CH> &a, int t, int k, 
         if (c == c2) v2 = a.v[c];
     }
     if (rk == 0) return v1;
-    const uint32_t send = (xl >= Lg - rk) ? v2 : v1;
-    return __shfl_sync(FULL, send, (xl - rk) & (Lg - 1), Lg);
+    const uint32_t send = (lm.xl >= lm.Lg - rk) ? v2 : v1;
+    const int src = lm.lane - rk + (lm.xl < rk ? lm.Lg : 0);
+    return __shfl_sync(FULL, send, src);
 }
 
 // acc <- min(acc, window of `lo:hi` at byte offset o) for one word position.
@@ -83,7 +93,7 @@ __device__ __forceinline__ void acc_window(uint32_t lo, uint32_t hi, int o, uint
 // JB > 0: shifts up to JB bytes, fully unrolled (jm * EB <= JB guaranteed by
 // the host); JB == 0: any shift (runtime loop, generic word fetch).
 template <int EB, int CH, int JB>
-__device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int xl, int Lg, int lglog,
+__device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, const LaneMap &lm,
                                              Words<CH> &ae, Words<CH> &ao)
 {
 #pragma unroll
@@ -91,11 +101,11 @@ __device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int x
     if (jm <= 0) return;
     Words<CH> w1, w2;
 #pragma unroll
-    for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur, t, 1, xl, Lg, lglog, 0xffffffffu);
+    for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur, t, 1, lm, 0xffffffffu);
     if (JB == 0 || JB > 4) {
         if (jm * EB > 4) {
 #pragma unroll
-            for (int t = 0; t < CH; ++t) w2.v[t] = word_left(cur, t, 2, xl, Lg, lglog, 0xffffffffu);
+            for (int t = 0; t < CH; ++t) w2.v[t] = word_left(cur, t, 2, lm, 0xffffffffu);
         }
     }
     if constexpr (JB > 0) {
@@ -123,8 +133,8 @@ __device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, int x
                 else if (db <= 8) acc_window<EB>(w2.v[t], w1.v[t], 8 - db, ae.v[t], ao.v[t]);
                 else {
                     const int k = (db + 3) >> 2;
-                    acc_window<EB>(word_left(cur, t, k, xl, Lg, lglog, 0xffffffffu),
-                                   word_left(cur, t, k - 1, xl, Lg, lglog, 0xffffffffu), 4 * k - db, ae.v[t], ao.v[t]);
+                    acc_window<EB>(word_left(cur, t, k, lm, 0xffffffffu), word_left(cur, t, k - 1, lm, 0xffffffffu),
+                                   4 * k - db, ae.v[t], ao.v[t]);
                 }
             }
         }
@@ -149,7 +159,7 @@ __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
-                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int lglog, int nsplit)
+                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int Lg, int nsplit)
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
@@ -179,10 +189,10 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     __syncthreads();
 
     const int lane = threadIdx.x & 31;
-    const int Lg = 1 << lglog;
-    const int grp = lane >> lglog;
-    const int xl = lane & (Lg - 1);
-    const int rpw = 32 >> lglog;
+    const int rpw = 32 / Lg;
+    const int grp = lane / Lg;          // grp >= rpw: idle lane
+    const int xl = lane - grp * Lg;
+    const LaneMap lm{lane, Lg, grp, xl};
     const unsigned gmask = Lg == 32 ? 0xffffffffu : ((1u << Lg) - 1u);
     // nsplit == 1: every warp owns its own rows.  nsplit > 1 (small row-levels):
     // the nsplit warps of a block share one set of rows, each walks every
@@ -203,25 +213,27 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     uint64_t npw[NW];
     {
         const int64_t slot = gw * rpw + grp;
+        const bool ok = grp < rpw && slot < slot_count;
 #pragma unroll
-        for (int w = 0; w < NW; ++w) npw[w] = slot < slot_count ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
-        if (slot < slot_count) nrb = rb[slot_begin + slot];
+        for (int w = 0; w < NW; ++w) npw[w] = ok ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
+        if (ok) nrb = rb[slot_begin + slot];
     }
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
     for (int64_t sb = gw * rpw; sb < slot_count; sb += nw * rpw) {
         {
             const int64_t slot = sb + grp;
-            const bool rowok = slot < slot_count;
+            const bool rowok = grp < rpw && slot < slot_count;
             int64_t rowbase = nrb;
             uint64_t pw[NW];
 #pragma unroll
             for (int w = 0; w < NW; ++w) pw[w] = npw[w];
             {   // prefetch the next row set's index entries
                 const int64_t ns = sb + nw * rpw + grp;
+                const bool ok = grp < rpw && ns < slot_count;
 #pragma unroll
-                for (int w = 0; w < NW; ++w) npw[w] = ns < slot_count ? pwa[(int64_t)w * pw_stride + slot_begin + ns] : 0;
-                nrb = ns < slot_count ? rb[slot_begin + ns] : 0;
+                for (int w = 0; w < NW; ++w) npw[w] = ok ? pwa[(int64_t)w * pw_stride + slot_begin + ns] : 0;
+                nrb = ok ? rb[slot_begin + ns] : 0;
             }
             // int32 word index of this lane's first word (the launcher guarantees < 2^31 words)
             const int rw = (int)(rowbase * EB / 4) + xl;
@@ -246,7 +258,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     for (int w = 0; w < NW; ++w)
                         dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
                 }
-                const unsigned m = (__ballot_sync(FULL, dom) >> (grp << lglog)) & gmask;
+                const unsigned bal = __ballot_sync(FULL, dom);
+                const unsigned m = grp < rpw ? (bal >> (grp * Lg)) & gmask : 0u;
                 const int cend = Lg < 4 ? Lg : ((np - base < Lg ? np - base : Lg) + 3) & ~3;
                 // 4 prefixes per step: their gathers are issued before any is consumed
                 for (int q0 = 0; q0 < cend; q0 += 4) {
@@ -264,7 +277,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                             curq[u].v[t] = (pd && wok[t]) ? __ldg(tab32 + (wi + Lg * t)) : 0xffffffffu;
                     }
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) relax_prefix<EB, CH, JB>(curq[u], jmq[u], xl, Lg, lglog, ae, ao);
+                    for (int u = 0; u < 4; ++u) relax_prefix<EB, CH, JB>(curq[u], jmq[u], lm, ae, ao);
                 }
             }
 
@@ -321,15 +334,15 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         if (JB == 0 && 2 * sa > 8) {
                             const int k = (2 * sa + 3) >> 2;
                             const Words<CH> &AA = odd ? oo : oe;
-                            plo = word_left(AA, t, k, xl, Lg, lglog, CFILL);
-                            phi = word_left(AA, t, k - 1, xl, Lg, lglog, CFILL);
+                            plo = word_left(AA, t, k, lm, CFILL);
+                            phi = word_left(AA, t, k - 1, lm, CFILL);
                             po = 4 * k - 2 * sa;
                         }
                         if (JB == 0 && 2 * sb > 8) {
                             const int k = (2 * sb + 3) >> 2;
                             const Words<CH> &BB = odd ? oe : oo;
-                            qlo = word_left(BB, t, k, xl, Lg, lglog, CFILL);
-                            qhi = word_left(BB, t, k - 1, xl, Lg, lglog, CFILL);
+                            qlo = word_left(BB, t, k, lm, CFILL);
+                            qhi = word_left(BB, t, k - 1, lm, CFILL);
                             qo = 4 * k - 2 * sb;
                         }
                         const uint32_t va = lane_shift(A0, A1, A2, 2 * sa, plo, phi, po);
@@ -341,8 +354,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         int po = 0;
                         if (JB == 0 && 2 * j > 8) {
                             const int k = (2 * j + 3) >> 2;
-                            plo = word_left(oe, t, k, xl, Lg, lglog, CFILL);
-                            phi = word_left(oe, t, k - 1, xl, Lg, lglog, CFILL);
+                            plo = word_left(oe, t, k, lm, CFILL);
+                            phi = word_left(oe, t, k - 1, lm, CFILL);
                             po = 4 * k - 2 * j;
                         }
                         const uint32_t va = lane_shift(oe.v[t], e1.v[t], e2.v[t], 2 * j, plo, phi, po);
@@ -358,16 +371,16 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 Words<CH> e1, o1, e2, o2;
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
-                    e1.v[t] = word_left(oe, t, 1, xl, Lg, lglog, CFILL);
-                    o1.v[t] = EB == 1 ? word_left(oo, t, 1, xl, Lg, lglog, CFILL) : 0u;
+                    e1.v[t] = word_left(oe, t, 1, lm, CFILL);
+                    o1.v[t] = EB == 1 ? word_left(oo, t, 1, lm, CFILL) : 0u;
                     e2.v[t] = e1.v[t];
                     o2.v[t] = o1.v[t];
                 }
                 if (chain_db > 4) {
 #pragma unroll
                     for (int t = 0; t < CH; ++t) {
-                        e2.v[t] = word_left(oe, t, 2, xl, Lg, lglog, CFILL);
-                        o2.v[t] = EB == 1 ? word_left(oo, t, 2, xl, Lg, lglog, CFILL) : 0u;
+                        e2.v[t] = word_left(oe, t, 2, lm, CFILL);
+                        o2.v[t] = EB == 1 ? word_left(oo, t, 2, lm, CFILL) : 0u;
                     }
                 }
                 Words<CH> ne = oe, no = oo;
@@ -420,18 +433,18 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
         for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
         if (rows_all * (int64_t)Lw >= ((int64_t)1 << 31)) return cudaErrorNotSupported;
     }
-    // words per lane (chunks, stride Lg): amortise the per-prefix cost over
-    // CH words; rows of <= 32 words use Lg = next_pow2(ceil(Lw / CH)).
+    // words per lane (chunks, stride Lg) and group width Lg (any 1..32):
+    // amortise the per-prefix cost over CH words while leaving few slots idle.
     int CH;
     const char *chs = std::getenv("PTAS_SWAR_CH");
     if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
     else if (chs && chs[0]) CH = std::atoi(chs);
     else CH = Lw >= 8 ? 2 : 1;
     if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
-    int lglog = 0;
-    while ((1 << lglog) * CH < Lw && lglog < 5) ++lglog;
-    if ((1 << lglog) * CH < Lw) return cudaErrorNotSupported;
-    const int rpw = 32 >> lglog;
+    int Lg = (Lw + CH - 1) / CH;
+    if (Lg < 1) Lg = 1;
+    if (Lg > 32) return cudaErrorNotSupported;
+    const int rpw = 32 / Lg;
     const int bs = 256;
     int64_t blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
     const int64_t cap = (int64_t)sm_count * 8;
@@ -471,7 +484,7 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
         cfg.attrs = attr;                                                                         \
         cfg.numAttrs = 1;                                                                         \
         err = cudaLaunchKernelEx(&cfg, kfn, (E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta,    \
-                                 J0, rho, slot_begin, slot_count, (E_ *)compact_out, lglog,       \
+                                 J0, rho, slot_begin, slot_count, (E_ *)compact_out, Lg,          \
                                  nsplit);                                                         \
         if (err != cudaSuccess) return err;                                                       \
     } while (0)

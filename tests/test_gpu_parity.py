@@ -181,6 +181,19 @@ def test_dp_fill_row_split_modes(P, monkeypatch, split):
     _check_table(P, np.array([30, 40, 300], np.int32), np.array([90, 70, 11], np.int64), 200)
 
 
+@pytest.mark.parametrize("ch", ["1", "2", "4", "8"])
+def test_dp_fill_lane_layouts(P, monkeypatch, ch):
+    # words per lane forced (group width Lg = ceil(words/CH), any value 1..32)
+    monkeypatch.setenv("PTAS_SWAR_CH", ch)
+    for W in (3, 5, 7, 13, 20, 29, 33, 61, 100, 127):
+        _check_table(P, np.array([3, 4, W - 1], np.int32), np.array([35, 50, 21], np.int64), 110)
+    rng = np.random.default_rng(int(ch))
+    for K in (4, 6):
+        for _ in range(3):
+            N, r, T = _rand_case(rng, K, {4: 12, 6: 6}[K])
+            _check_table(P, N, r, T)
+
+
 def test_dp_fill_very_long_rows(P):
     # rows longer than 1 KiB (uint16, W = 701) use the scalar kernel; W*e = 1024 B exactly uses 8 chunks
     _check_table(P, np.array([2, 700], np.int32), np.array([60, 13], np.int64), 120)
