@@ -201,8 +201,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     const int wid = threadIdx.x >> 5;
     const int64_t gw = nsplit > 1 ? (int64_t)blockIdx.x : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = nsplit > 1 ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int pbase0 = nsplit > 1 ? wid * Lg : 0;
-    const int pstep = nsplit > 1 ? nsplit * Lg : Lg;
+    const int pbase0 = nsplit > 1 ? wid * 32 : 0;
+    const int pstep = nsplit > 1 ? nsplit * 32 : 32;
     uint32_t *s_red = reinterpret_cast<uint32_t *>(s_w + (size_t)NW * np + 1);  // [warp][2][CH][32]
     const int Lw = (int)(g.Wp * EB / 4);  // words per (padded) row
     uint64_t guard[NW];
@@ -250,17 +250,22 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 ao.v[t] = 0xffffffffu;
             }
             for (int base = pbase0; base < np; base += pstep) {
-                const int c = base + xl;
-                bool dom = false;
-                if (rowok && c < np) {
-                    dom = true;
+                // dominance mask of prefixes base .. base+31 for this group's row:
+                // lane xl tests base + xl + k*Lg, ceil(32/Lg) ballots
+                unsigned m = 0;
+                for (int k0 = 0; k0 < 32; k0 += Lg) {
+                    const int c = base + k0 + xl;
+                    bool dom = false;
+                    if (rowok && xl + k0 < 32 && c < np) {
+                        dom = true;
 #pragma unroll
-                    for (int w = 0; w < NW; ++w)
-                        dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
+                        for (int w = 0; w < NW; ++w)
+                            dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
+                    }
+                    const unsigned bal = __ballot_sync(FULL, dom);
+                    if (grp < rpw) m |= ((bal >> (grp * Lg)) & gmask) << k0;
                 }
-                const unsigned bal = __ballot_sync(FULL, dom);
-                const unsigned m = grp < rpw ? (bal >> (grp * Lg)) & gmask : 0u;
-                const int cend = Lg < 4 ? Lg : ((np - base < Lg ? np - base : Lg) + 3) & ~3;
+                const int cend = ((np - base < 32 ? np - base : 32) + 3) & ~3;
                 // 4 prefixes per step: their gathers are issued before any is consumed
                 for (int q0 = 0; q0 < cend; q0 += 4) {
                     Words<CH> curq[4];
@@ -270,7 +275,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         const int q = q0 + u;
                         const int2 oj = s_oj[base + q];
                         const bool pd = (m >> q) & 1u;
-                        jmq[u] = (Lg < 4 && q >= Lg) ? -1 : oj.y;
+                        jmq[u] = oj.y;
                         const int wi = rw + oj.x;
 #pragma unroll
                         for (int t = 0; t < CH; ++t)
