@@ -69,6 +69,9 @@ typedef struct {
     int32_t layout;             /* 0 = internal class order chosen by the library
                                    (largest count fastest); 1 = classes in
                                    ascending-size order as classified             */
+    void *stream;               /* cudaStream_t for all device work of the call
+                                   (NULL = the library's own stream); the call
+                                   still returns only when its work is done       */
 } ptas_options;
 
 typedef struct {

@@ -26,7 +26,7 @@ vp = ctypes.c_void_p
 class PtasOptions(ctypes.Structure):
     _fields_ = [("probes_per_round", ctypes.c_int32), ("mode", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("comm", vp), ("table_budget_bytes", ctypes.c_int64), ("memoize", ctypes.c_int32),
-                ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32)]
+                ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32), ("stream", vp)]
 
 
 class PtasStats(ctypes.Structure):

@@ -37,6 +37,10 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objdir = os.path.join(HERE, "build")
     os.makedirs(objdir, exist_ok=True)
     hdr_t = max(os.path.getmtime(h) for h in _headers())
+    # stale objects of removed sources must not be linked
+    for o in glob.glob(os.path.join(objdir, "*.o")):
+        if os.path.basename(o)[:-2] not in {os.path.basename(x) for x in sources()}:
+            os.remove(o)
     flags = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I" + os.path.join(ROOT, "include")]
     if verbose:
         flags.append("-Xptxas=-v")
@@ -53,8 +57,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
         os.replace(tmp, obj)
         return obj
 
+    srcs = sorted(sources(), key=lambda x: -os.path.getsize(x))
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
-        objs = list(ex.map(compile_one, sources()))
+        objs = list(ex.map(compile_one, srcs))
     tmp = LIB + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-Xcompiler", "-fPIC", "-o", tmp, *objs, "-ldl"])
     os.replace(tmp, LIB)

@@ -86,6 +86,16 @@ cudaError_t Engine::sync_spin(cudaStream_t st)
     }
 }
 
+cudaError_t Engine::h2d(void *dst, const void *src, size_t bytes, cudaStream_t st)
+{
+    const size_t need = (pin_used_ + bytes + 255) & ~(size_t)255;
+    if (need > pin_cap_) return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, st);
+    unsigned char *h = pin_ + pin_used_;
+    std::memcpy(h, src, bytes);
+    pin_used_ = need;
+    return cudaMemcpyAsync(dst, h, bytes, cudaMemcpyHostToDevice, st);
+}
+
 int Engine::init(int device)
 {
     device_ = device;
@@ -97,6 +107,8 @@ int Engine::init(int device)
     PT_CK(cudaMalloc(&d_meta_, sizeof(DpMeta)));
     PT_CK(cudaMallocHost(&h_meta_, sizeof(DpMeta)));
     PT_CK(cudaMallocHost(&h_scalar_, 64));
+    pin_cap_ = (size_t)8 << 20;
+    PT_CK(cudaMallocHost((void **)&pin_, pin_cap_));
     return PTAS_OK;
 }
 
@@ -297,10 +309,10 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     for (int rho = 0; rho <= g.rho_max; ++rho) lstart[rho + 1] = lstart[rho] + cnt[rho];
     const size_t cnt_words = cnt.size() + lstart.size();
     PT_CK(cnt_.ensure(cnt_words * 8));
-    PT_CK(cudaMemcpyAsync(small_.p, small.data(), small_bytes, cudaMemcpyHostToDevice, st));
-    PT_CK(cudaMemcpyAsync(cnt_.p, cnt.data(), cnt.size() * 8, cudaMemcpyHostToDevice, st));
-    PT_CK(cudaMemcpyAsync((int64_t *)cnt_.p + cnt.size(), lstart.data(), lstart.size() * 8,
-                          cudaMemcpyHostToDevice, st));
+    pin_reset();
+    PT_CK(h2d(small_.p, small.data(), small_bytes, st));
+    PT_CK(h2d(cnt_.p, cnt.data(), cnt.size() * 8, st));
+    PT_CK(h2d((int64_t *)cnt_.p + cnt.size(), lstart.data(), lstart.size() * 8, st));
     o.h2d += (int64_t)(small_bytes + cnt_words * 8);
     // ---- a-4 level-ordered row index (row base + packed leading digits per row)
     const int NWk = g.nwords <= 1 ? 1 : 2;
@@ -343,6 +355,13 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     PT_CK(launch_build_prefix(K, (const uint16_t *)digits_.p, (const int64_t *)off_.p, nC, g,
                               N.data(), (PrefixEntry *)pref_.p, d_meta_, st));
     o.launches += 2;
+    // prefix offsets into the packed kernel's constant bank
+    PT_CK(cpstage_.ensure(const_prefix_staging_bytes()));
+    cudaError_t cpe = prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nC, e, g.nwords, cpstage_.p, st);
+    const char *ncp = std::getenv("PTAS_NO_CPREF");
+    const int cpref_ok = (cpe == cudaSuccess && !(ncp && ncp[0] == '1')) ? 1 : 0;
+    if (cpe != cudaSuccess && cpe != cudaErrorNotSupported) PT_CK(cpe);
+    ++o.launches;
     const int J0 = (int)std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
     const char *fs = std::getenv("PTAS_FORCE_SCALAR");
     const bool force_scalar = fs && fs[0] == '1';
@@ -357,7 +376,8 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
         cudaError_t err = cudaErrorNotSupported;
         if (!force_scalar) {
             err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC,
-                                       j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0);
+                                       j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0,
+                                       cpref_ok);
             if (err == cudaSuccess) prev_fill = true;
         }
         if (err == cudaErrorNotSupported) {
@@ -506,9 +526,10 @@ int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
     int32_t *d_N = d_rank + nC;
     int32_t *d_len = d_N + K;
     int32_t *d_out = d_len + 4;
-    PT_CK(cudaMemcpyAsync(d_stride, last_stride_.data(), (size_t)K * 8, cudaMemcpyHostToDevice, st));
-    PT_CK(cudaMemcpyAsync(d_rank, rank.data(), (size_t)nC * 4, cudaMemcpyHostToDevice, st));
-    PT_CK(cudaMemcpyAsync(d_N, last_N_.data(), (size_t)K * 4, cudaMemcpyHostToDevice, st));
+    pin_reset();
+    PT_CK(h2d(d_stride, last_stride_.data(), (size_t)K * 8, st));
+    PT_CK(h2d(d_rank, rank.data(), (size_t)nC * 4, st));
+    PT_CK(h2d(d_N, last_N_.data(), (size_t)K * 4, st));
     PT_CK(cudaMemsetAsync(&d_meta_->err, 0, 4, st));
     acc->h2d += (int64_t)(K * 8 + nC * 4 + K * 4);
     PT_CK(launch_traceback(last_e_, last_table_, K, d_N, d_stride, (const uint16_t *)digits_.p,

@@ -69,6 +69,11 @@ class Engine {
     int device() const { return device_; }
 
     cudaError_t sync_spin(cudaStream_t st);
+    // Host<->device copies of small host vectors through a pinned arena (no
+    // pageable bounce buffers in the driver); the arena is reset per DP, after
+    // the previous DP's final sync.
+    cudaError_t h2d(void *dst, const void *src, size_t bytes, cudaStream_t st);
+    void pin_reset() { pin_used_ = 0; }
 
   private:
     int init(int device);
@@ -85,7 +90,9 @@ class Engine {
     DpMeta *d_meta_ = nullptr;
     DpMeta *h_meta_ = nullptr;     // pinned
     int64_t *h_scalar_ = nullptr;  // pinned
-    Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_, rowidx_;
+    unsigned char *pin_ = nullptr;  // pinned arena
+    size_t pin_cap_ = 0, pin_used_ = 0;
+    Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_, rowidx_, cpstage_;
 
     // state of the last DP (for traceback)
     bool last_valid_ = false;

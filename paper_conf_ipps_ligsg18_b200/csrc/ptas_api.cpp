@@ -251,6 +251,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         rq.order = order.data();
         rq.shard = s;
         rq.budget = opt.table_budget_bytes;
+        rq.stream = (cudaStream_t)opt.stream;
         DpOutcome o;
         int r2 = eng->run_dp(rq, &o);
         if (r2) return r2;
@@ -306,7 +307,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             if (rank < np) mine[0] = optj[rank];
             int32_t *dbuf = nullptr;
             if (cudaMalloc(&dbuf, sizeof(int32_t) * world) != cudaSuccess) return PTAS_ENOMEM;
-            cudaStream_t st = eng->stream();
+            cudaStream_t st = opt.stream ? (cudaStream_t)opt.stream : eng->stream();
             cudaMemcpyAsync(dbuf + rank, mine.data(), 4, cudaMemcpyHostToDevice, st);
             int crc = comm_allgather(opt.comm, dbuf + rank, dbuf, 4, st);
             cudaMemcpyAsync(all.data(), dbuf, 4 * world, cudaMemcpyDeviceToHost, st);
@@ -439,6 +440,7 @@ void ptas_default_options(ptas_options *o)
     o->memoize = 1;
     o->virtual_shards = 1;
     o->layout = 0;
+    o->stream = nullptr;
 }
 
 const char *ptas_strerror(int s)
@@ -536,7 +538,7 @@ int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps, cons
     std::vector<int32_t> ha(n);
     {
         std::lock_guard<std::mutex> lk(eng->mu);
-        cudaStream_t st = eng->stream();
+        cudaStream_t st = (opt && opt->stream) ? (cudaStream_t)opt->stream : eng->stream();
         if (cudaMemcpyAsync(hp.data(), d_p, (size_t)n * 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
             eng->sync_spin(st) != cudaSuccess) {
             cudaGetLastError();
@@ -547,7 +549,7 @@ int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps, cons
                     (int64_t)n * 4, (int64_t)n * 8);
     if (rc) return rc;
     std::lock_guard<std::mutex> lk(eng->mu);
-    cudaStream_t st = eng->stream();
+    cudaStream_t st = (opt && opt->stream) ? (cudaStream_t)opt->stream : eng->stream();
     if (cudaMemcpyAsync(d_assignment, ha.data(), (size_t)n * 4, cudaMemcpyHostToDevice, st) != cudaSuccess ||
         eng->sync_spin(st) != cudaSuccess) {
         cudaGetLastError();
