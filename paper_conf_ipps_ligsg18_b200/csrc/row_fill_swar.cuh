@@ -516,7 +516,9 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     if (blocks > cap) blocks = cap;
     // small row-levels: split each row set's prefixes over the 8 warps of a block
     const char *sp = std::getenv("PTAS_SPLIT_ROWS");
-    const int64_t split_rows = sp ? std::atoll(sp) : (int64_t)sm_count * rpw * 2;
+    // (prefix batches are 32 wide: splitting pays only with several batches)
+    const int64_t np_ = nP_bound > 1 ? nP_bound - 1 : 0;
+    const int64_t split_rows = sp ? std::atoll(sp) : (np_ >= 128 ? (int64_t)sm_count * rpw * 2 : 0);
     int nsplit = 1;
     if (slot_count <= split_rows) {
         nsplit = bs / 32;
@@ -530,7 +532,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
     const int need = e == 1 ? ((J0 + 1) / 2 * 2 > J0 ? (J0 + 1) / 2 * 2 : J0) : 2 * J0;
     const int JBsel = need <= 4 ? 4 : (need <= 8 ? 8 : 0);
-    const bool cpref = np <= CP_MAX && cpref_ok;
+    const bool cpref = np <= CP_MAX && cpref_ok && np >= 64;
 #define PTAS_SWAR_JB(E_, NW_, CH_, JB_)                                                           \
     do {                                                                                          \
         auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, JB_, true, true>      \
