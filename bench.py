@@ -149,6 +149,13 @@ def cpu_oracle_sample(w, target_relax=2.0e9):
                       f"(full N={list(map(int, N))}); {relax:.3g} relaxations in {dt:.2f} s, 1 core"}
 
 
+def _config(w, **extra):
+    c = {"workload": w.name, "n": w.n, "m": w.m, "eps": w.eps, "P_jobs": w.P, "seed": w.seed,
+         "generator": "numpy default_rng(seed).integers(1, P_jobs, n, endpoint=True)"}
+    c.update(extra)
+    return c
+
+
 def run_reference(args, w):
     rank, _local, world = _dist_env()
     if rank != 0:
@@ -172,8 +179,8 @@ def run_reference(args, w):
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
-            "data": "synthetic", "config": {"workload": w.name, "n": w.n, "m": w.m, "eps": w.eps, "P": w.P,
-                                            "seed": w.seed},
+            "data": "synthetic", "config": _config(w, probes_per_round=1, mode="single",
+                                                   l2="flushed between steps (256 MiB write)"),
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
             "gpu_launches": 0}
@@ -285,11 +292,11 @@ def run_ours(args, w):
         "higher_is_better": True,
         "scaling": "strong" if (world > 1 and mode == P.MODE_LEVEL_SHARDED) else "weak",
         "vs_baseline": None, "dtype": args.dtype_label or "u8", "data": "synthetic",
-        "config": {"workload": w.name, "n": w.n, "m": w.m, "eps": w.eps, "P_jobs": w.P, "seed": w.seed,
-                   "probes_per_round": Pp, "mode": {0: "single", 1: "level_sharded", 2: "multi_probe"}[mode],
-                   "probes": st0["probes"], "unique_dps": st0["unique_dps"], "T_star": st0["T_star"],
-                   "sigma_max": st0["sigma_max"], "relax_per_step": relax_total / args.steps,
-                   "l2": "flushed between steps (256 MiB write)"},
+        "config": _config(w, probes_per_round=Pp,
+                          mode={0: "single", 1: "level_sharded", 2: "multi_probe"}[mode],
+                          l2="flushed between steps (256 MiB write)"),
+        "solve": {"probes": st0["probes"], "unique_dps": st0["unique_dps"], "T_star": st0["T_star"],
+                  "sigma_max": st0["sigma_max"], "relax_per_step": relax_total / args.steps},
         "solve_ms": 1e3 * t_total / args.steps,
         "solve_ms_median": statistics.median(dev_ms),
         "e2e": {"value": e2e_relax / e2e_t, "unit": UNIT,
@@ -298,7 +305,7 @@ def run_ours(args, w):
                 "solve_ms": 1e3 * e2e_t / args.steps},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "traffic_note": traffic_note,
-                     "kernel": "row_fill_kernel (level fill)",
+                     "kernel": "row_fill_swar_kernel (level fill, §8(a) a-5)",
                      "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)" if peak_kind == "measured" else "fallback",
                      "fill_ms_per_step": 1e3 * fill_s / args.steps,
                      "fill_launches_per_step": fill_launches / args.steps,
