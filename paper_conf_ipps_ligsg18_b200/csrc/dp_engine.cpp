@@ -32,7 +32,7 @@ namespace ptas {
         }                                                                          \
     } while (0)
 
-cudaError_t Engine::Buf::ensure(size_t bytes)
+cudaError_t DpSlot::Buf::ensure(size_t bytes)
 {
     if (p && bytes <= cap) return cudaSuccess;
     if (p) {
@@ -76,7 +76,7 @@ int Engine::get(int device, Engine **out)
 
 // The host driver waits for small readbacks many times per solve; a spin on
 // an event query avoids the scheduler wake-up latency of a blocking sync.
-cudaError_t Engine::sync_spin(cudaStream_t st)
+cudaError_t DpSlot::sync_spin(cudaStream_t st)
 {
     cudaError_t e = cudaEventRecord(ev_sync_, st);
     if (e != cudaSuccess) return e;
@@ -86,7 +86,7 @@ cudaError_t Engine::sync_spin(cudaStream_t st)
     }
 }
 
-cudaError_t Engine::h2d(void *dst, const void *src, size_t bytes, cudaStream_t st)
+cudaError_t DpSlot::h2d(void *dst, const void *src, size_t bytes, cudaStream_t st)
 {
     const size_t need = (pin_used_ + bytes + 255) & ~(size_t)255;
     if (need > pin_cap_) return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, st);
@@ -101,6 +101,32 @@ int Engine::init(int device)
     device_ = device;
     PT_CK(cudaSetDevice(device));
     PT_CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device));
+    DpSlot *s = nullptr;
+    return slot(0, &s);
+}
+
+int Engine::slot(int i, DpSlot **out)
+{
+    if (i < 0 || i >= MAX_SLOTS) return PTAS_EINVAL;
+    if (!slots_[i]) {
+        DpSlot *s = new DpSlot();
+        int rc = s->init(device_, sm_count_, i);
+        if (rc) {
+            delete s;
+            return rc;
+        }
+        slots_[i] = s;
+    }
+    *out = slots_[i];
+    return PTAS_OK;
+}
+
+int DpSlot::init(int device, int sm_count, int index)
+{
+    device_ = device;
+    sm_count_ = sm_count;
+    index_ = index;
+    PT_CK(cudaSetDevice(device));
     PT_CK(cudaStreamCreateWithFlags(&stream_, cudaStreamNonBlocking));
     for (auto &ev : ev_) PT_CK(cudaEventCreate(&ev));
     PT_CK(cudaEventCreateWithFlags(&ev_sync_, cudaEventDisableTiming));
@@ -112,7 +138,7 @@ int Engine::init(int device)
     return PTAS_OK;
 }
 
-int64_t Engine::free_budget()
+int64_t DpSlot::free_budget()
 {
     size_t fr = 0, tot = 0;
     if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) {
@@ -208,7 +234,7 @@ static double trace_now()
     return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
 
-int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
+int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
 {
     static const bool trace = [] {
         const char *t = std::getenv("PTAS_TRACE");
@@ -357,7 +383,9 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     o.launches += 2;
     // prefix offsets into the packed kernel's constant bank
     PT_CK(cpstage_.ensure(const_prefix_staging_bytes()));
-    cudaError_t cpe = prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nC, e, g.nwords, cpstage_.p, st);
+    cudaError_t cpe = index_ < 4 ? prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nC, e, g.nwords, index_,
+                                                   cpstage_.p, st)
+                                : cudaErrorNotSupported;
     const char *ncp = std::getenv("PTAS_NO_CPREF");
     const int cpref_ok = (cpe == cudaSuccess && !(ncp && ncp[0] == '1')) ? 1 : 0;
     if (cpe != cudaSuccess && cpe != cudaErrorNotSupported) PT_CK(cpe);
@@ -377,7 +405,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
         if (!force_scalar) {
             err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC,
                                        j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0,
-                                       cpref_ok);
+                                       cpref_ok ? index_ : -1);
             if (err == cudaSuccess) prev_fill = true;
         }
         if (err == cudaErrorNotSupported) {
@@ -498,7 +526,7 @@ int Engine::run_dp(const DpRequest &rq, DpOutcome *out)
     return PTAS_OK;
 }
 
-int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
+int DpSlot::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
 {
     if (!last_valid_) return PTAS_EINTERNAL;
     if (last_K_ == 0 || last_opt_ == 0) return PTAS_OK;
@@ -549,7 +577,7 @@ int Engine::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
     return PTAS_OK;
 }
 
-int Engine::copy_table_to_host(void *dst, int64_t bytes)
+int DpSlot::copy_table_to_host(void *dst, int64_t bytes)
 {
     if (!last_valid_) return PTAS_EINTERNAL;
     const void *src = last_table_;
@@ -564,7 +592,7 @@ int Engine::copy_table_to_host(void *dst, int64_t bytes)
     return PTAS_OK;
 }
 
-int Engine::configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits, int64_t *count)
+int DpSlot::configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits, int64_t *count)
 {
     // Runs a full DP on an engine-owned table is unnecessary: enumerate only.
     std::vector<int> order;
@@ -627,7 +655,7 @@ int Engine::configs_canonical(const DpRequest &rq, std::vector<int32_t> *digits,
     return PTAS_OK;
 }
 
-int Engine::row_index(const int32_t *Nc, int Kc, std::vector<int64_t> *level_start,
+int DpSlot::row_index(const int32_t *Nc, int Kc, std::vector<int64_t> *level_start,
                       std::vector<int64_t> *rowbase)
 {
     std::vector<int32_t> N;

@@ -49,11 +49,12 @@ struct DpOutcome {
 // one machine of the traceback: canonical digit vector s (length K canonical)
 using MachineCfg = std::vector<int32_t>;
 
-class Engine {
+// All per-DP device state: workspace buffers, stream, events, readback
+// buffers, and the description of the last DP (for traceback).  Several slots
+// run DPs concurrently (one host thread each) for the probes of one round.
+class DpSlot {
   public:
-    static int get(int device, Engine **out);
-    std::mutex mu;
-
+    int init(int device, int sm_count, int index);
     int run_dp(const DpRequest &rq, DpOutcome *out);
     // Traceback on the table of the last run_dp (engine-owned or the same
     // ext table); appends OPT(N) canonical configurations to machines.
@@ -66,7 +67,7 @@ class Engine {
     // D2H of the table of the last run_dp (engine-owned or ext).
     int copy_table_to_host(void *dst, int64_t bytes);
     cudaStream_t stream() const { return stream_; }
-    int device() const { return device_; }
+    bool last_valid() const { return last_valid_; }
 
     cudaError_t sync_spin(cudaStream_t st);
     // Host<->device copies of small host vectors through a pinned arena (no
@@ -76,7 +77,6 @@ class Engine {
     void pin_reset() { pin_used_ = 0; }
 
   private:
-    int init(int device);
     struct Buf {
         void *p = nullptr;
         size_t cap = 0;
@@ -84,6 +84,7 @@ class Engine {
     };
     int device_ = -1;
     int sm_count_ = 148;
+    int index_ = 0;  // slot index; constant-bank prefix area when < 4
     cudaStream_t stream_ = nullptr;
     cudaEvent_t ev_[4] = {nullptr, nullptr, nullptr, nullptr};
     cudaEvent_t ev_sync_ = nullptr;
@@ -105,6 +106,40 @@ class Engine {
     std::vector<int> last_order_;      // internal -> canonical
     std::vector<int32_t> last_N_;      // internal counts
     std::vector<int64_t> last_stride_; // internal strides
+};
+
+constexpr int MAX_SLOTS = 8;
+
+// Per-device engine: a lock serialising API calls on the device and up to
+// MAX_SLOTS DP slots.  Slot 0 serves every single-DP call.
+class Engine {
+  public:
+    static int get(int device, Engine **out);
+    std::mutex mu;
+    int device() const { return device_; }
+    int sm_count() const { return sm_count_; }
+    int slot(int i, DpSlot **out);
+    DpSlot *s0() { return slots_[0]; }
+    // forwards to slot 0
+    int run_dp(const DpRequest &rq, DpOutcome *out) { return slots_[0]->run_dp(rq, out); }
+    int traceback(std::vector<MachineCfg> *m, DpOutcome *acc) { return slots_[0]->traceback(m, acc); }
+    int configs_canonical(const DpRequest &rq, std::vector<int32_t> *d, int64_t *c)
+    {
+        return slots_[0]->configs_canonical(rq, d, c);
+    }
+    int row_index(const int32_t *N, int K, std::vector<int64_t> *ls, std::vector<int64_t> *rb)
+    {
+        return slots_[0]->row_index(N, K, ls, rb);
+    }
+    int copy_table_to_host(void *dst, int64_t bytes) { return slots_[0]->copy_table_to_host(dst, bytes); }
+    cudaStream_t stream() const { return slots_[0]->stream(); }
+    cudaError_t sync_spin(cudaStream_t st) { return slots_[0]->sync_spin(st); }
+
+  private:
+    int init(int device);
+    int device_ = -1;
+    int sm_count_ = 148;
+    DpSlot *slots_[MAX_SLOTS] = {};
 };
 
 // NCCL glue (comm.cpp)

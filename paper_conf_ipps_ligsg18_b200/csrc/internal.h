@@ -91,12 +91,12 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
                                  const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
                                  int J0, int rho, int64_t slot_begin, int64_t slot_count,
                                  void *compact_out, int sm_count, cudaStream_t st, int pdl,
-                                 int cpref_ok);
+                                 int cslot);
 // Copies the DP's prefix offsets/Jmax into the fill kernel's constant bank
 // (after build_prefix, before the fill loop); cudaErrorNotSupported when the
 // prefix list is too long (the kernels then read it from shared memory).
 cudaError_t prepare_const_prefix(const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound, int e,
-                                 int nwords, void *d_staging, cudaStream_t st);
+                                 int nwords, int cslot, void *d_staging, cudaStream_t st);
 size_t const_prefix_staging_bytes();
 // Copy rows of pitch Wp (src) to pitch W (dst), `rows` rows of e-byte entries.
 cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows, int64_t W,

@@ -7,10 +7,12 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <map>
 #include <queue>
+#include <thread>
 #include <vector>
 
 #include "engine.h"
@@ -235,14 +237,14 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     acc.s.h2d_bytes += extra_h2d;
     acc.s.d2h_bytes += extra_d2h;
     std::map<std::vector<int64_t>, int32_t> memo;
-    std::vector<int64_t> table_key;
-    bool table_valid = false;
     std::vector<ptas_probe> plog;
     int round = 0;
     Classified cl;
 
-    auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
-        std::vector<int> order = choose_order(c.N, opt.layout);
+    // which slot holds the table of which DP key (for the traceback at T*)
+    std::vector<std::vector<int64_t>> slot_key(MAX_SLOTS);
+    auto make_rq = [&](const Classified &c, int64_t T, const ShardCtx *s, const std::vector<int> &order,
+                       cudaStream_t st) {
         DpRequest rq;
         rq.K = (int)c.N.size();
         rq.N = c.N.data();
@@ -251,13 +253,61 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         rq.order = order.data();
         rq.shard = s;
         rq.budget = opt.table_budget_bytes;
-        rq.stream = (cudaStream_t)opt.stream;
+        rq.stream = st;
+        return rq;
+    };
+    auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
+        std::vector<int> order = choose_order(c.N, opt.layout);
+        DpRequest rq = make_rq(c, T, s, order, (cudaStream_t)opt.stream);
         DpOutcome o;
         int r2 = eng->run_dp(rq, &o);
         if (r2) return r2;
         acc.add(o);
         acc.s.unique_dps++;
         *opt_out = o.opt;
+        return PTAS_OK;
+    };
+    // Concurrent evaluation of several probes of one round (SINGLE mode): one
+    // host thread and one DP slot (own stream and workspace) per probe -- the
+    // quarter split of Alg 3 on one GPU.  With a caller
+    // stream, slot 0 uses it; the call is host-synchronous either way.
+    const char *ncs = std::getenv("PTAS_NO_CONCURRENT");
+    const bool concurrent = opt.mode == PTAS_MODE_SINGLE && !(ncs && ncs[0] == '1');
+    auto run_many = [&](std::vector<Classified> &cls_v, std::vector<int64_t> &T_v,
+                        std::vector<std::vector<int64_t>> &key_v, std::vector<int32_t> &opt_v) -> int {
+        const int nj = (int)cls_v.size();
+        for (int j0 = 0; j0 < nj; j0 += MAX_SLOTS) {
+            const int nb = std::min(MAX_SLOTS, nj - j0);
+            std::vector<DpSlot *> sl(nb);
+            for (int b = 0; b < nb; ++b) {
+                int r2 = eng->slot(b, &sl[b]);
+                if (r2) return r2;
+            }
+            std::vector<DpOutcome> outs(nb);
+            std::vector<int> rcs(nb, PTAS_OK);
+            std::vector<std::vector<int>> orders(nb);
+            for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, opt.layout);
+            auto work = [&](int b) {
+                if (cudaSetDevice(dev) != cudaSuccess) {
+                    rcs[b] = PTAS_ECUDA;
+                    return;
+                }
+                DpRequest rq = make_rq(cls_v[j0 + b], T_v[j0 + b], nullptr, orders[b],
+                                       b == 0 ? (cudaStream_t)opt.stream : nullptr);
+                rcs[b] = sl[b]->run_dp(rq, &outs[b]);
+            };
+            std::vector<std::thread> th;
+            for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
+            work(0);
+            for (auto &t : th) t.join();
+            for (int b = 0; b < nb; ++b) {
+                if (rcs[b]) return rcs[b];
+                acc.add(outs[b]);
+                acc.s.unique_dps++;
+                opt_v[j0 + b] = outs[b].opt;
+                slot_key[b] = key_v[j0 + b];
+            }
+        }
         return PTAS_OK;
     };
 
@@ -268,6 +318,11 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         std::vector<int32_t> optj(np, 0), hit(np, 0), who(np, 0), Kj(np, 0);
         std::vector<int64_t> sgj(np, 1);
         std::vector<std::vector<int64_t>> keys(np);
+        std::vector<int> pend_q;
+        std::vector<Classified> pend_cl;
+        std::vector<int64_t> pend_T;
+        std::vector<std::vector<int64_t>> pend_key;
+        std::vector<std::pair<int, int>> pend_alias;  // probe -> pending job
         for (int q = 0; q < np; ++q) {
             classify(p, n, Tj[q], k, &cl);
             Kj[q] = (int32_t)cl.N.size();
@@ -295,11 +350,36 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 optj[q] = -1;  // filled by the exchange
                 continue;
             }
+            if (concurrent) {
+                // deferred: evaluated below with the round's other probes
+                bool dup = false;
+                for (size_t jj = 0; jj < pend_key.size(); ++jj)
+                    if (pend_key[jj] == keys[q]) {
+                        pend_alias.push_back({q, (int)jj});
+                        dup = true;
+                        break;
+                    }
+                if (!dup) {
+                    pend_q.push_back(q);
+                    pend_cl.push_back(cl);
+                    pend_T.push_back(Tj[q]);
+                    pend_key.push_back(keys[q]);
+                    pend_alias.push_back({q, (int)pend_key.size() - 1});
+                }
+                continue;
+            }
             rc = run(cl, Tj[q], opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, &optj[q]);
             if (rc) return rc;
-            table_key = keys[q];
-            table_valid = true;
+            slot_key[0] = keys[q];
             if (opt.memoize) memo[keys[q]] = optj[q];
+        }
+        if (!pend_q.empty()) {
+            std::vector<int32_t> pend_opt(pend_q.size(), 0);
+            rc = run_many(pend_cl, pend_T, pend_key, pend_opt);
+            if (rc) return rc;
+            for (auto &qa : pend_alias) optj[qa.first] = pend_opt[qa.second];
+            if (opt.memoize)
+                for (size_t jj = 0; jj < pend_key.size(); ++jj) memo[pend_key[jj]] = pend_opt[jj];
         }
         if (opt.mode == PTAS_MODE_MULTI_PROBE) {
             // exchange OPT(N) of every rank's probe (int32 per rank) over NCCL
@@ -350,13 +430,23 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     int32_t opt_star = 0;
     if (!cl.N.empty()) {
         std::vector<int64_t> key = memo_key(cl, Ts);
-        if (!table_valid || key != table_key) {
+        int tslot = -1;
+        for (int b = 0; b < MAX_SLOTS; ++b)
+            if (slot_key[b] == key) {
+                tslot = b;
+                break;
+            }
+        if (tslot < 0) {
             rc = run(cl, Ts, opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, &opt_star);
             if (rc) return rc;
+            tslot = 0;
         }
+        DpSlot *tsl = nullptr;
+        rc = eng->slot(tslot, &tsl);
+        if (rc) return rc;
         std::vector<MachineCfg> machines;
         DpOutcome tb;
-        rc = eng->traceback(&machines, &tb);
+        rc = tsl->traceback(&machines, &tb);
         if (rc) return rc;
         acc.s.kernel_launches += tb.launches;
         acc.s.h2d_bytes += tb.h2d;

@@ -33,9 +33,9 @@ namespace ptas {
                                            const PrefixEntry *d_pref, const DpMeta *d_meta,               \
                                            int64_t nP_bound, int J0, int rho, int64_t slot_begin,         \
                                            int64_t slot_count, void *compact_out, int sm_count,           \
-                                           cudaStream_t st, int pdl, int cpref_ok);                       \
+                                           cudaStream_t st, int pdl, int cslot);                       \
     cudaError_t prepare_const_prefix_##tag(const PrefixEntry *d_pref, const DpMeta *d_meta,             \
-                                           int64_t nP_bound, int e, void *d_staging, cudaStream_t st);
+                                           int64_t nP_bound, int e, int cslot, void *d_staging, cudaStream_t st);
 PTAS_SWAR_DECL(u8_nw1)
 PTAS_SWAR_DECL(u8_nw2)
 PTAS_SWAR_DECL(u16_nw1)
@@ -45,12 +45,12 @@ PTAS_SWAR_DECL(u16_nw2)
 cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
                                  int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
                                  int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
-                                 void *compact_out, int sm_count, cudaStream_t st, int pdl, int cpref_ok)
+                                 void *compact_out, int sm_count, cudaStream_t st, int pdl, int cslot)
 {
     const bool two = g.nwords > 1;
 #define PTAS_SWAR_CALL(tag)                                                                             \
     return launch_row_fill_swar_##tag(e, table, g, rb, pw, pw_stride, d_pref, d_meta, nP_bound, J0, rho,     \
-                                      slot_begin, slot_count, compact_out, sm_count, st, pdl, cpref_ok)
+                                      slot_begin, slot_count, compact_out, sm_count, st, pdl, cslot)
     if (e == 1) {
         if (!two) PTAS_SWAR_CALL(u8_nw1);
         PTAS_SWAR_CALL(u8_nw2);
@@ -61,15 +61,15 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
 }
 
 cudaError_t prepare_const_prefix(const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound, int e, int nwords,
-                                 void *d_staging, cudaStream_t st)
+                                 int cslot, void *d_staging, cudaStream_t st)
 {
     const bool two = nwords > 1;
-    if (e == 1) return two ? prepare_const_prefix_u8_nw2(d_pref, d_meta, nP_bound, e, d_staging, st)
-                           : prepare_const_prefix_u8_nw1(d_pref, d_meta, nP_bound, e, d_staging, st);
-    return two ? prepare_const_prefix_u16_nw2(d_pref, d_meta, nP_bound, e, d_staging, st)
-               : prepare_const_prefix_u16_nw1(d_pref, d_meta, nP_bound, e, d_staging, st);
+    if (e == 1) return two ? prepare_const_prefix_u8_nw2(d_pref, d_meta, nP_bound, e, cslot, d_staging, st)
+                           : prepare_const_prefix_u8_nw1(d_pref, d_meta, nP_bound, e, cslot, d_staging, st);
+    return two ? prepare_const_prefix_u16_nw2(d_pref, d_meta, nP_bound, e, cslot, d_staging, st)
+               : prepare_const_prefix_u16_nw1(d_pref, d_meta, nP_bound, e, cslot, d_staging, st);
 }
 
-size_t const_prefix_staging_bytes() { return 8 + 8 * 4000; }
+size_t const_prefix_staging_bytes() { return 8 + 8 * 1000; }
 
 }  // namespace ptas

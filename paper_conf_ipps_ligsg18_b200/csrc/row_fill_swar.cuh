@@ -161,13 +161,14 @@ __device__ __forceinline__ uint32_t lane_shift(const uint32_t w0, const uint32_t
 // Prefix offsets/Jmax in constant memory: indexed by a warp-uniform loop
 // counter they load into uniform registers, so the j-branches are uniform
 // (no reconvergence barriers).  One DP is in flight per device (engine lock).
-constexpr int CP_MAX = 4000;
+constexpr int CP_MAX = 1000;   // per DP slot
+constexpr int CP_SLOTS = 4;
 struct ConstPref {
     int np;
     int pad;
     int2 oj[CP_MAX];
 };
-static __constant__ ConstPref c_pref;  // one copy per translation unit (no -rdc)
+static __constant__ ConstPref c_pref[CP_SLOTS];  // one copy per translation unit (no -rdc)
 
 static __global__ void pack_const_prefix_kernel(const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
                                          int eb, ConstPref *__restrict__ out)
@@ -189,15 +190,16 @@ static __global__ void pack_const_prefix_kernel(const PrefixEntry *__restrict__ 
 }
 
 static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
-                                           int e, void *d_staging, cudaStream_t st)
+                                           int e, int cslot, void *d_staging, cudaStream_t st)
 {
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    if (np > CP_MAX) return cudaErrorNotSupported;
+    if (np > CP_MAX || cslot < 0 || cslot >= CP_SLOTS) return cudaErrorNotSupported;
     pack_const_prefix_kernel<<<8, 256, 0, st>>>(d_pref, d_meta, e, (ConstPref *)d_staging);
     cudaError_t err = cudaGetLastError();
     if (err != cudaSuccess) return err;
     const size_t bytes = 8 + 8 * (size_t)((np + 31) & ~31 < CP_MAX ? ((np + 31) & ~31) : CP_MAX);
-    return cudaMemcpyToSymbolAsync(c_pref, d_staging, bytes, 0, cudaMemcpyDeviceToDevice, st);
+    return cudaMemcpyToSymbolAsync(c_pref, d_staging, bytes, (size_t)cslot * sizeof(ConstPref),
+                                   cudaMemcpyDeviceToDevice, st);
 }
 
 template <typename E, int NW, int CH, int JB, bool CPREF, bool SPLIT>
@@ -205,7 +207,7 @@ __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
-                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int Lg, int nsplit_arg)
+                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int Lg, int nsplit_arg, int cslot)
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
@@ -214,7 +216,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     // prologue now; everything before griddepcontrol.wait below reads only data
     // produced before the first fill launch of the DP (prefix table, row index).
     asm volatile("griddepcontrol.launch_dependents;");
-    const int np = CPREF ? c_pref.np : (int)(meta->nP - 1);
+    const ConstPref &cp = c_pref[CPREF ? cslot : 0];
+    const int np = CPREF ? cp.np : (int)(meta->nP - 1);
     // s_oj[c] = {-off(s') in words, Jmax(s')}: int32 offsets (the host routes
     // tables of 2^31 words or more to the scalar kernel)
     const int npad = (np + 31) & ~31;  // zero-padded: dummy slots never load and have Jmax 0
@@ -331,7 +334,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #pragma unroll
                     for (int u = 0; u < 4; ++u) {
                         const int q = q0 + u;
-                        const int2 oj = CPREF ? c_pref.oj[base + q] : s_oj[base + q];
+                        const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
                         const bool pd = (m >> q) & 1u;
                         jmq[u] = oj.y;
                         const int wi = rw + oj.x;
@@ -487,7 +490,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
                                  const uint64_t *pw, int64_t pw_stride, const PrefixEntry *d_pref,
                                  const DpMeta *d_meta, int64_t nP_bound, int J0, int rho,
                                  int64_t slot_begin, int64_t slot_count, void *compact_out, int sm_count,
-                                 cudaStream_t st, int pdl, int cpref_ok)
+                                 cudaStream_t st, int pdl, int cslot)
 {
     if (slot_count <= 0) return cudaSuccess;
     const int Lw = (int)(g.Wp * e / 4);
@@ -532,7 +535,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
     const int need = e == 1 ? ((J0 + 1) / 2 * 2 > J0 ? (J0 + 1) / 2 * 2 : J0) : 2 * J0;
     const int JBsel = need <= 4 ? 4 : (need <= 8 ? 8 : 0);
-    const bool cpref = np <= CP_MAX && cpref_ok && np >= 64;
+    const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && np >= 64;
 #define PTAS_SWAR_JB(E_, NW_, CH_, JB_)                                                           \
     do {                                                                                          \
         auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, JB_, true, true>      \
@@ -556,7 +559,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
         cfg.numAttrs = 1;                                                                         \
         err = cudaLaunchKernelEx(&cfg, kfn, (E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta,    \
                                  J0, rho, slot_begin, slot_count, (E_ *)compact_out, Lg,          \
-                                 nsplit);                                                         \
+                                 nsplit, cslot);                                                  \
         if (err != cudaSuccess) return err;                                                       \
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \

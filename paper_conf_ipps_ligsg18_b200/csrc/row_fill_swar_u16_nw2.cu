@@ -6,16 +6,16 @@ namespace ptas {
 cudaError_t launch_row_fill_swar_u16_nw2(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
                                  int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
                                  int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
-                                 void *compact_out, int sm_count, cudaStream_t st, int pdl, int cpref_ok)
+                                 void *compact_out, int sm_count, cudaStream_t st, int pdl, int cslot)
 {
     return swar::launch_swar_impl<uint16_t, 2>(e, table, g, rb, pw, pw_stride, d_pref, d_meta, nP_bound, J0, rho,
-                                          slot_begin, slot_count, compact_out, sm_count, st, pdl, cpref_ok);
+                                          slot_begin, slot_count, compact_out, sm_count, st, pdl, cslot);
 }
 
 cudaError_t prepare_const_prefix_u16_nw2(const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound, int e,
-                                  void *d_staging, cudaStream_t st)
+                                  int cslot, void *d_staging, cudaStream_t st)
 {
-    return swar::prepare_const_prefix_tu(d_pref, d_meta, nP_bound, e, d_staging, st);
+    return swar::prepare_const_prefix_tu(d_pref, d_meta, nP_bound, e, cslot, d_staging, st);
 }
 
 }  // namespace ptas

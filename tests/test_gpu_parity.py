@@ -260,6 +260,21 @@ def test_solve_layouts_and_memo(P):
                 _cmp_solve(P, p, 3, 0.25, 2, layout=layout, memoize=memo)
 
 
+def test_solve_concurrent_probes_identical(P, monkeypatch):
+    # P > 1 probes of a round run concurrently in separate DP slots; results and
+    # the probe log must equal the sequential evaluation and the oracle
+    for seed in range(6):
+        p = jobs(60, 1000, seed)
+        conc = _cmp_solve(P, p, 14, 0.3, 4)
+        monkeypatch.setenv("PTAS_NO_CONCURRENT", "1")
+        seq = P.ptas_solve(p, 14, 0.3, P=4)
+        monkeypatch.delenv("PTAS_NO_CONCURRENT")
+        assert seq["T_star"] == conc["T_star"] and (seq["assignment"] == conc["assignment"]).all()
+        assert [x[:5] for x in seq["probes"]] == [x[:5] for x in conc["probes"]]
+    p = jobs(40, 1000, 11)
+    _cmp_solve(P, p, 8, 0.25, 8)   # 8 concurrent slots
+
+
 def test_solve_g3_nonmonotone(P):
     g = json.load(open(os.path.join(GOLD, "g3_nonmonotone.json")))
     for Pp, want in g["by_P"].items():
