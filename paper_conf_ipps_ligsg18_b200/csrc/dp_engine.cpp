@@ -442,8 +442,20 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         PT_CK(stage_.ensure(mx));
     }
     PT_CK(cudaEventRecord(ev_[1], st));
+    // PTAS_LEVEL_TIMES=1: per-row-level device times (events between launches; diagnostics)
+    static const bool lvl_times = [] {
+        const char *t = std::getenv("PTAS_LEVEL_TIMES");
+        return t && t[0] == '1';
+    }();
+    std::vector<cudaEvent_t> lev;
+    if (lvl_times) {
+        lev.resize((size_t)g.rho_max + 2);
+        for (auto &ev : lev) PT_CK(cudaEventCreate(&ev));
+        PT_CK(cudaEventRecord(lev[0], st));
+    }
     for (int rho = 0; rho <= g.rho_max; ++rho) {
         const int64_t R = cnt[rho];
+        if (lvl_times && rho > 0) PT_CK(cudaEventRecord(lev[rho], st));
         if (R <= 0) continue;
         if (!sharded(R)) {
             PT_CK(fill(table, g, J0, rho, 0, R, nullptr));
@@ -474,6 +486,18 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         ++o.launches;
     }
     PT_CK(cudaEventRecord(ev_[2], st));
+    if (lvl_times) {
+        PT_CK(cudaEventRecord(lev[g.rho_max + 1], st));
+        PT_CK(cudaEventSynchronize(lev[g.rho_max + 1]));
+        std::fprintf(stderr, "[ptas] level times (us, rows) sigma=%lld:", (long long)sigma);
+        for (int rho = 0; rho <= g.rho_max; ++rho) {
+            float ms = 0;
+            cudaEventElapsedTime(&ms, lev[rho], lev[rho + 1]);
+            std::fprintf(stderr, " %.1f/%lld", ms * 1e3, (long long)cnt[rho]);
+        }
+        std::fprintf(stderr, "\n");
+        for (auto &ev : lev) cudaEventDestroy(ev);
+    }
     if (trace) tr_fillq = trace_now();
     o.launches += o.fill_launches;
     (void)ld;

@@ -505,9 +505,13 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // amortise the per-prefix cost over CH words while leaving few slots idle.
     int CH;
     const char *chs = std::getenv("PTAS_SWAR_CH");
+    // small row-levels are latency-bound: fewer words per lane (more lanes per
+    // row) shorten each lane's serial work
+    const char *cht = std::getenv("PTAS_SMALL_LEVEL_ROWS");
+    const int64_t small_rows = cht ? std::atoll(cht) : (int64_t)sm_count * 32;
     if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
     else if (chs && chs[0]) CH = std::atoi(chs);
-    else CH = Lw >= 8 ? 2 : 1;
+    else CH = (Lw >= 8 && slot_count > small_rows) ? 2 : 1;
     if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
     int Lg = (Lw + CH - 1) / CH;
     if (Lg < 1) Lg = 1;
