@@ -86,6 +86,10 @@ typedef struct {
     int32_t kernel_launches;/* kernels launched by the library in this call    */
     int32_t fill_launches;  /* of which level-fill launches                    */
     int64_t h2d_bytes, d2h_bytes; /* host<->device bytes moved by this call    */
+    double relax_executed;  /* (n, s') relaxations the fill kernels evaluated:
+                               the packed kernel takes one window per prefix
+                               s' (reading D5), so this is below
+                               `relaxations`; equal on the scalar kernel      */
 } ptas_stats;
 
 typedef struct {

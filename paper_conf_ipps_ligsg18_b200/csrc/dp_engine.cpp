@@ -169,7 +169,7 @@ static int build_geom(const std::vector<int32_t> &N, int e, bool pad, RowGeom *g
     std::memset(g, 0, sizeof(*g));
     g->K1 = K - 1;
     g->W = N[K - 1] + 1;
-    g->Wp = pad ? ((g->W * e + 3) / 4 * 4) / e : g->W;
+    g->Wp = pad ? row_pitch_words(g->W * e) * 4 / e : g->W;
     stride->assign(K, 1);
     if (K >= 2) (*stride)[K - 2] = g->Wp;
     for (int i = K - 3; i >= 0; --i) (*stride)[i] = (*stride)[i + 1] * (N[i + 1] + 1);
@@ -305,7 +305,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     const int64_t ibytes = rows * g.Wp * e;  // padded internal table
     // compute in the caller's buffer when its layout is the padded one
     void *table = nullptr;
-    const bool in_place = rq.ext_table && g.Wp == g.W && ((uintptr_t)rq.ext_table & 3) == 0;
+    const bool in_place = rq.ext_table && g.Wp == g.W && ((uintptr_t)rq.ext_table & 15) == 0;
     if (in_place) {
         table = rq.ext_table;
     } else {
@@ -324,6 +324,8 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         int64_t b = rq.T / r[i];
         hi[i] = (int32_t)(b < N[i] ? b : N[i]);
     }
+    // interior test of the fill kernel: rows p >= hi (leading dims) dominate every prefix
+    for (int i = 0; i < K - 1; ++i) g.maxs[g.word[i]] |= (uint64_t)hi[i] << g.shift[i];
     const size_t small_bytes = (size_t)K * (4 + 8 + 8);
     std::vector<unsigned char> small(small_bytes);
     std::memcpy(small.data(), r.data(), (size_t)K * 8);
@@ -396,6 +398,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     const char *pdls = std::getenv("PTAS_PDL");
     const bool use_pdl = !(pdls && pdls[0] == '0');
     bool prev_fill = false;  // the previous launch on st was a packed fill (PDL-safe)
+    bool used_scalar = false;  // some level ran on the scalar (uncollapsed) kernel
     // one row-level (or slice of it): packed-word kernel, scalar kernel as fallback
     auto fill = [&](void *tab, const RowGeom &gg, int j0, int rho_, int64_t b, int64_t c,
                     void *compact) -> cudaError_t {
@@ -412,6 +415,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC, j0,
                                   rho_, b, c, compact, sm_count_, st);
             prev_fill = false;
+            used_scalar = true;
         }
         return err;
     };
@@ -527,6 +531,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     }
     o.opt = h_meta_->opt;
     o.relax = (double)h_meta_->relax;
+    o.relax_exec = used_scalar ? o.relax : (double)h_meta_->relax_exec;
     o.nC = h_meta_->nC;
     o.nP = h_meta_->nP;
 

@@ -136,12 +136,12 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
 {
     __shared__ int64_t warp_sums[32];
     __shared__ int64_t carry;
-    __shared__ unsigned long long relax_acc;
+    __shared__ unsigned long long relax_acc, exec_acc;
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int K1 = K - 1;
-    if (tid == 0) { carry = 0; relax_acc = 0ull; }
+    if (tid == 0) { carry = 0; relax_acc = 0ull; exec_acc = 0ull; }
     __syncthreads();
-    unsigned long long my_relax = 0;
+    unsigned long long my_relax = 0, my_exec = 0;
     for (int64_t base = 0; base < nC; base += blockDim.x) {
         int64_t c = base + tid;
         bool valid = c < nC;
@@ -179,6 +179,16 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
                 e.jmax = 0;
                 e.pad = 0;
                 pref[id] = e;
+                // collapsed relaxations (D5): one per (row dominating s', x) for s' != 0,
+                // one per state with x >= 1 for the in-row term s' = 0
+                unsigned long long rows_dom = 1;
+                bool zero = true;
+                for (int i = 0; i < K1; ++i) {
+                    rows_dom *= (unsigned long long)(Nall.v[i] - dc[i] + 1);
+                    zero &= dc[i] == 0;
+                }
+                const unsigned long long Wl = (unsigned long long)Nall.v[K - 1] + 1;
+                my_exec += zero ? rows_dom * (Wl - 1) : rows_dom * Wl;
             }
             // closed-form relaxation count: prod_i (N_i - s_i + 1) states dominate s
             unsigned long long pr = 1;
@@ -194,11 +204,13 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
         __syncthreads();
     }
     atomicAdd(&relax_acc, my_relax);
+    atomicAdd(&exec_acc, my_exec);
     __syncthreads();
     if (tid == 0) {
         meta->nC = nC;
         meta->nP = carry;
         meta->relax = relax_acc;
+        meta->relax_exec = exec_acc;
     }
 }
 

@@ -40,6 +40,7 @@ struct DpOutcome {
     int e = 1;
     int Kint = 0;
     double relax = 0;
+    double relax_exec = 0;  // relaxations the kernels evaluated (collapsed form, or relax for the scalar kernel)
     int64_t nC = 0, nP = 0;
     double dp_s = 0, fill_s = 0;
     int launches = 0, fill_launches = 0;

@@ -6,8 +6,9 @@
 //            chosen by the driver; identity for dp_fill), last class fastest.
 //            A "row" is the run of W = N[K-1]+1 entries that share the K1 = K-1
 //            leading digits p; rows are stored with pitch Wp (W*e rounded up
-//            to a multiple of 4 bytes) so every row and every off(s') is word
-//            aligned.  Rows are filled in row-level order rho = sum(p) (the
+//            to a multiple of 4 bytes, and of 4*CH bytes for rows of 8 or
+//            more words, CH = the fill kernel's words per lane) so every row
+//            and every off(s') is aligned for the kernel's vector loads.  Rows are filled in row-level order rho = sum(p) (the
 //            wavefront).  The caller's layout (pitch W) is produced by a
 //            compaction copy when Wp != W.
 //   configs: C(T) in internal lexicographic order: uint16
@@ -37,21 +38,34 @@ struct RowGeom {
     int32_t K1;                 // number of leading classes (K-1)
     int32_t rho_max;            // sum of leading counts
     int64_t W;                  // row length N[K-1]+1
-    int64_t Wp;                 // padded row pitch (entries): W*e rounded up to 4 bytes
+    int64_t Wp;                 // padded row pitch (entries), see row_pitch_words()
     int32_t N[MAXK];            // leading counts
     int32_t maxsuf[MAXK + 1];   // maxsuf[i] = sum_{d >= i} N[d] (leading dims)
     int64_t stride[MAXK];       // element strides of the leading dims
     uint8_t word[MAXK];         // packed word index of leading digit i
     uint8_t shift[MAXK];        // bit offset of leading digit i
     uint64_t guard[MAXW];       // guard bit per field, per word
+    uint64_t maxs[MAXW];        // packed hi_i = min(N_i, T / r_i): the digit-wise max over the prefixes of C(T)
     int32_t nwords;
 };
+
+// Padded row pitch in 32-bit words for a row of `bytes` bytes: a multiple of
+// the packed fill kernel's words per lane (2 up to 64 words, 4 up to 128, 8
+// beyond), so each lane's chunk is one aligned vector load.
+inline int64_t row_pitch_words(int64_t bytes)
+{
+    const int64_t w = (bytes + 3) / 4;
+    const int64_t ch = w < 8 ? 1 : (w <= 64 ? 2 : (w <= 128 ? 4 : 8));
+    return (w + ch - 1) / ch * ch;
+}
 
 // Device-side summary written by the planning kernels and read back once.
 struct DpMeta {
     int64_t nC;            // |C|
     int64_t nP;            // number of prefix entries (incl. the zero prefix)
     unsigned long long relax;  // closed-form relaxations sum_{s in C} prod(N_i - s_i + 1)
+    unsigned long long relax_exec;  // (n, s') pairs the packed kernel evaluates (reading D5):
+                                    // sum_{s' != 0} prod_{i<K-1}(N_i - s'_i + 1) * W + rows * (W - 1)
     int32_t opt;           // OPT(N)
     int32_t err;           // device-detected error (traceback)
 };

@@ -155,6 +155,7 @@ struct Acc {
     void add(const DpOutcome &o)
     {
         s.relaxations += o.relax;
+        s.relax_executed += o.relax_exec;
         s.dp_seconds += o.dp_s;
         s.fill_seconds += o.fill_s;
         s.alg_bytes += (o.relax + (double)o.sigma) * o.e;

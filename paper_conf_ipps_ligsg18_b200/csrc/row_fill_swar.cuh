@@ -1,31 +1,35 @@
 // row_fill_swar.cuh — packed-word level fill kernel template (see row_fill_swar.cu).
 // Included by the four instantiation units row_fill_swar_<E>_nw<NW>.cu so the
-// 48 variants of each (entry type, digit words) pair compile in parallel.
+// variants of each (entry type, digit words) pair compile in parallel.
 #pragma once
 //
-// Same recurrence and row-wavefront as row_fill_kernel (dp_kernels.cu), Eq. 1
-// of PAPER.md:74-79, but every lane owns one 32-bit word of a row: 4 uint8
-// states or 2 uint16 states.  Rows are padded to a multiple of 4 bytes
-// (RowGeom::Wp), so every row and every off(s') is word aligned:
+// Eq. 1 of PAPER.md:74-79 on the row wavefront (row-level rho = sum of the
+// K-1 leading digits p of n = (p, x)), with the result-identical reduction of
+// SURVEY.md §8(f)-1 (reading D5): OPT is monotone under dominance,
+// so for a prefix s' of C(T) (the leading K-1 digits of configurations s)
 //
-//   * the source row p - s' of a prefix is read with ONE coalesced 32-bit
-//     load per lane;
-//   * the j-shifted windows (s = (s', j), j = 0..Jmax(s')) come from the
-//     lane's word and its left neighbours (warp shuffles) through one PRMT
-//     each; uint8 windows are split into even/odd uint16 lanes with the
-//     sign-replicating PRMT mode (v < 128 -> v, v >= 128 -> 0xFF00|v, a
-//     monotone encoding), so VIMNMX.U16x2 takes two minima per instruction;
-//   * all row groups of a warp walk the prefix list in lockstep (uniform
-//     loop, uniform Jmax), each with its own dominance predicate s' <= p.
+//     min_{0 <= j <= min(x, Jmax(s'))} OPT(p - s', x - j) = OPT(p - s', x - min(x, Jmax(s')))
 //
-// The in-row term (s' = 0, j = 1..J0) is then resolved on packed uint16
-// lanes by Bellman-Ford rounds (shift, +1, min) until no lane changes.
-// Every (n, s) with s in C, s <= n is relaxed exactly once, so the closed
-// form relaxation count still holds.  Entries in the row padding and in
-// lanes past the row end are computed but never read as sources.
+// and the in-row configurations (0, j), 1 <= j <= J0, reduce to the single
+// term OPT(p, x - min(x, J0)).  Per (row, prefix) the kernel therefore takes
+// ONE shifted window of the source row instead of Jmax(s') + 1 of them; the
+// value is bit-identical to the plain recurrence (pinned by the parity tests).
+//
+// Lane layout: a row of Lw 32-bit words (pitch padded by the driver to a
+// multiple of CH words) is owned by a group of Lg = Lw / CH lanes; lane xl of
+// the group holds the CH consecutive words xl*CH .. xl*CH+CH-1 (one vector
+// load per source row).  uint8 windows are split into even/odd uint16 lanes
+// with the sign-replicating PRMT mode (v < 128 -> v, v >= 128 -> 0xFF00|v, a
+// monotone encoding) so VIMNMX.U16x2 takes two minima per instruction.  All
+// row groups of a warp walk the prefix list in lockstep (uniform loop,
+// uniform shift), each with its own dominance mask s' <= p; a warp whose rows
+// all dominate every prefix (p >= hi digit-wise, "interior") skips the mask.
+// Positions x - J < 0 take the row's first entry (the clamp min(x, J)).
 #include <cstdint>
 #include <cstdlib>
 #include <cuda_runtime.h>
+#include <mutex>
+#include <unordered_map>
 
 #include "device_common.cuh"
 #include "internal.h"
@@ -49,118 +53,116 @@ struct Words {
     uint32_t v[CH];
 };
 
-// Lane geometry: a row is owned by a group of Lg lanes (any 1 <= Lg <= 32,
-// rows per warp = 32 / Lg, trailing lanes idle); lane xl of group grp holds
-// the row's words w = xl + Lg * t, t < CH.
-struct LaneMap {
-    int lane, Lg, grp, xl;
-};
-
-// Word k positions to the left of the lane's word of chunk t.  With
-// k = qk * Lg + rk, word w - k lives in lane (xl - rk) mod Lg of the same
-// group, chunk t - qk (or t - qk - 1 when the lane index wraps).  Chunks
-// before 0 are outside the row and read as `fill`.
 template <int CH>
-__device__ __forceinline__ uint32_t word_left(const Words<CH> &a, int t, int k, const LaneMap &lm, uint32_t fill)
+__device__ __forceinline__ void fill_words(Words<CH> &w, uint32_t x)
 {
-    int qk = 0, rk = k;
-    if (k >= lm.Lg) {
-        qk = k / lm.Lg;
-        rk = k - qk * lm.Lg;
-    }
-    const int c1 = t - qk, c2 = c1 - 1;
-    uint32_t v1 = fill, v2 = fill;
 #pragma unroll
-    for (int c = 0; c < CH; ++c) {
-        if (c == c1) v1 = a.v[c];
-        if (c == c2) v2 = a.v[c];
-    }
-    if (rk == 0) return v1;
-    const uint32_t send = (lm.xl >= lm.Lg - rk) ? v2 : v1;
-    const int src = lm.lane - rk + (lm.xl < rk ? lm.Lg : 0);
-    return __shfl_sync(FULL, send, src);
+    for (int t = 0; t < CH; ++t) w.v[t] = x;
 }
 
-// acc <- min(acc, window of `lo:hi` at byte offset o) for one word position.
-template <int EB>
-__device__ __forceinline__ void acc_window(uint32_t lo, uint32_t hi, int o, uint32_t &ae, uint32_t &ao)
+// CH consecutive words at p (4*CH-byte aligned: the pitch is a multiple of CH words)
+template <int CH>
+__device__ __forceinline__ Words<CH> load_words(const uint32_t *p)
 {
-    if constexpr (EB == 1) {
-        ae = vmin2(ae, prmt(lo, hi, 0xA280u + 0x1111u * o));
-        ao = vmin2(ao, prmt(lo, hi, 0xB391u + 0x1111u * o));
+    Words<CH> w;
+    if constexpr (CH == 1) {
+        w.v[0] = __ldg(p);
+    } else if constexpr (CH == 2) {
+        const uint2 a = __ldg(reinterpret_cast<const uint2 *>(p));
+        w.v[0] = a.x;
+        w.v[1] = a.y;
     } else {
-        ae = vmin2(ae, prmt(lo, hi, 0x3210u + 0x1111u * o));
+#pragma unroll
+        for (int c = 0; c < CH; c += 4) {
+            const uint4 a = __ldg(reinterpret_cast<const uint4 *>(p + c));
+            w.v[c] = a.x;
+            w.v[c + 1] = a.y;
+            w.v[c + 2] = a.z;
+            w.v[c + 3] = a.w;
+        }
+    }
+    return w;
+}
+
+template <int CH>
+__device__ __forceinline__ void store_words(uint32_t *p, const Words<CH> &w)
+{
+    if constexpr (CH == 1) {
+        p[0] = w.v[0];
+    } else if constexpr (CH == 2) {
+        *reinterpret_cast<uint2 *>(p) = make_uint2(w.v[0], w.v[1]);
+    } else {
+#pragma unroll
+        for (int c = 0; c < CH; c += 4)
+            *reinterpret_cast<uint4 *>(p + c) = make_uint4(w.v[c], w.v[c + 1], w.v[c + 2], w.v[c + 3]);
     }
 }
 
-// All relaxations (s', j), j = 0..jm, of one prefix on the lane's words.
-// JB > 0: shifts up to JB bytes, fully unrolled (jm * EB <= JB guaranteed by
-// the host); JB == 0: any shift (runtime loop, generic word fetch).
-template <int EB, int CH, int JB>
-__device__ __forceinline__ void relax_prefix(const Words<CH> &cur, int jm, const LaneMap &lm,
-                                             Words<CH> &ae, Words<CH> &ao)
+// Word w - k of the row for the lane's slot t (w = xl*CH + t), k >= 0 warp-uniform;
+// `fill` for w - k < 0.  Every lane of the warp must call it (shuffle).
+template <int CH>
+__device__ __forceinline__ uint32_t word_back(const Words<CH> &a, int t, int k, int xl, uint32_t fill)
 {
+    const int d = k - t;  // > 0: the word lives in a lane to the left
+    if (d <= 0) {
+        uint32_t r = a.v[0];
 #pragma unroll
-    for (int t = 0; t < CH; ++t) acc_window<EB>(cur.v[t], cur.v[t], 0, ae.v[t], ao.v[t]);
-    if (jm <= 0) return;
-    Words<CH> w1, w2;
-#pragma unroll
-    for (int t = 0; t < CH; ++t) w1.v[t] = word_left(cur, t, 1, lm, 0xffffffffu);
-    if (JB == 0 || JB > 4) {
-        if (jm * EB > 4) {
-#pragma unroll
-            for (int t = 0; t < CH; ++t) w2.v[t] = word_left(cur, t, 2, lm, 0xffffffffu);
-        }
+        for (int c = 1; c < CH; ++c)
+            if (c == t - k) r = a.v[c];
+        return r;
     }
-    if constexpr (JB > 0) {
-        // jm is warp-uniform (all groups walk the same prefix): leave the
-        // unrolled sequence with a uniform branch instead of predicating the
-        // remaining steps
+    const int dl = (d + CH - 1) / CH;
+    const int slot = dl * CH - d;
+    uint32_t send = a.v[0];
 #pragma unroll
-        for (int j = 1; j <= JB / EB; ++j) {
-            if (j > jm) break;
-            {
-                const int db = j * EB;
+    for (int c = 1; c < CH; ++c)
+        if (c == slot) send = a.v[c];
+    const uint32_t got = __shfl_up_sync(FULL, send, dl > 31 ? 31 : dl);
+    return xl >= dl ? got : fill;
+}
+
+// Operands of the 4-byte window that starts db bytes left of each of the
+// lane's words: PRMT(lo, hi) at byte offset o = (4 - db % 4) % 4, with
+// lo = word w - k1, hi = word w - k1 + 1, k1 = ceil(db / 4) (db > 0; the
+// caller uses the word itself for db = 0).  Fast form (db <= 4): the only
+// word needed from another lane is the left neighbour's last one (one
+// shuffle).  Words before the row read `fill`.
+template <int CH, bool GEN>
+__device__ __forceinline__ void windows(const Words<CH> &a, int db, int xl, uint32_t fill, Words<CH> &lo,
+                                        Words<CH> &hi)
+{
+    if (!GEN || db <= 4) {
+        const uint32_t left = __shfl_up_sync(FULL, a.v[CH - 1], 1);
 #pragma unroll
-                for (int t = 0; t < CH; ++t) {
-                    if (db <= 4) acc_window<EB>(w1.v[t], cur.v[t], 4 - db, ae.v[t], ao.v[t]);
-                    else acc_window<EB>(w2.v[t], w1.v[t], 8 - db, ae.v[t], ao.v[t]);
-                }
-            }
+        for (int t = 0; t < CH; ++t) {
+            lo.v[t] = t == 0 ? (xl == 0 ? fill : left) : a.v[t - 1];
+            hi.v[t] = a.v[t];
         }
     } else {
-        for (int j = 1; j <= jm; ++j) {
-            const int db = j * EB;
+        const int k1 = (db + 3) >> 2;
 #pragma unroll
-            for (int t = 0; t < CH; ++t) {
-                if (db <= 4) acc_window<EB>(w1.v[t], cur.v[t], 4 - db, ae.v[t], ao.v[t]);
-                else if (db <= 8) acc_window<EB>(w2.v[t], w1.v[t], 8 - db, ae.v[t], ao.v[t]);
-                else {
-                    const int k = (db + 3) >> 2;
-                    acc_window<EB>(word_left(cur, t, k, lm, 0xffffffffu), word_left(cur, t, k - 1, lm, 0xffffffffu),
-                                   4 * k - db, ae.v[t], ao.v[t]);
-                }
-            }
+        for (int t = 0; t < CH; ++t) {
+            lo.v[t] = word_back(a, t, k1, xl, fill);
+            hi.v[t] = word_back(a, t, k1 - 1, xl, fill);
         }
     }
 }
 
-// u16-lane window of a packed array shifted right by s u16 positions
-// (byte shift db = 2s) given the words 1 and 2 to the left.
-__device__ __forceinline__ uint32_t lane_shift(const uint32_t w0, const uint32_t w1, const uint32_t w2, int db,
-                                               uint32_t prevk_lo, uint32_t prevk_hi, int ok)
+// Kernel-side prefix entry: x = -off(s') in words, y = PRMT selector of the
+// window (low 16 bits; the odd-byte selector is y + 0x1111) | db << 16, where
+// db = Jmax(s') * e is the window's byte shift (db = 0: the word itself).
+__device__ __forceinline__ int2 oj_entry(const PrefixEntry &pe, int eb)
 {
-    if (db == 0) return w0;
-    if (db <= 4) return prmt(w1, w0, 0x3210u + 0x1111u * (4 - db));
-    if (db <= 8) return prmt(w2, w1, 0x3210u + 0x1111u * (8 - db));
-    return prmt(prevk_lo, prevk_hi, 0x3210u + 0x1111u * ok);
+    const int db = pe.jmax * eb;
+    const int o = (4 - (db & 3)) & 3;
+    const int sel = (eb == 1 ? 0xA280 : 0x3210) + 0x1111 * o;
+    return make_int2(-(int)((uint64_t)pe.off * eb / 4), sel | (db << 16));
 }
 
 }  // namespace
 
 // Prefix offsets/Jmax in constant memory: indexed by a warp-uniform loop
-// counter they load into uniform registers, so the j-branches are uniform
-// (no reconvergence barriers).  One DP is in flight per device (engine lock).
+// counter they load into uniform registers.  One slot per DP slot of the engine.
 constexpr int CP_MAX = 1000;   // per DP slot
 constexpr int CP_SLOTS = 4;
 struct ConstPref {
@@ -182,9 +184,9 @@ static __global__ void pack_const_prefix_kernel(const PrefixEntry *__restrict__ 
          i += gridDim.x * blockDim.x) {
         if (i < np) {
             const PrefixEntry pe = gpref[1 + i];
-            out->oj[i] = make_int2(-(int)((uint64_t)pe.off * eb / 4), pe.jmax);
+            out->oj[i] = oj_entry(pe, eb);
         } else {
-            out->oj[i] = make_int2(0, 0);
+            out->oj[i] = make_int2(0, eb == 1 ? 0xA280 : 0x3210);
         }
     }
 }
@@ -202,7 +204,11 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
                                    cudaMemcpyDeviceToDevice, st);
 }
 
-template <typename E, int NW, int CH, int JB, bool CPREF, bool SPLIT>
+// E: uint8_t / uint16_t entries; NW: 64-bit words of packed leading digits;
+// CH: words per lane; GEN: shifts beyond one word occur (J0 * e > 4);
+// CPREF: prefix offsets from the constant bank; SPLIT: the warps of a block
+// share rows (small row-levels with long prefix lists).
+template <typename E, int NW, int CH, bool GEN, bool CPREF, bool SPLIT>
 __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
@@ -218,26 +224,19 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     asm volatile("griddepcontrol.launch_dependents;");
     const ConstPref &cp = c_pref[CPREF ? cslot : 0];
     const int np = CPREF ? cp.np : (int)(meta->nP - 1);
-    // s_oj[c] = {-off(s') in words, Jmax(s')}: int32 offsets (the host routes
-    // tables of 2^31 words or more to the scalar kernel)
-    const int npad = (np + 31) & ~31;  // zero-padded: dummy slots never load and have Jmax 0
+    // s_oj[c] = oj_entry: int32 offsets (the host routes tables of 2^31 words
+    // or more to the scalar kernel); s_w: packed digits
+    const int npad = (np + 31) & ~31;  // zero-padded: dummy slots are never loaded (mask bit 0)
     int2 *s_oj = reinterpret_cast<int2 *>(smem_raw);
     uint64_t *s_w = reinterpret_cast<uint64_t *>(s_oj + npad);
     for (int i = threadIdx.x; i < npad; i += blockDim.x) {
-        if (CPREF) {
-            if (i < np) {
-#pragma unroll
-                for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = gpref[1 + i].w[w];
-            }
-        } else if (i < np) {
+        if (i < np) {
             const PrefixEntry pe = gpref[1 + i];
-            // off(s') in words (a multiple of the padded row, hence of 4 bytes)
-            const uint64_t offw = (uint64_t)pe.off * EB / 4;
-            s_oj[i] = make_int2(-(int)offw, pe.jmax);
+            if (!CPREF) s_oj[i] = oj_entry(pe, EB);
 #pragma unroll
             for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
-        } else {
-            s_oj[i] = make_int2(0, 0);
+        } else if (!CPREF) {
+            s_oj[i] = make_int2(0, EB == 1 ? 0xA280 : 0x3210);
         }
     }
     __syncthreads();
@@ -246,23 +245,23 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     const int rpw = 32 / Lg;
     const int grp = lane / Lg;          // grp >= rpw: idle lane
     const int xl = lane - grp * Lg;
-    const LaneMap lm{lane, Lg, grp, xl};
-    const unsigned gmask = Lg == 32 ? 0xffffffffu : ((1u << Lg) - 1u);
     // nsplit == 1: every warp owns its own rows.  nsplit > 1 (small row-levels):
     // the nsplit warps of a block share one set of rows, each walks every
-    // nsplit-th prefix batch, and warp 0 combines the partial minima (shared
-    // memory) before the chain -- the per-row latency drops by ~nsplit.
+    // nsplit-th 32-prefix chunk, and warp 0 combines the partial minima (shared
+    // memory) before the chain.
     const int nsplit = SPLIT ? nsplit_arg : 1;
     const int wid = threadIdx.x >> 5;
     const int64_t gw = SPLIT ? (int64_t)blockIdx.x : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = SPLIT ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int pbase0 = SPLIT ? wid * 32 : 0;  // non-split: a provably uniform prefix index
+    const int pbase0 = SPLIT ? wid * 32 : 0;
     const int pstep = SPLIT ? nsplit * 32 : 32;
     uint32_t *s_red = reinterpret_cast<uint32_t *>(s_w + (size_t)NW * np + 1);  // [warp][2][CH][32]
-    const int Lw = (int)(g.Wp * EB / 4);  // words per (padded) row
-    uint64_t guard[NW];
+    uint64_t guard[NW], maxs[NW];
 #pragma unroll
-    for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
+    for (int w = 0; w < NW; ++w) {
+        guard[w] = g.guard[w];
+        maxs[w] = g.maxs[w];
+    }
     // first row set's index entries, loaded before waiting on the previous level
     int64_t nrb = 0;
     uint64_t npw[NW];
@@ -275,100 +274,132 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     }
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
+    const uint32_t *tab32 = reinterpret_cast<const uint32_t *>(table);
     // uniform trip count (every warp of the grid runs the same number of row
-    // sets; the tail ones are idle) keeps the prefix loop in uniform control
-    // flow, so the constant-bank prefix loads and the j-branches are uniform
+    // sets; the tail ones are idle) keeps the prefix loop in uniform control flow
     const int64_t nsets = (slot_count + rpw - 1) / rpw;
     const int64_t iters = (nsets + nw - 1) / nw;
     for (int64_t it = 0; it < iters; ++it) {
         const int64_t sb = (it * nw + gw) * rpw;
-        {
-            const int64_t slot = sb + grp;
-            const bool rowok = grp < rpw && slot < slot_count;
-            int64_t rowbase = nrb;
-            uint64_t pw[NW];
+        const int64_t slot = sb + grp;
+        const bool rowok = grp < rpw && slot < slot_count;
+        const int64_t rowbase = nrb;
+        uint64_t pw[NW];
 #pragma unroll
-            for (int w = 0; w < NW; ++w) pw[w] = npw[w];
-            {   // prefetch the next row set's index entries
-                const int64_t ns = sb + nw * rpw + grp;
-                const bool ok = grp < rpw && ns < slot_count;
+        for (int w = 0; w < NW; ++w) pw[w] = npw[w];
+        {   // prefetch the next row set's index entries
+            const int64_t ns = sb + nw * rpw + grp;
+            const bool ok = grp < rpw && ns < slot_count;
 #pragma unroll
-                for (int w = 0; w < NW; ++w) npw[w] = ok ? pwa[(int64_t)w * pw_stride + slot_begin + ns] : 0;
-                nrb = ok ? rb[slot_begin + ns] : 0;
-            }
-            // int32 word index of this lane's first word (the launcher guarantees < 2^31 words)
-            const int rw = (int)(rowbase * EB / 4) + xl;
-            const uint32_t *tab32 = reinterpret_cast<const uint32_t *>(table);
-            bool wok[CH];
+            for (int w = 0; w < NW; ++w) npw[w] = ok ? pwa[(int64_t)w * pw_stride + slot_begin + ns] : 0;
+            nrb = ok ? rb[slot_begin + ns] : 0;
+        }
+        // the lane's first word (int32 word index: the launcher guarantees < 2^31 words)
+        const uint32_t *src = tab32 + ((int)(rowbase * EB / 4) + xl * CH);
+        // opaque to the compiler: keeps the pointer in registers instead of
+        // re-deriving it from the kernel parameters at every gather
+        asm volatile("" : "+l"(src));
+        // every prefix dominated by every row of the warp?
+        bool interior = rowok;
 #pragma unroll
-            for (int t = 0; t < CH; ++t) wok[t] = rowok && (xl + Lg * t) < Lw;
+        for (int w = 0; w < NW; ++w) interior &= (((pw[w] | guard[w]) - maxs[w]) & guard[w]) == guard[w];
+        const bool allint = __all_sync(FULL, grp >= rpw || interior);
 
-            // ---- cross-row relaxations
-            Words<CH> ae, ao;
+        // ---- cross-row relaxations: acc = min over s' <= p of OPT(p - s', x - min(x, Jmax(s')))
+        Words<CH> ae, ao;
+        fill_words(ae, 0xffffffffu);
+        fill_words(ao, 0xffffffffu);
+        for (int base = pbase0; base < np; base += pstep) {
+            const int cnt = np - base < 32 ? np - base : 32;
+            unsigned m;
+            if (allint) {
+                m = !rowok ? 0u : (cnt == 32 ? FULL : ((1u << cnt) - 1u));  // idle lanes load nothing
+            } else {
+                // lane xl tests prefixes base + xl + k*Lg for its group's row (uniform
+                // trip count), then an OR all-reduce over the group by rotations
+                // (after the step with distance d every lane holds the OR of 2d
+                // consecutive group lanes; OR is idempotent, so overlaps are harmless)
+                unsigned bits = 0;
+                const int kmax = (cnt + Lg - 1) / Lg;
+                for (int k = 0; k < kmax; ++k) {
+                    const int c = xl + k * Lg;
+                    const bool in = rowok && c < cnt;
+                    const int ci = base + (in ? c : 0);
+                    bool dom = in;
 #pragma unroll
-            for (int t = 0; t < CH; ++t) {
-                ae.v[t] = 0xffffffffu;
-                ao.v[t] = 0xffffffffu;
+                    for (int w = 0; w < NW; ++w)
+                        dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + ci]) & guard[w]) == guard[w];
+                    bits |= dom ? (1u << c) : 0u;
+                }
+                for (int d = 1; d < Lg; d <<= 1) {
+                    const int xs = xl + d >= Lg ? xl + d - Lg : xl + d;
+                    bits |= __shfl_sync(FULL, bits, lane - xl + xs);
+                }
+                m = rowok ? bits : 0u;  // idle lanes (past 32 / Lg groups) may have read foreign bits
             }
-            for (int base = pbase0; base < np; base += pstep) {
-                // dominance mask of prefixes base .. base+31 for this group's row:
-                // lane xl tests base + xl + k*Lg, ceil(32/Lg) ballots
-                unsigned m = 0;
-                for (int k0 = 0; k0 < 32; k0 += Lg) {
-                    const int c = base + k0 + xl;
-                    bool dom = false;
-                    if (rowok && xl + k0 < 32 && c < np) {
-                        dom = true;
+            const int cend = (cnt + 3) & ~3;
+            // 4 prefixes per step: their gathers are issued before any is consumed
+            for (int q0 = 0; q0 < cend; q0 += 4) {
+                Words<CH> cur[4];
+                int sj[4];
 #pragma unroll
-                        for (int w = 0; w < NW; ++w)
-                            dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
-                    }
-                    const unsigned bal = __ballot_sync(FULL, dom);
-                    if (grp < rpw) m |= ((bal >> (grp * Lg)) & gmask) << k0;
+                for (int u = 0; u < 4; ++u) {
+                    const int q = q0 + u;
+                    const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
+                    sj[u] = oj.y;
+                    const uint32_t *p = src + oj.x;
+                    if ((m >> q) & 1u) cur[u] = load_words<CH>(p);
+                    else fill_words(cur[u], 0xffffffffu);
                 }
-                const int cend = ((np - base < 32 ? np - base : 32) + 3) & ~3;
-                // 4 prefixes per step: their gathers are issued before any is consumed
-                for (int q0 = 0; q0 < cend; q0 += 4) {
-                    Words<CH> curq[4];
-                    int jmq[4];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const int q = q0 + u;
-                        const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
-                        const bool pd = (m >> q) & 1u;
-                        jmq[u] = oj.y;
-                        const int wi = rw + oj.x;
-#pragma unroll
-                        for (int t = 0; t < CH; ++t)
-                            curq[u].v[t] = (pd && wok[t]) ? __ldg(tab32 + (wi + Lg * t)) : 0xffffffffu;
+                for (int u = 0; u < 4; ++u) {
+                    const uint32_t sel = (uint32_t)sj[u];   // warp-uniform
+                    Words<CH> lo, hi;
+                    if (sel < 0x10000u) {   // Jmax(s') = 0: the window is the word itself
+                        lo = cur[u];
+                        hi = cur[u];
+                    } else {
+                        // positions before the row read its first entry (clamp to x = 0)
+                        uint32_t f;
+                        if (GEN) f = __shfl_sync(FULL, cur[u].v[0], lane - xl);
+                        else f = cur[u].v[0];
+                        f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
+                        windows<CH, GEN>(cur[u], (int)(sel >> 16), xl, f, lo, hi);
                     }
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) relax_prefix<EB, CH, JB>(curq[u], jmq[u], lm, ae, ao);
-                }
-            }
-
-            if (SPLIT) {
-#pragma unroll
-                for (int t = 0; t < CH; ++t) {
-                    s_red[((wid * 2 + 0) * CH + t) * 32 + lane] = ae.v[t];
-                    s_red[((wid * 2 + 1) * CH + t) * 32 + lane] = ao.v[t];
-                }
-                __syncthreads();
-                if (wid == 0) {
-                    for (int w2 = 1; w2 < nsplit; ++w2) {
-#pragma unroll
-                        for (int t = 0; t < CH; ++t) {
-                            ae.v[t] = vmin2(ae.v[t], s_red[((w2 * 2 + 0) * CH + t) * 32 + lane]);
-                            ao.v[t] = vmin2(ao.v[t], s_red[((w2 * 2 + 1) * CH + t) * 32 + lane]);
+                    for (int t = 0; t < CH; ++t) {
+                        if constexpr (EB == 1) {
+                            ae.v[t] = vmin2(ae.v[t], prmt(lo.v[t], hi.v[t], sel));
+                            ao.v[t] = vmin2(ao.v[t], prmt(lo.v[t], hi.v[t], sel + 0x1111u));
+                        } else {
+                            ae.v[t] = vmin2(ae.v[t], prmt(lo.v[t], hi.v[t], sel));
                         }
                     }
                 }
             }
-            if (!SPLIT || wid == 0) {
-            // ---- in-row chain on plain uint16 lanes: opt = 1 + min(acc, opt(x - j))
+        }
+
+        if (SPLIT) {
+#pragma unroll
+            for (int t = 0; t < CH; ++t) {
+                s_red[((wid * 2 + 0) * CH + t) * 32 + lane] = ae.v[t];
+                s_red[((wid * 2 + 1) * CH + t) * 32 + lane] = ao.v[t];
+            }
+            __syncthreads();
+            if (wid == 0) {
+                for (int w2 = 1; w2 < nsplit; ++w2) {
+#pragma unroll
+                    for (int t = 0; t < CH; ++t) {
+                        ae.v[t] = vmin2(ae.v[t], s_red[((w2 * 2 + 0) * CH + t) * 32 + lane]);
+                        ao.v[t] = vmin2(ao.v[t], s_red[((w2 * 2 + 1) * CH + t) * 32 + lane]);
+                    }
+                }
+            }
+        }
+        if (!SPLIT || wid == 0) {
+            // ---- in-row term on plain uint16 lanes: opt(x) = min(1 + acc(x), 1 + opt(x - min(x, J0)))
             // uint8: E holds x = 4w, 4w+2; O holds x = 4w+1, 4w+3.  uint16: E holds 2w, 2w+1.
             Words<CH> oe, oo;
-            constexpr uint32_t CFILL = (EB == 1) ? 0x01ff01ffu : 0xfffefffeu;  // "outside the row"
 #pragma unroll
             for (int t = 0; t < CH; ++t) {
                 if constexpr (EB == 1) {
@@ -380,111 +411,93 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 }
             }
             if (rho == 0 && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
-            // one Bellman-Ford step for shift j: ne/no <- min(ne/no, opt(x - j) + 1)
-            auto chain_step = [&](int j, const Words<CH> &e1, const Words<CH> &o1, const Words<CH> &e2,
-                                  const Words<CH> &o2, Words<CH> &ne, Words<CH> &no) {
-#pragma unroll
-                for (int t = 0; t < CH; ++t) {
-                    if constexpr (EB == 1) {
-                        // even dest x = 2i: j even -> E shifted j/2; j odd -> O shifted (j+1)/2
-                        // odd dest  x = 2i+1: j even -> O shifted j/2; j odd -> E shifted (j-1)/2
-                        const bool odd = j & 1;
-                        const int sa = odd ? (j + 1) >> 1 : j >> 1;
-                        const int sb = odd ? (j - 1) >> 1 : j >> 1;
-                        const uint32_t A0 = odd ? oo.v[t] : oe.v[t], A1 = odd ? o1.v[t] : e1.v[t],
-                                       A2 = odd ? o2.v[t] : e2.v[t];
-                        const uint32_t B0 = odd ? oe.v[t] : oo.v[t], B1 = odd ? e1.v[t] : o1.v[t],
-                                       B2 = odd ? e2.v[t] : o2.v[t];
-                        uint32_t plo = 0, phi = 0, qlo = 0, qhi = 0;
-                        int po = 0, qo = 0;
-                        if (JB == 0 && 2 * sa > 8) {
-                            const int k = (2 * sa + 3) >> 2;
-                            const Words<CH> &AA = odd ? oo : oe;
-                            plo = word_left(AA, t, k, lm, CFILL);
-                            phi = word_left(AA, t, k - 1, lm, CFILL);
-                            po = 4 * k - 2 * sa;
-                        }
-                        if (JB == 0 && 2 * sb > 8) {
-                            const int k = (2 * sb + 3) >> 2;
-                            const Words<CH> &BB = odd ? oe : oo;
-                            qlo = word_left(BB, t, k, lm, CFILL);
-                            qhi = word_left(BB, t, k - 1, lm, CFILL);
-                            qo = 4 * k - 2 * sb;
-                        }
-                        const uint32_t va = lane_shift(A0, A1, A2, 2 * sa, plo, phi, po);
-                        const uint32_t vb = lane_shift(B0, B1, B2, 2 * sb, qlo, qhi, qo);
-                        ne.v[t] = vmin2(ne.v[t], va + ONES);
-                        no.v[t] = vmin2(no.v[t], vb + ONES);
-                    } else {
-                        uint32_t plo = 0, phi = 0;
-                        int po = 0;
-                        if (JB == 0 && 2 * j > 8) {
-                            const int k = (2 * j + 3) >> 2;
-                            plo = word_left(oe, t, k, lm, CFILL);
-                            phi = word_left(oe, t, k - 1, lm, CFILL);
-                            po = 4 * k - 2 * j;
-                        }
-                        const uint32_t va = lane_shift(oe.v[t], e1.v[t], e2.v[t], 2 * j, plo, phi, po);
-                        ne.v[t] = vmin2(ne.v[t], vmin2(va, 0xfffefffeu) + ONES);
-                    }
-                }
-            };
-            // largest u16-lane shift the chain needs: u8 (J0+1)/2, u16 J0 -> bytes
-            const int chain_db = EB == 1 ? 2 * ((J0 + 1) >> 1) : 2 * J0;
+            // opt(p, 0) is final (no in-row term at x = 0): the clamp value
+            uint32_t f0 = __shfl_sync(FULL, oe.v[0], lane - xl);
+            f0 = prmt(f0, 0u, 0x1010u);
+            // u16-lane shifts of the two arrays: dest parity d <- source array, shift in u16 lanes
+            //   uint8, J0 even: E <- E >> J0/2, O <- O >> J0/2
+            //   uint8, J0 odd : E <- O >> (J0+1)/2, O <- E >> (J0-1)/2
+            //   uint16        : E <- E >> J0
+            const bool odd = EB == 1 && (J0 & 1);
+            const int dbe = EB == 1 ? 2 * (odd ? (J0 + 1) >> 1 : J0 >> 1) : 2 * J0;
+            const int dbo = EB == 1 ? 2 * (odd ? (J0 - 1) >> 1 : J0 >> 1) : 0;
+            const uint32_t oe_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbe & 3)) & 3u);
+            const uint32_t oo_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbo & 3)) & 3u);
             bool changed = true;
             while (__any_sync(FULL, changed)) {
                 changed = false;
-                Words<CH> e1, o1, e2, o2;
+                const Words<CH> &se = odd ? oo : oe;   // source of the even destinations
+                const Words<CH> &so = odd ? oe : oo;   // source of the odd destinations
+                Words<CH> le, he, lo2, ho2;
+                windows<CH, GEN>(se, dbe, xl, f0, le, he);
+                if (dbe == 0) {
 #pragma unroll
-                for (int t = 0; t < CH; ++t) {
-                    e1.v[t] = word_left(oe, t, 1, lm, CFILL);
-                    o1.v[t] = EB == 1 ? word_left(oo, t, 1, lm, CFILL) : 0u;
-                    e2.v[t] = e1.v[t];
-                    o2.v[t] = o1.v[t];
+                    for (int t = 0; t < CH; ++t) le.v[t] = se.v[t];
                 }
-                if (chain_db > 4) {
+                if constexpr (EB == 1) {
+                    windows<CH, GEN>(so, dbo, xl, f0, lo2, ho2);
+                    if (dbo == 0) {
 #pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        e2.v[t] = word_left(oe, t, 2, lm, CFILL);
-                        o2.v[t] = EB == 1 ? word_left(oo, t, 2, lm, CFILL) : 0u;
+                        for (int t = 0; t < CH; ++t) lo2.v[t] = so.v[t];
                     }
                 }
-                Words<CH> ne = oe, no = oo;
-                if constexpr (JB > 0) {
+                Words<CH> ne, no;
 #pragma unroll
-                    for (int j = 1; j <= JB / EB; ++j)
-                        if (j <= J0) chain_step(j, e1, o1, e2, o2, ne, no);
-                } else {
-                    for (int j = 1; j <= J0; ++j) chain_step(j, e1, o1, e2, o2, ne, no);
+                for (int t = 0; t < CH; ++t) {
+                    const uint32_t ve = prmt(le.v[t], he.v[t], oe_sel);
+                    if constexpr (EB == 1) {
+                        const uint32_t vo = prmt(lo2.v[t], ho2.v[t], oo_sel);
+                        ne.v[t] = vmin2(oe.v[t], ve + ONES);
+                        no.v[t] = vmin2(oo.v[t], vo + ONES);
+                    } else {
+                        ne.v[t] = vmin2(oe.v[t], vmin2(ve, 0xfffefffeu) + ONES);
+                        no.v[t] = 0;
+                    }
                 }
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
-                    if (wok[t] && (ne.v[t] != oe.v[t] || (EB == 1 && no.v[t] != oo.v[t]))) changed = true;
+                    if (rowok && (ne.v[t] != oe.v[t] || (EB == 1 && no.v[t] != oo.v[t]))) changed = true;
                     oe.v[t] = ne.v[t];
                     oo.v[t] = no.v[t];
                 }
             }
             // ---- store the packed row (padding bytes receive don't-care values)
-            uint32_t *out32 = compact ? reinterpret_cast<uint32_t *>(compact + slot * g.Wp)
-                                      : reinterpret_cast<uint32_t *>(table + rowbase);
+            if (rowok) {
+                uint32_t *out32 = compact ? reinterpret_cast<uint32_t *>(compact + slot * g.Wp)
+                                          : reinterpret_cast<uint32_t *>(table + rowbase);
+                Words<CH> wv;
 #pragma unroll
-            for (int t = 0; t < CH; ++t) {
-                if (!wok[t]) continue;
-                uint32_t wv;
-                if constexpr (EB == 1) wv = prmt(oe.v[t], oo.v[t], 0x6240u);
-                else wv = oe.v[t];
-                out32[xl + Lg * t] = wv;
+                for (int t = 0; t < CH; ++t) {
+                    if constexpr (EB == 1) wv.v[t] = prmt(oe.v[t], oo.v[t], 0x6240u);
+                    else wv.v[t] = oe.v[t];
+                }
+                store_words<CH>(out32 + xl * CH, wv);
             }
             __syncwarp();
-            }  // chain + store (warp 0 in split mode)
-            if (SPLIT) __syncthreads();  // s_red reused by the next row set
-        }
+        }  // chain + store (warp 0 in split mode)
+        if (SPLIT) __syncthreads();  // s_red reused by the next row set
     }
 }
 
+// Resident blocks per SM of a kernel variant at a dynamic smem size (cached).
+template <typename K>
+static int occupancy_of(K kfn, size_t smem, int bs)
+{
+    static std::mutex mu;
+    static std::unordered_map<uint64_t, int> cache;
+    const uint64_t key = (uint64_t)(uintptr_t)(const void *)kfn ^ ((uint64_t)smem << 40);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kfn, bs, smem) != cudaSuccess || occ < 1) occ = 1;
+    cache[key] = occ;
+    return occ;
+}
+
 // Host launcher body for one (E, NW): returns cudaErrorNotSupported when the
-// geometry needs the scalar kernel (row longer than 1 KiB, or shifts beyond one
-// chunk).
+// geometry needs the scalar kernel (row longer than 1 KiB, pitch not a
+// multiple of the lane chunk, or a table of 2^31 words or more).
 template <typename E, int NW>
 static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const int64_t *rb,
                                  const uint64_t *pw, int64_t pw_stride, const PrefixEntry *d_pref,
@@ -495,61 +508,63 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     if (slot_count <= 0) return cudaSuccess;
     const int Lw = (int)(g.Wp * e / 4);
     if ((g.Wp * e) % 4 != 0 || Lw > 256 || J0 * e > 124) return cudaErrorNotSupported;
+    if (compact_out && ((uintptr_t)compact_out & 15)) return cudaErrorNotSupported;
     // int32 word offsets: the table (incl. padding) must stay below 2^31 words
     {
         int64_t rows_all = 1;
         for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
         if (rows_all * (int64_t)Lw >= ((int64_t)1 << 31)) return cudaErrorNotSupported;
     }
-    // words per lane (chunks, stride Lg) and group width Lg (any 1..32):
-    // amortise the per-prefix cost over CH words while leaving few slots idle.
+    // words per lane CH (group width Lg = Lw / CH <= 32): amortise the
+    // per-prefix cost over CH words; small row-levels are latency-bound and
+    // use CH = 1 (more lanes per row, shorter serial work per lane)
     int CH;
     const char *chs = std::getenv("PTAS_SWAR_CH");
-    // small row-levels are latency-bound: fewer words per lane (more lanes per
-    // row) shorten each lane's serial work
     const char *cht = std::getenv("PTAS_SMALL_LEVEL_ROWS");
     const int64_t small_rows = cht ? std::atoll(cht) : (int64_t)sm_count * 32;
     if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
     else if (chs && chs[0]) CH = std::atoi(chs);
     else CH = (Lw >= 8 && slot_count > small_rows) ? 2 : 1;
     if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
-    int Lg = (Lw + CH - 1) / CH;
-    if (Lg < 1) Lg = 1;
-    if (Lg > 32) return cudaErrorNotSupported;
+    if (Lw % CH != 0) {
+        if (Lw > 32) return cudaErrorNotSupported;
+        CH = 1;
+    }
+    const int Lg = Lw / CH;
+    if (Lg < 1 || Lg > 32) return cudaErrorNotSupported;
     const int rpw = 32 / Lg;
     const int bs = 256;
-    int64_t blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);
-    const int64_t cap = (int64_t)sm_count * 8;
-    if (blocks > cap) blocks = cap;
-    // small row-levels: split each row set's prefixes over the 8 warps of a block
-    const char *sp = std::getenv("PTAS_SPLIT_ROWS");
-    // (prefix batches are 32 wide: splitting pays only with several batches)
-    const int64_t np_ = nP_bound > 1 ? nP_bound - 1 : 0;
-    const int64_t split_rows = sp ? std::atoll(sp) : (np_ >= 128 ? (int64_t)sm_count * rpw * 2 : 0);
-    int nsplit = 1;
-    if (slot_count <= split_rows) {
-        nsplit = bs / 32;
-        blocks = (slot_count + rpw - 1) / rpw;
-    }
-    const int NWk = NW;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NWk + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
+    // small row-levels with long prefix lists: split each row set's prefixes over the 8 warps of a block
+    const char *sp = std::getenv("PTAS_SPLIT_ROWS");
+    const int64_t split_rows = sp ? std::atoll(sp) : (np >= 128 ? (int64_t)sm_count * rpw * 2 : 0);
+    const int nsplit = slot_count <= split_rows ? bs / 32 : 1;
+    const size_t smem = (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
-    cudaError_t err;
-    // static shift window: chain needs u16-lane shifts up to (J0+1)/2 (u8) or J0 (u16)
-    const int need = e == 1 ? ((J0 + 1) / 2 * 2 > J0 ? (J0 + 1) / 2 * 2 : J0) : 2 * J0;
-    const int JBsel = need <= 4 ? 4 : (need <= 8 ? 8 : 0);
+    // shifts beyond one word: prefix windows J * e (J <= J0) or chain u16-lane shifts
+    const int chain_db = e == 1 ? 2 * ((J0 + 1) / 2) : 2 * J0;
+    const bool gen = J0 * e > 4 || chain_db > 4;
     const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && np >= 64;
-#define PTAS_SWAR_JB(E_, NW_, CH_, JB_)                                                           \
+    cudaError_t err;
+#define PTAS_SWAR_GO(E_, NW_, CH_, GEN_)                                                          \
     do {                                                                                          \
-        auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, JB_, true, true>      \
-                                       : row_fill_swar_kernel<E_, NW_, CH_, JB_, true, false>)    \
-                         : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, JB_, false, true>     \
-                                       : row_fill_swar_kernel<E_, NW_, CH_, JB_, false, false>);                                            \
+        auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, GEN_, true, true>     \
+                                       : row_fill_swar_kernel<E_, NW_, CH_, GEN_, true, false>)   \
+                         : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, GEN_, false, true>    \
+                                       : row_fill_swar_kernel<E_, NW_, CH_, GEN_, false, false>); \
         if (smem > 48 * 1024) {                                                                   \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
                                        (int)smem);                                                \
             if (err != cudaSuccess) return err;                                                   \
+        }                                                                                         \
+        int64_t blocks;                                                                           \
+        if (nsplit > 1) {                                                                         \
+            blocks = (slot_count + rpw - 1) / rpw;                                                \
+        } else {                                                                                  \
+            /* one resident wave: every warp loops over row sets */                               \
+            blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);   \
+            const int64_t cap = (int64_t)sm_count * occupancy_of(kfn, smem, bs);                  \
+            if (blocks > cap) blocks = cap;                                                       \
         }                                                                                         \
         cudaLaunchConfig_t cfg = {};                                                              \
         cudaLaunchAttribute attr[1];                                                              \
@@ -568,21 +583,15 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
     do {                                                                                          \
-        if (JBsel == 4) PTAS_SWAR_JB(E_, NW_, CH_, 4);                                            \
-        else if (JBsel == 8) PTAS_SWAR_JB(E_, NW_, CH_, 8);                                       \
-        else PTAS_SWAR_JB(E_, NW_, CH_, 0);                                                       \
+        if (gen) PTAS_SWAR_GO(E_, NW_, CH_, true);                                                \
+        else PTAS_SWAR_GO(E_, NW_, CH_, false);                                                   \
     } while (0)
-#define PTAS_SWAR_CH(E_, NW_)                                                                     \
-    do {                                                                                          \
-        if (CH == 1) PTAS_SWAR_CASE(E_, NW_, 1);                                                  \
-        else if (CH == 2) PTAS_SWAR_CASE(E_, NW_, 2);                                             \
-        else if (CH == 4) PTAS_SWAR_CASE(E_, NW_, 4);                                             \
-        else PTAS_SWAR_CASE(E_, NW_, 8);                                                          \
-    } while (0)
-    PTAS_SWAR_CH(E, NW);
-#undef PTAS_SWAR_CH
+    if (CH == 1) PTAS_SWAR_CASE(E, NW, 1);
+    else if (CH == 2) PTAS_SWAR_CASE(E, NW, 2);
+    else if (CH == 4) PTAS_SWAR_CASE(E, NW, 4);
+    else PTAS_SWAR_CASE(E, NW, 8);
 #undef PTAS_SWAR_CASE
-#undef PTAS_SWAR_JB
+#undef PTAS_SWAR_GO
     return cudaGetLastError();
 }
 
