@@ -260,6 +260,8 @@ def run_ours(args, w):
     t_total = sum(dev_ms) / 1e3
     fill_s = sum(s["fill_seconds"] for s in stats)
     alg_bytes = sum(s["alg_bytes"] for s in stats)
+    exec_bytes = sum(s["exec_bytes"] for s in stats)
+    relax_exec = sum(s["relax_executed"] for s in stats)
     fill_launches = sum(s["fill_launches"] for s in stats)
     launches = sum(s["kernel_launches"] for s in stats)
     e2e_relax = sum(s["relaxations"] for s in e2e_stats)
@@ -310,6 +312,11 @@ def run_ours(args, w):
                      "fill_ms_per_step": 1e3 * fill_s / args.steps,
                      "fill_launches_per_step": fill_launches / args.steps,
                      "alg_bytes_per_step": alg_bytes / args.steps,
+                     # the kernel takes one window per (row, prefix) (D5): the
+                     # bytes it actually gathers, and their rate, next to the algorithmic ones
+                     "relax_executed_per_step": relax_exec / args.steps,
+                     "executed_bytes_per_step": exec_bytes / args.steps,
+                     "executed_gbs": exec_bytes / fill_s / 1e9 if fill_s > 0 else None,
                      "fill_relax_per_s": relax_total / fill_s if fill_s > 0 else None},
         "step_ms": [round(x, 3) for x in dev_ms],
         "step_dp_ms": [round(1e3 * st["dp_seconds"], 3) for st in stats],

@@ -90,6 +90,8 @@ typedef struct {
                                the packed kernel takes one window per prefix
                                s' (reading D5), so this is below
                                `relaxations`; equal on the scalar kernel      */
+    double exec_bytes;      /* sum (relax_executed + sigma) * e: the table bytes
+                               the fill kernels gather and write              */
 } ptas_stats;
 
 typedef struct {

@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libptas_b200.so")
+LIB_PATH = os.environ.get("PTAS_LIB") or os.path.join(_HERE, "libptas_b200.so")
 
 PTAS_OK, PTAS_EINVAL, PTAS_ETOOBIG, PTAS_ENOMEM, PTAS_ECUDA, PTAS_ENCCL, PTAS_EINTERNAL = 0, -1, -2, -3, -4, -5, -6
 MODE_SINGLE, MODE_LEVEL_SHARDED, MODE_MULTI_PROBE = 0, 1, 2
@@ -36,7 +36,8 @@ class PtasStats(ctypes.Structure):
                 ("dp_seconds", ctypes.c_double), ("fill_seconds", ctypes.c_double),
                 ("total_seconds", ctypes.c_double), ("alg_bytes", ctypes.c_double), ("states", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int32), ("fill_launches", ctypes.c_int32),
-                ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64), ("relax_executed", ctypes.c_double)]
+                ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64), ("relax_executed", ctypes.c_double),
+                ("exec_bytes", ctypes.c_double)]
 
     def to_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

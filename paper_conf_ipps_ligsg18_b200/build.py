@@ -9,6 +9,12 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libptas_b200.so")
+# experiment builds (A/B of compile-time knobs): PTAS_VARIANT=<name> with
+# PTAS_EXTRA_FLAGS="-DX=Y ..." writes variants/<name>/libptas_b200.so; load it
+# with PTAS_LIB=<path> (paper_conf_ipps_ligsg18_b200/_native.py)
+VARIANT = os.environ.get("PTAS_VARIANT")
+if VARIANT:
+    LIB = os.path.join(ROOT, "variants", VARIANT, "libptas_b200.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -34,14 +40,15 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
     from concurrent.futures import ThreadPoolExecutor
-    objdir = os.path.join(HERE, "build")
+    objdir = os.path.join(os.path.dirname(LIB), "build") if VARIANT else os.path.join(HERE, "build")
     os.makedirs(objdir, exist_ok=True)
     hdr_t = max(os.path.getmtime(h) for h in _headers())
     # stale objects of removed sources must not be linked
     for o in glob.glob(os.path.join(objdir, "*.o")):
         if os.path.basename(o)[:-2] not in {os.path.basename(x) for x in sources()}:
             os.remove(o)
-    flags = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I" + os.path.join(ROOT, "include")]
+    flags = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I" + os.path.join(ROOT, "include"),
+             *os.environ.get("PTAS_EXTRA_FLAGS", "").split()]
     if verbose:
         flags.append("-Xptxas=-v")
 

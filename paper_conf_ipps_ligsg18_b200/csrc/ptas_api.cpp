@@ -156,6 +156,7 @@ struct Acc {
     {
         s.relaxations += o.relax;
         s.relax_executed += o.relax_exec;
+        s.exec_bytes += (o.relax_exec + (double)o.sigma) * o.e;
         s.dp_seconds += o.dp_s;
         s.fill_seconds += o.fill_s;
         s.alg_bytes += (o.relax + (double)o.sigma) * o.e;

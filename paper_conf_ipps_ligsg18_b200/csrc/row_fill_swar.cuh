@@ -217,6 +217,13 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
+#ifndef PTAS_PB1
+#define PTAS_PB1 16
+#endif
+#ifndef PTAS_PB2
+#define PTAS_PB2 4
+#endif
+    constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);   // gathers in flight per lane (prefix batch)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     // Programmatic dependent launch: let the next row-level's grid start its
     // prologue now; everything before griddepcontrol.wait below reads only data
@@ -337,13 +344,13 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 }
                 m = rowok ? bits : 0u;  // idle lanes (past 32 / Lg groups) may have read foreign bits
             }
-            const int cend = (cnt + 3) & ~3;
-            // 4 prefixes per step: their gathers are issued before any is consumed
-            for (int q0 = 0; q0 < cend; q0 += 4) {
-                Words<CH> cur[4];
-                int sj[4];
+            const int cend = (cnt + PB - 1) & ~(PB - 1);
+            // PB prefixes per step: their gathers are issued before any is consumed
+            for (int q0 = 0; q0 < cend; q0 += PB) {
+                Words<CH> cur[PB];
+                int sj[PB];
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
+                for (int u = 0; u < PB; ++u) {
                     const int q = q0 + u;
                     const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
                     sj[u] = oj.y;
@@ -352,7 +359,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     else fill_words(cur[u], 0xffffffffu);
                 }
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
+                for (int u = 0; u < PB; ++u) {
                     const uint32_t sel = (uint32_t)sj[u];   // warp-uniform
                     Words<CH> lo, hi;
                     if (sel < 0x10000u) {   // Jmax(s') = 0: the window is the word itself

@@ -84,6 +84,21 @@ def test_row_index_complete(P):
 
 
 # ------------------------------------------------------------------ a-5
+def _collapsed_relax(N, r, T):
+    """Closed form of the (n, s') pairs the packed kernel evaluates (DESIGN.md
+    D5): one window per (row dominating s' != 0, x), plus the in-row term for
+    every state with x >= 1.  Internal order = the non-empty classes."""
+    nz = np.asarray(N) > 0
+    Nn, rn = np.asarray(N)[nz].astype(np.int64), np.asarray(r)[nz]
+    if len(Nn) == 0:
+        return 0.0
+    W = float(Nn[-1] + 1)
+    rows = float(np.prod((Nn[:-1] + 1).astype(np.float64)))
+    C = oracle.configs(Nn.astype(np.int32), rn, T)
+    pre = {tuple(int(x) for x in c[:-1]) for c in C} - {tuple([0] * (len(Nn) - 1))}
+    return sum(float(np.prod((Nn[:-1] - np.array(s) + 1).astype(np.float64))) * W for s in pre) + rows * (W - 1)
+
+
 def _check_table(P, N, r, T):
     opt, tab, st = P.dp_fill(N, r, T)
     want, relax = oracle.dp(N, r, T)
@@ -92,6 +107,13 @@ def _check_table(P, N, r, T):
     assert len(bad) == 0, (N.tolist(), r.tolist(), T, bad[:5].tolist())
     assert opt == int(want[tuple(N)]) if len(N) else opt == 0
     assert st["relaxations"] == relax
+    # executed relaxations: the collapsed count on the packed kernel, the full one on the scalar kernel
+    assert st["relax_executed"] in (relax, _collapsed_relax(N, r, T)), (st["relax_executed"], relax)
+    nz = np.asarray(N)[np.asarray(N) > 0]
+    if os.environ.get("PTAS_FORCE_SCALAR") == "1":
+        assert st["relax_executed"] == relax
+    elif len(nz) and (int(nz[-1]) + 1) * (1 if nz.sum() <= 255 else 2) <= 124:
+        assert st["relax_executed"] == _collapsed_relax(N, r, T)   # packed kernel for sure
     return tab
 
 
