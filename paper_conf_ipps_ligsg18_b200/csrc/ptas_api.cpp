@@ -8,6 +8,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstdlib>
+#include <cstdio>
 #include <cstring>
 #include <functional>
 #include <map>
@@ -448,8 +449,12 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         if (rc) return rc;
         std::vector<MachineCfg> machines;
         DpOutcome tb;
+        const double ttb0 = now_s();
         rc = tsl->traceback(&machines, &tb);
         if (rc) return rc;
+        if (std::getenv("PTAS_TRACE"))
+            std::fprintf(stderr, "[ptas] traceback at T*=%lld: %zu machines, %.3f ms (slot %d)\n", (long long)Ts,
+                         machines.size(), 1e3 * (now_s() - ttb0), tslot);
         acc.s.kernel_launches += tb.launches;
         acc.s.h2d_bytes += tb.h2d;
         acc.s.d2h_bytes += tb.d2h;

@@ -254,14 +254,18 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     const int xl = lane - grp * Lg;
     // nsplit == 1: every warp owns its own rows.  nsplit > 1 (small row-levels):
     // the nsplit warps of a block share one set of rows, each walks every
-    // nsplit-th 32-prefix chunk, and warp 0 combines the partial minima (shared
+    // nsplit-th 32-prefix chunk (long prefix lists) or every nsplit-th batch of
+    // PB prefixes within each chunk (short lists), and warp 0 combines the partial minima (shared
     // memory) before the chain.
     const int nsplit = SPLIT ? nsplit_arg : 1;
     const int wid = threadIdx.x >> 5;
     const int64_t gw = SPLIT ? (int64_t)blockIdx.x : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = SPLIT ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int pbase0 = SPLIT ? wid * 32 : 0;
-    const int pstep = SPLIT ? nsplit * 32 : 32;
+    const bool split_chunks = SPLIT && np >= 32 * nsplit;
+    const int pbase0 = split_chunks ? wid * 32 : 0;
+    const int pstep = split_chunks ? nsplit * 32 : 32;
+    const int qbase0 = (SPLIT && !split_chunks) ? wid * PB : 0;
+    const int qstep = (SPLIT && !split_chunks) ? nsplit * PB : PB;
     uint32_t *s_red = reinterpret_cast<uint32_t *>(s_w + (size_t)NW * np + 1);  // [warp][2][CH][32]
     uint64_t guard[NW], maxs[NW];
 #pragma unroll
@@ -346,7 +350,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
             }
             const int cend = (cnt + PB - 1) & ~(PB - 1);
             // PB prefixes per step: their gathers are issued before any is consumed
-            for (int q0 = 0; q0 < cend; q0 += PB) {
+            for (int q0 = qbase0; q0 < cend; q0 += qstep) {
                 Words<CH> cur[PB];
                 int sj[PB];
 #pragma unroll
@@ -544,7 +548,9 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
     // small row-levels with long prefix lists: split each row set's prefixes over the 8 warps of a block
     const char *sp = std::getenv("PTAS_SPLIT_ROWS");
-    const int64_t split_rows = sp ? std::atoll(sp) : (np >= 128 ? (int64_t)sm_count * rpw * 2 : 0);
+    // (worth it when a row's prefix walk has several batches of gathers in series)
+    const int PBh = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);
+    const int64_t split_rows = sp ? std::atoll(sp) : ((np + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
     const int nsplit = slot_count <= split_rows ? bs / 32 : 1;
     const size_t smem = (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
