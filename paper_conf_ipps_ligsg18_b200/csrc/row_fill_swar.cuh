@@ -124,19 +124,34 @@ __device__ __forceinline__ uint32_t word_back(const Words<CH> &a, int t, int k, 
 // Operands of the 4-byte window that starts db bytes left of each of the
 // lane's words: PRMT(lo, hi) at byte offset o = (4 - db % 4) % 4, with
 // lo = word w - k1, hi = word w - k1 + 1, k1 = ceil(db / 4) (db > 0; the
-// caller uses the word itself for db = 0).  Fast form (db <= 4): the only
-// word needed from another lane is the left neighbour's last one (one
-// shuffle).  Words before the row read `fill`.
-template <int CH, bool GEN>
+// caller uses the word itself for db = 0).  db <= 4: the only word needed
+// from another lane is the left neighbour's last one (one shuffle); db <= 8:
+// two shuffles; longer shifts: word_back.  WIN = the largest db the caller
+// can pass (4, 8, or 0 = any), so the unneeded forms are not compiled.  Words before
+// the row read `fill`.
+template <int CH, int WIN>
 __device__ __forceinline__ void windows(const Words<CH> &a, int db, int xl, uint32_t fill, Words<CH> &lo,
                                         Words<CH> &hi)
 {
-    if (!GEN || db <= 4) {
-        const uint32_t left = __shfl_up_sync(FULL, a.v[CH - 1], 1);
+    const uint32_t left = __shfl_up_sync(FULL, a.v[CH - 1], 1);
+    const uint32_t l1 = xl >= 1 ? left : fill;   // word w - 1 of slot 0
+    if (WIN == 4 || db <= 4) {
 #pragma unroll
         for (int t = 0; t < CH; ++t) {
-            lo.v[t] = t == 0 ? (xl == 0 ? fill : left) : a.v[t - 1];
+            lo.v[t] = t == 0 ? l1 : a.v[t - 1];
             hi.v[t] = a.v[t];
+        }
+    } else if (WIN == 8 || db <= 8) {
+        // word w - 2 of slot 0: lane xl-1's slot CH-2 (CH >= 2) or lane xl-2 (CH = 1)
+        const uint32_t left2 = __shfl_up_sync(FULL, a.v[CH >= 2 ? CH - 2 : 0], CH >= 2 ? 1 : 2);
+        const uint32_t l2 = xl >= (CH >= 2 ? 1 : 2) ? left2 : fill;
+        const bool two = db > 4;   // k1 = 2
+#pragma unroll
+        for (int t = 0; t < CH; ++t) {
+            const uint32_t w1 = t == 0 ? l1 : a.v[t - 1];
+            const uint32_t w2 = t >= 2 ? a.v[t - 2] : (t == 1 ? l1 : l2);
+            lo.v[t] = two ? w2 : w1;
+            hi.v[t] = two ? w1 : a.v[t];
         }
     } else {
         const int k1 = (db + 3) >> 2;
@@ -145,6 +160,21 @@ __device__ __forceinline__ void windows(const Words<CH> &a, int db, int xl, uint
             lo.v[t] = word_back(a, t, k1, xl, fill);
             hi.v[t] = word_back(a, t, k1 - 1, xl, fill);
         }
+    }
+}
+
+// Same operands from a copy of the group's row in shared memory (row word r
+// at srow[r]), any db > 0: used by the in-row closure's long shifts.
+template <int CH>
+__device__ __forceinline__ void windows_smem(const uint32_t *srow, int db, int xl, uint32_t fill, Words<CH> &lo,
+                                             Words<CH> &hi)
+{
+    const int k1 = (db + 3) >> 2;
+#pragma unroll
+    for (int t = 0; t < CH; ++t) {
+        const int w = xl * CH + t - k1;
+        lo.v[t] = w >= 0 ? srow[w] : fill;
+        hi.v[t] = w + 1 >= 0 ? srow[w + 1] : fill;
     }
 }
 
@@ -205,10 +235,11 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
 }
 
 // E: uint8_t / uint16_t entries; NW: 64-bit words of packed leading digits;
-// CH: words per lane; GEN: shifts beyond one word occur (J0 * e > 4);
+// CH: words per lane; WIN: largest prefix window shift in bytes the kernel
+// supports (J0 * e <= 4, <= 8, or 0 = any);
 // CPREF: prefix offsets from the constant bank; SPLIT: the warps of a block
 // share rows (small row-levels with long prefix lists).
-template <typename E, int NW, int CH, bool GEN, bool CPREF, bool SPLIT>
+template <typename E, int NW, int CH, int WIN, bool CPREF, bool SPLIT>
 __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
@@ -371,11 +402,11 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         hi = cur[u];
                     } else {
                         // positions before the row read its first entry (clamp to x = 0)
-                        uint32_t f;
-                        if (GEN) f = __shfl_sync(FULL, cur[u].v[0], lane - xl);
-                        else f = cur[u].v[0];
+                        // (db <= 4: only lane xl = 0 reads it, from its own word 0)
+                        uint32_t f = cur[u].v[0];
+                        if (WIN != 4 && (sel >> 16) > 4u) f = __shfl_sync(FULL, f, lane - xl);
                         f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
-                        windows<CH, GEN>(cur[u], (int)(sel >> 16), xl, f, lo, hi);
+                        windows<CH, WIN>(cur[u], (int)(sel >> 16), xl, f, lo, hi);
                     }
 #pragma unroll
                     for (int t = 0; t < CH; ++t) {
@@ -425,52 +456,74 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
             // opt(p, 0) is final (no in-row term at x = 0): the clamp value
             uint32_t f0 = __shfl_sync(FULL, oe.v[0], lane - xl);
             f0 = prmt(f0, 0u, 0x1010u);
-            // u16-lane shifts of the two arrays: dest parity d <- source array, shift in u16 lanes
-            //   uint8, J0 even: E <- E >> J0/2, O <- O >> J0/2
-            //   uint8, J0 odd : E <- O >> (J0+1)/2, O <- E >> (J0-1)/2
-            //   uint16        : E <- E >> J0
-            const bool odd = EB == 1 && (J0 & 1);
-            const int dbe = EB == 1 ? 2 * (odd ? (J0 + 1) >> 1 : J0 >> 1) : 2 * J0;
-            const int dbo = EB == 1 ? 2 * (odd ? (J0 - 1) >> 1 : J0 >> 1) : 0;
-            const uint32_t oe_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbe & 3)) & 3u);
-            const uint32_t oo_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbo & 3)) & 3u);
-            bool changed = true;
-            while (__any_sync(FULL, changed)) {
-                changed = false;
-                const Words<CH> &se = odd ? oo : oe;   // source of the even destinations
-                const Words<CH> &so = odd ? oe : oo;   // source of the odd destinations
+            // Closure of opt(x) = min(v(x), 1 + opt(max(0, x - J0))) by doubling:
+            // round k relaxes opt(x) against opt(x - S) + 2^k with S = 2^k * J0,
+            // positions before the row holding opt(p, 0).  After round k every x
+            // has the minimum over paths of fewer than 2^(k+1) in-row steps; a
+            // round without change means the closure is complete (a later round
+            // can only repeat a path already covered), and S >= W ends it.
+            // u16-lane shifts: uint8, S even: E <- E >> S/2, O <- O >> S/2;
+            // S odd: E <- O >> (S+1)/2, O <- E >> (S-1)/2; uint16: E <- E >> S.
+            int S = J0;
+            uint32_t inc = 1;
+            for (;;) {
+                const bool odd = EB == 1 && (S & 1);
+                const int dbe = EB == 1 ? 2 * (odd ? (S + 1) >> 1 : S >> 1) : 2 * S;
+                const int dbo = EB == 1 ? 2 * (odd ? (S - 1) >> 1 : S >> 1) : 0;
+                const uint32_t oe_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbe & 3)) & 3u);
+                const uint32_t oo_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbo & 3)) & 3u);
                 Words<CH> le, he, lo2, ho2;
-                windows<CH, GEN>(se, dbe, xl, f0, le, he);
-                if (dbe == 0) {
+                if (dbe <= 8 && dbo <= 8) {
+                    Words<CH> se, so;   // sources of the even / odd destinations (registers, no aliasing)
 #pragma unroll
-                    for (int t = 0; t < CH; ++t) le.v[t] = se.v[t];
-                }
-                if constexpr (EB == 1) {
-                    windows<CH, GEN>(so, dbo, xl, f0, lo2, ho2);
-                    if (dbo == 0) {
+                    for (int t = 0; t < CH; ++t) {
+                        se.v[t] = odd ? oo.v[t] : oe.v[t];
+                        so.v[t] = odd ? oe.v[t] : oo.v[t];
+                    }
+                    windows<CH, 8>(se, dbe, xl, f0, le, he);
+                    if (dbe == 0) le = se;
+                    if constexpr (EB == 1) {
+                        windows<CH, 8>(so, dbo, xl, f0, lo2, ho2);
+                        if (dbo == 0) lo2 = so;
+                    }
+                } else {
+                    // long shift: through this warp's slice of s_red ([2][CH * 32] words)
+                    uint32_t *sE = s_red + (size_t)wid * 2 * CH * 32 + grp * Lg * CH;
+                    uint32_t *sO = sE + CH * 32;
+                    __syncwarp();
 #pragma unroll
-                        for (int t = 0; t < CH; ++t) lo2.v[t] = so.v[t];
+                    for (int t = 0; t < CH; ++t) {
+                        sE[xl * CH + t] = oe.v[t];
+                        if (EB == 1) sO[xl * CH + t] = oo.v[t];
+                    }
+                    __syncwarp();
+                    windows_smem<CH>(odd ? sO : sE, dbe, xl, f0, le, he);
+                    if constexpr (EB == 1) {
+                        if (dbo == 0) lo2 = odd ? oe : oo;
+                        else windows_smem<CH>(odd ? sE : sO, dbo, xl, f0, lo2, ho2);
                     }
                 }
-                Words<CH> ne, no;
+                const uint32_t incw = inc * ONES;
+                const uint32_t capw = (0xffffu - inc) * ONES;   // saturating + inc on uint16 lanes
+                bool changed = false;
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
                     const uint32_t ve = prmt(le.v[t], he.v[t], oe_sel);
+                    uint32_t ne, no = 0;
                     if constexpr (EB == 1) {
                         const uint32_t vo = prmt(lo2.v[t], ho2.v[t], oo_sel);
-                        ne.v[t] = vmin2(oe.v[t], ve + ONES);
-                        no.v[t] = vmin2(oo.v[t], vo + ONES);
+                        ne = vmin2(oe.v[t], ve + incw);   // uint8 values stay below 0x200
+                        no = vmin2(oo.v[t], vo + incw);
                     } else {
-                        ne.v[t] = vmin2(oe.v[t], vmin2(ve, 0xfffefffeu) + ONES);
-                        no.v[t] = 0;
+                        ne = vmin2(oe.v[t], vmin2(ve, capw) + incw);
                     }
+                    if (rowok && (ne != oe.v[t] || (EB == 1 && no != oo.v[t]))) changed = true;
+                    oe.v[t] = ne;
+                    oo.v[t] = no;
                 }
-#pragma unroll
-                for (int t = 0; t < CH; ++t) {
-                    if (rowok && (ne.v[t] != oe.v[t] || (EB == 1 && no.v[t] != oo.v[t]))) changed = true;
-                    oe.v[t] = ne.v[t];
-                    oo.v[t] = no.v[t];
-                }
+                if (!__any_sync(FULL, changed) || (int64_t)S >= g.W) break;
+                S *= 2;
+                inc *= 2;
             }
             // ---- store the packed row (padding bytes receive don't-care values)
             if (rowok) {
@@ -555,16 +608,17 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     const size_t smem = (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     // shifts beyond one word: prefix windows J * e (J <= J0) or chain u16-lane shifts
-    const int chain_db = e == 1 ? 2 * ((J0 + 1) / 2) : 2 * J0;
-    const bool gen = J0 * e > 4 || chain_db > 4;
+    // prefix windows beyond two words (J * e > 8, J <= J0) need the generic word fetch;
+    // the in-row closure handles any shift (registers up to 8 bytes, else shared memory)
+    const int win = J0 * e <= 4 ? 4 : (J0 * e <= 8 ? 8 : 0);
     const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && np >= 64;
     cudaError_t err;
-#define PTAS_SWAR_GO(E_, NW_, CH_, GEN_)                                                          \
+#define PTAS_SWAR_GO(E_, NW_, CH_, WIN_)                                                          \
     do {                                                                                          \
-        auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, GEN_, true, true>     \
-                                       : row_fill_swar_kernel<E_, NW_, CH_, GEN_, true, false>)   \
-                         : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, GEN_, false, true>    \
-                                       : row_fill_swar_kernel<E_, NW_, CH_, GEN_, false, false>); \
+        auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true>     \
+                                       : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false>)   \
+                         : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true>    \
+                                       : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false>); \
         if (smem > 48 * 1024) {                                                                   \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
                                        (int)smem);                                                \
@@ -596,8 +650,9 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
     do {                                                                                          \
-        if (gen) PTAS_SWAR_GO(E_, NW_, CH_, true);                                                \
-        else PTAS_SWAR_GO(E_, NW_, CH_, false);                                                   \
+        if (win == 4) PTAS_SWAR_GO(E_, NW_, CH_, 4);                                              \
+        else if (win == 8) PTAS_SWAR_GO(E_, NW_, CH_, 8);                                         \
+        else PTAS_SWAR_GO(E_, NW_, CH_, 0);                                                       \
     } while (0)
     if (CH == 1) PTAS_SWAR_CASE(E, NW, 1);
     else if (CH == 2) PTAS_SWAR_CASE(E, NW, 2);
