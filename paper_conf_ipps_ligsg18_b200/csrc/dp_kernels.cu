@@ -222,33 +222,71 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
 // with the suffix-count table, and stores the row base index and the packed
 // leading digits used by the dominance test.
 template <int NW>
-__global__ void build_row_index_kernel(const RowGeom g, const int64_t *__restrict__ cnt,
-                                       const int64_t *__restrict__ level_start, int64_t rows,
-                                       int64_t *__restrict__ rb, uint64_t *__restrict__ pw)
+__global__ void build_row_index_kernel(const RowGeom g, const int64_t *__restrict__ cnt_g,
+                                       const int64_t *__restrict__ level_start_g, int64_t rows,
+                                       int64_t *__restrict__ rb, uint64_t *__restrict__ pw, int R,
+                                       int tables_in_smem)
 {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= rows) return;
-    int lo = 0, hi = g.rho_max;  // largest rho with level_start[rho] <= t
-    while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (level_start[mid] <= t) lo = mid;
-        else hi = mid - 1;
+    // Each thread produces R consecutive slots: one unranking (binary search +
+    // suffix-count walk), then the lexicographic successor within the level.
+    // Results are staged in shared memory and written out coalesced; the
+    // suffix-count table and level_start are staged too when they fit.
+    extern __shared__ int64_t s_tab[];
+    const int ld = g.rho_max + 1;
+    const int64_t ncnt = (int64_t)(g.K1 + 1) * ld;
+    const int64_t *cnt = cnt_g, *level_start = level_start_g;
+    int64_t *s_out = s_tab + (tables_in_smem ? ncnt + ld + 1 : 0);   // [R * blockDim][1 + NW]
+    if (tables_in_smem) {
+        for (int64_t i = threadIdx.x; i < ncnt + ld + 1; i += blockDim.x)
+            s_tab[i] = i < ncnt ? cnt_g[i] : level_start_g[i - ncnt];
+        __syncthreads();
+        cnt = s_tab;
+        level_start = s_tab + ncnt;
     }
-    int32_t d[MAXK];
-    unrank_digits(g, cnt, lo, t - level_start[lo], d);
-    int64_t base = 0;
-    uint64_t w[NW];
+    const int64_t span = (int64_t)R * blockDim.x;
+    const int64_t b0 = (int64_t)blockIdx.x * span;
+    const int64_t t0 = b0 + (int64_t)threadIdx.x * R;
+    if (t0 < rows) {
+        int lo = 0, hi = g.rho_max;  // largest rho with level_start[rho] <= t0
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (level_start[mid] <= t0) lo = mid;
+            else hi = mid - 1;
+        }
+        int32_t d[MAXK];
+        unrank_digits(g, cnt, lo, t0 - level_start[lo], d);
+        int64_t next_level = level_start[lo + 1];
+        const int64_t tend = t0 + R < rows ? t0 + R : rows;
+        for (int64_t t = t0; t < tend; ++t) {
+            if (t == next_level) {   // first row of the next level
+                ++lo;
+                unrank_digits(g, cnt, lo, 0, d);
+                next_level = level_start[lo + 1];
+            }
+            int64_t base = 0;
+            uint64_t w[NW];
 #pragma unroll
-    for (int q = 0; q < NW; ++q) w[q] = 0;
-    for (int i = 0; i < g.K1; ++i) {
-        base += (int64_t)d[i] * g.stride[i];
+            for (int q = 0; q < NW; ++q) w[q] = 0;
+            for (int i = 0; i < g.K1; ++i) {
+                base += (int64_t)d[i] * g.stride[i];
 #pragma unroll
-        for (int q = 0; q < NW; ++q)
-            if (g.word[i] == q) w[q] |= (uint64_t)d[i] << g.shift[i];
+                for (int q = 0; q < NW; ++q)
+                    if (g.word[i] == q) w[q] |= (uint64_t)d[i] << g.shift[i];
+            }
+            const int64_t k = t - b0;
+            s_out[k] = base;
+#pragma unroll
+            for (int q = 0; q < NW; ++q) s_out[(q + 1) * span + k] = (int64_t)w[q];
+            if (t + 1 < next_level) next_in_level(g, d);
+        }
     }
-    rb[t] = base;
+    __syncthreads();
+    const int64_t n = rows - b0 < span ? rows - b0 : span;
+    for (int64_t k = threadIdx.x; k < n; k += blockDim.x) {
+        rb[b0 + k] = s_out[k];
 #pragma unroll
-    for (int q = 0; q < NW; ++q) pw[(int64_t)q * rows + t] = w[q];
+        for (int q = 0; q < NW; ++q) pw[(int64_t)q * rows + b0 + k] = (uint64_t)s_out[(q + 1) * span + k];
+    }
 }
 
 // ------------------------------------------------------------------ a-5
@@ -519,11 +557,18 @@ cudaError_t launch_build_row_index(const RowGeom &g, const int64_t *d_cnt, const
 {
     if (rows <= 0) return cudaSuccess;
     const int bs = 128;
-    const int64_t blocks = (rows + bs - 1) / bs;
+    const int R = rows >= (int64_t)1 << 16 ? 8 : 1;   // slots per thread
+    const int64_t threads = (rows + R - 1) / R;
+    const int64_t blocks = (threads + bs - 1) / bs;
+    const int NWk = g.nwords <= 1 ? 1 : 2;
+    const size_t out_bytes = (size_t)R * bs * 8 * (1 + NWk);
+    const size_t tab = ((size_t)(g.K1 + 1) * (g.rho_max + 1) + g.rho_max + 2) * 8;
+    const int in_smem = tab + out_bytes <= 48 * 1024 ? 1 : 0;
+    const size_t smem = (in_smem ? tab : 0) + out_bytes;
     if (g.nwords <= 1)
-        build_row_index_kernel<1><<<(unsigned)blocks, bs, 0, st>>>(g, d_cnt, d_level_start, rows, d_rb, d_pw);
+        build_row_index_kernel<1><<<(unsigned)blocks, bs, smem, st>>>(g, d_cnt, d_level_start, rows, d_rb, d_pw, R, in_smem);
     else
-        build_row_index_kernel<2><<<(unsigned)blocks, bs, 0, st>>>(g, d_cnt, d_level_start, rows, d_rb, d_pw);
+        build_row_index_kernel<2><<<(unsigned)blocks, bs, smem, st>>>(g, d_cnt, d_level_start, rows, d_rb, d_pw, R, in_smem);
     return cudaGetLastError();
 }
 
