@@ -23,9 +23,27 @@
 
 namespace ptas {
 
+// PTAS_SLOW_CALLS=<ms> (diagnostics): report every checked call slower than
+// <ms> milliseconds of host time, with its source line.
+static double slow_call_ms()
+{
+    static const double v = [] {
+        const char *t = std::getenv("PTAS_SLOW_CALLS");
+        return t ? std::atof(t) : 0.0;
+    }();
+    return v;
+}
+static double host_ms()
+{
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
 #define PT_CK(x)                                                                   \
     do {                                                                           \
+        const double t0__ = slow_call_ms() > 0 ? host_ms() : 0.0;                  \
         cudaError_t e__ = (x);                                                     \
+        if (t0__ > 0 && host_ms() - t0__ > slow_call_ms())                         \
+            std::fprintf(stderr, "[ptas] slow call %.2f ms at dp_engine.cpp:%d: %s\n", \
+                         host_ms() - t0__, __LINE__, #x);                            \
         if (e__ != cudaSuccess) {                                                  \
             cudaGetLastError();                                                    \
             return e__ == cudaErrorMemoryAllocation ? PTAS_ENOMEM : PTAS_ECUDA;    \
