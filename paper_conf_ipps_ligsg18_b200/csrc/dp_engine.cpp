@@ -327,8 +327,12 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     if (in_place) {
         table = rq.ext_table;
     } else {
-        int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
-        if (ibytes > budget) return PTAS_ETOOBIG;
+        // auto budget: query free HBM only when the table has to grow
+        // (cudaMemGetInfo costs ~0.1 ms per call)
+        if (rq.budget > 0 || (size_t)ibytes > table_.cap) {
+            const int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
+            if (ibytes > budget) return PTAS_ETOOBIG;
+        }
         PT_CK(table_.ensure((size_t)ibytes));
         table = table_.p;
     }
@@ -463,6 +467,104 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         }
         PT_CK(stage_.ensure(mx));
     }
+    // ---- dataflow runs (D7): runs of row-levels filled by ONE
+    // launch each.  PTAS_DF = 0: off (one launch per row-level); 1: the whole
+    // DP in one launch, one row set per warp; 2: maximal runs of row-levels
+    // with at most PTAS_DF_ROWS rows (default 2 * 32 * SMs) in one launch
+    // each, the other levels one launch each; 3: the whole DP in dataflow
+    // launches, runs of levels with at most PTAS_DF_SPLIT_ROWS rows with one
+    // row set per block (the 8 warps split the prefix walk: shorter latency
+    // per row for the narrow levels on the critical path), the others with
+    // one row set per warp (the default).  Only for unsharded DPs on the packed kernel.
+    struct DfRun {
+        int rho0, rho1;        // levels rho0 .. rho1 (inclusive)
+        int nsplit;
+        int64_t max_rows;
+        int64_t total_sets;
+        size_t plan_off;       // int32 offset into dfplan_
+    };
+    std::vector<DfRun> runs;
+    {
+        const char *dfs = std::getenv("PTAS_DF");
+        const int df_mode = dfs && dfs[0] ? std::atoi(dfs) : 3;
+        const char *dfr = std::getenv("PTAS_DF_ROWS");
+        const char *dsr = std::getenv("PTAS_DF_SPLIT_ROWS");
+        const int64_t df_rows = df_mode == 1 ? INT64_MAX
+                                             : (dfr && dfr[0] ? std::atoll(dfr) : (int64_t)2 * 32 * sm_count_);
+        // (measured on M2s/M3s/M4s/M5s: 600..8000 within a few %, 2000 best overall)
+        const int64_t split_rows = dsr && dsr[0] ? std::atoll(dsr) : 2000;
+        if (df_mode > 0 && G == 1 && !force_scalar && g.rho_max >= 1) {
+            if (df_mode == 3) {
+                for (int rho = 0; rho <= g.rho_max;) {
+                    const bool sp = cnt[rho] <= split_rows;
+                    int r1 = rho;
+                    while (r1 + 1 <= g.rho_max && (cnt[r1 + 1] <= split_rows) == sp) ++r1;
+                    runs.push_back({rho, r1, sp ? 8 : 1, 0, 0, 0});
+                    rho = r1 + 1;
+                }
+            } else {
+                for (int rho = 0; rho <= g.rho_max;) {
+                    if (cnt[rho] > df_rows) {
+                        ++rho;
+                        continue;
+                    }
+                    int r1 = rho;
+                    while (r1 + 1 <= g.rho_max && cnt[r1 + 1] <= df_rows) ++r1;
+                    if (r1 > rho) runs.push_back({rho, r1, 1, 0, 0, 0});
+                    rho = r1 + 1;
+                }
+            }
+        }
+        std::vector<int32_t> plan;
+        std::vector<DfRun> ok;
+        for (DfRun rn : runs) {
+            for (int rho = rn.rho0; rho <= rn.rho1; ++rho) rn.max_rows = std::max(rn.max_rows, cnt[rho]);
+            const int rpw = swar_df_rows_per_set(e, g, J0, rn.max_rows, sm_count_);
+            if (rpw <= 0) continue;
+            const int nl = rn.rho1 - rn.rho0 + 1;
+            rn.plan_off = plan.size();
+            int64_t sets = 0;
+            plan.resize(plan.size() + 2 * (size_t)(nl + 1));
+            int32_t *ss = plan.data() + rn.plan_off, *sl = ss + nl + 1;
+            for (int l = 0; l <= nl; ++l) {
+                ss[l] = (int32_t)sets;
+                sl[l] = (int32_t)lstart[rn.rho0 + l];
+                if (l < nl) sets += (cnt[rn.rho0 + l] + rpw - 1) / rpw;
+            }
+            rn.total_sets = sets;
+            ok.push_back(rn);
+        }
+        runs.swap(ok);
+        if (!runs.empty()) {
+            PT_CK(dfplan_.ensure(plan.size() * 4));
+            PT_CK(h2d(dfplan_.p, plan.data(), plan.size() * 4, st));
+            o.h2d += (int64_t)plan.size() * 4;
+            void *old = flags_.p;
+            PT_CK(flags_.ensure((size_t)rows * 4));
+            if (flags_.p != old || df_epoch_ + runs.size() + 1 < df_epoch_) {
+                PT_CK(cudaMemsetAsync(flags_.p, 0, flags_.cap, st));
+                df_epoch_ = 0;
+            }
+            if (!ticket_.p) {
+                PT_CK(ticket_.ensure(8));
+                PT_CK(cudaMemsetAsync(ticket_.p, 0, 8, st));
+                ticket_base_ = 0;
+            }
+        }
+    }
+    DfArgs dfa;
+    std::memset(&dfa, 0, sizeof(dfa));
+    if (!runs.empty()) {
+        dfa.flags = (uint32_t *)flags_.p;
+        dfa.ticket = (unsigned long long *)ticket_.p;
+        for (int i = 0; i < K - 1; ++i) {
+            dfa.rstride[i] = (int32_t)(stride[i] / g.Wp);
+            const int w = bits_of(N[i]) + 1;
+            dfa.dmask[i] = (((uint64_t)1 << (w - 1)) - 1) << g.shift[i];
+        }
+    }
+    size_t next_run = 0;
+
     PT_CK(cudaEventRecord(ev_[1], st));
     // PTAS_LEVEL_TIMES=1: per-row-level device times (events between launches; diagnostics)
     static const bool lvl_times = [] {
@@ -479,6 +581,56 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         const int64_t R = cnt[rho];
         if (lvl_times && rho > 0) PT_CK(cudaEventRecord(lev[rho], st));
         if (R <= 0) continue;
+        if (next_run < runs.size() && runs[next_run].rho0 == rho) {
+            const DfRun &rn = runs[next_run++];
+            dfa.plan = (const int32_t *)dfplan_.p + rn.plan_off;
+            dfa.nlev = rn.rho1 - rn.rho0 + 1;
+            dfa.total_sets = rn.total_sets;
+            dfa.base = ticket_base_;
+            dfa.epoch = ++df_epoch_;
+            dfa.nsplit = rn.nsplit;
+            // PTAS_DF_PROF=1 (with a PTAS_DF_PROFILE=1 build): per-level set timings of the run
+            static const bool df_prof = [] {
+                const char *t = std::getenv("PTAS_DF_PROF");
+                return t && t[0] == '1';
+            }();
+            std::vector<unsigned long long> prof_h;
+            if (df_prof) {
+                prof_h.assign((size_t)6 * dfa.nlev, 0);
+                for (int l = 0; l < dfa.nlev; ++l) prof_h[6 * l + 4] = ~0ull;
+                PT_CK(dfprof_.ensure(prof_h.size() * 8));
+                PT_CK(cudaMemcpyAsync(dfprof_.p, prof_h.data(), prof_h.size() * 8, cudaMemcpyHostToDevice, st));
+                dfa.prof = (unsigned long long *)dfprof_.p;
+            }
+            cudaError_t err = launch_row_fill_swar_df(e, table, g, d_rb, d_pw, rows, (const PrefixEntry *)pref_.p,
+                                                      d_meta_, nC, J0, rn.max_rows, dfa, &ticket_base_, sm_count_,
+                                                      st, (use_pdl && prev_fill) ? 1 : 0, cpref_ok ? index_ : -1);
+            if (err == cudaSuccess && df_prof) {
+                PT_CK(cudaMemcpyAsync(prof_h.data(), dfprof_.p, prof_h.size() * 8, cudaMemcpyDeviceToHost, st));
+                PT_CK(cudaStreamSynchronize(st));
+                const unsigned long long g0 = prof_h[4];
+                std::fprintf(stderr, "[ptas] df run rho %d..%d split %d sigma=%lld: lvl rows sets wait/walk/tail(cyc) ready..done(us)\n",
+                             rn.rho0, rn.rho1, rn.nsplit, (long long)sigma);
+                for (int l = 0; l < dfa.nlev; ++l) {
+                    const unsigned long long *q = prof_h.data() + 6 * l;
+                    const double c = q[0] ? (double)q[0] : 1.0;
+                    std::fprintf(stderr, "  %3d %8lld %7llu %7.0f %7.0f %7.0f %9.2f %9.2f\n", rn.rho0 + l,
+                                 (long long)cnt[rn.rho0 + l], q[0], q[1] / c, q[2] / c, q[3] / c,
+                                 (q[4] - g0) * 1e-3, (q[5] - g0) * 1e-3);
+                }
+                dfa.prof = nullptr;
+            }
+            if (err == cudaSuccess) {
+                prev_fill = true;
+                ++o.fill_launches;
+                if (lvl_times)
+                    for (int r2 = rho + 1; r2 <= rn.rho1; ++r2) PT_CK(cudaEventRecord(lev[r2], st));
+                rho = rn.rho1;
+                continue;
+            }
+            if (err != cudaErrorNotSupported) PT_CK(err);
+            // unsupported geometry: fill the run level by level
+        }
         if (!sharded(R)) {
             PT_CK(fill(table, g, J0, rho, 0, R, nullptr));
             ++o.fill_launches;

@@ -95,6 +95,10 @@ class DpSlot {
     unsigned char *pin_ = nullptr;  // pinned arena
     size_t pin_cap_ = 0, pin_used_ = 0;
     Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_, rowidx_, cpstage_;
+    // dataflow fill (D7): per-row ready flags, ticket counter, run plans
+    Buf flags_, ticket_, dfplan_, dfprof_;
+    uint32_t df_epoch_ = 0;
+    unsigned long long ticket_base_ = 0;
 
     // state of the last DP (for traceback)
     bool last_valid_ = false;

@@ -59,6 +59,24 @@ inline int64_t row_pitch_words(int64_t bytes)
     return (w + ch - 1) / ch * ch;
 }
 
+// Dataflow wavefront (one launch for a run of row-levels rho0 .. rho0+nlev-1,
+// DESIGN.md D7): warps take row sets in level order from a ticket counter and
+// wait only for the ready flags of each row's unit predecessors p - e_i.
+// Row sets never straddle a level (a set never waits on itself).
+struct DfArgs {
+    const int32_t *plan;          // device: [nlev+1] first set of each level, then [nlev+1] first slot
+    uint32_t *flags;              // device: one ready flag per row (row-major row id)
+    unsigned long long *ticket;   // device: monotone ticket counter of the slot
+    unsigned long long base;      // ticket value of set 0 of this launch
+    int64_t total_sets;
+    int32_t nlev;
+    uint32_t epoch;               // flag value meaning "row done in this launch"
+    int32_t nsplit;               // 1: one row set per warp; 8: per block (the warps split the prefix walk)
+    unsigned long long *prof;     // diagnostics build (PTAS_DF_PROFILE): 6 counters per level, else null
+    int32_t rstride[MAXK];        // rows between p and p - e_i (leading digit i)
+    uint64_t dmask[MAXK];         // bits of leading digit i inside its packed word g.word[i]
+};
+
 // Device-side summary written by the planning kernels and read back once.
 struct DpMeta {
     int64_t nC;            // |C|
@@ -106,6 +124,17 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
                                  int J0, int rho, int64_t slot_begin, int64_t slot_count,
                                  void *compact_out, int sm_count, cudaStream_t st, int pdl,
                                  int cslot);
+// Dataflow launch over a run of row-levels (D7).  rb/pw are the
+// DP's whole row index (slot 0 = row-level 0).  rows_per_set: see
+// swar_df_rows_per_set.  *ticket_base advances by the ticket grabs of the
+// launch.  cudaErrorNotSupported -> fill the run level by level instead.
+cudaError_t launch_row_fill_swar_df(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
+                                    int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                    int64_t nP_bound, int J0, int64_t max_level_rows, const DfArgs &df,
+                                    unsigned long long *ticket_base, int sm_count, cudaStream_t st, int pdl,
+                                    int cslot);
+// Rows per row set the dataflow kernel will use for this geometry (0 = unsupported).
+int swar_df_rows_per_set(int e, const RowGeom &g, int J0, int64_t max_level_rows, int sm_count);
 // Copies the DP's prefix offsets/Jmax into the fill kernel's constant bank
 // (after build_prefix, before the fill loop); cudaErrorNotSupported when the
 // prefix list is too long (the kernels then read it from shared memory).

@@ -42,6 +42,19 @@ PTAS_SWAR_DECL(u16_nw1)
 PTAS_SWAR_DECL(u16_nw2)
 #undef PTAS_SWAR_DECL
 
+#define PTAS_SWAR_DF_DECL(tag)                                                                        \
+    cudaError_t launch_row_fill_swar_df_##tag(int e, void *table, const RowGeom &g, const int64_t *rb,     \
+                                              const uint64_t *pw, int64_t pw_stride,                       \
+                                              const PrefixEntry *d_pref, const DpMeta *d_meta,              \
+                                              int64_t nP_bound, int J0, int64_t max_level_rows,             \
+                                              const DfArgs &df, unsigned long long *ticket_base,            \
+                                              int sm_count, cudaStream_t st, int pdl, int cslot);
+PTAS_SWAR_DF_DECL(u8_nw1)
+PTAS_SWAR_DF_DECL(u8_nw2)
+PTAS_SWAR_DF_DECL(u16_nw1)
+PTAS_SWAR_DF_DECL(u16_nw2)
+#undef PTAS_SWAR_DF_DECL
+
 cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
                                  int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
                                  int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
@@ -58,6 +71,25 @@ cudaError_t launch_row_fill_swar(int e, void *table, const RowGeom &g, const int
     if (!two) PTAS_SWAR_CALL(u16_nw1);
     PTAS_SWAR_CALL(u16_nw2);
 #undef PTAS_SWAR_CALL
+}
+
+cudaError_t launch_row_fill_swar_df(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
+                                    int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                    int64_t nP_bound, int J0, int64_t max_level_rows, const DfArgs &df,
+                                    unsigned long long *ticket_base, int sm_count, cudaStream_t st, int pdl,
+                                    int cslot)
+{
+    const bool two = g.nwords > 1;
+#define PTAS_SWAR_DF_CALL(tag)                                                                            \
+    return launch_row_fill_swar_df_##tag(e, table, g, rb, pw, pw_stride, d_pref, d_meta, nP_bound, J0,     \
+                                         max_level_rows, df, ticket_base, sm_count, st, pdl, cslot)
+    if (e == 1) {
+        if (!two) PTAS_SWAR_DF_CALL(u8_nw1);
+        PTAS_SWAR_DF_CALL(u8_nw2);
+    }
+    if (!two) PTAS_SWAR_DF_CALL(u16_nw1);
+    PTAS_SWAR_DF_CALL(u16_nw2);
+#undef PTAS_SWAR_DF_CALL
 }
 
 cudaError_t prepare_const_prefix(const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound, int e, int nwords,

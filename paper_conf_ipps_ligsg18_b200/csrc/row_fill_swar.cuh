@@ -27,6 +27,7 @@
 // Positions x - J < 0 take the row's first entry (the clamp min(x, J)).
 #include <cstdint>
 #include <cstdlib>
+#include <cstring>
 #include <cuda_runtime.h>
 #include <mutex>
 #include <unordered_map>
@@ -60,12 +61,73 @@ __device__ __forceinline__ void fill_words(Words<CH> &w, uint32_t x)
     for (int t = 0; t < CH; ++t) w.v[t] = x;
 }
 
+#ifndef PTAS_DF_PROFILE
+#define PTAS_DF_PROFILE 0
+#endif
+#ifndef PTAS_DF_LD_CG
+#define PTAS_DF_LD_CG 0
+#endif
+// Coherent 32-bit loads of table words for the dataflow kernel (the table is
+// written during the launch, so the read-only path is not allowed): ordinary
+// weak loads, kept after the flag acquire by `volatile` (the acquire
+// invalidates L1); PTAS_DF_LD_CG=1 reads through L2 only.
+__device__ __forceinline__ uint32_t ld_co(const uint32_t *p)
+{
+    uint32_t v;
+    if (PTAS_DF_LD_CG) asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    else asm volatile("ld.global.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint2 ld_co2(const uint32_t *p)
+{
+    uint2 v;
+    if (PTAS_DF_LD_CG) asm volatile("ld.global.cg.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
+    else asm volatile("ld.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint4 ld_co4(const uint32_t *p)
+{
+    uint4 v;
+    if (PTAS_DF_LD_CG)
+        asm volatile("ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    else
+        asm volatile("ld.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
 // CH consecutive words at p (4*CH-byte aligned: the pitch is a multiple of CH words)
-template <int CH>
+template <int CH, bool CO = false>
 __device__ __forceinline__ Words<CH> load_words(const uint32_t *p)
 {
     Words<CH> w;
-    if constexpr (CH == 1) {
+    if constexpr (CO) {
+        if constexpr (CH == 1) {
+            w.v[0] = ld_co(p);
+        } else if constexpr (CH == 2) {
+            const uint2 a = ld_co2(p);
+            w.v[0] = a.x;
+            w.v[1] = a.y;
+        } else {
+#pragma unroll
+            for (int c = 0; c < CH; c += 4) {
+                const uint4 a = ld_co4(p + c);
+                w.v[c] = a.x;
+                w.v[c + 1] = a.y;
+                w.v[c + 2] = a.z;
+                w.v[c + 3] = a.w;
+            }
+        }
+    } else if constexpr (CH == 1) {
         w.v[0] = __ldg(p);
     } else if constexpr (CH == 2) {
         const uint2 a = __ldg(reinterpret_cast<const uint2 *>(p));
@@ -238,13 +300,16 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
 // CH: words per lane; WIN: largest prefix window shift in bytes the kernel
 // supports (J0 * e <= 4, <= 8, or 0 = any);
 // CPREF: prefix offsets from the constant bank; SPLIT: the warps of a block
-// share rows (small row-levels with long prefix lists).
-template <typename E, int NW, int CH, int WIN, bool CPREF, bool SPLIT>
+// share rows (small row-levels with long prefix lists); DF: dataflow launch
+// over a run of row-levels (D7; rho, slot_begin and slot_count
+// are unused, the row sets come from df).
+template <typename E, int NW, int CH, int WIN, bool CPREF, bool SPLIT, bool DF>
 __global__ void __launch_bounds__(256)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
-                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int Lg, int nsplit_arg, int cslot)
+                     int rho, int64_t slot_begin, int64_t slot_count, E *compact, int Lg, int nsplit_arg, int cslot,
+                     const DfArgs df)
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
@@ -252,7 +317,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #define PTAS_PB1 16
 #endif
 #ifndef PTAS_PB2
-#define PTAS_PB2 4
+#define PTAS_PB2 8
 #endif
     constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);   // gathers in flight per lane (prefix batch)
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -304,10 +369,20 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         guard[w] = g.guard[w];
         maxs[w] = g.maxs[w];
     }
+    // DF: per-level first set / first slot of the run, in shared memory
+    int32_t *s_set = reinterpret_cast<int32_t *>(s_red + (size_t)(256 / 32) * 2 * 8 * 32);
+    int32_t *s_sl = s_set + (DF ? df.nlev + 1 : 0);
+    // DF + SPLIT: the block's ticket (8-byte aligned after the plan)
+    unsigned long long *s_tk =
+        reinterpret_cast<unsigned long long *>(s_set + ((DF ? 2 * (df.nlev + 1) : 0) + 1) / 2 * 2);
+    if constexpr (DF) {
+        for (int i = threadIdx.x; i < 2 * (df.nlev + 1); i += blockDim.x) s_set[i] = df.plan[i];
+        __syncthreads();
+    }
     // first row set's index entries, loaded before waiting on the previous level
     int64_t nrb = 0;
     uint64_t npw[NW];
-    {
+    if constexpr (!DF) {
         const int64_t slot = gw * rpw + grp;
         const bool ok = grp < rpw && slot < slot_count;
 #pragma unroll
@@ -316,20 +391,59 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     }
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
+    // DF row sets: tickets in level order; set t of level lv covers slots
+    // s_sl[lv] + (t - s_set[lv]) * rpw + grp (< s_sl[lv+1])
+    int df_lv = 0;            // level (within the run) of the last mapped ticket
+    int64_t tk = 0;          // current ticket
+    int cur_lv = 0;
+    int64_t cur_slot = 0, nxt_slot = 0;
+    bool cur_ok = false, nxt_ok = false;
+    const uint32_t Lw = (uint32_t)(g.Wp * EB / 4);
+    auto df_map = [&](int64_t t, int64_t &slot, bool &ok) {
+        while (t >= s_set[df_lv + 1]) ++df_lv;
+        slot = (int64_t)s_sl[df_lv] + (t - s_set[df_lv]) * rpw + grp;
+        ok = grp < rpw && slot < s_sl[df_lv + 1];
+    };
+    if constexpr (DF) {
+        unsigned long long t0 = 0;
+        if (SPLIT) {
+            if (threadIdx.x == 0) *s_tk = atomicAdd(df.ticket, 1ull);
+            __syncthreads();
+            t0 = *s_tk;
+            __syncthreads();   // every warp has read it before thread 0 stores the next ticket
+        } else {
+            if (lane == 0) t0 = atomicAdd(df.ticket, 1ull);
+            t0 = __shfl_sync(FULL, t0, 0);
+        }
+        tk = (int64_t)(t0 - df.base);
+        if (tk < df.total_sets) {
+            df_map(tk, cur_slot, cur_ok);
+            cur_lv = df_lv;
+#pragma unroll
+            for (int w = 0; w < NW; ++w) npw[w] = cur_ok ? pwa[(int64_t)w * pw_stride + cur_slot] : 0;
+            if (cur_ok) nrb = rb[cur_slot];
+        }
+    }
+
     const uint32_t *tab32 = reinterpret_cast<const uint32_t *>(table);
     // uniform trip count (every warp of the grid runs the same number of row
     // sets; the tail ones are idle) keeps the prefix loop in uniform control flow
     const int64_t nsets = (slot_count + rpw - 1) / rpw;
-    const int64_t iters = (nsets + nw - 1) / nw;
-    for (int64_t it = 0; it < iters; ++it) {
+    const int64_t iters = DF ? 0 : (nsets + nw - 1) / nw;
+    for (int64_t it = 0;; ++it) {
+        if (DF ? tk >= df.total_sets : it >= iters) break;
         const int64_t sb = (it * nw + gw) * rpw;
-        const int64_t slot = sb + grp;
-        const bool rowok = grp < rpw && slot < slot_count;
+        const int64_t slot = DF ? cur_slot : sb + grp;
+        const bool rowok = DF ? cur_ok : (grp < rpw && slot < slot_count);
         const int64_t rowbase = nrb;
         uint64_t pw[NW];
 #pragma unroll
         for (int w = 0; w < NW; ++w) pw[w] = npw[w];
-        {   // prefetch the next row set's index entries
+        unsigned long long tnext = 0;
+        if constexpr (DF) {
+            // next ticket now; its value is consumed after the prefix walk
+            if (SPLIT ? threadIdx.x == 0 : lane == 0) tnext = atomicAdd(df.ticket, 1ull);
+        } else {   // prefetch the next row set's index entries
             const int64_t ns = sb + nw * rpw + grp;
             const bool ok = grp < rpw && ns < slot_count;
 #pragma unroll
@@ -341,12 +455,42 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         // opaque to the compiler: keeps the pointer in registers instead of
         // re-deriving it from the kernel parameters at every gather
         asm volatile("" : "+l"(src));
+        uint32_t rid = 0;   // DF: row-major row id of the group's row (flag index)
+#if PTAS_DF_PROFILE
+        long long pf_t0 = clock64(), pf_t1 = 0, pf_t2 = 0;
+#endif
+        if constexpr (DF) {
+            rid = rowok ? (uint32_t)(rowbase * EB / 4) / Lw : 0u;
+            if (cur_lv > 0) {
+                // wait until every unit predecessor p - e_i (p_i >= 1) is done; by
+                // induction that covers every dominated row, i.e. every source
+                // row p - s' of the prefix walk (rows of the run's first level
+                // read only rows filled before the launch)
+                for (;;) {
+                    bool ok = true;
+                    if (rowok) {
+                        for (int i = xl; i < g.K1; i += Lg) {
+                            const uint64_t wv = NW == 1 ? pw[0] : (g.word[i] ? pw[NW - 1] : pw[0]);
+                            if (wv & df.dmask[i]) ok &= ld_acquire(df.flags + (rid - (uint32_t)df.rstride[i])) == df.epoch;
+                        }
+                    }
+                    if (__all_sync(FULL, ok)) break;
+                    __nanosleep(64);
+                }
+                __syncwarp();
+            }
+        }
         // every prefix dominated by every row of the warp?
         bool interior = rowok;
 #pragma unroll
         for (int w = 0; w < NW; ++w) interior &= (((pw[w] | guard[w]) - maxs[w]) & guard[w]) == guard[w];
         const bool allint = __all_sync(FULL, grp >= rpw || interior);
 
+#if PTAS_DF_PROFILE
+        pf_t1 = clock64();
+        unsigned long long pf_g1 = 0;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(pf_g1));
+#endif
         // ---- cross-row relaxations: acc = min over s' <= p of OPT(p - s', x - min(x, Jmax(s')))
         Words<CH> ae, ao;
         fill_words(ae, 0xffffffffu);
@@ -390,7 +534,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
                     sj[u] = oj.y;
                     const uint32_t *p = src + oj.x;
-                    if ((m >> q) & 1u) cur[u] = load_words<CH>(p);
+                    if ((m >> q) & 1u) cur[u] = load_words<CH, DF>(p);
                     else fill_words(cur[u], 0xffffffffu);
                 }
 #pragma unroll
@@ -421,13 +565,30 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
             }
         }
 
+        // DF: next row set -- map the ticket and start its index loads (they
+        // land during the in-row closure)
+        auto df_next = [&](unsigned long long t) {
+            const int64_t tn = (int64_t)(t - df.base);
+            nxt_ok = false;
+            if (tn < df.total_sets) df_map(tn, nxt_slot, nxt_ok);
+#pragma unroll
+            for (int w = 0; w < NW; ++w) npw[w] = nxt_ok ? pwa[(int64_t)w * pw_stride + nxt_slot] : 0;
+            nrb = nxt_ok ? rb[nxt_slot] : 0;
+            tk = tn;
+        };
+#if PTAS_DF_PROFILE
+        pf_t2 = clock64();
+#endif
+        if constexpr (DF && !SPLIT) df_next(__shfl_sync(FULL, tnext, 0));
         if (SPLIT) {
 #pragma unroll
             for (int t = 0; t < CH; ++t) {
                 s_red[((wid * 2 + 0) * CH + t) * 32 + lane] = ae.v[t];
                 s_red[((wid * 2 + 1) * CH + t) * 32 + lane] = ao.v[t];
             }
+            if (DF && threadIdx.x == 0) *s_tk = tnext;
             __syncthreads();
+            if constexpr (DF) df_next(*s_tk);
             if (wid == 0) {
                 for (int w2 = 1; w2 < nsplit; ++w2) {
 #pragma unroll
@@ -452,7 +613,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     oo.v[t] = 0;
                 }
             }
-            if (rho == 0 && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
+            if ((DF ? rowbase == 0 : rho == 0) && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
             // opt(p, 0) is final (no in-row term at x = 0): the clamp value
             uint32_t f0 = __shfl_sync(FULL, oe.v[0], lane - xl);
             f0 = prmt(f0, 0u, 0x1010u);
@@ -537,9 +698,34 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 }
                 store_words<CH>(out32 + xl * CH, wv);
             }
+            if constexpr (DF) {
+                // release: the row's words are visible at gpu scope before its flag
+                __threadfence();
+                __syncwarp();
+                if (rowok && xl == 0) st_relaxed(df.flags + rid, df.epoch);
+#if PTAS_DF_PROFILE
+                // per level (of the run): sets, wait, walk, tail cycles, first ready, last done (ns)
+                if (df.prof && lane == 0) {
+                    unsigned long long g2;
+                    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g2));
+                    unsigned long long *pr = df.prof + 6 * (size_t)cur_lv;
+                    atomicAdd(pr + 0, 1ull);
+                    atomicAdd(pr + 1, (unsigned long long)(pf_t1 - pf_t0));
+                    atomicAdd(pr + 2, (unsigned long long)(pf_t2 - pf_t1));
+                    atomicAdd(pr + 3, (unsigned long long)(clock64() - pf_t2));
+                    atomicMin(pr + 4, pf_g1);
+                    atomicMax(pr + 5, g2);
+                }
+#endif
+            }
             __syncwarp();
         }  // chain + store (warp 0 in split mode)
         if (SPLIT) __syncthreads();  // s_red reused by the next row set
+        if constexpr (DF) {
+            cur_slot = nxt_slot;
+            cur_ok = nxt_ok;
+            cur_lv = df_lv;
+        }
     }
 }
 
@@ -559,43 +745,60 @@ static int occupancy_of(K kfn, size_t smem, int bs)
     return occ;
 }
 
+// Words per lane CH for a row of Lw words (group width Lg = Lw / CH <= 32),
+// 0 = the packed kernel does not support the geometry.  CH amortises the
+// per-prefix cost over CH words; small row-levels are latency-bound and use
+// CH = 1 (more lanes per row, shorter serial work per lane).  `rows` = rows
+// of the level (per-level launches) or of the largest level of the run (DF).
+static int plan_ch(int e, const RowGeom &g, int J0, int64_t rows, int sm_count, bool df)
+{
+    const int Lw = (int)(g.Wp * e / 4);
+    if ((g.Wp * e) % 4 != 0 || Lw > 256 || J0 * e > 124) return 0;
+    // int32 word offsets: the table (incl. padding) must stay below 2^31 words
+    int64_t rows_all = 1;
+    for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
+    if (rows_all * (int64_t)Lw >= ((int64_t)1 << 31)) return 0;
+    int CH;
+    const char *chs = std::getenv(df ? "PTAS_DF_CH" : "PTAS_SWAR_CH");
+    const char *cht = std::getenv("PTAS_SMALL_LEVEL_ROWS");
+    const int64_t small_rows = cht ? std::atoll(cht) : (int64_t)sm_count * 32;
+    if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
+    else if (chs && chs[0]) CH = std::atoi(chs);
+    else CH = (Lw >= 8 && rows > small_rows) ? 2 : 1;
+    if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
+    if (Lw % CH != 0) {
+        if (Lw > 32) return 0;
+        CH = 1;
+    }
+    const int Lg = Lw / CH;
+    if (Lg < 1 || Lg > 32) return 0;
+    return CH;
+}
+
+static size_t swar_smem(int64_t np, int NW, int nlev_df)
+{
+    return (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * 8 * 32 * 4 +
+           (nlev_df > 0 ? (size_t)8 * (nlev_df + 1) + 16 : 0);
+}
+
 // Host launcher body for one (E, NW): returns cudaErrorNotSupported when the
 // geometry needs the scalar kernel (row longer than 1 KiB, pitch not a
 // multiple of the lane chunk, or a table of 2^31 words or more).
+// df != nullptr: one dataflow launch over the run described by *df.
 template <typename E, int NW>
 static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const int64_t *rb,
                                  const uint64_t *pw, int64_t pw_stride, const PrefixEntry *d_pref,
                                  const DpMeta *d_meta, int64_t nP_bound, int J0, int rho,
                                  int64_t slot_begin, int64_t slot_count, void *compact_out, int sm_count,
-                                 cudaStream_t st, int pdl, int cslot)
+                                 cudaStream_t st, int pdl, int cslot, const DfArgs *df = nullptr,
+                                 unsigned long long *ticket_base = nullptr)
 {
     if (slot_count <= 0) return cudaSuccess;
-    const int Lw = (int)(g.Wp * e / 4);
-    if ((g.Wp * e) % 4 != 0 || Lw > 256 || J0 * e > 124) return cudaErrorNotSupported;
     if (compact_out && ((uintptr_t)compact_out & 15)) return cudaErrorNotSupported;
-    // int32 word offsets: the table (incl. padding) must stay below 2^31 words
-    {
-        int64_t rows_all = 1;
-        for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
-        if (rows_all * (int64_t)Lw >= ((int64_t)1 << 31)) return cudaErrorNotSupported;
-    }
-    // words per lane CH (group width Lg = Lw / CH <= 32): amortise the
-    // per-prefix cost over CH words; small row-levels are latency-bound and
-    // use CH = 1 (more lanes per row, shorter serial work per lane)
-    int CH;
-    const char *chs = std::getenv("PTAS_SWAR_CH");
-    const char *cht = std::getenv("PTAS_SMALL_LEVEL_ROWS");
-    const int64_t small_rows = cht ? std::atoll(cht) : (int64_t)sm_count * 32;
-    if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
-    else if (chs && chs[0]) CH = std::atoi(chs);
-    else CH = (Lw >= 8 && slot_count > small_rows) ? 2 : 1;
-    if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
-    if (Lw % CH != 0) {
-        if (Lw > 32) return cudaErrorNotSupported;
-        CH = 1;
-    }
+    const int CH = plan_ch(e, g, J0, slot_count, sm_count, df != nullptr);
+    if (CH == 0) return cudaErrorNotSupported;
+    const int Lw = (int)(g.Wp * e / 4);
     const int Lg = Lw / CH;
-    if (Lg < 1 || Lg > 32) return cudaErrorNotSupported;
     const int rpw = 32 / Lg;
     const int bs = 256;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
@@ -604,49 +807,62 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // (worth it when a row's prefix walk has several batches of gathers in series)
     const int PBh = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);
     const int64_t split_rows = sp ? std::atoll(sp) : ((np + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
-    const int nsplit = slot_count <= split_rows ? bs / 32 : 1;
-    const size_t smem = (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(bs / 32) * 2 * 8 * 32 * 4;
+    const int nsplit = df ? (df->nsplit > 1 ? bs / 32 : 1) : (slot_count <= split_rows ? bs / 32 : 1);
+    const size_t smem = swar_smem(np, NW, df ? df->nlev : 0);
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     // shifts beyond one word: prefix windows J * e (J <= J0) or chain u16-lane shifts
     // prefix windows beyond two words (J * e > 8, J <= J0) need the generic word fetch;
     // the in-row closure handles any shift (registers up to 8 bytes, else shared memory)
     const int win = J0 * e <= 4 ? 4 : (J0 * e <= 8 ? 8 : 0);
     const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && np >= 64;
+    DfArgs dfa;
+    if (df) dfa = *df;
+    else std::memset(&dfa, 0, sizeof(dfa));
     cudaError_t err;
-#define PTAS_SWAR_GO(E_, NW_, CH_, WIN_)                                                          \
-    do {                                                                                          \
-        auto kfn = cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true>     \
-                                       : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false>)   \
-                         : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true>    \
-                                       : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false>); \
-        if (smem > 48 * 1024) {                                                                   \
-            err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
-                                       (int)smem);                                                \
-            if (err != cudaSuccess) return err;                                                   \
-        }                                                                                         \
-        int64_t blocks;                                                                           \
-        if (nsplit > 1) {                                                                         \
-            blocks = (slot_count + rpw - 1) / rpw;                                                \
-        } else {                                                                                  \
-            /* one resident wave: every warp loops over row sets */                               \
-            blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);   \
-            const int64_t cap = (int64_t)sm_count * occupancy_of(kfn, smem, bs);                  \
-            if (blocks > cap) blocks = cap;                                                       \
-        }                                                                                         \
-        cudaLaunchConfig_t cfg = {};                                                              \
-        cudaLaunchAttribute attr[1];                                                              \
-        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;                          \
-        attr[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;                         \
-        cfg.gridDim = dim3((unsigned)blocks);                                                     \
-        cfg.blockDim = dim3(bs);                                                                  \
-        cfg.dynamicSmemBytes = smem;                                                              \
-        cfg.stream = st;                                                                          \
-        cfg.attrs = attr;                                                                         \
-        cfg.numAttrs = 1;                                                                         \
-        err = cudaLaunchKernelEx(&cfg, kfn, (E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta,    \
-                                 J0, rho, slot_begin, slot_count, (E_ *)compact_out, Lg,          \
-                                 nsplit, cslot);                                                  \
-        if (err != cudaSuccess) return err;                                                       \
+#define PTAS_SWAR_GO(E_, NW_, CH_, WIN_)                                                                  \
+    do {                                                                                                  \
+        auto kfn = df ? (cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true, true>  \
+                                             : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, true>) \
+                               : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true, true> \
+                                             : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, true>)) \
+               : cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true, false>        \
+                                     : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, false>)      \
+                       : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true, false>       \
+                                     : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, false>);    \
+        if (smem > 48 * 1024) {                                                                           \
+            err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);      \
+            if (err != cudaSuccess) return err;                                                           \
+        }                                                                                                 \
+        int64_t blocks;                                                                                   \
+        const int64_t cap = (int64_t)sm_count * occupancy_of(kfn, smem, bs);                              \
+        if (df) {                                                                                         \
+            /* persistent: every block resident, row sets from the ticket counter */                     \
+            const int spb = nsplit > 1 ? 1 : bs / 32;   /* row sets in flight per block */                \
+            blocks = (df->total_sets + spb - 1) / spb;                                                    \
+            if (blocks > cap) blocks = cap;                                                               \
+        } else if (nsplit > 1) {                                                                          \
+            blocks = (slot_count + rpw - 1) / rpw;                                                        \
+        } else {                                                                                          \
+            /* one resident wave: every warp loops over row sets */                                       \
+            blocks = (slot_count + (int64_t)(bs / 32) * rpw - 1) / ((int64_t)(bs / 32) * rpw);           \
+            if (blocks > cap) blocks = cap;                                                               \
+        }                                                                                                 \
+        cudaLaunchConfig_t cfg = {};                                                                      \
+        cudaLaunchAttribute attr[1];                                                                      \
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;                                  \
+        attr[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;                                 \
+        cfg.gridDim = dim3((unsigned)blocks);                                                             \
+        cfg.blockDim = dim3(bs);                                                                          \
+        cfg.dynamicSmemBytes = smem;                                                                      \
+        cfg.stream = st;                                                                                  \
+        cfg.attrs = attr;                                                                                 \
+        cfg.numAttrs = 1;                                                                                 \
+        err = cudaLaunchKernelEx(&cfg, kfn, (E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta, J0, rho,   \
+                                 slot_begin, slot_count, (E_ *)compact_out, Lg, nsplit, cslot, dfa);      \
+        if (err != cudaSuccess) return err;                                                               \
+        /* every grabbing warp (block in split mode) ends with exactly one failed grab */               \
+        if (df && ticket_base) *ticket_base += (unsigned long long)df->total_sets +                       \
+                                               (unsigned long long)blocks * (nsplit > 1 ? 1 : bs / 32);   \
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
     do {                                                                                          \
@@ -661,6 +877,18 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
 #undef PTAS_SWAR_CASE
 #undef PTAS_SWAR_GO
     return cudaGetLastError();
+}
+
+template <typename E, int NW>
+static cudaError_t launch_swar_df_impl(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
+                                       int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                       int64_t nP_bound, int J0, int64_t max_level_rows, const DfArgs &df,
+                                       unsigned long long *ticket_base, int sm_count, cudaStream_t st, int pdl,
+                                       int cslot)
+{
+    if (df.total_sets <= 0) return cudaSuccess;
+    return launch_swar_impl<E, NW>(e, table, g, rb, pw, pw_stride, d_pref, d_meta, nP_bound, J0, 0, 0,
+                                   max_level_rows, nullptr, sm_count, st, pdl, cslot, &df, ticket_base);
 }
 
 }  // namespace swar

@@ -18,4 +18,14 @@ cudaError_t prepare_const_prefix_u8_nw2(const PrefixEntry *d_pref, const DpMeta 
     return swar::prepare_const_prefix_tu(d_pref, d_meta, nP_bound, e, cslot, d_staging, st);
 }
 
+cudaError_t launch_row_fill_swar_df_u8_nw2(int e, void *table, const RowGeom &g, const int64_t *rb,
+                                    const uint64_t *pw, int64_t pw_stride, const PrefixEntry *d_pref,
+                                    const DpMeta *d_meta, int64_t nP_bound, int J0, int64_t max_level_rows,
+                                    const DfArgs &df, unsigned long long *ticket_base, int sm_count,
+                                    cudaStream_t st, int pdl, int cslot)
+{
+    return swar::launch_swar_df_impl<uint8_t, 2>(e, table, g, rb, pw, pw_stride, d_pref, d_meta, nP_bound, J0,
+                                              max_level_rows, df, ticket_base, sm_count, st, pdl, cslot);
+}
+
 }  // namespace ptas

@@ -125,8 +125,17 @@ def test_g1_golden(P):
     assert opt == 2
 
 
+@pytest.fixture(params=["default", "0"], ids=["df-default", "level-launches"])
+def fillmode(request, monkeypatch):
+    """default: the library's fill schedule (dataflow runs, DESIGN.md D7);
+    "0": one launch per row-level."""
+    if request.param != "default":
+        monkeypatch.setenv("PTAS_DF", request.param)
+    return request.param
+
+
 @pytest.mark.parametrize("K", [1, 2, 3, 4, 5, 6, 7, 8, 9])
-def test_dp_fill_random_uint8(P, K):
+def test_dp_fill_random_uint8(P, K, fillmode):
     rng = np.random.default_rng(1000 + K)
     maxN = {1: 200, 2: 60, 3: 25, 4: 12, 5: 8, 6: 6, 7: 4, 8: 3, 9: 3}[K]
     for _ in range(12):
@@ -135,7 +144,7 @@ def test_dp_fill_random_uint8(P, K):
 
 
 @pytest.mark.parametrize("K", [1, 2, 3, 4])
-def test_dp_fill_random_uint16(P, K):
+def test_dp_fill_random_uint16(P, K, fillmode):
     rng = np.random.default_rng(2000 + K)
     for _ in range(4):
         N = rng.integers(1, {1: 300, 2: 200, 3: 60, 4: 20}[K], K).astype(np.int32)
@@ -146,7 +155,7 @@ def test_dp_fill_random_uint16(P, K):
         _check_table(P, N, r, T)
 
 
-def test_dp_fill_long_rows_ragged(P):
+def test_dp_fill_long_rows_ragged(P, fillmode):
     # W = 71 (3 chunks of 32, ragged), small last size -> long in-row chains (J0 large)
     _check_table(P, np.array([5, 4, 70], np.int32), np.array([90, 70, 11], np.int64), 200)
     _check_table(P, np.array([3, 3, 3, 100], np.int32), np.array([50, 60, 70, 7], np.int64), 250)
@@ -194,6 +203,7 @@ def test_dp_fill_scalar_kernel(P, monkeypatch):
 def test_dp_fill_row_split_modes(P, monkeypatch, split):
     # small-level mode (8 warps share a row set) forced on / off for every level
     monkeypatch.setenv("PTAS_SPLIT_ROWS", split)
+    monkeypatch.setenv("PTAS_DF", "0")   # one launch per row-level (the knob is theirs)
     rng = np.random.default_rng(57)
     for K in (2, 3, 5, 7):
         for _ in range(3):
@@ -207,6 +217,7 @@ def test_dp_fill_row_split_modes(P, monkeypatch, split):
 def test_dp_fill_lane_layouts(P, monkeypatch, ch):
     # words per lane forced (group width Lg = ceil(words/CH), any value 1..32)
     monkeypatch.setenv("PTAS_SWAR_CH", ch)
+    monkeypatch.setenv("PTAS_DF", "0")   # one launch per row-level (the knob is theirs)
     for W in (3, 5, 7, 13, 20, 29, 33, 61, 100, 127):
         _check_table(P, np.array([3, 4, W - 1], np.int32), np.array([35, 50, 21], np.int64), 110)
     rng = np.random.default_rng(int(ch))
@@ -223,7 +234,7 @@ def test_dp_fill_very_long_rows(P):
     _check_table(P, np.array([1, 1, 300], np.int32), np.array([50, 40, 7], np.int64), 120)
 
 
-def test_dp_fill_padding_pitches(P):
+def test_dp_fill_padding_pitches(P, fillmode):
     # row byte lengths 1..9 (u8) and odd u16 lengths: every padding case of the packed kernel
     for W in range(1, 10):
         _check_table(P, np.array([4, 3, W - 1], np.int32), np.array([35, 50, 21], np.int64), 110)
@@ -245,7 +256,7 @@ def test_dp_fill_device_torch(P):
     assert opt == want[tuple(N)]
 
 
-def test_dp_fill_two_word_packing(P, monkeypatch):
+def test_dp_fill_two_word_packing(P, fillmode, monkeypatch):
     # force the leading digits into two 64-bit words (exercises the NW=2 kernels)
     monkeypatch.setenv("PTAS_FORCE_TWO_WORDS", "1")
     rng = np.random.default_rng(77)
@@ -312,7 +323,7 @@ def test_solve_g2(P):
     assert got["assignment"].tolist() == g["assignment"]
 
 
-def test_solve_medium_instances(P):
+def test_solve_medium_instances(P, fillmode):
     # shaped like the paper's workloads but small enough for the oracle
     for (n, m, eps, seed) in [(40, 8, 0.3, 1), (60, 14, 0.3, 2), (50, 10, 0.2, 3), (30, 5, 0.15, 4)]:
         p = jobs(n, 1000, seed)
@@ -368,7 +379,7 @@ def _subbox(N, cap_sigma=2_000_000):
 
 
 @pytest.mark.parametrize("name", ["M2s", "M4s", "M3s"])
-def test_full_size_dp_sampled(P, name):
+def test_full_size_dp_sampled(P, fillmode, name):
     """Full-size DP of the workload at T = LB (its largest probe): exact parity
     on a sub-box (the DP restricted to n <= N' equals the oracle's DP on N'),
     Eq. 1 re-checked at sampled states, and invariants on the whole table."""

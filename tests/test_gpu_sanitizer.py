@@ -1,5 +1,5 @@
 """compute-sanitizer over the fill kernels (memcheck; racecheck on the split
-mode's shared-memory reduction).  Small geometries that exercise every lane
+mode's shared-memory reduction and the dataflow kernel's block ticket).  Small geometries that exercise every lane
 layout: group widths that do not divide 32 (idle lanes), multi-word shifts
 (GEN path), vector chunks CH = 1/2/4/8, uint8 and uint16 tables, split mode.
 Parity of the same cases is checked in test_gpu_parity.py; here only memory
@@ -61,9 +61,22 @@ def test_memcheck_fill_layouts():
 
 @pytest.mark.timeout(1200)
 def test_memcheck_split_mode_and_forced_chunks():
-    _run("memcheck", {"PTAS_SPLIT_ROWS": "1000000000", "PTAS_SWAR_CH": "2"})
+    _run("memcheck", {"PTAS_SPLIT_ROWS": "1000000000", "PTAS_SWAR_CH": "2", "PTAS_DF": "0"})
 
 
 @pytest.mark.timeout(1800)
 def test_racecheck_split_mode():
-    _run("racecheck", {"PTAS_SPLIT_ROWS": "1000000000"})
+    _run("racecheck", {"PTAS_SPLIT_ROWS": "1000000000", "PTAS_DF": "0"})
+
+
+# dataflow launches (D7): warp row sets, block row sets (shared-memory ticket), mixed runs
+@pytest.mark.timeout(1200)
+@pytest.mark.parametrize("env", [{"PTAS_DF": "1"}, {"PTAS_DF": "3", "PTAS_DF_SPLIT_ROWS": "1000000000"},
+                                 {"PTAS_DF": "3", "PTAS_DF_SPLIT_ROWS": "3"}])
+def test_memcheck_dataflow(env):
+    _run("memcheck", env)
+
+
+@pytest.mark.timeout(1800)
+def test_racecheck_dataflow_split():
+    _run("racecheck", {"PTAS_DF": "3", "PTAS_DF_SPLIT_ROWS": "1000000000"})
