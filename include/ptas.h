@@ -72,6 +72,12 @@ typedef struct {
     void *stream;               /* cudaStream_t for all device work of the call
                                    (NULL = the library's own stream); the call
                                    still returns only when its work is done       */
+    int32_t speculate;          /* P = 1, SINGLE mode: evaluate the next levels of
+                                   Alg 1's bisection tree concurrently while the
+                                   DPs are small (-1 = library default, 0 = off,
+                                   d = up to 2^d - 1 probes in flight).  The probe
+                                   sequence, T* and the schedule are those of
+                                   Alg 1 (D8); only time changes.      */
 } ptas_options;
 
 typedef struct {
@@ -92,6 +98,9 @@ typedef struct {
                                `relaxations`; equal on the scalar kernel      */
     double exec_bytes;      /* sum (relax_executed + sigma) * e: the table bytes
                                the fill kernels gather and write              */
+    int32_t spec_dps;       /* DPs evaluated speculatively (options.speculate) */
+    int32_t spec_wasted;    /* of which never probed by the search (their work
+                               is not counted in the fields above)            */
 } ptas_stats;
 
 typedef struct {

@@ -20,7 +20,8 @@ __all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "dp_t
 
 
 def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, budget: int = 0,
-            memoize: bool = True, virtual_shards: int = 1, layout: int = 0, stream=None) -> PtasOptions:
+            memoize: bool = True, virtual_shards: int = 1, layout: int = 0, stream=None,
+            speculate: int = -1) -> PtasOptions:
     o = PtasOptions()
     lib().ptas_default_options(ctypes.byref(o))
     o.probes_per_round = int(P)
@@ -31,6 +32,7 @@ def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, bu
     o.memoize = int(bool(memoize))
     o.virtual_shards = int(virtual_shards)
     o.layout = int(layout)
+    o.speculate = int(speculate)
     o.stream = None if stream is None else ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
     return o
 

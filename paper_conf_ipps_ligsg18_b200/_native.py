@@ -26,7 +26,8 @@ vp = ctypes.c_void_p
 class PtasOptions(ctypes.Structure):
     _fields_ = [("probes_per_round", ctypes.c_int32), ("mode", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("comm", vp), ("table_budget_bytes", ctypes.c_int64), ("memoize", ctypes.c_int32),
-                ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32), ("stream", vp)]
+                ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32), ("stream", vp),
+                ("speculate", ctypes.c_int32)]
 
 
 class PtasStats(ctypes.Structure):
@@ -37,7 +38,7 @@ class PtasStats(ctypes.Structure):
                 ("total_seconds", ctypes.c_double), ("alg_bytes", ctypes.c_double), ("states", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int32), ("fill_launches", ctypes.c_int32),
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64), ("relax_executed", ctypes.c_double),
-                ("exec_bytes", ctypes.c_double)]
+                ("exec_bytes", ctypes.c_double), ("spec_dps", ctypes.c_int32), ("spec_wasted", ctypes.c_int32)]
 
     def to_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

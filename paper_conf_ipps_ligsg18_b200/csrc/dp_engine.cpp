@@ -148,6 +148,9 @@ int DpSlot::init(int device, int sm_count, int index)
     PT_CK(cudaStreamCreateWithFlags(&stream_, cudaStreamNonBlocking));
     for (auto &ev : ev_) PT_CK(cudaEventCreate(&ev));
     PT_CK(cudaEventCreateWithFlags(&ev_sync_, cudaEventDisableTiming));
+    PT_CK(cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking));
+    PT_CK(cudaEventCreateWithFlags(&ev_fork_, cudaEventDisableTiming));
+    PT_CK(cudaEventCreateWithFlags(&ev_join_, cudaEventDisableTiming));
     PT_CK(cudaMalloc(&d_meta_, sizeof(DpMeta)));
     PT_CK(cudaMallocHost(&h_meta_, sizeof(DpMeta)));
     PT_CK(cudaMallocHost(&h_scalar_, 64));
@@ -369,8 +372,12 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     PT_CK(rowidx_.ensure((size_t)rows * 8 * (1 + NWk)));
     int64_t *d_rb = (int64_t *)rowidx_.p;
     uint64_t *d_pw = (uint64_t *)(d_rb + rows);
+    // on the side stream: overlaps the enumeration below and its host round trip
+    PT_CK(cudaEventRecord(ev_fork_, st));
+    PT_CK(cudaStreamWaitEvent(side_, ev_fork_, 0));
     PT_CK(launch_build_row_index(g, (const int64_t *)cnt_.p, (const int64_t *)cnt_.p + cnt.size(), rows, d_rb,
-                                 d_pw, st));
+                                 d_pw, side_));
+    PT_CK(cudaEventRecord(ev_join_, side_));
     ++o.launches;
     const int64_t *d_r = (const int64_t *)small_.p;
     const int64_t *d_stride = (const int64_t *)((unsigned char *)small_.p + K * 8);
@@ -565,6 +572,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     }
     size_t next_run = 0;
 
+    PT_CK(cudaStreamWaitEvent(st, ev_join_, 0));   // row index ready
     PT_CK(cudaEventRecord(ev_[1], st));
     // PTAS_LEVEL_TIMES=1: per-row-level device times (events between launches; diagnostics)
     static const bool lvl_times = [] {
@@ -589,6 +597,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             dfa.base = ticket_base_;
             dfa.epoch = ++df_epoch_;
             dfa.nsplit = rn.nsplit;
+            dfa.grid_div = rq.grid_div > 1 ? rq.grid_div : 1;
             // PTAS_DF_PROF=1 (with a PTAS_DF_PROFILE=1 build): per-level set timings of the run
             static const bool df_prof = [] {
                 const char *t = std::getenv("PTAS_DF_PROF");

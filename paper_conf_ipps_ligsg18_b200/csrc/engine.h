@@ -32,6 +32,7 @@ struct DpRequest {
     cudaStream_t stream = nullptr;  // nullptr = engine stream
     const ShardCtx *shard = nullptr;
     int64_t budget = 0;           // bytes allowed for the table (0 = auto)
+    int grid_div = 1;             // >1: this many DPs run concurrently; persistent grids take 1/grid_div of the GPU
 };
 
 struct DpOutcome {
@@ -89,6 +90,10 @@ class DpSlot {
     cudaStream_t stream_ = nullptr;
     cudaEvent_t ev_[4] = {nullptr, nullptr, nullptr, nullptr};
     cudaEvent_t ev_sync_ = nullptr;
+    // side stream: the a-4 row index is built concurrently with the a-3
+    // enumeration and its host round trip (fork/join events)
+    cudaStream_t side_ = nullptr;
+    cudaEvent_t ev_fork_ = nullptr, ev_join_ = nullptr;
     DpMeta *d_meta_ = nullptr;
     DpMeta *h_meta_ = nullptr;     // pinned
     int64_t *h_scalar_ = nullptr;  // pinned

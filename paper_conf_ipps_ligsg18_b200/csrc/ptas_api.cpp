@@ -276,6 +276,44 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     // stream, slot 0 uses it; the call is host-synchronous either way.
     const char *ncs = std::getenv("PTAS_NO_CONCURRENT");
     const bool concurrent = opt.mode == PTAS_MODE_SINGLE && !(ncs && ncs[0] == '1');
+    // Runs the jobs concurrently (slots 0..), outcomes in outs; grid_div > 0:
+    // persistent fill grids take 1/(jobs in flight) of the GPU each.
+    auto run_jobs = [&](std::vector<Classified> &cls_v, std::vector<int64_t> &T_v,
+                        std::vector<std::vector<int64_t>> &key_v, std::vector<DpOutcome> &outs_all,
+                        bool share_grid) -> int {
+        const int nj = (int)cls_v.size();
+        outs_all.assign(nj, DpOutcome());
+        for (int j0 = 0; j0 < nj; j0 += MAX_SLOTS) {
+            const int nb = std::min(MAX_SLOTS, nj - j0);
+            std::vector<DpSlot *> sl(nb);
+            for (int b = 0; b < nb; ++b) {
+                int r2 = eng->slot(b, &sl[b]);
+                if (r2) return r2;
+            }
+            std::vector<int> rcs(nb, PTAS_OK);
+            std::vector<std::vector<int>> orders(nb);
+            for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, opt.layout);
+            auto work = [&](int b) {
+                if (cudaSetDevice(dev) != cudaSuccess) {
+                    rcs[b] = PTAS_ECUDA;
+                    return;
+                }
+                DpRequest rq = make_rq(cls_v[j0 + b], T_v[j0 + b], nullptr, orders[b],
+                                       b == 0 ? (cudaStream_t)opt.stream : nullptr);
+                rq.grid_div = share_grid ? nb : 1;
+                rcs[b] = sl[b]->run_dp(rq, &outs_all[j0 + b]);
+            };
+            std::vector<std::thread> th;
+            for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
+            work(0);
+            for (auto &t : th) t.join();
+            for (int b = 0; b < nb; ++b) {
+                if (rcs[b]) return rcs[b];
+                slot_key[b] = key_v[j0 + b];
+            }
+        }
+        return PTAS_OK;
+    };
     auto run_many = [&](std::vector<Classified> &cls_v, std::vector<int64_t> &T_v,
                         std::vector<std::vector<int64_t>> &key_v, std::vector<int32_t> &opt_v) -> int {
         const int nj = (int)cls_v.size();
@@ -314,9 +352,92 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         return PTAS_OK;
     };
 
+    // ---- speculative bisection (D8).  With P = 1 the probes are
+    // Alg 1's; when the next probe's DP is not known yet, the next `depth`
+    // levels of the bisection tree below [LB, UB] (both outcomes of every
+    // probe) whose tables are small are evaluated concurrently with it.  A
+    // speculative result is used only when Alg 1 actually probes that key,
+    // and only then is its work counted; the search itself is unchanged.
+    struct SpecRes {
+        int32_t opt;
+        DpOutcome o;
+    };
+    std::map<std::vector<int64_t>, SpecRes> spec;
+    int spec_depth = opt.speculate < 0 ? 3 : opt.speculate;
+    int64_t spec_sigma = (int64_t)1 << 24;
+    {
+        const char *sd = std::getenv("PTAS_SPEC_DEPTH");
+        if (sd && sd[0] && opt.speculate < 0) spec_depth = std::atoi(sd);
+        const char *ss = std::getenv("PTAS_SPEC_SIGMA");
+        if (ss && ss[0]) spec_sigma = std::atoll(ss);
+        if (spec_depth > 3) spec_depth = 3;   // 2^3 - 1 = 7 DPs in flight (MAX_SLOTS slots)
+    }
+    const bool spec_on = spec_depth >= 1 && P == 1 && concurrent && opt.memoize && opt.mode == PTAS_MODE_SINGLE;
+    auto speculate = [&](int64_t lb0, int64_t ub0) -> int {
+        struct Node {
+            int64_t lb, ub;
+            int d;
+        };
+        std::vector<Node> q{{lb0, ub0, 0}};
+        std::vector<Classified> cls_v;
+        std::vector<int64_t> T_v;
+        std::vector<std::vector<int64_t>> key_v;
+        for (size_t h = 0; h < q.size(); ++h) {
+            const Node nd = q[h];
+            if (nd.lb >= nd.ub) continue;
+            std::vector<int64_t> t1;
+            probe_targets(nd.lb, nd.ub, 1, &t1);
+            const int64_t T = t1[0];
+            Classified c;
+            classify(p, n, T, k, &c);
+            bool take = false;
+            std::vector<int64_t> key;
+            if (!c.N.empty()) {
+                key = memo_key(c, T);
+                __int128 sg = 1;
+                for (int32_t x : c.N) {
+                    sg *= (x + 1);
+                    if (sg > (__int128)spec_sigma) break;
+                }
+                const bool known = memo.count(key) || spec.count(key) ||
+                                   std::find(key_v.begin(), key_v.end(), key) != key_v.end();
+                // a large next probe runs alone (throughput-bound: nothing to overlap)
+                if (nd.d == 0 && sg > (__int128)spec_sigma) return PTAS_OK;
+                take = !known && sg <= (__int128)spec_sigma;
+            }
+            if (take) {
+                cls_v.push_back(c);
+                T_v.push_back(T);
+                key_v.push_back(key);
+            }
+            if (nd.d + 1 < spec_depth && (int)cls_v.size() < MAX_SLOTS) {
+                q.push_back({nd.lb, T, nd.d + 1});        // T feasible
+                q.push_back({T + 1, nd.ub, nd.d + 1});    // T infeasible
+            }
+            if ((int)cls_v.size() >= MAX_SLOTS) break;
+        }
+        if (cls_v.empty()) return PTAS_OK;
+        std::vector<DpOutcome> outs;
+        int r2 = run_jobs(cls_v, T_v, key_v, outs, true);
+        if (r2) return r2;
+        for (size_t j = 0; j < cls_v.size(); ++j) spec[key_v[j]] = SpecRes{outs[j].opt, outs[j]};
+        acc.s.spec_dps += (int32_t)cls_v.size();
+        return PTAS_OK;
+    };
+
     while (LB < UB) {
         std::vector<int64_t> Tj;
         probe_targets(LB, UB, P, &Tj);
+        if (spec_on) {
+            classify(p, n, Tj[0], k, &cl);
+            if (!cl.N.empty()) {
+                const std::vector<int64_t> key = memo_key(cl, Tj[0]);
+                if (!memo.count(key) && !spec.count(key)) {
+                    rc = speculate(LB, UB);
+                    if (rc) return rc;
+                }
+            }
+        }
         const int np = (int)Tj.size();
         std::vector<int32_t> optj(np, 0), hit(np, 0), who(np, 0), Kj(np, 0);
         std::vector<int64_t> sgj(np, 1);
@@ -345,6 +466,15 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             if (it != memo.end()) {
                 optj[q] = it->second;
                 hit[q] = 1;
+                continue;
+            }
+            auto sp = spec.find(keys[q]);
+            if (sp != spec.end()) {   // evaluated speculatively: now it is the search's own DP
+                optj[q] = sp->second.opt;
+                acc.add(sp->second.o);
+                acc.s.unique_dps++;
+                memo[keys[q]] = optj[q];
+                spec.erase(sp);
                 continue;
             }
             const bool mine = opt.mode != PTAS_MODE_MULTI_PROBE || q == rank;
@@ -498,6 +628,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     }
     if (log_len) *log_len = (int32_t)plog.size();
     if (stats) {
+        acc.s.spec_wasted = (int32_t)spec.size();
         acc.s.probes = (int32_t)plog.size();
         acc.s.rounds = round;
         acc.s.K_at_Tstar = (int32_t)cl.N.size();
@@ -538,6 +669,7 @@ void ptas_default_options(ptas_options *o)
     o->virtual_shards = 1;
     o->layout = 0;
     o->stream = nullptr;
+    o->speculate = -1;
 }
 
 const char *ptas_strerror(int s)

@@ -25,6 +25,7 @@
 // uniform shift), each with its own dominance mask s' <= p; a warp whose rows
 // all dominate every prefix (p >= hi digit-wise, "interior") skips the mask.
 // Positions x - J < 0 take the row's first entry (the clamp min(x, J)).
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -815,6 +816,8 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // the in-row closure handles any shift (registers up to 8 bytes, else shared memory)
     const int win = J0 * e <= 4 ? 4 : (J0 * e <= 8 ? 8 : 0);
     const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && np >= 64;
+    const char *dwv = std::getenv("PTAS_DF_WAVE");
+    const int64_t df_wave = dwv && dwv[0] ? std::max(1, std::atoi(dwv)) : 2;
     DfArgs dfa;
     if (df) dfa = *df;
     else std::memset(&dfa, 0, sizeof(dfa));
@@ -838,8 +841,11 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
         if (df) {                                                                                         \
             /* persistent: every block resident, row sets from the ticket counter */                     \
             const int spb = nsplit > 1 ? 1 : bs / 32;   /* row sets in flight per block */                \
-            blocks = (df->total_sets + spb - 1) / spb;                                                    \
-            if (blocks > cap) blocks = cap;                                                               \
+            /* enough row sets in flight for `wave` of the run's widest levels: more would only spin */   \
+            const int64_t inflight = std::min<int64_t>(df->total_sets, df_wave * ((slot_count + rpw - 1) / rpw)); \
+            blocks = (inflight + spb - 1) / spb;                                                          \
+            const int64_t capd = df->grid_div > 1 ? std::max<int64_t>(1, cap / df->grid_div) : cap;      \
+            if (blocks > capd) blocks = capd;                                                             \
         } else if (nsplit > 1) {                                                                          \
             blocks = (slot_count + rpw - 1) / rpw;                                                        \
         } else {                                                                                          \

@@ -408,3 +408,29 @@ def test_full_size_dp_sampled(P, fillmode, name):
         d = np.diff(t64, axis=ax)
         assert d.min() >= 0 and d.max() <= 1
     assert opt == t64[tuple(N)]
+
+
+# ------------------------------------------------------------------ speculative bisection (D8)
+def test_speculation_preserves_alg1(P):
+    """P = 1 with the next levels of the bisection tree evaluated concurrently:
+    same probe log, T*, makespan and assignment as without speculation and as
+    the oracle; the counted work is that of the probed DPs only."""
+    cases = [(jobs(60, 1000, s), 14, 0.3) for s in range(4)] + [(jobs(12, 100, s), 3, 0.3) for s in range(20)]
+    cases.append((WORKLOADS["M2s"].p(), WORKLOADS["M2s"].m, WORKLOADS["M2s"].eps))
+    used = 0
+    for p, m, eps in cases:
+        ref = P.ptas_solve(p, m, eps, P=1, speculate=0)
+        assert ref["stats"]["spec_dps"] == 0
+        for d in (1, 2, 3):
+            got = P.ptas_solve(p, m, eps, P=1, speculate=d)
+            assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
+            assert (got["assignment"] == ref["assignment"]).all()
+            assert got["probes"] == ref["probes"]   # incl. memo hits: speculation is not a memo hit
+            st, rs = got["stats"], ref["stats"]
+            assert st["relaxations"] == rs["relaxations"] and st["unique_dps"] == rs["unique_dps"]
+            assert st["spec_wasted"] <= st["spec_dps"]
+            used += st["spec_dps"]
+        if len(p) <= 12:
+            want = oracle.ptas(p, m, eps, 1)
+            assert ref["T_star"] == want["T_star"] and ref["assignment"].tolist() == want["assignment"].tolist()
+    assert used > 0
