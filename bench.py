@@ -298,7 +298,11 @@ def run_ours(args, w):
                           mode={0: "single", 1: "level_sharded", 2: "multi_probe"}[mode],
                           l2="flushed between steps (256 MiB write)"),
         "solve": {"probes": st0["probes"], "unique_dps": st0["unique_dps"], "T_star": st0["T_star"],
-                  "sigma_max": st0["sigma_max"], "relax_per_step": relax_total / args.steps},
+                  "sigma_max": st0["sigma_max"], "K_at_Tstar": st0["K_at_Tstar"],
+                  "relax_per_step": relax_total / args.steps,
+                  # speculative bisection (D8): DPs evaluated ahead of Alg 1 /
+                  # never probed (their work is not in `value`)
+                  "spec_dps": st0["spec_dps"], "spec_wasted": st0["spec_wasted"]},
         "solve_ms": 1e3 * t_total / args.steps,
         "solve_ms_median": statistics.median(dev_ms),
         "e2e": {"value": e2e_relax / e2e_t, "unit": UNIT,
@@ -307,7 +311,7 @@ def run_ours(args, w):
                 "solve_ms": 1e3 * e2e_t / args.steps},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "traffic_note": traffic_note,
-                     "kernel": "row_fill_swar_kernel (level fill, §8(a) a-5)",
+                     "kernel": "row_fill_swar_kernel (level fill, §8(a) a-5; dataflow launches, DESIGN.md D7)",
                      "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)" if peak_kind == "measured" else "fallback",
                      "fill_ms_per_step": 1e3 * fill_s / args.steps,
                      "fill_launches_per_step": fill_launches / args.steps,

@@ -482,7 +482,9 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // launches, runs of levels with at most PTAS_DF_SPLIT_ROWS rows with one
     // row set per block (the 8 warps split the prefix walk: shorter latency
     // per row for the narrow levels on the critical path), the others with
-    // one row set per warp (the default).  Only for unsharded DPs on the packed kernel.
+    // one row set per warp (the default); 4: as 3, with the narrow runs filled by
+    // ONE thread-block cluster in lockstep (cluster barrier per level, no flags).
+    // Only for unsharded DPs on the packed kernel.
     struct DfRun {
         int rho0, rho1;        // levels rho0 .. rho1 (inclusive)
         int nsplit;
@@ -501,12 +503,12 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         // (measured on M2s/M3s/M4s/M5s: 600..8000 within a few %, 2000 best overall)
         const int64_t split_rows = dsr && dsr[0] ? std::atoll(dsr) : 2000;
         if (df_mode > 0 && G == 1 && !force_scalar && g.rho_max >= 1) {
-            if (df_mode == 3) {
+            if (df_mode == 3 || df_mode == 4) {
                 for (int rho = 0; rho <= g.rho_max;) {
                     const bool sp = cnt[rho] <= split_rows;
                     int r1 = rho;
                     while (r1 + 1 <= g.rho_max && (cnt[r1 + 1] <= split_rows) == sp) ++r1;
-                    runs.push_back({rho, r1, sp ? 8 : 1, 0, 0, 0});
+                    runs.push_back({rho, r1, sp ? (df_mode == 4 ? 0 : 8) : 1, 0, 0, 0});
                     rho = r1 + 1;
                 }
             } else {

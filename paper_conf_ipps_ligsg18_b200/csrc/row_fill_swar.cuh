@@ -62,6 +62,9 @@ __device__ __forceinline__ void fill_words(Words<CH> &w, uint32_t x)
     for (int t = 0; t < CH; ++t) w.v[t] = x;
 }
 
+#ifndef PTAS_DF_NOACQ
+#define PTAS_DF_NOACQ 0
+#endif
 #ifndef PTAS_DF_PROFILE
 #define PTAS_DF_PROFILE 0
 #endif
@@ -304,8 +307,11 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
 // share rows (small row-levels with long prefix lists); DF: dataflow launch
 // over a run of row-levels (D7; rho, slot_begin and slot_count
 // are unused, the row sets come from df).
-template <typename E, int NW, int CH, int WIN, bool CPREF, bool SPLIT, bool DF>
-__global__ void __launch_bounds__(256)
+#ifndef PTAS_MINB
+#define PTAS_MINB 1
+#endif
+template <typename E, int NW, int CH, int WIN, bool CPREF, bool SPLIT, int DFM>
+__global__ void __launch_bounds__(256, PTAS_MINB)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,
@@ -314,6 +320,12 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
+    // DFM = 0: one row-level per launch; 1: dataflow run (tickets + ready flags,
+    // DESIGN.md D7); 2: cluster run (the CTAs of ONE thread-block cluster fill
+    // a run of narrow row-levels in lockstep, one cluster barrier per level)
+    constexpr bool DF = DFM == 1;
+    constexpr bool CL = DFM == 2;
+    constexpr bool RUN = DFM != 0;
 #ifndef PTAS_PB1
 #define PTAS_PB1 16
 #endif
@@ -372,18 +384,44 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     }
     // DF: per-level first set / first slot of the run, in shared memory
     int32_t *s_set = reinterpret_cast<int32_t *>(s_red + (size_t)(256 / 32) * 2 * 8 * 32);
-    int32_t *s_sl = s_set + (DF ? df.nlev + 1 : 0);
+    int32_t *s_sl = s_set + (RUN ? df.nlev + 1 : 0);
     // DF + SPLIT: the block's ticket (8-byte aligned after the plan)
     unsigned long long *s_tk =
-        reinterpret_cast<unsigned long long *>(s_set + ((DF ? 2 * (df.nlev + 1) : 0) + 1) / 2 * 2);
-    if constexpr (DF) {
+        reinterpret_cast<unsigned long long *>(s_set + ((RUN ? 2 * (df.nlev + 1) : 0) + 1) / 2 * 2);
+    if constexpr (RUN) {
         for (int i = threadIdx.x; i < 2 * (df.nlev + 1); i += blockDim.x) s_set[i] = df.plan[i];
         __syncthreads();
     }
     // first row set's index entries, loaded before waiting on the previous level
     int64_t nrb = 0;
     uint64_t npw[NW];
-    if constexpr (!DF) {
+    // CL: warp gwc of the cluster takes sets gwc, gwc + nwc, ... of each level
+    int c_lv = 0, n_lv = 0, bars = 0;
+    int64_t c_t = 0, n_t = 0;
+    int gwc = 0, nwc = 1;
+    auto cl_norm = [&](int &lv, int64_t &t) {
+        while (lv < df.nlev && t >= (int64_t)(s_set[lv + 1] - s_set[lv])) {
+            ++lv;
+            t = gwc;
+        }
+    };
+    auto cl_load = [&](int lv, int64_t t) {
+        const int64_t sl = (int64_t)s_sl[lv] + t * rpw + grp;
+        const bool ok = grp < rpw && sl < s_sl[lv + 1];
+#pragma unroll
+        for (int w = 0; w < NW; ++w) npw[w] = ok ? pwa[(int64_t)w * pw_stride + sl] : 0;
+        nrb = ok ? rb[sl] : 0;
+    };
+    if constexpr (CL) {
+        uint32_t r, nr;
+        asm("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+        asm("mov.u32 %0, %%cluster_nctarank;" : "=r"(nr));
+        gwc = (int)r * (int)(blockDim.x >> 5) + wid;
+        nwc = (int)nr * (int)(blockDim.x >> 5);
+        c_t = gwc;
+        cl_norm(c_lv, c_t);
+        if (c_lv < df.nlev) cl_load(c_lv, c_t);
+    } else if constexpr (!DF) {
         const int64_t slot = gw * rpw + grp;
         const bool ok = grp < rpw && slot < slot_count;
 #pragma unroll
@@ -430,18 +468,30 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     // uniform trip count (every warp of the grid runs the same number of row
     // sets; the tail ones are idle) keeps the prefix loop in uniform control flow
     const int64_t nsets = (slot_count + rpw - 1) / rpw;
-    const int64_t iters = DF ? 0 : (nsets + nw - 1) / nw;
+    const int64_t iters = RUN ? 0 : (nsets + nw - 1) / nw;
     for (int64_t it = 0;; ++it) {
-        if (DF ? tk >= df.total_sets : it >= iters) break;
+        if (CL ? c_lv >= df.nlev : (DF ? tk >= df.total_sets : it >= iters)) break;
         const int64_t sb = (it * nw + gw) * rpw;
-        const int64_t slot = DF ? cur_slot : sb + grp;
-        const bool rowok = DF ? cur_ok : (grp < rpw && slot < slot_count);
+        const int64_t slot = CL ? (int64_t)s_sl[c_lv] + c_t * rpw + grp : (DF ? cur_slot : sb + grp);
+        const bool rowok = CL ? (grp < rpw && slot < s_sl[CL ? c_lv + 1 : 0]) : (DF ? cur_ok : (grp < rpw && slot < slot_count));
         const int64_t rowbase = nrb;
         uint64_t pw[NW];
 #pragma unroll
         for (int w = 0; w < NW; ++w) pw[w] = npw[w];
         unsigned long long tnext = 0;
-        if constexpr (DF) {
+        if constexpr (CL) {
+            // next set of this warp (possibly levels ahead) and its index entries
+            n_lv = c_lv;
+            n_t = c_t + nwc;
+            cl_norm(n_lv, n_t);
+            if (n_lv < df.nlev) cl_load(n_lv, n_t);
+            // every level below c_lv is complete in the whole cluster
+            // (release/acquire at cluster scope orders the table stores)
+            while (bars < c_lv) {
+                asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+                ++bars;
+            }
+        } else if constexpr (DF) {
             // next ticket now; its value is consumed after the prefix walk
             if (SPLIT ? threadIdx.x == 0 : lane == 0) tnext = atomicAdd(df.ticket, 1ull);
         } else {   // prefetch the next row set's index entries
@@ -472,7 +522,16 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     if (rowok) {
                         for (int i = xl; i < g.K1; i += Lg) {
                             const uint64_t wv = NW == 1 ? pw[0] : (g.word[i] ? pw[NW - 1] : pw[0]);
-                            if (wv & df.dmask[i]) ok &= ld_acquire(df.flags + (rid - (uint32_t)df.rstride[i])) == df.epoch;
+                            if (wv & df.dmask[i]) {
+                                const uint32_t *f = df.flags + (rid - (uint32_t)df.rstride[i]);
+#if PTAS_DF_NOACQ   // measurement only (not a correct protocol): flags without acquire
+                                uint32_t fv;
+                                asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(fv) : "l"(f) : "memory");
+                                ok &= fv == df.epoch;
+#else
+                                ok &= ld_acquire(f) == df.epoch;
+#endif
+                            }
                         }
                     }
                     if (__all_sync(FULL, ok)) break;
@@ -535,7 +594,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
                     sj[u] = oj.y;
                     const uint32_t *p = src + oj.x;
-                    if ((m >> q) & 1u) cur[u] = load_words<CH, DF>(p);
+                    if ((m >> q) & 1u) cur[u] = load_words<CH, RUN>(p);
                     else fill_words(cur[u], 0xffffffffu);
                 }
 #pragma unroll
@@ -614,7 +673,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     oo.v[t] = 0;
                 }
             }
-            if ((DF ? rowbase == 0 : rho == 0) && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
+            if ((RUN ? rowbase == 0 : rho == 0) && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
             // opt(p, 0) is final (no in-row term at x = 0): the clamp value
             uint32_t f0 = __shfl_sync(FULL, oe.v[0], lane - xl);
             f0 = prmt(f0, 0u, 0x1010u);
@@ -727,6 +786,17 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
             cur_ok = nxt_ok;
             cur_lv = df_lv;
         }
+        if constexpr (CL) {
+            c_lv = n_lv;
+            c_t = n_t;
+        }
+    }
+    if constexpr (CL) {
+        // every thread of the cluster passes the same nlev - 1 barriers
+        while (bars < df.nlev - 1) {
+            asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+            ++bars;
+        }
     }
 }
 
@@ -808,6 +878,10 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // (worth it when a row's prefix walk has several batches of gathers in series)
     const int PBh = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);
     const int64_t split_rows = sp ? std::atoll(sp) : ((np + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
+    // df->nsplit: 1 = warp row sets, 8 = block row sets, 0 = one cluster in lockstep
+    const bool cl = df && df->nsplit == 0;
+    const char *cls = std::getenv("PTAS_CL_SIZE");
+    const int cl_size = cl ? (cls && cls[0] ? std::max(1, std::min(16, std::atoi(cls))) : 16) : 1;
     const int nsplit = df ? (df->nsplit > 1 ? bs / 32 : 1) : (slot_count <= split_rows ? bs / 32 : 1);
     const size_t smem = swar_smem(np, NW, df ? df->nlev : 0);
     if (smem > 220 * 1024) return cudaErrorNotSupported;
@@ -824,21 +898,29 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     cudaError_t err;
 #define PTAS_SWAR_GO(E_, NW_, CH_, WIN_)                                                                  \
     do {                                                                                                  \
-        auto kfn = df ? (cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true, true>  \
-                                             : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, true>) \
-                               : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true, true> \
-                                             : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, true>)) \
-               : cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true, false>        \
-                                     : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, false>)      \
-                       : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true, false>       \
-                                     : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, false>);    \
+        auto kfn = cl ? (cpref ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, 2>                 \
+                               : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, 2>)               \
+                 : df ? (cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true, 1>    \
+                                             : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, 1>)  \
+                               : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true, 1>   \
+                                             : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, 1>)) \
+               : cpref ? (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, true, 0>            \
+                                     : row_fill_swar_kernel<E_, NW_, CH_, WIN_, true, false, 0>)          \
+                       : (nsplit > 1 ? row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, true, 0>           \
+                                     : row_fill_swar_kernel<E_, NW_, CH_, WIN_, false, false, 0>);        \
         if (smem > 48 * 1024) {                                                                           \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);      \
             if (err != cudaSuccess) return err;                                                           \
         }                                                                                                 \
+        if (cl && cl_size > 8) {                                                                          \
+            err = cudaFuncSetAttribute(kfn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);           \
+            if (err != cudaSuccess) return err;                                                           \
+        }                                                                                                 \
         int64_t blocks;                                                                                   \
         const int64_t cap = (int64_t)sm_count * occupancy_of(kfn, smem, bs);                              \
-        if (df) {                                                                                         \
+        if (cl) {                                                                                         \
+            blocks = cl_size;   /* one cluster */                                                         \
+        } else if (df) {                                                                                  \
             /* persistent: every block resident, row sets from the ticket counter */                     \
             const int spb = nsplit > 1 ? 1 : bs / 32;   /* row sets in flight per block */                \
             /* enough row sets in flight for `wave` of the run's widest levels: more would only spin */   \
@@ -854,21 +936,25 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
             if (blocks > cap) blocks = cap;                                                               \
         }                                                                                                 \
         cudaLaunchConfig_t cfg = {};                                                                      \
-        cudaLaunchAttribute attr[1];                                                                      \
+        cudaLaunchAttribute attr[2];                                                                      \
         attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;                                  \
         attr[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;                                 \
+        attr[1].id = cudaLaunchAttributeClusterDimension;                                                 \
+        attr[1].val.clusterDim.x = (unsigned)cl_size;                                                     \
+        attr[1].val.clusterDim.y = 1;                                                                     \
+        attr[1].val.clusterDim.z = 1;                                                                     \
         cfg.gridDim = dim3((unsigned)blocks);                                                             \
         cfg.blockDim = dim3(bs);                                                                          \
         cfg.dynamicSmemBytes = smem;                                                                      \
         cfg.stream = st;                                                                                  \
         cfg.attrs = attr;                                                                                 \
-        cfg.numAttrs = 1;                                                                                 \
+        cfg.numAttrs = cl ? 2 : 1;                                                                        \
         err = cudaLaunchKernelEx(&cfg, kfn, (E_ *)table, g, rb, pw, pw_stride, d_pref, d_meta, J0, rho,   \
                                  slot_begin, slot_count, (E_ *)compact_out, Lg, nsplit, cslot, dfa);      \
         if (err != cudaSuccess) return err;                                                               \
         /* every grabbing warp (block in split mode) ends with exactly one failed grab */               \
-        if (df && ticket_base) *ticket_base += (unsigned long long)df->total_sets +                       \
-                                               (unsigned long long)blocks * (nsplit > 1 ? 1 : bs / 32);   \
+        if (df && !cl && ticket_base) *ticket_base += (unsigned long long)df->total_sets +                \
+                                                      (unsigned long long)blocks * (nsplit > 1 ? 1 : bs / 32); \
     } while (0)
 #define PTAS_SWAR_CASE(E_, NW_, CH_)                                                              \
     do {                                                                                          \

@@ -2,9 +2,10 @@
 row-levels, row sets from a ticket counter, per-row ready flags.
 
 Same bit-exact comparisons against the oracle as test_gpu_parity.py, with
-PTAS_DF = 1 (the whole DP in one launch) and PTAS_DF = 2 (runs of small
+PTAS_DF = 1 (the whole DP in one launch), PTAS_DF = 2 (runs of small
 row-levels between per-level launches; a tiny PTAS_DF_ROWS splits every DP
-into several runs).
+into several runs), PTAS_DF = 3 (block row sets for narrow levels) and
+PTAS_DF = 4 (narrow levels by one thread-block cluster in lockstep).
 """
 from __future__ import annotations
 
@@ -19,7 +20,8 @@ pytestmark = pytest.mark.gpu
 
 # (PTAS_DF, PTAS_DF_ROWS, PTAS_DF_SPLIT_ROWS)
 MODES = [("1", None, None), ("2", "40", None), ("2", "3000", None),
-         ("3", None, None), ("3", None, "20"), ("3", None, "1000000000")]
+         ("3", None, None), ("3", None, "20"), ("3", None, "1000000000"),
+         ("4", None, None), ("4", None, "1000000000"), ("4c2", None, "1000000000")]
 
 
 @pytest.fixture(scope="module")
@@ -31,6 +33,9 @@ def P():
 @pytest.fixture(params=MODES, ids=lambda m: f"df{m[0]}-rows{m[1]}-split{m[2]}")
 def df(request, monkeypatch):
     mode, rows, split = request.param
+    if mode == "4c2":   # cluster runs with a 2-CTA cluster: many sets per warp and level
+        mode = "4"
+        monkeypatch.setenv("PTAS_CL_SIZE", "2")
     monkeypatch.setenv("PTAS_DF", mode)
     if rows is not None:
         monkeypatch.setenv("PTAS_DF_ROWS", rows)
@@ -129,7 +134,7 @@ def test_df_matches_level_launches_on_solve(P, monkeypatch):
     w = WORKLOADS["M2s"]
     monkeypatch.setenv("PTAS_DF", "0")
     ref = P.ptas_solve(w.p(), w.m, w.eps, P=1)
-    for mode in ("1", "2", "3"):
+    for mode in ("1", "2", "3", "4"):
         monkeypatch.setenv("PTAS_DF", mode)
         got = P.ptas_solve(w.p(), w.m, w.eps, P=1)
         assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
