@@ -101,6 +101,11 @@ typedef struct {
     int32_t spec_dps;       /* DPs evaluated speculatively (options.speculate) */
     int32_t spec_wasted;    /* of which never probed by the search (their work
                                is not counted in the fields above)            */
+    double fill_wall_seconds; /* device time during which at least one level-
+                               fill loop ran: union of the DPs' fill intervals
+                               (CUDA events on one time axis).  Equals
+                               fill_seconds when DPs run one at a time; below it
+                               when speculative / concurrent DPs overlap       */
 } ptas_stats;
 
 typedef struct {

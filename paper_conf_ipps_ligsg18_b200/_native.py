@@ -38,7 +38,8 @@ class PtasStats(ctypes.Structure):
                 ("total_seconds", ctypes.c_double), ("alg_bytes", ctypes.c_double), ("states", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int32), ("fill_launches", ctypes.c_int32),
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64), ("relax_executed", ctypes.c_double),
-                ("exec_bytes", ctypes.c_double), ("spec_dps", ctypes.c_int32), ("spec_wasted", ctypes.c_int32)]
+                ("exec_bytes", ctypes.c_double), ("spec_dps", ctypes.c_int32), ("spec_wasted", ctypes.c_int32),
+                ("fill_wall_seconds", ctypes.c_double)]
 
     def to_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

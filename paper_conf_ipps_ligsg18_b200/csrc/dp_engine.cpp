@@ -123,6 +123,15 @@ int Engine::init(int device)
     return slot(0, &s);
 }
 
+int Engine::mark_reference(cudaStream_t st, cudaEvent_t *out)
+{
+    if (!ref_ev_) PT_CK(cudaEventCreate(&ref_ev_));
+    PT_CK(cudaEventRecord(ref_ev_, st ? st : stream()));
+    PT_CK(cudaEventSynchronize(ref_ev_));
+    *out = ref_ev_;
+    return PTAS_OK;
+}
+
 int Engine::slot(int i, DpSlot **out)
 {
     if (i < 0 || i >= MAX_SLOTS) return PTAS_EINVAL;
@@ -703,6 +712,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     o.dp_s = ms * 1e-3;
     PT_CK(cudaEventElapsedTime(&ms, ev_[1], ev_[2]));
     o.fill_s = ms * 1e-3;
+    if (rq.ref_event) {
+        float a = 0, b = 0;
+        PT_CK(cudaEventElapsedTime(&a, rq.ref_event, ev_[1]));
+        PT_CK(cudaEventElapsedTime(&b, rq.ref_event, ev_[2]));
+        o.fill_t0 = a * 1e-3;
+        o.fill_t1 = b * 1e-3;
+    }
     if (trace) {
         const double t3 = trace_now();
         std::fprintf(stderr, "[ptas] dp sigma=%lld K=%d levels=%d host: setup+enum-sync %.3f ms, fill enqueue %.3f ms, "

@@ -33,6 +33,7 @@ struct DpRequest {
     const ShardCtx *shard = nullptr;
     int64_t budget = 0;           // bytes allowed for the table (0 = auto)
     int grid_div = 1;             // >1: this many DPs run concurrently; persistent grids take 1/grid_div of the GPU
+    cudaEvent_t ref_event = nullptr;  // completed timing event: fill interval reported relative to it
 };
 
 struct DpOutcome {
@@ -44,6 +45,7 @@ struct DpOutcome {
     double relax_exec = 0;  // relaxations the kernels evaluated (collapsed form, or relax for the scalar kernel)
     int64_t nC = 0, nP = 0;
     double dp_s = 0, fill_s = 0;
+    double fill_t0 = -1, fill_t1 = -1;   // fill interval in seconds after rq.ref_event (-1: none)
     int launches = 0, fill_launches = 0;
     int64_t h2d = 0, d2h = 0;
 };
@@ -143,6 +145,9 @@ class Engine {
     }
     int copy_table_to_host(void *dst, int64_t bytes) { return slots_[0]->copy_table_to_host(dst, bytes); }
     cudaStream_t stream() const { return slots_[0]->stream(); }
+    // timing reference of one call: recorded on st and waited for, so the
+    // DPs' fill intervals (events on any stream) can be placed on one axis
+    int mark_reference(cudaStream_t st, cudaEvent_t *out);
     cudaError_t sync_spin(cudaStream_t st) { return slots_[0]->sync_spin(st); }
 
   private:
@@ -150,6 +155,7 @@ class Engine {
     int device_ = -1;
     int sm_count_ = 148;
     DpSlot *slots_[MAX_SLOTS] = {};
+    cudaEvent_t ref_ev_ = nullptr;
 };
 
 // NCCL glue (comm.cpp)

@@ -152,9 +152,32 @@ double now_s()
 
 struct Acc {
     ptas_stats s;
+    std::vector<std::pair<double, double>> iv;   // fill intervals of every DP run (incl. unused speculative ones)
     Acc() { std::memset(&s, 0, sizeof(s)); }
+    void interval(const DpOutcome &o)
+    {
+        if (o.fill_t0 >= 0 && o.fill_t1 > o.fill_t0) iv.emplace_back(o.fill_t0, o.fill_t1);
+    }
+    // device time during which at least one level-fill loop ran
+    void finish_wall()
+    {
+        std::sort(iv.begin(), iv.end());
+        double tot = 0, a = -1, b = -1;
+        for (auto &x : iv) {
+            if (x.first > b) {
+                if (b > a) tot += b - a;
+                a = x.first;
+                b = x.second;
+            } else {
+                b = std::max(b, x.second);
+            }
+        }
+        if (b > a) tot += b - a;
+        s.fill_wall_seconds = tot;
+    }
     void add(const DpOutcome &o)
     {
+        interval(o);
         s.relaxations += o.relax;
         s.relax_executed += o.relax_exec;
         s.exec_bytes += (o.relax_exec + (double)o.sigma) * o.e;
@@ -239,6 +262,11 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     Acc acc;
     acc.s.h2d_bytes += extra_h2d;
     acc.s.d2h_bytes += extra_d2h;
+    cudaEvent_t ref_ev = nullptr;   // time axis of the DPs' fill intervals (fill_wall_seconds)
+    {
+        const int r2 = eng->mark_reference((cudaStream_t)opt.stream, &ref_ev);
+        if (r2) return r2;
+    }
     std::map<std::vector<int64_t>, int32_t> memo;
     std::vector<ptas_probe> plog;
     int round = 0;
@@ -257,6 +285,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         rq.shard = s;
         rq.budget = opt.table_budget_bytes;
         rq.stream = st;
+        rq.ref_event = ref_ev;
         return rq;
     };
     auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
@@ -629,6 +658,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     if (log_len) *log_len = (int32_t)plog.size();
     if (stats) {
         acc.s.spec_wasted = (int32_t)spec.size();
+        for (auto &kv : spec) acc.interval(kv.second.o);
+        acc.finish_wall();
         acc.s.probes = (int32_t)plog.size();
         acc.s.rounds = round;
         acc.s.K_at_Tstar = (int32_t)cl.N.size();
@@ -840,6 +871,7 @@ static int dp_fill_common(const int32_t *counts, const int64_t *sizes, int32_t K
     if (rc) return rc;
     Acc acc;
     acc.add(o);
+    acc.s.fill_wall_seconds = o.fill_s;
     if (host_out) {
         // engine-owned table; identity order => caller's layout
         rc = eng->copy_table_to_host(host_out, sigma * e);

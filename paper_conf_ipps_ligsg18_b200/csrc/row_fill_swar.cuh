@@ -307,11 +307,18 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
 // share rows (small row-levels with long prefix lists); DF: dataflow launch
 // over a run of row-levels (D7; rho, slot_begin and slot_count
 // are unused, the row sets come from df).
-#ifndef PTAS_MINB
-#define PTAS_MINB 1
+// Resident blocks per SM the compiler must allow (register cap 65536 / (256 * MINB)):
+// uint16 tables 4 (64 registers: M3s 8.8 -> 8.1 ms, M5s-0.15 21.8 -> 20.3 ms fill,
+// measured), uint8 tables 1 (capping their kernels at 64 registers spills:
+// M2s 3.40 -> 3.59 ms).
+#ifndef PTAS_MINB_U8
+#define PTAS_MINB_U8 1
+#endif
+#ifndef PTAS_MINB_U16
+#define PTAS_MINB_U16 4
 #endif
 template <typename E, int NW, int CH, int WIN, bool CPREF, bool SPLIT, int DFM>
-__global__ void __launch_bounds__(256, PTAS_MINB)
+__global__ void __launch_bounds__(256, sizeof(E) == 1 ? PTAS_MINB_U8 : PTAS_MINB_U16)
 row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                      const uint64_t *__restrict__ pwa, int64_t pw_stride,
                      const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta, int J0,

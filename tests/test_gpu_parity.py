@@ -434,3 +434,18 @@ def test_speculation_preserves_alg1(P):
             want = oracle.ptas(p, m, eps, 1)
             assert ref["T_star"] == want["T_star"] and ref["assignment"].tolist() == want["assignment"].tolist()
     assert used > 0
+
+
+def test_fill_wall_time(P):
+    """stats.fill_wall_seconds (union of the DPs' fill intervals): equal to the
+    per-DP sum when DPs run one at a time, at most the sum (and at least the
+    longest DP's fill) when speculative DPs overlap."""
+    w = WORKLOADS["M2s"]
+    for d in (0, 3):
+        st = P.ptas_solve(w.p(), w.m, w.eps, P=1, speculate=d)["stats"]
+        assert st["fill_wall_seconds"] > 0
+        assert st["fill_wall_seconds"] <= st["fill_seconds"] * (1 + 1e-6) + 1e-6
+        if d == 0:
+            assert abs(st["fill_wall_seconds"] - st["fill_seconds"]) <= 0.02 * st["fill_seconds"] + 2e-5
+    st = P.dp_fill(np.array([5, 4, 30], np.int32), np.array([60, 45, 17], np.int64), 160)[2]
+    assert st["fill_wall_seconds"] == st["fill_seconds"]
