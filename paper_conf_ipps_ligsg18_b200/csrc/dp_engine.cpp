@@ -406,24 +406,46 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     PT_CK(launch_enum_configs(0, K, D, nprefix, d_hi, d_r, rq.T, d_stride, d_counts, nullptr,
                               nullptr, nullptr, st));
     PT_CK(launch_exclusive_scan(d_counts, d_offsets, nprefix, d_offsets + nprefix, st));
-    PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
-    PT_CK(sync_spin(st));
-    o.d2h += 8;
     o.launches += 2;
-    const int64_t nC = h_scalar_[0];
+    // |C| is needed on the host only to size buffers and shared-memory tables.
+    // Once this slot has run a DP, the DP is enqueued without waiting for it:
+    // buffers preallocated for nc_cap_ configurations, prefix tables sized for
+    // NP_CAP, launch heuristics from the previous DP's prefix count; the
+    // kernels exit and the DP is redone synchronously if a bound is exceeded
+    // (meta->ovf), which then grows the bounds.
+    const char *es = std::getenv("PTAS_ENUM_SYNC");
+    const bool nosync = np_hint_ >= 0 && nc_cap_ > 0 && !force_sync_enum_ && !(es && es[0] == '1');
+    int64_t nC;        // |C| (synchronous) or its bound
+    int64_t nP_bound;  // bound of the prefix list incl. the zero prefix (smem sizing)
+    // test knobs: PTAS_NC_CAP / PTAS_NP_CAP lower the bounds (exercise the redo path)
+    const char *ncc = std::getenv("PTAS_NC_CAP");
+    const char *npc = std::getenv("PTAS_NP_CAP");
+    const int64_t np_cap = npc && npc[0] ? std::min<int64_t>(NP_CAP, std::atoll(npc)) : NP_CAP;
+    if (nosync) {
+        nC = ncc && ncc[0] ? std::min<int64_t>(nc_cap_, std::max<int64_t>(1, std::atoll(ncc))) : nc_cap_;
+        nP_bound = NP_CAP + 1;
+    } else {
+        PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
+        PT_CK(sync_spin(st));
+        o.d2h += 8;
+        nC = h_scalar_[0];
+        if (nC <= 0) return PTAS_EINTERNAL;  // (0,..,0,1) is always feasible
+        nC_cap_grow(nC);
+        nP_bound = nC;
+    }
     if (trace) tr_enum = trace_now();
-    if (nC <= 0) return PTAS_EINTERNAL;  // (0,..,0,1) is always feasible
     PT_CK(digits_.ensure((size_t)nC * K * 2));
     PT_CK(off_.ensure((size_t)nC * 8));
     PT_CK(pref_.ensure((size_t)nC * sizeof(PrefixEntry)));
     PT_CK(launch_enum_configs(1, K, D, nprefix, d_hi, d_r, rq.T, d_stride, d_counts, d_offsets,
-                              (uint16_t *)digits_.p, (int64_t *)off_.p, st));
-    PT_CK(launch_build_prefix(K, (const uint16_t *)digits_.p, (const int64_t *)off_.p, nC, g,
-                              N.data(), (PrefixEntry *)pref_.p, d_meta_, st));
+                              (uint16_t *)digits_.p, (int64_t *)off_.p, st, nC));
+    PT_CK(launch_build_prefix(K, (const uint16_t *)digits_.p, (const int64_t *)off_.p, d_offsets + nprefix, nC,
+                              nosync ? np_cap : INT64_MAX, g, N.data(), (PrefixEntry *)pref_.p, d_meta_, st));
     o.launches += 2;
+    tl_np_hint = nosync ? np_hint_ : -1;
     // prefix offsets into the packed kernel's constant bank
     PT_CK(cpstage_.ensure(const_prefix_staging_bytes()));
-    cudaError_t cpe = index_ < 4 ? prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nC, e, g.nwords, index_,
+    cudaError_t cpe = index_ < 4 ? prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nP_bound, e, g.nwords, index_,
                                                    cpstage_.p, st)
                                 : cudaErrorNotSupported;
     const char *ncp = std::getenv("PTAS_NO_CPREF");
@@ -444,13 +466,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         const uint64_t *pwl = d_pw + lstart[rho_];
         cudaError_t err = cudaErrorNotSupported;
         if (!force_scalar) {
-            err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC,
+            err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
                                        j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0,
                                        cpref_ok ? index_ : -1);
             if (err == cudaSuccess) prev_fill = true;
         }
         if (err == cudaErrorNotSupported) {
-            err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nC, j0,
+            err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound, j0,
                                   rho_, b, c, compact, sm_count_, st);
             prev_fill = false;
             used_scalar = true;
@@ -623,7 +645,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                 dfa.prof = (unsigned long long *)dfprof_.p;
             }
             cudaError_t err = launch_row_fill_swar_df(e, table, g, d_rb, d_pw, rows, (const PrefixEntry *)pref_.p,
-                                                      d_meta_, nC, J0, rn.max_rows, dfa, &ticket_base_, sm_count_,
+                                                      d_meta_, nP_bound, J0, rn.max_rows, dfa, &ticket_base_, sm_count_,
                                                       st, (use_pdl && prev_fill) ? 1 : 0, cpref_ok ? index_ : -1);
             if (err == cudaSuccess && df_prof) {
                 PT_CK(cudaMemcpyAsync(prof_h.data(), dfprof_.p, prof_h.size() * 8, cudaMemcpyDeviceToHost, st));
@@ -726,6 +748,21 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                      (long long)sigma, K, g.rho_max + 1, 1e3 * (tr_enum - tr0), 1e3 * (tr_fillq - tr_enum),
                      1e3 * (t3 - tr_fillq), 1e3 * o.dp_s, 1e3 * o.fill_s);
     }
+    tl_np_hint = -1;
+    if (h_meta_->ovf) {
+        // a bound of the round-trip-free enumeration was exceeded: nothing was
+        // filled; redo synchronously (exact sizes) and keep the larger bounds
+        nC_cap_grow(h_meta_->nC);
+        if (ticket_.p) {   // the exited dataflow launches took no tickets: restart the counter
+            PT_CK(cudaMemsetAsync(ticket_.p, 0, 8, st));
+            ticket_base_ = 0;
+        }
+        force_sync_enum_ = true;
+        const int rc2 = run_dp(rq, out);
+        force_sync_enum_ = false;
+        return rc2;
+    }
+    np_hint_ = h_meta_->nP - 1;
     o.opt = h_meta_->opt;
     o.relax = (double)h_meta_->relax;
     o.relax_exec = used_scalar ? o.relax : (double)h_meta_->relax_exec;
@@ -739,7 +776,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     last_Kcanon_ = rq.K;
     last_e_ = e;
     last_sigma_ = sigma;
-    last_nC_ = nC;
+    last_nC_ = h_meta_->nC;
     last_opt_ = o.opt;
     last_order_ = order;
     last_N_ = N;

@@ -19,6 +19,9 @@
 
 namespace ptas {
 
+thread_local int64_t tl_np_hint = -1;
+
+
 namespace {
 
 // ------------------------------------------------------------------ a-3
@@ -31,10 +34,11 @@ __global__ void enum_configs_kernel(int pass, int K, int D, int64_t nprefix,
                                     const int32_t *__restrict__ hi, const int64_t *__restrict__ r,
                                     int64_t T, const int64_t *__restrict__ stride,
                                     int64_t *__restrict__ counts, const int64_t *__restrict__ offsets,
-                                    uint16_t *__restrict__ digits, int64_t *__restrict__ off)
+                                    uint16_t *__restrict__ digits, int64_t *__restrict__ off, int64_t cap)
 {
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= nprefix) return;
+    if (pass == 1 && offsets[nprefix] > cap) return;   // buffers too small: build_prefix flags it
     int32_t s[MAXK];
     uint64_t load = 0;
     bool over = false;
@@ -130,10 +134,20 @@ __device__ __forceinline__ bool same_lead(const uint16_t *a, const uint16_t *b, 
 struct NallArg { int32_t v[MAXK]; };
 
 __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
-                                    const int64_t *__restrict__ off, int64_t nC, RowGeom g,
+                                    const int64_t *__restrict__ off, const int64_t *__restrict__ d_nC,
+                                    int64_t nc_cap, int64_t np_cap, RowGeom g,
                                     NallArg Nall, PrefixEntry *__restrict__ pref,
                                     DpMeta *__restrict__ meta)
 {
+    const int64_t nC = *d_nC;
+    if (nC > nc_cap) {   // uniform: the buffers were sized for nc_cap configurations
+        if (threadIdx.x == 0) {
+            meta->nC = nC;
+            meta->nP = 0;
+            meta->ovf = 1;
+        }
+        return;
+    }
     __shared__ int64_t warp_sums[32];
     __shared__ int64_t carry;
     __shared__ unsigned long long relax_acc, exec_acc;
@@ -211,6 +225,7 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
         meta->nP = carry;
         meta->relax = relax_acc;
         meta->relax_exec = exec_acc;
+        meta->ovf = carry - 1 > np_cap ? 1 : 0;
     }
 }
 
@@ -307,6 +322,7 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
                 int J0, int rho, int64_t slot_begin, int64_t slot_count, E *compact, int wlog)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    if (meta->ovf) return;   // enumeration overflowed its bounds: the host redoes the DP
     const int np = (int)(meta->nP - 1);      // cross-row prefixes (entry 0 is s' = 0)
     uint64_t *s_oj = reinterpret_cast<uint64_t *>(smem_raw);
     uint64_t *s_w = s_oj + np;
@@ -526,12 +542,12 @@ int wlog_for(int64_t W)
 cudaError_t launch_enum_configs(int pass, int K, int D, int64_t nprefix, const int32_t *hi,
                                 const int64_t *r, int64_t T, const int64_t *stride,
                                 int64_t *d_counts, const int64_t *d_offsets, uint16_t *d_digits,
-                                int64_t *d_off, cudaStream_t st)
+                                int64_t *d_off, cudaStream_t st, int64_t cap)
 {
     const int bs = 128;
     int64_t blocks = (nprefix + bs - 1) / bs;
     enum_configs_kernel<<<(unsigned)blocks, bs, 0, st>>>(pass, K, D, nprefix, hi, r, T, stride,
-                                                         d_counts, d_offsets, d_digits, d_off);
+                                                         d_counts, d_offsets, d_digits, d_off, cap);
     return cudaGetLastError();
 }
 
@@ -542,13 +558,13 @@ cudaError_t launch_exclusive_scan(const int64_t *d_in, int64_t *d_out, int64_t n
     return cudaGetLastError();
 }
 
-cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off, int64_t nC,
-                                const RowGeom &g, const int32_t *Nall, PrefixEntry *d_pref,
-                                DpMeta *d_meta, cudaStream_t st)
+cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off, const int64_t *d_nC,
+                                int64_t nc_cap, int64_t np_cap, const RowGeom &g, const int32_t *Nall,
+                                PrefixEntry *d_pref, DpMeta *d_meta, cudaStream_t st)
 {
     NallArg na;
     for (int i = 0; i < MAXK; ++i) na.v[i] = i < K ? Nall[i] : 0;
-    build_prefix_kernel<<<1, 1024, 0, st>>>(K, d_digits, d_off, nC, g, na, d_pref, d_meta);
+    build_prefix_kernel<<<1, 1024, 0, st>>>(K, d_digits, d_off, d_nC, nc_cap, np_cap, g, na, d_pref, d_meta);
     return cudaGetLastError();
 }
 

@@ -98,6 +98,13 @@ class DpSlot {
     cudaEvent_t ev_fork_ = nullptr, ev_join_ = nullptr;
     DpMeta *d_meta_ = nullptr;
     DpMeta *h_meta_ = nullptr;     // pinned
+    // enumeration without a host round trip (D9): configuration
+    // buffers preallocated for nc_cap_ configurations; prefix-list length of
+    // this slot's last DP (launch heuristics; -1 = none yet: synchronous path)
+    int64_t nc_cap_ = 0;
+    int64_t np_hint_ = -1;
+    bool force_sync_enum_ = false;
+    void nC_cap_grow(int64_t nC) { nc_cap_ = std::max<int64_t>(nc_cap_, std::max<int64_t>(4096, 2 * nC)); }
     int64_t *h_scalar_ = nullptr;  // pinned
     unsigned char *pin_ = nullptr;  // pinned arena
     size_t pin_cap_ = 0, pin_used_ = 0;

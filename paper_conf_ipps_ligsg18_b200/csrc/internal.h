@@ -87,20 +87,34 @@ struct DpMeta {
                                     // sum_{s' != 0} prod_{i<K-1}(N_i - s'_i + 1) * W + rows * (W - 1)
     int32_t opt;           // OPT(N)
     int32_t err;           // device-detected error (traceback)
+    int32_t ovf;           // enumeration without a host round trip: |C| or the prefix
+                           // list exceeded the preallocated bounds (the fill kernels
+                           // then do nothing and the host redoes the DP synchronously)
+    int32_t pad_;
 };
+
+// Prefix-list bound of a DP enumerated without a host round trip (= the
+// constant bank's CP_MAX): shared-memory tables are sized for it.
+constexpr int64_t NP_CAP = 1000;
+// Heuristic hint for the fill launchers (prefix-list length estimate of the
+// calling DP slot's thread; -1 = use the bound they are given).
+extern thread_local int64_t tl_np_hint;
 
 // ---------------------------------------------------------------- launchers
 // All launchers enqueue on `st` and return cudaGetLastError().
+// pass 1 writes nothing when the total |C| (offsets[nprefix]) exceeds cap
 cudaError_t launch_enum_configs(int pass, int K, int D, int64_t nprefix,
                                 const int32_t *hi, const int64_t *r, int64_t T,
                                 const int64_t *stride, int64_t *d_counts,
                                 const int64_t *d_offsets, uint16_t *d_digits,
-                                int64_t *d_off, cudaStream_t st);
+                                int64_t *d_off, cudaStream_t st, int64_t cap = INT64_MAX);
 cudaError_t launch_exclusive_scan(const int64_t *d_in, int64_t *d_out, int64_t n,
                                   int64_t *d_total, cudaStream_t st);
+// |C| = *d_nC (device); nc_cap / np_cap: bounds of the buffers / of the fill
+// kernels' prefix tables (exceeded: meta->ovf = 1 and nothing else is written)
 cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off,
-                                int64_t nC, const RowGeom &g, const int32_t *Nall,
-                                PrefixEntry *d_pref, DpMeta *d_meta, cudaStream_t st);
+                                const int64_t *d_nC, int64_t nc_cap, int64_t np_cap, const RowGeom &g,
+                                const int32_t *Nall, PrefixEntry *d_pref, DpMeta *d_meta, cudaStream_t st);
 // One row-level of the level fill.  e = 1 or 2.  Rows [slot_begin, slot_begin+slot_count)
 // of row-level rho; results go to the table (compact_out == NULL) or to
 // compact_out[(slot - slot_begin) * Wp + x].

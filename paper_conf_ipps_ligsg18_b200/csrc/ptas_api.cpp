@@ -329,7 +329,12 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 }
                 DpRequest rq = make_rq(cls_v[j0 + b], T_v[j0 + b], nullptr, orders[b],
                                        b == 0 ? (cudaStream_t)opt.stream : nullptr);
-                rq.grid_div = share_grid ? nb : 1;
+                // PTAS_GRID_DIV (experiment knob): 0 = every launch may take the whole GPU
+                static const int gd_env = [] {
+                    const char *t = std::getenv("PTAS_GRID_DIV");
+                    return t && t[0] ? std::atoi(t) : -1;
+                }();
+                rq.grid_div = gd_env == 0 ? 1 : (share_grid ? nb : 1);
                 rcs[b] = sl[b]->run_dp(rq, &outs_all[j0 + b]);
             };
             std::vector<std::thread> th;

@@ -271,6 +271,7 @@ static __constant__ ConstPref c_pref[CP_SLOTS];  // one copy per translation uni
 static __global__ void pack_const_prefix_kernel(const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
                                          int eb, ConstPref *__restrict__ out)
 {
+    if (meta->ovf) return;   // enumeration overflowed its bounds (the fill kernels exit too)
     const int np = (int)(meta->nP - 1);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         out->np = np;
@@ -295,7 +296,7 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
     pack_const_prefix_kernel<<<8, 256, 0, st>>>(d_pref, d_meta, e, (ConstPref *)d_staging);
     cudaError_t err = cudaGetLastError();
     if (err != cudaSuccess) return err;
-    const size_t bytes = 8 + 8 * (size_t)((np + 31) & ~31 < CP_MAX ? ((np + 31) & ~31) : CP_MAX);
+    const size_t bytes = 8 + 8 * (size_t)std::min<int64_t>((np + 31) & ~(int64_t)31, CP_MAX);   // within the slot
     return cudaMemcpyToSymbolAsync(c_pref, d_staging, bytes, (size_t)cslot * sizeof(ConstPref),
                                    cudaMemcpyDeviceToDevice, st);
 }
@@ -345,6 +346,9 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     // prologue now; everything before griddepcontrol.wait below reads only data
     // produced before the first fill launch of the DP (prefix table, row index).
     asm volatile("griddepcontrol.launch_dependents;");
+    // enumeration without a host round trip overflowed its bounds (grid-uniform):
+    // nothing is filled and the host redoes the DP synchronously
+    if (meta->ovf) return;
     const ConstPref &cp = c_pref[CPREF ? cslot : 0];
     const int np = CPREF ? cp.np : (int)(meta->nP - 1);
     // s_oj[c] = oj_entry: int32 offsets (the host routes tables of 2^31 words
@@ -879,12 +883,14 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     const int Lg = Lw / CH;
     const int rpw = 32 / Lg;
     const int bs = 256;
-    const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
+    const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;   // bound: sizes the shared-memory tables
+    // heuristics use the caller's estimate when the exact length is not known on the host
+    const int64_t nph = tl_np_hint >= 0 ? std::min<int64_t>(tl_np_hint, np) : np;
     // small row-levels with long prefix lists: split each row set's prefixes over the 8 warps of a block
     const char *sp = std::getenv("PTAS_SPLIT_ROWS");
     // (worth it when a row's prefix walk has several batches of gathers in series)
     const int PBh = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);
-    const int64_t split_rows = sp ? std::atoll(sp) : ((np + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
+    const int64_t split_rows = sp ? std::atoll(sp) : ((nph + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
     // df->nsplit: 1 = warp row sets, 8 = block row sets, 0 = one cluster in lockstep
     const bool cl = df && df->nsplit == 0;
     const char *cls = std::getenv("PTAS_CL_SIZE");
@@ -896,7 +902,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // prefix windows beyond two words (J * e > 8, J <= J0) need the generic word fetch;
     // the in-row closure handles any shift (registers up to 8 bytes, else shared memory)
     const int win = J0 * e <= 4 ? 4 : (J0 * e <= 8 ? 8 : 0);
-    const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && np >= 64;
+    const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && nph >= 64;
     const char *dwv = std::getenv("PTAS_DF_WAVE");
     const int64_t df_wave = dwv && dwv[0] ? std::max(1, std::atoi(dwv)) : 2;
     DfArgs dfa;

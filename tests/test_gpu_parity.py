@@ -449,3 +449,20 @@ def test_fill_wall_time(P):
             assert abs(st["fill_wall_seconds"] - st["fill_seconds"]) <= 0.02 * st["fill_seconds"] + 2e-5
     st = P.dp_fill(np.array([5, 4, 30], np.int32), np.array([60, 45, 17], np.int64), 160)[2]
     assert st["fill_wall_seconds"] == st["fill_seconds"]
+
+
+@pytest.mark.parametrize("env", [{}, {"PTAS_ENUM_SYNC": "1"}, {"PTAS_NC_CAP": "5"}, {"PTAS_NP_CAP": "3"}])
+def test_enumeration_without_round_trip(P, monkeypatch, env):
+    """DPs after a slot's first are enqueued without reading |C| back (DESIGN.md
+    D9): bit-exact tables on a sequence of DPs of varying size on one slot, with
+    the bounds forced below |C| or the prefix count (every DP overflows, the
+    kernels exit, the DP is redone synchronously) and with the synchronous path."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    rng = np.random.default_rng(91)
+    for it in range(14):
+        K = int(rng.integers(2, 7))
+        N, r, T = _rand_case(rng, K, {2: 40, 3: 20, 4: 9, 5: 6, 6: 4}[K])
+        _check_table(P, N, r, T)
+    for seed in range(6):
+        _cmp_solve(P, jobs(40, 1000, seed), 8, 0.3, 1)
