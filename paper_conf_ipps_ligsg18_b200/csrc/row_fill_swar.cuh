@@ -246,12 +246,15 @@ __device__ __forceinline__ void windows_smem(const uint32_t *srow, int db, int x
 
 // Kernel-side prefix entry: x = -off(s') in words, y = PRMT selector of the
 // window (low 16 bits; the odd-byte selector is y + 0x1111) | db << 16, where
-// db = Jmax(s') * e is the window's byte shift (db = 0: the word itself).
+// db = Jmax(s') * e is the window's byte shift.  db = 0 (the word itself)
+// takes byte offset 4, i.e. the selector reads the high operand (the word)
+// only, so every prefix runs the same branch-free window code.
+constexpr int SEL_U8 = 0xA280, SEL_U16 = 0x3210, SEL_SELF = 0x4444;
 __device__ __forceinline__ int2 oj_entry(const PrefixEntry &pe, int eb)
 {
     const int db = pe.jmax * eb;
-    const int o = (4 - (db & 3)) & 3;
-    const int sel = (eb == 1 ? 0xA280 : 0x3210) + 0x1111 * o;
+    const int o = db == 0 ? 4 : (4 - (db & 3)) & 3;
+    const int sel = (eb == 1 ? SEL_U8 : SEL_U16) + 0x1111 * o;
     return make_int2(-(int)((uint64_t)pe.off * eb / 4), sel | (db << 16));
 }
 
@@ -283,7 +286,7 @@ static __global__ void pack_const_prefix_kernel(const PrefixEntry *__restrict__ 
             const PrefixEntry pe = gpref[1 + i];
             out->oj[i] = oj_entry(pe, eb);
         } else {
-            out->oj[i] = make_int2(0, eb == 1 ? 0xA280 : 0x3210);
+            out->oj[i] = make_int2(0, (eb == 1 ? SEL_U8 : SEL_U16) + SEL_SELF);
         }
     }
 }
@@ -363,7 +366,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #pragma unroll
             for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
         } else if (!CPREF) {
-            s_oj[i] = make_int2(0, EB == 1 ? 0xA280 : 0x3210);
+            s_oj[i] = make_int2(0, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF);
         }
     }
     __syncthreads();
@@ -612,17 +615,13 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 for (int u = 0; u < PB; ++u) {
                     const uint32_t sel = (uint32_t)sj[u];   // warp-uniform
                     Words<CH> lo, hi;
-                    if (sel < 0x10000u) {   // Jmax(s') = 0: the window is the word itself
-                        lo = cur[u];
-                        hi = cur[u];
-                    } else {
-                        // positions before the row read its first entry (clamp to x = 0)
-                        // (db <= 4: only lane xl = 0 reads it, from its own word 0)
-                        uint32_t f = cur[u].v[0];
-                        if (WIN != 4 && (sel >> 16) > 4u) f = __shfl_sync(FULL, f, lane - xl);
-                        f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
-                        windows<CH, WIN>(cur[u], (int)(sel >> 16), xl, f, lo, hi);
-                    }
+                    // positions before the row read its first entry (clamp to x = 0)
+                    // (db <= 4: only lane xl = 0 reads it, from its own word 0).
+                    // Jmax(s') = 0 needs no window: its selector reads `hi` only.
+                    uint32_t f = cur[u].v[0];
+                    if (WIN != 4 && (sel >> 16) > 4u) f = __shfl_sync(FULL, f, lane - xl);
+                    f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
+                    windows<CH, WIN>(cur[u], (int)(sel >> 16), xl, f, lo, hi);
 #pragma unroll
                     for (int t = 0; t < CH; ++t) {
                         if constexpr (EB == 1) {
