@@ -580,9 +580,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 // (after the step with distance d every lane holds the OR of 2d
                 // consecutive group lanes; OR is idempotent, so overlaps are harmless)
                 unsigned bits = 0;
-                const int kmax = (cnt + Lg - 1) / Lg;
-                for (int k = 0; k < kmax; ++k) {
-                    const int c = xl + k * Lg;
+                for (int c0 = 0; c0 < cnt; c0 += Lg) {   // ceil(cnt / Lg) steps, no division
+                    const int c = xl + c0;
                     const bool in = rowok && c < cnt;
                     const int ci = base + (in ? c : 0);
                     bool dom = in;
