@@ -443,6 +443,28 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                               nosync ? np_cap : INT64_MAX, g, N.data(), (PrefixEntry *)pref_.p, d_meta_, st));
     o.launches += 2;
     tl_np_hint = nosync ? np_hint_ : -1;
+    // dominance table of the prefix chunks (D10) when it fits the
+    // shared-memory budget for the prefix-list bound; PTAS_DOMTAB=0: off
+    {
+        int ts = 0;
+        for (int i = 0; i < K - 1; ++i) {
+            g.hi[i] = hi[i];
+            g.dbase[i] = ts;
+            ts += hi[i] + 1;
+        }
+        const int64_t nch = (std::max<int64_t>(nP_bound - 1, 0) + 31) / 32;
+        const char *dt = std::getenv("PTAS_DOMTAB");
+        // (K - 1 >= 4: many leading digits, so few interior rows and long per-row
+        // dominance tests; with 1-3 digits the lane-parallel test is as fast)
+        const bool want = e == 1 && (dt && dt[0] ? dt[0] != '0' : K - 1 >= 4);   // (uint8 kernels only)
+        if (K > 1 && want && (int64_t)ts * nch * 4 <= DOMTAB_MAX_BYTES) {
+            PT_CK(domtab_.ensure((size_t)DOMTAB_MAX_BYTES));
+            g.TS = ts;
+            g.domtab = (const uint32_t *)domtab_.p;
+            PT_CK(launch_build_dom_table((const PrefixEntry *)pref_.p, d_meta_, g, (uint32_t *)domtab_.p, st));
+            ++o.launches;
+        }
+    }
     // prefix offsets into the packed kernel's constant bank
     PT_CK(cpstage_.ensure(const_prefix_staging_bytes()));
     cudaError_t cpe = index_ < 4 ? prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nP_bound, e, g.nwords, index_,

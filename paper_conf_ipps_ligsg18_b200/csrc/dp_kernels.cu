@@ -558,6 +558,43 @@ cudaError_t launch_exclusive_scan(const int64_t *d_in, int64_t *d_out, int64_t n
     return cudaGetLastError();
 }
 
+// Dominance table (D10): word c * TS + dbase[i] + v holds the bits j
+// of prefix chunk c (fill-kernel prefix index 32c + j = entry 1 + 32c + j)
+// whose leading digit i is <= v.  A row p dominates prefix s' iff every digit
+// s'_i <= min(p_i, hi_i), so the row's mask of a chunk is the AND over i of the
+// words at v = min(p_i, hi_i).
+__global__ void build_dom_table_kernel(const PrefixEntry *__restrict__ pref, const DpMeta *__restrict__ meta,
+                                       const RowGeom g, uint32_t *__restrict__ tab)
+{
+    if (meta->ovf) return;
+    const int np = (int)(meta->nP - 1);
+    const int nch = (np + 31) / 32;
+    const int n = nch * g.TS;
+    for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
+        const int c = e / g.TS, r = e - c * g.TS;
+        int i = 0;
+        while (i + 1 < g.K1 && g.dbase[i + 1] <= r) ++i;
+        const int v = r - g.dbase[i];
+        const uint64_t gw = g.guard[g.word[i]] >> g.shift[i];
+        const uint64_t fm = (gw & (~gw + 1)) - 1;   // bits below the field's guard bit
+        uint32_t bits = 0;
+        for (int j = 0; j < 32; ++j) {
+            const int q = 32 * c + j;
+            if (q >= np) break;
+            const uint64_t d = (pref[1 + q].w[g.word[i]] >> g.shift[i]) & fm;
+            if (d <= (uint64_t)v) bits |= 1u << j;
+        }
+        tab[e] = bits;
+    }
+}
+
+cudaError_t launch_build_dom_table(const PrefixEntry *d_pref, const DpMeta *d_meta, const RowGeom &g,
+                                   uint32_t *d_tab, cudaStream_t st)
+{
+    build_dom_table_kernel<<<4, 256, 0, st>>>(d_pref, d_meta, g, d_tab);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off, const int64_t *d_nC,
                                 int64_t nc_cap, int64_t np_cap, const RowGeom &g, const int32_t *Nall,
                                 PrefixEntry *d_pref, DpMeta *d_meta, cudaStream_t st)

@@ -47,7 +47,15 @@ struct RowGeom {
     uint64_t guard[MAXW];       // guard bit per field, per word
     uint64_t maxs[MAXW];        // packed hi_i = min(N_i, T / r_i): the digit-wise max over the prefixes of C(T)
     int32_t nwords;
+    // dominance table (D10): for each 32-prefix chunk, digit i and
+    // value v <= hi_i, the bits of the chunk's prefixes s' with s'_i <= v, at
+    // word chunk * TS + dbase[i] + v.  TS = sum_i (hi_i + 1); 0 = no table.
+    int32_t TS;
+    int32_t hi[MAXK];
+    int32_t dbase[MAXK];
+    const uint32_t *domtab;     // device table (TS > 0)
 };
+constexpr int64_t DOMTAB_MAX_BYTES = 16384;
 
 // Padded row pitch in 32-bit words for a row of `bytes` bytes: a multiple of
 // the packed fill kernel's words per lane (2 up to 64 words, 4 up to 128, 8
@@ -110,6 +118,9 @@ cudaError_t launch_enum_configs(int pass, int K, int D, int64_t nprefix,
                                 int64_t *d_off, cudaStream_t st, int64_t cap = INT64_MAX);
 cudaError_t launch_exclusive_scan(const int64_t *d_in, int64_t *d_out, int64_t n,
                                   int64_t *d_total, cudaStream_t st);
+// Dominance table of the DP's prefixes (g.TS > 0; exits when meta->ovf).
+cudaError_t launch_build_dom_table(const PrefixEntry *d_pref, const DpMeta *d_meta, const RowGeom &g,
+                                   uint32_t *d_tab, cudaStream_t st);
 // |C| = *d_nC (device); nc_cap / np_cap: bounds of the buffers / of the fill
 // kernels' prefix tables (exceeded: meta->ovf = 1 and nothing else is written)
 cudaError_t launch_build_prefix(int K, const uint16_t *d_digits, const int64_t *d_off,

@@ -313,10 +313,10 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
 // are unused, the row sets come from df).
 // Resident blocks per SM the compiler must allow (register cap 65536 / (256 * MINB)):
 // uint16 tables 4 (64 registers: M3s 8.8 -> 8.1 ms, M5s-0.15 21.8 -> 20.3 ms fill,
-// measured), uint8 tables 1 (capping their kernels at 64 registers spills:
-// M2s 3.40 -> 3.59 ms).
+// measured), uint8 tables 3 (80 registers; 64 spills: M2s 3.40 -> 3.59 ms;
+// uncapped, the dominance-table code takes 90-96 and 2 blocks/SM: M4s +13%).
 #ifndef PTAS_MINB_U8
-#define PTAS_MINB_U8 1
+#define PTAS_MINB_U8 3
 #endif
 #ifndef PTAS_MINB_U16
 #define PTAS_MINB_U16 4
@@ -402,6 +402,22 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     // DF + SPLIT: the block's ticket (8-byte aligned after the plan)
     unsigned long long *s_tk =
         reinterpret_cast<unsigned long long *>(s_set + ((RUN ? 2 * (df.nlev + 1) : 0) + 1) / 2 * 2);
+    // dominance table (g.TS > 0, D10): per-digit selectors, then the
+    // chunk words (copied from the DP's table built after the prefix list)
+    int4 *s_dsel = reinterpret_cast<int4 *>(((uintptr_t)(s_tk + 1) + 15) & ~(uintptr_t)15);
+    uint32_t *s_tab = reinterpret_cast<uint32_t *>(s_dsel + g.K1);
+    // (uint8 kernels only: in the 64-register uint16 kernels the extra code
+    // costs more than it saves, measured)
+    const bool use_tab = EB == 1 && g.TS > 0;
+    if (EB == 1 && use_tab) {
+        for (int i = threadIdx.x; i < g.K1; i += blockDim.x) {
+            const uint64_t gw = g.guard[g.word[i]] >> g.shift[i];
+            s_dsel[i] = make_int4(g.shift[i] | (g.word[i] << 8), (int)((gw & (~gw + 1)) - 1), g.hi[i], g.dbase[i]);
+        }
+        const int n = ((np + 31) >> 5) * g.TS;
+        for (int e = threadIdx.x; e < n; e += blockDim.x) s_tab[e] = g.domtab[e];
+        __syncthreads();
+    }
     if constexpr (RUN) {
         for (int i = threadIdx.x; i < 2 * (df.nlev + 1); i += blockDim.x) s_set[i] = df.plan[i];
         __syncthreads();
@@ -580,7 +596,24 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 // (after the step with distance d every lane holds the OR of 2d
                 // consecutive group lanes; OR is idempotent, so overlaps are harmless)
                 unsigned bits = 0;
-                for (int c0 = 0; c0 < cnt; c0 += Lg) {   // ceil(cnt / Lg) steps, no division
+                if (EB == 1 && use_tab) {
+                    // AND over the row's digits of the chunk's table words, the digits
+                    // spread over the group's lanes, then an AND all-reduce over the group
+                    bits = 0xffffffffu;
+                    const uint32_t *tb = s_tab + (base >> 5) * g.TS;
+                    for (int i = xl; i < g.K1; i += Lg) {
+                        const int4 d = s_dsel[i];
+                        const uint64_t wv = NW == 1 ? pw[0] : ((d.x >> 8) ? pw[NW - 1] : pw[0]);
+                        const int v = min((int)((uint32_t)(wv >> (d.x & 0xff)) & (uint32_t)d.y), d.z);
+                        bits &= tb[d.w + v];
+                    }
+                    for (int d = 1; d < Lg; d <<= 1) {
+                        const int xs = xl + d >= Lg ? xl + d - Lg : xl + d;
+                        bits &= __shfl_sync(FULL, bits, lane - xl + xs);
+                    }
+                    bits &= cnt == 32 ? FULL : ((1u << cnt) - 1u);
+                }
+                for (int c0 = 0; c0 < (use_tab ? 0 : cnt); c0 += Lg) {   // ceil(cnt / Lg) steps, no division
                     const int c = xl + c0;
                     const bool in = rowok && c < cnt;
                     const int ci = base + (in ? c : 0);
@@ -590,7 +623,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + ci]) & guard[w]) == guard[w];
                     bits |= dom ? (1u << c) : 0u;
                 }
-                for (int d = 1; d < Lg; d <<= 1) {
+                for (int d = 1; d < (use_tab ? 1 : Lg); d <<= 1) {
                     const int xs = xl + d >= Lg ? xl + d - Lg : xl + d;
                     bits |= __shfl_sync(FULL, bits, lane - xl + xs);
                 }
@@ -855,10 +888,12 @@ static int plan_ch(int e, const RowGeom &g, int J0, int64_t rows, int sm_count, 
     return CH;
 }
 
-static size_t swar_smem(int64_t np, int NW, int nlev_df)
+static size_t swar_smem(int64_t np, int NW, int nlev_df, const RowGeom &g)
 {
+    // s_oj | s_w | pad | s_red | DF plan | ticket (16 B) | dominance selectors + table
     return (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * 8 * 32 * 4 +
-           (nlev_df > 0 ? (size_t)8 * (nlev_df + 1) + 16 : 0);
+           (size_t)8 * (nlev_df + 1) + 32 +
+           (g.TS > 0 ? (size_t)16 * g.K1 + (size_t)((np + 31) / 32) * g.TS * 4 : 0);
 }
 
 // Host launcher body for one (E, NW): returns cudaErrorNotSupported when the
@@ -894,7 +929,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     const char *cls = std::getenv("PTAS_CL_SIZE");
     const int cl_size = cl ? (cls && cls[0] ? std::max(1, std::min(16, std::atoi(cls))) : 16) : 1;
     const int nsplit = df ? (df->nsplit > 1 ? bs / 32 : 1) : (slot_count <= split_rows ? bs / 32 : 1);
-    const size_t smem = swar_smem(np, NW, df ? df->nlev : 0);
+    const size_t smem = swar_smem(np, NW, df ? df->nlev : 0, g);
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     // shifts beyond one word: prefix windows J * e (J <= J0) or chain u16-lane shifts
     // prefix windows beyond two words (J * e > 8, J <= J0) need the generic word fetch;

@@ -466,3 +466,22 @@ def test_enumeration_without_round_trip(P, monkeypatch, env):
         _check_table(P, N, r, T)
     for seed in range(6):
         _cmp_solve(P, jobs(40, 1000, seed), 8, 0.3, 1)
+
+
+@pytest.mark.parametrize("domtab", ["0", "1"])
+def test_dominance_table_modes(P, monkeypatch, domtab):
+    """Per-row dominance masks from the DP's digit-threshold table (DESIGN.md
+    D10, forced on for every K, uint8) or from the lane-parallel packed-digit
+    test (forced off): bit-exact tables either way, in per-level and dataflow
+    launches, including two-word digit packing."""
+    monkeypatch.setenv("PTAS_DOMTAB", domtab)
+    rng = np.random.default_rng(4242)
+    for K in (2, 3, 5, 7, 9):
+        for _ in range(3):
+            N, r, T = _rand_case(rng, K, {2: 60, 3: 25, 5: 8, 7: 4, 9: 3}[K])
+            _check_table(P, N, r, T)
+    monkeypatch.setenv("PTAS_DF", "0")
+    monkeypatch.setenv("PTAS_FORCE_TWO_WORDS", "1")
+    for K in (3, 6):
+        N, r, T = _rand_case(rng, K, {3: 20, 6: 5}[K])
+        _check_table(P, N, r, T)
