@@ -652,6 +652,14 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             dfa.base = ticket_base_;
             dfa.epoch = ++df_epoch_;
             dfa.nsplit = rn.nsplit;
+            // PTAS_DF_SLEEP=a:b: poll backoff from a ns doubling up to b ns
+            {
+                const char *sl = std::getenv("PTAS_DF_SLEEP");
+                int a = 64, b = 64;
+                if (sl && sl[0]) std::sscanf(sl, "%d:%d", &a, &b);
+                dfa.sleep0 = std::max(0, a);
+                dfa.sleep_max = std::max(dfa.sleep0, b);
+            }
             dfa.grid_div = rq.grid_div > 1 ? rq.grid_div : 1;
             // PTAS_DF_PROF=1 (with a PTAS_DF_PROFILE=1 build): per-level set timings of the run
             static const bool df_prof = [] {

@@ -81,6 +81,7 @@ struct DfArgs {
     uint32_t epoch;               // flag value meaning "row done in this launch"
     int32_t nsplit;               // 1: one row set per warp; 8: per block (the warps split the prefix walk)
     int32_t grid_div;             // >1: concurrent DPs, the launch takes 1/grid_div of the resident blocks
+    int32_t sleep0, sleep_max;    // flag-poll backoff (ns): first sleep, cap
     unsigned long long *prof;     // diagnostics build (PTAS_DF_PROFILE): 6 counters per level, else null
     int32_t rstride[MAXK];        // rows between p and p - e_i (leading digit i)
     uint64_t dmask[MAXK];         // bits of leading digit i inside its packed word g.word[i]

@@ -543,6 +543,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         if constexpr (DF) {
             rid = rowok ? (uint32_t)(rowbase * EB / 4) / Lw : 0u;
             if (cur_lv > 0) {
+                uint32_t sleep_ns = (uint32_t)df.sleep0;
                 // wait until every unit predecessor p - e_i (p_i >= 1) is done; by
                 // induction that covers every dominated row, i.e. every source
                 // row p - s' of the prefix walk (rows of the run's first level
@@ -565,7 +566,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                         }
                     }
                     if (__all_sync(FULL, ok)) break;
-                    __nanosleep(64);
+                    __nanosleep(sleep_ns);
+                    if (sleep_ns < df.sleep_max) sleep_ns *= 2;   // backoff (fewer polls, fewer L1 invalidations)
                 }
                 __syncwarp();
             }
