@@ -64,6 +64,7 @@ def _load():
                                       i32p, ctypes.POINTER(ctypes.c_double)]
             lib.oracle_ptas.argtypes = [i64p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double, ctypes.c_int32,
                                         i64p, i64p, i32p, ctypes.POINTER(OracleProbe), ctypes.c_int32, i32p]
+            lib.oracle_hmbp.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, i32p, ctypes.c_int32]
             _lib = lib
     return _lib
 
@@ -151,3 +152,19 @@ def ptas(p, m: int, eps: float, P: int = 1, log_cap: int = 4096):
     probes = [(log[i].T, log[i].round, log[i].feasible, log[i].K, log[i].opt, log[i].sigma)
               for i in range(min(nlog.value, log_cap))]
     return {"T_star": ts.value, "makespan": ms.value, "assignment": asg, "probes": probes}
+
+
+def hmbp(N, r, T: int):
+    """High-multiplicity bin packing (Eq. 1 with capacity T): (bins, packing[bins, K])
+    with the traceback of reading R11 (oracle_hmbp)."""
+    N = np.ascontiguousarray(N, dtype=np.int32)
+    r = np.ascontiguousarray(r, dtype=np.int64)
+    K = len(N)
+    mx = max(int(N.sum()), 1)
+    pk = np.zeros((mx, max(K, 1)), np.int32)
+    bins = ctypes.c_int32()
+    rc = _load().oracle_hmbp(_p(N, ctypes.c_int32), _p(r, ctypes.c_int64), K, int(T), ctypes.byref(bins),
+                             _p(pk, ctypes.c_int32), mx)
+    if rc:
+        raise ValueError(f"oracle_hmbp rc={rc}")
+    return bins.value, pk[:bins.value, :K].copy()

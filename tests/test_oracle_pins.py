@@ -404,3 +404,42 @@ def test_empty_dp_path_literal_configs():
         # with no long jobs the schedule is the greedy list schedule: makespan <= A + max p
         LB, UB = oracle.bounds(p, w.m)
         assert res["makespan"] <= UB
+
+
+# ---------------------------------------------------------------- high-multiplicity bin packing
+def test_hmbp_bins_equal_exhaustive_and_packing_valid():
+    """oracle.hmbp: the bin count equals the exhaustive
+    set-partition optimum, and the packing is a valid partition: every bin
+    holds at most T, no bin is empty, per-class totals equal N."""
+    rng = np.random.default_rng(71)
+    for _ in range(50):
+        K = int(rng.integers(1, 5))
+        N = rng.integers(0, 4, K)
+        while N.sum() > 10 or N.sum() == 0:
+            N = rng.integers(0, 4, K)
+        r = rng.integers(5, 60, K)
+        T = int(rng.integers(int(r.max()), 150))
+        bins, pk = oracle.hmbp(N, r, T)
+        items = [int(r[i]) for i in range(K) for _ in range(int(N[i]))]
+        assert bins == _min_bins_all_subsets(items, T)[(1 << len(items)) - 1]
+        assert pk.shape == (bins, K)
+        assert (pk.sum(axis=0) == N).all()
+        assert ((pk * r).sum(axis=1) <= T).all() and (pk.sum(axis=1) > 0).all()
+
+
+def test_hmbp_closed_forms_and_edges():
+    # K = 1: ceil(N / floor(T / r)) bins; reading R11 takes the smallest s that
+    # keeps OPT(n - s) = OPT(n) - 1 first (2 of 17, then full bins of 3)
+    bins, pk = oracle.hmbp([17], [30], 100)
+    assert bins == 6 and pk[:, 0].tolist() == [2, 3, 3, 3, 3, 3]
+    # zero counts and an all-zero instance
+    assert oracle.hmbp([0, 0], [5, 7], 10)[0] == 0
+    bins, pk = oracle.hmbp([0, 4], [50, 5], 10)
+    assert bins == 2 and (pk[:, 0] == 0).all()
+    # load bound ceil(32 / 10) = 4 is met: {6,4} {6,4} {3,3,3} {3}
+    bins, _ = oracle.hmbp([2, 2, 4], [6, 4, 3], 10)
+    assert bins == 4
+    # 3 items of 5 and 3 of 4, capacity 9: every bin holds at most one 5 => 3 bins
+    assert oracle.hmbp([3, 3], [5, 4], 9)[0] == 3
+    with pytest.raises(ValueError):
+        oracle.hmbp([1], [11], 10)   # an item larger than the capacity
