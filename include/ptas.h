@@ -177,6 +177,26 @@ int dp_fill(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T,
             void *table_out, int64_t table_bytes, int32_t *opt_N_out,
             ptas_stats *stats);
 
+/* High-multiplicity bin packing on the same level-fill engine (SURVEY.md
+ * §8(f)-4; the paper's future work on other higher-dimensional DPs,
+ * PAPER.md:472).  Eq. 1 with T = capacity and r = sizes is
+ * exactly this problem: OPT(N) is the minimum number of bins of capacity
+ * `capacity` that hold counts[i] items of size sizes[i].
+ *   counts[K], sizes[K] : host arrays (caller order; zero counts allowed)
+ *   bins_out            : host, receives OPT(N) (minimum number of bins)
+ *   packing_out         : host, nullable; [max_bins][K] int32, row b = items
+ *                         of each class in bin b, bins in traceback order
+ *                         (reading R11: first configuration in lexicographic
+ *                         order of the caller's class order)
+ *   max_bins            : rows of packing_out; must be >= sum(counts)
+ *   stats               : nullable, as dp_fill (+ traceback launches)
+ * The table is laid out internally by ascending count (D2); the
+ * result does not depend on it.  Errors: as dp_fill (EINVAL for a size >
+ * capacity with a positive count, capacity < 1, ...), EINVAL if packing_out
+ * is given with max_bins < sum(counts).  Nothing is written on error. */
+int hmbp_solve(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t capacity,
+               int32_t *bins_out, int32_t *packing_out, int32_t max_bins, ptas_stats *stats);
+
 /* As dp_fill, into a caller-owned device buffer d_table (>= sigma*e bytes,
  * e.g. a torch uint8/uint16 tensor) on the current device, enqueued on
  * cuda_stream (a cudaStream_t; NULL = legacy default stream).  The call

@@ -13,7 +13,7 @@ import numpy as np
 from ._native import (MODE_LEVEL_SHARDED, MODE_MULTI_PROBE, MODE_SINGLE, EXPORTS, PtasError, PtasOptions,
                       PtasProbe, PtasStats, _a, _chk, _ptr, lib, strerror)
 
-__all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "dp_table_shape", "dp_configs",
+__all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
            "dp_row_index", "ptas_k", "ptas_bounds", "ptas_classify", "ptas_probe_targets",
            "ptas_interval_update", "ptas_shard_range", "Comm", "init_comm", "options", "lib", "strerror",
            "PtasError", "EXPORTS", "MODE_SINGLE", "MODE_LEVEL_SHARDED", "MODE_MULTI_PROBE"]
@@ -94,6 +94,23 @@ def dp_fill(counts, sizes, T: int, table: bool = True):
     if table:
         out = out.reshape(tuple(int(x) + 1 for x in c)) if len(c) else out.reshape(())
     return opt.value, out, st.to_dict()
+
+
+def hmbp_solve(counts, sizes, capacity: int, packing: bool = True):
+    """High-multiplicity bin packing on the level-fill engine (include/ptas.h):
+    (bins, packing[bins, K] int32 or None, stats)."""
+    c = _a(counts, np.int32)
+    s = _a(sizes, np.int64)
+    K = len(c)
+    mx = max(int(c.sum()), 1)
+    pk = np.zeros((mx, max(K, 1)), np.int32) if packing else None
+    bins = ctypes.c_int32()
+    st = PtasStats()
+    rc = lib().hmbp_solve(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), K, int(capacity), ctypes.byref(bins),
+                          pk.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)) if packing else None, mx,
+                          ctypes.byref(st))
+    _chk("hmbp_solve", rc)
+    return bins.value, (pk[:bins.value, :K].copy() if packing else None), st.to_dict()
 
 
 def dp_fill_device(counts, sizes, T: int, table_dev, stream=None) -> int:

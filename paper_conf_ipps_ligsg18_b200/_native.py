@@ -55,7 +55,7 @@ EXPORTS = [
     "ptas_default_options", "ptas_solve", "ptas_solve_ex", "ptas_solve_device", "dp_table_shape", "dp_fill",
     "dp_fill_device", "ptas_get_unique_id", "ptas_comm_init", "ptas_comm_destroy", "ptas_strerror", "ptas_k",
     "ptas_bounds", "ptas_classify", "ptas_probe_targets", "ptas_interval_update", "ptas_shard_range",
-    "dp_configs", "dp_row_index",
+    "dp_configs", "dp_row_index", "hmbp_solve",
 ]
 
 _lib = None
@@ -99,6 +99,8 @@ def lib():
     L.ptas_interval_update.argtypes = [i64p, i64p, i64p, i32p, ctypes.c_int32]
     L.ptas_shard_range.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, i64p, i64p]
     L.dp_configs.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, ctypes.c_int64, i64p]
+    L.hmbp_solve.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, i32p, ctypes.c_int32,
+                             ctypes.POINTER(PtasStats)]
     L.dp_row_index.argtypes = [i32p, ctypes.c_int32, i64p, ctypes.c_int64, i64p, ctypes.c_int64]
     _lib = L
     return L

@@ -892,6 +892,74 @@ static int dp_fill_common(const int32_t *counts, const int64_t *sizes, int32_t K
     return PTAS_OK;
 }
 
+int hmbp_solve(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t capacity, int32_t *bins_out,
+               int32_t *packing_out, int32_t max_bins, ptas_stats *stats)
+{
+    const double t0 = now_s();
+    int rc = validate_dp(counts, sizes, K, capacity);
+    if (rc) return rc;
+    if (!bins_out) return PTAS_EINVAL;
+    int64_t total = 0;
+    std::vector<int32_t> N(counts, counts + K);
+    for (int32_t x : N) total += x;
+    if (packing_out && max_bins < total) return PTAS_EINVAL;
+    Acc acc;
+    if (total == 0) {
+        *bins_out = 0;
+        if (stats) {
+            acc.s.total_seconds = now_s() - t0;
+            *stats = acc.s;
+        }
+        return PTAS_OK;
+    }
+    int64_t sigma;
+    int32_t e;
+    rc = dp_table_shape(counts, K, &sigma, &e);
+    if (rc) return rc;
+    int dev;
+    rc = resolve_device(-1, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+    // internal layout: the non-empty classes by ascending count (D2)
+    std::vector<int> order;
+    for (int i = 0; i < K; ++i)
+        if (N[i] > 0) order.push_back(i);
+    std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return N[a] < N[b]; });
+    DpRequest rq;
+    rq.K = K;
+    rq.N = counts;
+    rq.r = sizes;
+    rq.T = capacity;
+    rq.order = order.data();
+    DpOutcome o;
+    rc = eng->run_dp(rq, &o);
+    if (rc) return rc;
+    acc.add(o);
+    acc.s.fill_wall_seconds = o.fill_s;
+    std::vector<MachineCfg> bins;   // canonical (caller-order) digit vectors, traceback order
+    DpOutcome tb;
+    rc = eng->traceback(&bins, &tb);
+    if (rc) return rc;
+    if ((int32_t)bins.size() != o.opt) return PTAS_EINTERNAL;
+    acc.s.kernel_launches += tb.launches;
+    acc.s.h2d_bytes += tb.h2d;
+    acc.s.d2h_bytes += tb.d2h;
+    if (packing_out)
+        for (size_t b = 0; b < bins.size(); ++b)
+            for (int i = 0; i < K; ++i) packing_out[(int64_t)b * K + i] = bins[b][i];
+    *bins_out = o.opt;
+    if (stats) {
+        acc.s.unique_dps = 1;
+        acc.s.opt_at_Tstar = o.opt;
+        acc.s.total_seconds = now_s() - t0;
+        *stats = acc.s;
+    }
+    return PTAS_OK;
+}
+
 int dp_fill(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, void *table_out,
             int64_t table_bytes, int32_t *opt_N_out, ptas_stats *stats)
 {

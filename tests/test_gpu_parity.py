@@ -485,3 +485,34 @@ def test_dominance_table_modes(P, monkeypatch, domtab):
     for K in (3, 6):
         N, r, T = _rand_case(rng, K, {3: 20, 6: 5}[K])
         _check_table(P, N, r, T)
+
+
+def test_hmbp_parity(P):
+    """High-multiplicity bin packing (include/ptas.h hmbp_solve):
+    bin count and packing identical to oracle.hmbp (same R11 traceback) on
+    random instances incl. zero counts, uint16 tables and K = 1; a valid
+    packing with the load bound at a larger size."""
+    rng = np.random.default_rng(808)
+    for it in range(40):
+        K = int(rng.integers(1, 7))
+        N = rng.integers(0, {1: 300, 2: 40, 3: 16, 4: 8, 5: 5, 6: 4}[K], K).astype(np.int32)
+        if it % 5 == 0:
+            N[rng.integers(0, K)] = 0
+        if N.sum() == 0:
+            N[0] = 3
+        r = rng.integers(5, 100, K).astype(np.int64)
+        T = int(rng.integers(int(r.max()), int(r.max()) * 4))
+        bins, pk, st = P.hmbp_solve(N, r, T)
+        wb, wpk = oracle.hmbp(N, r, T)
+        assert bins == wb and pk.tolist() == wpk.tolist(), (N, r, T)
+        assert st["kernel_launches"] > 0
+    assert P.hmbp_solve([0, 0], [3, 4], 10)[0] == 0
+    with pytest.raises(P.PtasError):
+        P.hmbp_solve([1], [11], 10)
+    # larger instance: validity + load bound (no oracle call on the full size)
+    N = np.array([30, 25, 17, 20, 19, 13], np.int32)
+    r = np.array([244, 355, 423, 511, 592, 677], np.int64)
+    bins, pk, _ = P.hmbp_solve(N, r, 1674)
+    assert (pk.sum(axis=0) == N).all() and ((pk * r).sum(axis=1) <= 1674).all()
+    assert bins >= -(-int((N * r).sum()) // 1674)
+    assert bins == P.dp_fill(N, r, 1674, table=False)[0]
