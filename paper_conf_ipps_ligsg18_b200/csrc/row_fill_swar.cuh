@@ -404,7 +404,9 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         reinterpret_cast<unsigned long long *>(s_set + ((RUN ? 2 * (df.nlev + 1) : 0) + 1) / 2 * 2);
     // dominance table (g.TS > 0, D10): per-digit selectors, then the
     // chunk words (copied from the DP's table built after the prefix list)
-    int4 *s_dsel = reinterpret_cast<int4 *>(((uintptr_t)(s_tk + 1) + 15) & ~(uintptr_t)15);
+    // (offset arithmetic from smem_raw keeps the shared state space: LDS, not generic loads)
+    int4 *s_dsel = reinterpret_cast<int4 *>(
+        smem_raw + ((reinterpret_cast<unsigned char *>(s_tk + 1) - smem_raw + 15) & ~(ptrdiff_t)15));
     uint32_t *s_tab = reinterpret_cast<uint32_t *>(s_dsel + g.K1);
     // (uint8 kernels only: in the 64-register uint16 kernels the extra code
     // costs more than it saves, measured)
