@@ -397,7 +397,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         maxs[w] = g.maxs[w];
     }
     // DF: per-level first set / first slot of the run, in shared memory
-    int32_t *s_set = reinterpret_cast<int32_t *>(s_red + (size_t)(256 / 32) * 2 * 8 * 32);
+    int32_t *s_set = reinterpret_cast<int32_t *>(s_red + (size_t)(256 / 32) * 2 * CH * 32);
     int32_t *s_sl = s_set + (RUN ? df.nlev + 1 : 0);
     // DF + SPLIT: the block's ticket (8-byte aligned after the plan)
     unsigned long long *s_tk =
@@ -892,10 +892,11 @@ static int plan_ch(int e, const RowGeom &g, int J0, int64_t rows, int sm_count, 
     return CH;
 }
 
-static size_t swar_smem(int64_t np, int NW, int nlev_df, const RowGeom &g)
+static size_t swar_smem(int64_t np, int NW, int nlev_df, const RowGeom &g, int CH)
 {
     // s_oj | s_w | pad | s_red | DF plan | ticket (16 B) | dominance selectors + table
-    return (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * 8 * 32 * 4 +
+    // (s_red sized for the kernel's lane chunk: smem left over is L1 for the gathers)
+    return (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * CH * 32 * 4 +
            (size_t)8 * (nlev_df + 1) + 32 +
            (g.TS > 0 ? (size_t)16 * g.K1 + (size_t)((np + 31) / 32) * g.TS * 4 : 0);
 }
@@ -933,7 +934,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     const char *cls = std::getenv("PTAS_CL_SIZE");
     const int cl_size = cl ? (cls && cls[0] ? std::max(1, std::min(16, std::atoi(cls))) : 16) : 1;
     const int nsplit = df ? (df->nsplit > 1 ? bs / 32 : 1) : (slot_count <= split_rows ? bs / 32 : 1);
-    const size_t smem = swar_smem(np, NW, df ? df->nlev : 0, g);
+    const size_t smem = swar_smem(np, NW, df ? df->nlev : 0, g, CH);
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     // shifts beyond one word: prefix windows J * e (J <= J0) or chain u16-lane shifts
     // prefix windows beyond two words (J * e > 8, J <= J0) need the generic word fetch;
@@ -961,6 +962,11 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
         if (smem > 48 * 1024) {                                                                           \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);      \
             if (err != cudaSuccess) return err;                                                           \
+        }                                                                                                 \
+        {   /* PTAS_CARVEOUT=<pct> (experiment): preferred shared-memory carveout */                     \
+            static const int co = [] { const char *t = std::getenv("PTAS_CARVEOUT");                     \
+                                       return t && t[0] ? std::atoi(t) : -1; }();                          \
+            if (co >= 0) cudaFuncSetAttribute(kfn, cudaFuncAttributePreferredSharedMemoryCarveout, co);    \
         }                                                                                                 \
         if (cl && cl_size > 8) {                                                                          \
             err = cudaFuncSetAttribute(kfn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);           \
