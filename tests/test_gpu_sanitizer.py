@@ -55,6 +55,14 @@ def _run(tool, extra_env=None, timeout=900):
 
 
 @pytest.mark.timeout(1200)
+@pytest.mark.parametrize("env", [{"PTAS_DOMTAB": "1"}, {"PTAS_NC_CAP": "5"}, {"PTAS_NP_CAP": "2"}])
+def test_memcheck_domtab_and_round_trip_free_enumeration(env):
+    # dominance table forced for every geometry (D10); enumeration
+    # bounds forced below |C| / the prefix count (D9: kernels exit, DP redone)
+    _run("memcheck", env)
+
+
+@pytest.mark.timeout(1200)
 def test_memcheck_fill_layouts():
     _run("memcheck")
 
