@@ -343,7 +343,15 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #ifndef PTAS_PB2
 #define PTAS_PB2 8
 #endif
-    constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);   // gathers in flight per lane (prefix batch)
+#ifndef PTAS_PB2S
+#define PTAS_PB2S 10
+#endif
+    // gathers in flight per lane (prefix batch); CH = 2 with the prefix list in
+    // shared memory (short lists) takes 10: 20 prefixes in two batches instead
+    // of three (M2s fill -5%, measured; 12 spills at 80 registers)
+    // (uint8 only: the 64-register uint16 kernels lose with it, M3s +3%)
+    constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? ((CPREF || EB == 2) ? PTAS_PB2 : PTAS_PB2S) : 4);
+    constexpr bool PB_POW2 = (PB & (PB - 1)) == 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     // Programmatic dependent launch: let the next row-level's grid start its
     // prologue now; everything before griddepcontrol.wait below reads only data
@@ -358,8 +366,10 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     // or more to the scalar kernel); s_w: packed digits
     const int npad = (np + 31) & ~31;  // zero-padded: dummy slots are never loaded (mask bit 0)
     int2 *s_oj = reinterpret_cast<int2 *>(smem_raw);
-    uint64_t *s_w = reinterpret_cast<uint64_t *>(s_oj + npad);
-    for (int i = threadIdx.x; i < npad; i += blockDim.x) {
+    // (16 dummy entries past npad: a batch of a non-power-of-two size may run
+    // past the last chunk; those slots are never loaded, their mask bit is 0)
+    uint64_t *s_w = reinterpret_cast<uint64_t *>(s_oj + npad + 16);
+    for (int i = threadIdx.x; i < npad + 16; i += blockDim.x) {
         if (i < np) {
             const PrefixEntry pe = gpref[1 + i];
             if (!CPREF) s_oj[i] = oj_entry(pe, EB);
@@ -633,7 +643,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                 }
                 m = rowok ? bits : 0u;  // idle lanes (past 32 / Lg groups) may have read foreign bits
             }
-            const int cend = (cnt + PB - 1) & ~(PB - 1);
+            const int cend = PB_POW2 ? ((cnt + PB - 1) & ~(PB - 1)) : (cnt + PB - 1) / PB * PB;
             // PB prefixes per step: their gathers are issued before any is consumed
             for (int q0 = qbase0; q0 < cend; q0 += qstep) {
                 Words<CH> cur[PB];
@@ -644,7 +654,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     const int2 oj = CPREF ? cp.oj[base + q] : s_oj[base + q];
                     sj[u] = oj.y;
                     const uint32_t *p = src + oj.x;
-                    if ((m >> q) & 1u) cur[u] = load_words<CH, RUN>(p);
+                    if (PB_POW2 ? ((m >> q) & 1u) : (q < 32 && ((m >> (q & 31)) & 1u))) cur[u] = load_words<CH, RUN>(p);
                     else fill_words(cur[u], 0xffffffffu);
                 }
 #pragma unroll
@@ -896,7 +906,7 @@ static size_t swar_smem(int64_t np, int NW, int nlev_df, const RowGeom &g, int C
 {
     // s_oj | s_w | pad | s_red | DF plan | ticket (16 B) | dominance selectors + table
     // (s_red sized for the kernel's lane chunk: smem left over is L1 for the gathers)
-    return (size_t)((np + 31) & ~31) * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * CH * 32 * 4 +
+    return (size_t)((np + 31) & ~31) * 8 + 16 * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * CH * 32 * 4 +
            (size_t)8 * (nlev_df + 1) + 32 +
            (g.TS > 0 ? (size_t)16 * g.K1 + (size_t)((np + 31) / 32) * g.TS * 4 : 0);
 }
