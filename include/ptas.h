@@ -72,10 +72,12 @@ typedef struct {
     void *stream;               /* cudaStream_t for all device work of the call
                                    (NULL = the library's own stream); the call
                                    still returns only when its work is done       */
-    int32_t speculate;          /* P = 1, SINGLE mode: evaluate the next levels of
-                                   Alg 1's bisection tree concurrently while the
-                                   DPs are small (-1 = library default, 0 = off,
-                                   d = up to 2^d - 1 probes in flight).  The probe
+    int32_t speculate;          /* P = 1, SINGLE mode: evaluate upcoming probes of
+                                   Alg 1 concurrently while the DPs are small
+                                   (-1 = library default: the next 4 probes on
+                                   the all-feasible path; 0 = off; d > 0 = the
+                                   whole bisection tree d levels deep, up to
+                                   2^d - 1 probes in flight).  The probe
                                    sequence, T* and the schedule are those of
                                    Alg 1 (D8); only time changes.      */
 } ptas_options;

@@ -421,7 +421,7 @@ def test_speculation_preserves_alg1(P):
     for p, m, eps in cases:
         ref = P.ptas_solve(p, m, eps, P=1, speculate=0)
         assert ref["stats"]["spec_dps"] == 0
-        for d in (1, 2, 3):
+        for d in (1, 2, 3, -1):   # -1: the default feasible-branch chain
             got = P.ptas_solve(p, m, eps, P=1, speculate=d)
             assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
             assert (got["assignment"] == ref["assignment"]).all()
