@@ -365,32 +365,40 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     std::memcpy(small.data(), r.data(), (size_t)K * 8);
     std::memcpy(small.data() + K * 8, stride.data(), (size_t)K * 8);
     std::memcpy(small.data() + K * 16, hi.data(), (size_t)K * 4);
-    PT_CK(small_.ensure(small_bytes));
-    // cnt table followed by level_start[rho_max + 2] (prefix sums of the row counts)
+    // one upload (one API call): [r | stride | hi] (8-byte padded), then the
+    // cnt table and level_start[rho_max + 2] (prefix sums of the row counts)
     std::vector<int64_t> lstart((size_t)g.rho_max + 2, 0);
     for (int rho = 0; rho <= g.rho_max; ++rho) lstart[rho + 1] = lstart[rho] + cnt[rho];
     const size_t cnt_words = cnt.size() + lstart.size();
-    PT_CK(cnt_.ensure(cnt_words * 8));
+    const size_t small_pad = (small_bytes + 7) & ~(size_t)7;
+    small.resize(small_pad + cnt_words * 8, 0);
+    std::memcpy(small.data() + small_pad, cnt.data(), cnt.size() * 8);
+    std::memcpy(small.data() + small_pad + cnt.size() * 8, lstart.data(), lstart.size() * 8);
+    PT_CK(cnt_.ensure(small.size()));
     pin_reset();
-    PT_CK(h2d(small_.p, small.data(), small_bytes, st));
-    PT_CK(h2d(cnt_.p, cnt.data(), cnt.size() * 8, st));
-    PT_CK(h2d((int64_t *)cnt_.p + cnt.size(), lstart.data(), lstart.size() * 8, st));
-    o.h2d += (int64_t)(small_bytes + cnt_words * 8);
+    PT_CK(h2d(cnt_.p, small.data(), small.size(), st));
+    o.h2d += (int64_t)small.size();
+    void *const d_small = cnt_.p;
+    const int64_t *d_cnt = (const int64_t *)((unsigned char *)cnt_.p + small_pad);
     // ---- a-4 level-ordered row index (row base + packed leading digits per row)
     const int NWk = g.nwords <= 1 ? 1 : 2;
     PT_CK(rowidx_.ensure((size_t)rows * 8 * (1 + NWk)));
     int64_t *d_rb = (int64_t *)rowidx_.p;
     uint64_t *d_pw = (uint64_t *)(d_rb + rows);
     // on the side stream: overlaps the enumeration below and its host round trip
-    PT_CK(cudaEventRecord(ev_fork_, st));
-    PT_CK(cudaStreamWaitEvent(side_, ev_fork_, 0));
-    PT_CK(launch_build_row_index(g, (const int64_t *)cnt_.p, (const int64_t *)cnt_.p + cnt.size(), rows, d_rb,
-                                 d_pw, side_));
-    PT_CK(cudaEventRecord(ev_join_, side_));
+    // (PTAS_ROWIDX_MAIN=1: on the DP's own stream, three API calls fewer)
+    const char *rim = std::getenv("PTAS_ROWIDX_MAIN");
+    const bool ri_main = rim && rim[0] == '1';
+    if (!ri_main) {
+        PT_CK(cudaEventRecord(ev_fork_, st));
+        PT_CK(cudaStreamWaitEvent(side_, ev_fork_, 0));
+    }
+    PT_CK(launch_build_row_index(g, d_cnt, d_cnt + cnt.size(), rows, d_rb, d_pw, ri_main ? st : side_));
+    if (!ri_main) PT_CK(cudaEventRecord(ev_join_, side_));
     ++o.launches;
-    const int64_t *d_r = (const int64_t *)small_.p;
-    const int64_t *d_stride = (const int64_t *)((unsigned char *)small_.p + K * 8);
-    const int32_t *d_hi = (const int32_t *)((unsigned char *)small_.p + K * 16);
+    const int64_t *d_r = (const int64_t *)d_small;
+    const int64_t *d_stride = (const int64_t *)((unsigned char *)d_small + K * 8);
+    const int32_t *d_hi = (const int32_t *)((unsigned char *)d_small + K * 16);
 
     // ---- a-3 configuration enumeration
     int D = 0;
@@ -627,7 +635,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     }
     size_t next_run = 0;
 
-    PT_CK(cudaStreamWaitEvent(st, ev_join_, 0));   // row index ready
+    if (!ri_main) PT_CK(cudaStreamWaitEvent(st, ev_join_, 0));   // row index ready
     PT_CK(cudaEventRecord(ev_[1], st));
     // PTAS_LEVEL_TIMES=1: per-row-level device times (events between launches; diagnostics)
     static const bool lvl_times = [] {
@@ -757,7 +765,11 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     }
     PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
     PT_CK(cudaEventRecord(ev_[3], st));
-    PT_CK(sync_spin(st));
+    for (;;) {   // spin on the end event itself (one event record fewer than sync_spin)
+        const cudaError_t q = cudaEventQuery(ev_[3]);
+        if (q == cudaSuccess) break;
+        if (q != cudaErrorNotReady) PT_CK(q);
+    }
     o.d2h += sizeof(DpMeta);
     float ms = 0;
     PT_CK(cudaEventElapsedTime(&ms, ev_[0], ev_[3]));

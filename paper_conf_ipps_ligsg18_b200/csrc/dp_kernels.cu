@@ -12,6 +12,7 @@
 // Integer-only; no tensor cores (the DP is a min over gathers, not a
 // contraction).  See DESIGN.md for the roofline of each kernel.
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "internal.h"
@@ -511,6 +512,65 @@ traceback_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__
     if (tid == 0) *len = mu;
 }
 
+// Same traceback by ONE warp with the configurations staged in shared memory:
+// no block barriers and no global reads besides the two table entries per
+// step (OPT(n) and OPT(n - s), issued together), so a step is about one L2
+// round trip.  The canonical ranks are unique, so the warp minimum of the
+// candidate ranks names exactly one configuration.
+template <typename E>
+__global__ void __launch_bounds__(32)
+traceback_warp_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__ N,
+                      const uint16_t *__restrict__ digits, const int64_t *__restrict__ off,
+                      const int32_t *__restrict__ rank, int nC, int64_t idx_start, int32_t *__restrict__ out,
+                      int32_t max_out, int32_t *__restrict__ len, DpMeta *meta)
+{
+    extern __shared__ __align__(16) unsigned char tb_smem[];
+    int64_t *s_off = reinterpret_cast<int64_t *>(tb_smem);
+    int32_t *s_rank = reinterpret_cast<int32_t *>(s_off + nC);
+    int32_t *s_cur = s_rank + nC;
+    uint16_t *s_dig = reinterpret_cast<uint16_t *>(s_cur + K);
+    const int lane = threadIdx.x;
+    for (int c = lane; c < nC; c += 32) {
+        s_off[c] = off[c];
+        s_rank[c] = rank[c];
+    }
+    for (int i = lane; i < nC * K; i += 32) s_dig[i] = digits[i];
+    for (int i = lane; i < K; i += 32) s_cur[i] = N[i];
+    __syncwarp();
+    int64_t idx = idx_start;
+    int32_t mu = 0;
+    bool err = false;
+    while (idx != 0) {
+        const int v = (int)table[idx];
+        uint32_t bestr = 0xffffffffu;
+        int bestc = -1;
+        for (int c = lane; c < nC; c += 32) {
+            bool dom = true;
+            for (int i = 0; i < K; ++i) dom &= s_dig[c * K + i] <= s_cur[i];
+            if (dom && (int)table[idx - s_off[c]] == v - 1 && (uint32_t)s_rank[c] < bestr) {
+                bestr = (uint32_t)s_rank[c];
+                bestc = c;
+            }
+        }
+        const uint32_t m = __reduce_min_sync(FULL, bestr);
+        if (m == 0xffffffffu || mu >= max_out) {
+            err = true;
+            break;
+        }
+        const int c = __shfl_sync(FULL, bestc, __ffs(__ballot_sync(FULL, bestr == m)) - 1);
+        if (lane == 0) out[mu] = c;
+        ++mu;
+        idx -= s_off[c];
+        __syncwarp();
+        for (int i = lane; i < K; i += 32) s_cur[i] -= s_dig[c * K + i];
+        __syncwarp();
+    }
+    if (lane == 0) {
+        *len = mu;
+        if (err) meta->err = 1;
+    }
+}
+
 template <typename E>
 __global__ void compact_rows_kernel(const E *__restrict__ src, E *__restrict__ dst, int64_t rows, int64_t W,
                                     int64_t Wp)
@@ -697,6 +757,19 @@ cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N
                              const int32_t *d_rank, int64_t nC, int64_t idx_start, int32_t *d_out,
                              int32_t max_out, int32_t *d_len, DpMeta *d_meta, cudaStream_t st)
 {
+    // one warp with the configurations in shared memory when they fit (48 KB)
+    const size_t smem = (size_t)nC * (8 + 4) + (size_t)K * 4 + (size_t)nC * K * 2 + 16;
+    const char *tbb = std::getenv("PTAS_TB_BLOCK");   // tests: force the block kernel
+    if (smem <= 48 * 1024 && !(tbb && tbb[0] == '1')) {
+        if (e == 1)
+            traceback_warp_kernel<uint8_t><<<1, 32, smem, st>>>((const uint8_t *)table, K, d_N, d_digits, d_off, d_rank,
+                                                                (int)nC, idx_start, d_out, max_out, d_len, d_meta);
+        else
+            traceback_warp_kernel<uint16_t><<<1, 32, smem, st>>>((const uint16_t *)table, K, d_N, d_digits, d_off,
+                                                                 d_rank, (int)nC, idx_start, d_out, max_out, d_len,
+                                                                 d_meta);
+        return cudaGetLastError();
+    }
     if (e == 1)
         traceback_kernel<uint8_t><<<1, 256, 0, st>>>((const uint8_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, idx_start, d_out, max_out, d_len, d_meta);
     else

@@ -516,3 +516,23 @@ def test_hmbp_parity(P):
     assert (pk.sum(axis=0) == N).all() and ((pk * r).sum(axis=1) <= 1674).all()
     assert bins >= -(-int((N * r).sum()) // 1674)
     assert bins == P.dp_fill(N, r, 1674, table=False)[0]
+
+
+@pytest.mark.parametrize("tb", ["0", "1"])
+def test_traceback_kernels(P, monkeypatch, tb):
+    """Warp traceback (configurations in shared memory) and the block kernel:
+    identical schedules, equal to the oracle's (reading R11)."""
+    monkeypatch.setenv("PTAS_TB_BLOCK", tb)
+    for seed in range(12):
+        _cmp_solve(P, jobs(12, 100, seed), 3, 0.3, 1)
+    for (n, m, eps, seed) in [(40, 8, 0.3, 1), (60, 14, 0.3, 2), (50, 10, 0.2, 3)]:
+        _cmp_solve(P, jobs(n, 1000, seed), m, eps, 1)
+    rng = np.random.default_rng(99)
+    for _ in range(6):
+        K = int(rng.integers(2, 6))
+        N = rng.integers(1, 9, K).astype(np.int32)
+        r = rng.integers(5, 80, K).astype(np.int64)
+        T = int(rng.integers(int(r.max()), int(r.max()) * 3))
+        bins, pk, _ = P.hmbp_solve(N, r, T)
+        wb, wpk = oracle.hmbp(N, r, T)
+        assert bins == wb and pk.tolist() == wpk.tolist()
