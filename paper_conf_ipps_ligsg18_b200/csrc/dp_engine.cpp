@@ -838,6 +838,41 @@ int DpSlot::traceback(std::vector<MachineCfg> *machines, DpOutcome *acc)
     const int K = last_K_;
     const int64_t nC = last_nC_;
     cudaStream_t st = last_stream_;
+    {
+        // device ranking + canonical output: one upload, two kernels, one readback
+        const int Kc = last_Kcanon_;
+        std::vector<int32_t> up((size_t)K + Kc, -1);
+        std::copy(last_N_.begin(), last_N_.end(), up.begin());
+        for (int i = 0; i < K; ++i) up[(size_t)K + last_order_[i]] = i;
+        const size_t tb_bytes = ((size_t)nC + K + Kc + 4 + (size_t)last_opt_ * (1 + Kc)) * 4 + 16;
+        PT_CK(tb_.ensure(tb_bytes));
+        int32_t *d_N = (int32_t *)tb_.p;
+        int32_t *d_inv = d_N + K;
+        int32_t *d_rank = d_inv + Kc;
+        int32_t *d_len = d_rank + nC;   // [4] then d_out[opt], then d_out_dig[opt][Kc]
+        int32_t *d_out = d_len + 4;
+        int32_t *d_out_dig = d_out + last_opt_;
+        pin_reset();
+        PT_CK(h2d(d_N, up.data(), up.size() * 4, st));
+        PT_CK(cudaMemsetAsync(&d_meta_->err, 0, 4, st));
+        const cudaError_t le = launch_traceback_canon(last_e_, last_table_, K, d_N, (const uint16_t *)digits_.p,
+                                                      (const int64_t *)off_.p, d_rank, nC, d_inv, Kc, last_idxN_,
+                                                      d_out, d_out_dig, last_opt_, d_len, d_meta_, st);
+        if (le == cudaSuccess) {
+            acc->h2d += (int64_t)up.size() * 4;
+            acc->launches += 2;
+            std::vector<int32_t> outv(4 + (size_t)last_opt_ * (1 + Kc));
+            PT_CK(cudaMemcpyAsync(outv.data(), d_len, outv.size() * 4, cudaMemcpyDeviceToHost, st));
+            PT_CK(cudaMemcpyAsync(h_meta_, d_meta_, sizeof(DpMeta), cudaMemcpyDeviceToHost, st));
+            PT_CK(sync_spin(st));
+            acc->d2h += (int64_t)outv.size() * 4 + (int64_t)sizeof(DpMeta);
+            if (h_meta_->err || outv[0] != last_opt_) return PTAS_EINTERNAL;
+            const int32_t *dg = outv.data() + 4 + last_opt_;
+            for (int q = 0; q < last_opt_; ++q) machines->emplace_back(dg + (size_t)q * Kc, dg + (size_t)(q + 1) * Kc);
+            return PTAS_OK;
+        }
+        if (le != cudaErrorNotSupported) PT_CK(le);
+    }
     std::vector<uint16_t> dig((size_t)nC * K);
     PT_CK(cudaMemcpyAsync(dig.data(), digits_.p, dig.size() * 2, cudaMemcpyDeviceToHost, st));
     PT_CK(sync_spin(st));

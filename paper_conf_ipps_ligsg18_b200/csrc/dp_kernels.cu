@@ -522,7 +522,8 @@ __global__ void __launch_bounds__(32)
 traceback_warp_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__ N,
                       const uint16_t *__restrict__ digits, const int64_t *__restrict__ off,
                       const int32_t *__restrict__ rank, int nC, int64_t idx_start, int32_t *__restrict__ out,
-                      int32_t max_out, int32_t *__restrict__ len, DpMeta *meta)
+                      int32_t max_out, int32_t *__restrict__ len, DpMeta *meta,
+                      const int32_t *__restrict__ inv = nullptr, int Kc = 0, int32_t *__restrict__ out_dig = nullptr)
 {
     extern __shared__ __align__(16) unsigned char tb_smem[];
     int64_t *s_off = reinterpret_cast<int64_t *>(tb_smem);
@@ -559,6 +560,8 @@ traceback_warp_kernel(const E *__restrict__ table, int K, const int32_t *__restr
         }
         const int c = __shfl_sync(FULL, bestc, __ffs(__ballot_sync(FULL, bestr == m)) - 1);
         if (lane == 0) out[mu] = c;
+        if (out_dig)   // the machine's configuration in canonical class order
+            for (int j = lane; j < Kc; j += 32) out_dig[(size_t)mu * Kc + j] = inv[j] < 0 ? 0 : s_dig[c * K + inv[j]];
         ++mu;
         idx -= s_off[c];
         __syncwarp();
@@ -569,6 +572,28 @@ traceback_warp_kernel(const E *__restrict__ table, int K, const int32_t *__restr
         *len = mu;
         if (err) meta->err = 1;
     }
+}
+
+// Canonical lexicographic rank of every configuration (reading R11): rank(c)
+// = #{c' : key(c') < key(c)}, key = the digits in canonical class order
+// (inv[j] = internal position of canonical class j, -1 = empty class, digit 0).
+__global__ void rank_configs_kernel(const uint16_t *__restrict__ digits, int nC, int K,
+                                    const int32_t *__restrict__ inv, int Kc, int32_t *__restrict__ rank)
+{
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nC) return;
+    int32_t rk = 0;
+    for (int c2 = 0; c2 < nC; ++c2) {
+        int cmp = 0;   // key(c2) vs key(c)
+        for (int j = 0; j < Kc && cmp == 0; ++j) {
+            const int i = inv[j];
+            if (i < 0) continue;
+            const int a = digits[(size_t)c2 * K + i], b = digits[(size_t)c * K + i];
+            cmp = a < b ? -1 : (a > b ? 1 : 0);
+        }
+        rk += cmp < 0;
+    }
+    rank[c] = rk;
 }
 
 template <typename E>
@@ -774,6 +799,26 @@ cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N
         traceback_kernel<uint8_t><<<1, 256, 0, st>>>((const uint8_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, idx_start, d_out, max_out, d_len, d_meta);
     else
         traceback_kernel<uint16_t><<<1, 256, 0, st>>>((const uint16_t *)table, K, d_N, d_stride, d_digits, d_off, d_rank, nC, idx_start, d_out, max_out, d_len, d_meta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_traceback_canon(int e, const void *table, int K, const int32_t *d_N, const uint16_t *d_digits,
+                                   const int64_t *d_off, int32_t *d_rank, int64_t nC, const int32_t *d_inv, int Kc,
+                                   int64_t idx_start, int32_t *d_out, int32_t *d_out_dig, int32_t max_out,
+                                   int32_t *d_len, DpMeta *d_meta, cudaStream_t st)
+{
+    const size_t smem = (size_t)nC * (8 + 4) + (size_t)K * 4 + (size_t)nC * K * 2 + 16;
+    const char *tbb = std::getenv("PTAS_TB_BLOCK");
+    if (smem > 48 * 1024 || nC > (1 << 20) || (tbb && tbb[0] == '1')) return cudaErrorNotSupported;
+    rank_configs_kernel<<<(unsigned)((nC + 127) / 128), 128, 0, st>>>(d_digits, (int)nC, K, d_inv, Kc, d_rank);
+    if (e == 1)
+        traceback_warp_kernel<uint8_t><<<1, 32, smem, st>>>((const uint8_t *)table, K, d_N, d_digits, d_off, d_rank,
+                                                            (int)nC, idx_start, d_out, max_out, d_len, d_meta, d_inv,
+                                                            Kc, d_out_dig);
+    else
+        traceback_warp_kernel<uint16_t><<<1, 32, smem, st>>>((const uint16_t *)table, K, d_N, d_digits, d_off, d_rank,
+                                                             (int)nC, idx_start, d_out, max_out, d_len, d_meta, d_inv,
+                                                             Kc, d_out_dig);
     return cudaGetLastError();
 }
 

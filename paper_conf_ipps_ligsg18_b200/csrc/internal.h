@@ -168,6 +168,13 @@ int swar_df_rows_per_set(int e, const RowGeom &g, int J0, int64_t max_level_rows
 cudaError_t prepare_const_prefix(const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound, int e,
                                  int nwords, int cslot, void *d_staging, cudaStream_t st);
 size_t const_prefix_staging_bytes();
+// Traceback with the canonical ranks computed on the device and the machines'
+// configurations written in canonical class order (d_out_dig[max_out][Kc]);
+// cudaErrorNotSupported when the configurations do not fit shared memory.
+cudaError_t launch_traceback_canon(int e, const void *table, int K, const int32_t *d_N, const uint16_t *d_digits,
+                                   const int64_t *d_off, int32_t *d_rank, int64_t nC, const int32_t *d_inv, int Kc,
+                                   int64_t idx_start, int32_t *d_out, int32_t *d_out_dig, int32_t max_out,
+                                   int32_t *d_len, DpMeta *d_meta, cudaStream_t st);
 // Copy rows of pitch Wp (src) to pitch W (dst), `rows` rows of e-byte entries.
 cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows, int64_t W,
                                 int64_t Wp, cudaStream_t st);
