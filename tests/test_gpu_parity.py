@@ -536,3 +536,59 @@ def test_traceback_kernels(P, monkeypatch, tb):
         bins, pk, _ = P.hmbp_solve(N, r, T)
         wb, wpk = oracle.hmbp(N, r, T)
         assert bins == wb and pk.tolist() == wpk.tolist()
+
+
+@pytest.mark.parametrize("name", ["M4x", "M3g"])
+def test_full_size_dp_sampled_device(P, name):
+    """The two largest tables (M4x: K = 8, 1.75 GB uint8; M3g: 5.5 GB uint16)
+    filled on the device at T = LB in the bench's launch configuration and
+    checked there: exact parity with the oracle on a sub-box, Eq. 1 re-checked
+    at 4000 sampled states (all configurations gathered at once), OPT(0) = 0,
+    OPT(N) = the returned value, and monotonicity / +1 Lipschitz along every
+    axis over the whole table (on the GPU)."""
+    import torch
+    w = WORKLOADS[name]
+    p = w.p()
+    k = oracle.k_of(w.eps)
+    LB, _ = oracle.bounds(p, w.m)
+    u, r, N, _ = oracle.classify(p, LB, k)
+    N = np.asarray(N, np.int64)
+    sg, e = P.dp_table_shape(N)
+    t = torch.empty(sg, dtype=torch.uint8 if e == 1 else torch.int16, device="cuda:0")
+    opt = P.dp_fill_device(N.astype(np.int32), r, LB, t)
+    torch.cuda.synchronize()
+    shape = tuple(int(x) + 1 for x in N)
+    stride = np.ones(len(N), np.int64)
+    for i in range(len(N) - 2, -1, -1):
+        stride[i] = stride[i + 1] * shape[i + 1]
+    tv = t.view(shape)
+
+    def at(idx):   # int64 flat indices -> values (host)
+        return t[torch.as_tensor(idx, device="cuda:0")].to(torch.int64).cpu().numpy() & (0xff if e == 1 else 0xffff)
+
+    # sub-box parity
+    Nc = _subbox(N, cap_sigma=150000)
+    want, _ = oracle.dp(Nc, r, LB)
+    grids = np.meshgrid(*[np.arange(int(x) + 1) for x in Nc], indexing="ij")
+    flat = sum(g.astype(np.int64) * s for g, s in zip(grids, stride))
+    assert (at(flat.ravel()).reshape(want.shape) == want).all()
+    # Eq. 1 at sampled states
+    C = oracle.configs(N, r, LB).astype(np.int64)
+    off = C @ stride
+    rng = np.random.default_rng(5)
+    ns = np.stack([rng.integers(0, int(x) + 1, 4000) for x in N], axis=1)
+    ns = ns[ns.any(axis=1)]
+    idx = ns @ stride
+    dom = (C[None, :, :] <= ns[:, None, :]).all(axis=2)          # [samples, |C|]
+    src = np.where(dom, idx[:, None] - off[None, :], 0)
+    vals = at(src.ravel()).reshape(src.shape)
+    best = np.where(dom, vals, 1 << 30).min(axis=1)
+    assert (at(idx) == best + 1).all()
+    assert at(np.array([0]))[0] == 0 and opt == at(np.array([int(N @ stride)]))[0]
+    # monotone and +1 Lipschitz along every axis (whole table, on the GPU)
+    for ax in range(len(N)):
+        a = tv.narrow(ax, 1, shape[ax] - 1).to(torch.int32)
+        b = tv.narrow(ax, 0, shape[ax] - 1).to(torch.int32)
+        d = a - b
+        assert int(d.min()) >= 0 and int(d.max()) <= 1
+        del a, b, d
