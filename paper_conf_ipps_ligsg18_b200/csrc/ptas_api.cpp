@@ -413,7 +413,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     // speculate = d > 0: the full tree of depth d.  PTAS_SPEC_CHAIN=0 / 1 forces.
     const char *sch = std::getenv("PTAS_SPEC_CHAIN");
     const bool spec_chain = sch && sch[0] ? sch[0] == '1' : opt.speculate < 0;
-    if (spec_chain) {
+    if (spec_chain && spec_depth > 0) {   // (PTAS_SPEC_DEPTH=0 still turns speculation off)
         const char *scd = std::getenv("PTAS_SPEC_CHAIN_DEPTH");
         spec_depth = scd && scd[0] ? std::max(1, std::min(MAX_SLOTS, std::atoi(scd))) : 4;
     }

@@ -346,11 +346,14 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #ifndef PTAS_PB2S
 #define PTAS_PB2S 10
 #endif
+#ifndef PTAS_PB2U16
+#define PTAS_PB2U16 8
+#endif
     // gathers in flight per lane (prefix batch); CH = 2 with the prefix list in
     // shared memory (short lists) takes 10: 20 prefixes in two batches instead
     // of three (M2s fill -5%, measured; 12 spills at 80 registers)
     // (uint8 only: the 64-register uint16 kernels lose with it, M3s +3%)
-    constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? ((CPREF || EB == 2) ? PTAS_PB2 : PTAS_PB2S) : 4);
+    constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? (EB == 2 ? PTAS_PB2U16 : (CPREF ? PTAS_PB2 : PTAS_PB2S)) : 4);
     constexpr bool PB_POW2 = (PB & (PB - 1)) == 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     // Programmatic dependent launch: let the next row-level's grid start its
