@@ -12,6 +12,7 @@ Functions (each cites its PAPER.md passage in ptas_oracle.c):
   configs(N, r, T)                PAPER.md:68, Alg 2 l.17
   dp(N, r, T)                     Eq. 1; Alg 2
   ptas(p, m, eps, P)              Alg 1 / Alg 3
+  dp_omp(N, r, T)                 Alg 2 level-parallel comparator, OpenMP
 """
 from __future__ import annotations
 
@@ -168,3 +169,58 @@ def hmbp(N, r, T: int):
     if rc:
         raise ValueError(f"oracle_hmbp rc={rc}")
     return bins.value, pk[:bins.value, :K].copy()
+
+
+# ---------------------------------------------------------------------------
+# The paper's CPU comparator shape (Alg 2, OpenMP level-parallel)
+# in its own file, ptas_oracle_omp.c, for bench.py's all-core cpu_baseline.
+_SRC_OMP = os.path.join(_HERE, "ptas_oracle_omp.c")
+_LIB_OMP = os.path.join(_HERE, "libptas_oracle_omp.so")
+_lib_omp = None
+
+
+def build_omp(force: bool = False) -> str:
+    """Compile the Alg-2 comparator with gcc -O2 -fopenmp."""
+    if force or not os.path.exists(_LIB_OMP) or os.path.getmtime(_LIB_OMP) < os.path.getmtime(_SRC_OMP):
+        tmp = _LIB_OMP + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fopenmp", "-shared", "-fPIC", "-o", tmp, _SRC_OMP])
+        os.replace(tmp, _LIB_OMP)
+    return _LIB_OMP
+
+
+def _load_omp():
+    global _lib_omp
+    with _lock:
+        if _lib_omp is None:
+            lib = ctypes.CDLL(build_omp())
+            i32p = ctypes.POINTER(ctypes.c_int32)
+            i64p = ctypes.POINTER(ctypes.c_int64)
+            lib.oracle_omp_threads.restype = ctypes.c_int
+            lib.oracle_dp_omp.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, ctypes.c_int64,
+                                          i32p, ctypes.POINTER(ctypes.c_double)]
+            _lib_omp = lib
+    return _lib_omp
+
+
+def omp_threads() -> int:
+    return int(_load_omp().oracle_omp_threads())
+
+
+def dp_omp(N, r, T: int):
+    """Same contract as dp(): (table, relax), computed by Alg 2's level-parallel
+    loop on all OpenMP threads."""
+    N = np.ascontiguousarray(N, dtype=np.int32)
+    r = np.ascontiguousarray(r, dtype=np.int64)
+    K = len(N)
+    sg = sigma(N)
+    if sg < 0:
+        raise OverflowError("sigma overflows int64")
+    tab = np.zeros(sg, np.int32)
+    opt = ctypes.c_int32()
+    relax = ctypes.c_double()
+    rc = _load_omp().oracle_dp_omp(_p(N, ctypes.c_int32), _p(r, ctypes.c_int64), K, int(T),
+                                   _p(tab, ctypes.c_int32), sg, ctypes.byref(opt), ctypes.byref(relax))
+    if rc:
+        raise ValueError(f"oracle_dp_omp rc={rc}")
+    shape = tuple(int(x) + 1 for x in N) if K else ()
+    return tab.reshape(shape) if K else tab.reshape(()), relax.value

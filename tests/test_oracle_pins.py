@@ -443,3 +443,51 @@ def test_hmbp_closed_forms_and_edges():
     assert oracle.hmbp([3, 3], [5, 4], 9)[0] == 3
     with pytest.raises(ValueError):
         oracle.hmbp([1], [11], 10)   # an item larger than the capacity
+
+
+# --- Alg 2 comparator (oracle/ptas_oracle_omp.c, bench.py's all-core cpu_baseline) ---
+
+def test_dp_omp_equals_exhaustive_bin_packing():
+    # pinned directly to bin packing, not only to oracle_dp
+    rng = np.random.default_rng(17)
+    for _ in range(30):
+        K = int(rng.integers(1, 5))
+        N = rng.integers(0, 4, K)
+        while N.sum() > 10 or N.sum() == 0:
+            N = rng.integers(0, 4, K)
+        r = rng.integers(5, 60, K)
+        T = int(rng.integers(int(r.max()), 150))
+        tab, _ = oracle.dp_omp(N, r, T)
+        items, first = [], []
+        for i in range(K):
+            first.append(len(items))
+            items += [int(r[i])] * int(N[i])
+        best = _min_bins_all_subsets(items, T)
+        for n in itertools.product(*[range(int(x) + 1) for x in N]):
+            mask = 0
+            for i in range(K):
+                for t in range(n[i]):
+                    mask |= 1 << (first[i] + t)
+            assert tab[n] == best[mask], (N, r, T, n)
+
+
+@pytest.mark.parametrize("N,r,T", [(17, 30, 100), (255, 11, 100), (0, 3, 3)])
+def test_dp_omp_K1_closed_form(N, r, T):
+    tab, _ = oracle.dp_omp([N], [r], T)
+    per = T // r
+    assert [int(v) for v in tab] == [math.ceil(x / per) for x in range(N + 1)]
+
+
+def test_dp_omp_equals_oracle_dp_and_relax_closed_form():
+    rng = np.random.default_rng(23)
+    for _ in range(12):
+        K = int(rng.integers(2, 7))
+        N = rng.integers(1, 9, K)
+        r = rng.integers(20, 120, K)
+        T = int(rng.integers(int(r.max()) * 2, 500))
+        a, ra = oracle.dp(N, r, T)
+        b, rb = oracle.dp_omp(N, r, T)
+        assert np.array_equal(a, b)
+        C = oracle.configs(N, r, T)
+        assert ra == rb == sum(int(np.prod(N - s + 1)) for s in C)
+    assert oracle.omp_threads() >= 1
