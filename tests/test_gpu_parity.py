@@ -592,3 +592,13 @@ def test_full_size_dp_sampled_device(P, name):
         d = a - b
         assert int(d.min()) >= 0 and int(d.max()) <= 1
         del a, b, d
+
+
+@pytest.mark.parametrize("k", [4, 5, 7])
+def test_dstar_shapes_full_table(P, k):
+    # the D* roofline-sweep geometry (synth.dstar) at sizes the
+    # oracle finishes in seconds: every entry vs the oracle, K = 3..8
+    from synth import dstar
+    for K in range(3, 9):
+        N, r, T = dstar(K, 3.0e4 if k < 7 else 1.2e4, k)
+        _check_table(P, N, r, T)
