@@ -217,11 +217,14 @@ def run_ours(args, w):
     if world > 1:
         mode = P.MODE_MULTI_PROBE if args.mode == "multiprobe" else P.MODE_LEVEL_SHARDED
         Pp = world if mode == P.MODE_MULTI_PROBE else args.P
+    elif args.virtual_shards > 1:
+        mode, Pp = P.MODE_LEVEL_SHARDED, args.P
     else:
         mode, Pp = P.MODE_SINGLE, args.P
     # all library work on this stream, so the CUDA events below bracket it exactly
     lib_stream = torch.cuda.Stream(device=local)
-    opts = P.options(P=Pp, mode=mode, device=local, comm=comm, stream=lib_stream)
+    opts = P.options(P=Pp, mode=mode, device=local, comm=comm, stream=lib_stream,
+                     virtual_shards=args.virtual_shards if world == 1 else 1)
 
     p = w.p()
     n = len(p)
@@ -315,6 +318,7 @@ def run_ours(args, w):
         "vs_baseline": None, "dtype": args.dtype_label or "u8", "data": "synthetic",
         "config": _config(w, probes_per_round=Pp,
                           mode={0: "single", 1: "level_sharded", 2: "multi_probe"}[mode],
+                          **({"virtual_shards": args.virtual_shards} if world == 1 and args.virtual_shards > 1 else {}),
                           l2="flushed between steps (256 MiB write)"),
         "solve": {"probes": st0["probes"], "unique_dps": st0["unique_dps"], "T_star": st0["T_star"],
                   "sigma_max": st0["sigma_max"], "K_at_Tstar": st0["K_at_Tstar"],
@@ -371,6 +375,9 @@ def main():
     ap.add_argument("--workload", default="M2s", choices=sorted(WORKLOADS))
     ap.add_argument("--P", type=int, default=1, help="probes per round (single GPU)")
     ap.add_argument("--mode", choices=["sharded", "multiprobe"], default="sharded", help="N>1 mode")
+    ap.add_argument("--virtual-shards", type=int, default=1,
+                    help="N=1 only: run LEVEL_SHARDED with G logical shards on one GPU (slice fill + "
+                         "gather copy + scatter per level, no NCCL) to measure the exchange overhead")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--dtype-label", default=None)
     args = ap.parse_args()
