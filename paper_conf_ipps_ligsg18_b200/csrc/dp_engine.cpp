@@ -484,7 +484,10 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     ++o.launches;
     const int J0 = (int)std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
     const char *fs = std::getenv("PTAS_FORCE_SCALAR");
-    const bool force_scalar = fs && fs[0] == '1';
+    // PTAS_FORCE_SCALAR=1: the full-relaxation scalar kernel for every level;
+    // =2: the long-row two-launch path for every level (test coverage)
+    const bool force_scalar = fs && (fs[0] == '1' || fs[0] == '2');
+    const bool force_long = fs && fs[0] == '2';
     const char *pdls = std::getenv("PTAS_PDL");
     const bool use_pdl = !(pdls && pdls[0] == '0');
     bool prev_fill = false;  // the previous launch on st was a packed fill (PDL-safe)
@@ -500,6 +503,15 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                        j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0,
                                        cpref_ok ? index_ : -1);
             if (err == cudaSuccess) prev_fill = true;
+        }
+        if (err == cudaErrorNotSupported && compact == nullptr && (force_long || !force_scalar)) {
+            err = launch_row_fill_long(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
+                                       j0, rho_, b, c, sm_count_, st);
+            if (err == cudaSuccess) {
+                prev_fill = false;
+                return err;
+            }
+            if (err == cudaErrorInvalidValue) err = cudaErrorNotSupported;
         }
         if (err == cudaErrorNotSupported) {
             err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound, j0,

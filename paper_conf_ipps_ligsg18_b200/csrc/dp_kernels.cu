@@ -5,6 +5,7 @@
 //  build_prefix_kernel   a-3: group C by leading digits, packed words, off(s'),
 //                        closed-form relaxation count
 //  row_fill_kernel       a-5: Eq. 1 for one row-level
+//  row_cross_kernel / row_chain_kernel  a-5 for rows longer than 1 KiB (D5, two launches)
 //  row_scatter_kernel    §8(e): gathered compact rows -> mixed-radix table
 //  build_row_index_kernel a-4: level-ordered row index (row base + packed digits)
 //  traceback_kernel      a-8: schedule of the rounded long jobs from DP(T*)
@@ -436,6 +437,125 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
     }
 }
 
+// Long rows (W > 1 KiB, beyond the packed kernel's one-row-per-group layout):
+// the row-level is filled in two launches so that a long row is spread over
+// many warps instead of one.
+//  row_cross_kernel: one warp per (row, 32-entry chunk); for each state
+//    acc(x) = min over prefixes s' != 0, s' <= p of OPT(p - s', x - min(x, Jmax(s')))
+//    (the window min of reading D5: OPT is monotone in x), written to the
+//    state's own entry as a provisional value (sentinel = the all-ones E value:
+//    every finite acc is an OPT of a smaller state, <= sum N - 1).
+//  row_chain_kernel: one warp per row, chunks in order; in-row term of D5
+//    OPT(p, x) = 1 + min(acc(x), OPT(p, x - min(x, J0))), x >= 1, resolved
+//    inside a chunk by Bellman-Ford over shuffles (<= 32 / J0 + 1 rounds),
+//    from earlier chunks by a plain read of the stored final value.
+// Executed relaxations equal the collapsed count of the packed kernel.
+template <typename E, int NW>
+__global__ void __launch_bounds__(256)
+row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const uint64_t *__restrict__ pwa,
+                 int64_t pw_stride, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
+                 int64_t slot_count, int64_t nch)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    if (meta->ovf) return;
+    const int np = (int)(meta->nP - 1);
+    uint64_t *s_oj = reinterpret_cast<uint64_t *>(smem_raw);
+    uint64_t *s_w = s_oj + np;
+    for (int i = threadIdx.x; i < np; i += blockDim.x) {
+        const PrefixEntry pe = gpref[1 + i];
+        s_oj[i] = ((uint64_t)(uint32_t)pe.jmax << 48) | (uint64_t)pe.off;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) s_w[(size_t)w * np + i] = pe.w[w];
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    uint64_t guard[NW];
+#pragma unroll
+    for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
+    const E SENT = (E)~(E)0;
+    for (int64_t task = gw; task < slot_count * nch; task += nw) {
+        const int64_t slot = task / nch;
+        const int64_t x = (task - slot * nch) * 32 + lane;
+        const bool act = x < g.W;
+        uint64_t pw[NW];
+#pragma unroll
+        for (int w = 0; w < NW; ++w) pw[w] = pwa[(int64_t)w * pw_stride + slot];
+        const int64_t rowbase = rb[slot];
+        const E *rowp = table + rowbase + x;
+        int acc = INF;
+        for (int base = 0; base < np; base += 32) {
+            const int c = base + lane;
+            bool dom = c < np;
+            if (dom) {
+#pragma unroll
+                for (int w = 0; w < NW; ++w)
+                    dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
+            }
+            unsigned m = __ballot_sync(FULL, dom);
+            while (m) {
+                int v[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    v[q] = INF;
+                    if (m) {
+                        const int b = __ffs(m) - 1;
+                        m &= m - 1;
+                        const uint64_t oj = s_oj[base + b];
+                        const int64_t jm = (int64_t)(oj >> 48);
+                        const int64_t J = jm < x ? jm : x;
+                        if (act) v[q] = rowp[-(int64_t)(oj & 0xffffffffffffull) - J];
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q) acc = v[q] < acc ? v[q] : acc;
+            }
+        }
+        if (act) table[rowbase + x] = acc >= INF ? SENT : (E)acc;
+    }
+}
+
+template <typename E>
+__global__ void __launch_bounds__(256)
+row_chain_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const DpMeta *__restrict__ meta,
+                 int J0, int rho, int64_t slot_count)
+{
+    if (meta->ovf) return;
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const E SENT = (E)~(E)0;
+    for (int64_t slot = gw; slot < slot_count; slot += nw) {
+        E *out = table + rb[slot];
+        for (int64_t x0 = 0; x0 < g.W; x0 += 32) {
+            const int64_t x = x0 + lane;
+            const bool act = x < g.W;
+            int opt = INF;
+            if (act) {
+                const int a = out[x];
+                opt = (rho == 0 && x == 0) ? 0 : (a == (int)SENT ? INF : a + 1);
+            }
+            const int64_t src = act && x > 0 ? x - (J0 < x ? J0 : x) : -1;
+            if (src >= 0 && src < x0) {          // earlier chunk: already final
+                const int v = out[src] + 1;
+                opt = v < opt ? v : opt;
+            }
+            const bool inchunk = src >= x0;
+            const int sl = inchunk ? (int)(src - x0) : lane;
+            bool changed = true;
+            while (__any_sync(FULL, changed)) {
+                const int t = __shfl_sync(FULL, opt, sl);
+                const int nopt = inchunk && t + 1 < opt ? t + 1 : opt;
+                changed = nopt < opt;
+                opt = nopt;
+            }
+            if (act) out[x] = (E)opt;
+            __syncwarp();
+        }
+    }
+}
+
 // §8(e): write gathered compact rows (slot-major, pitch Wp) into the table.
 template <typename E>
 __global__ void __launch_bounds__(256)
@@ -753,6 +873,47 @@ cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t 
     }
 #undef PTAS_FILL_JU
 #undef PTAS_FILL_CASE
+    return cudaGetLastError();
+}
+
+cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
+                                 int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                 int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
+                                 int sm_count, cudaStream_t st)
+{
+    if (slot_count <= 0) return cudaSuccess;
+    const int NWk = g.nwords <= 1 ? 1 : 2;
+    const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
+    const size_t smem = (size_t)np * (8 + 8 * NWk) + 16;
+    if (smem > 220 * 1024) return cudaErrorInvalidValue;
+    const int64_t nch = (g.W + 31) / 32;
+    const int bs = 256;
+    const int64_t cap = (int64_t)sm_count * 8;
+    int64_t blocks = (slot_count * nch + 7) / 8;
+    if (blocks > cap) blocks = cap;
+    const int64_t *rbl = rb + slot_begin;
+    const uint64_t *pwl = pw + slot_begin;
+    cudaError_t err;
+#define PTAS_LONG_CASE(E_, NW_)                                                                    \
+    do {                                                                                           \
+        auto kfn = row_cross_kernel<E_, NW_>;                                                      \
+        if (smem > 48 * 1024) {                                                                    \
+            err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); \
+            if (err != cudaSuccess) return err;                                                    \
+        }                                                                                          \
+        kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, rbl, pwl, pw_stride, d_pref, d_meta, \
+                                                slot_count, nch);                                  \
+        int64_t b2 = (slot_count + 7) / 8;                                                         \
+        if (b2 > cap) b2 = cap;                                                                    \
+        row_chain_kernel<E_><<<(unsigned)b2, bs, 0, st>>>((E_ *)table, g, rbl, d_meta, J0, rho,     \
+                                                          slot_count);                             \
+    } while (0)
+    if (e == 1) {
+        if (NWk == 1) PTAS_LONG_CASE(uint8_t, 1); else PTAS_LONG_CASE(uint8_t, 2);
+    } else {
+        if (NWk == 1) PTAS_LONG_CASE(uint16_t, 1); else PTAS_LONG_CASE(uint16_t, 2);
+    }
+#undef PTAS_LONG_CASE
     return cudaGetLastError();
 }
 

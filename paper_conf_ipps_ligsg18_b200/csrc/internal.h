@@ -137,6 +137,14 @@ cudaError_t launch_row_fill(int e, void *table, const RowGeom &g, const int64_t 
                             const PrefixEntry *d_pref, const DpMeta *d_meta, int64_t nP_bound,
                             int J0, int rho, int64_t slot_begin, int64_t slot_count,
                             void *compact_out, int sm_count, cudaStream_t st);
+// Rows longer than the packed kernel takes (> 1 KiB): cross-row window minima
+// (one warp per 32-entry chunk) then the in-row chain (one warp per row).
+// Table output only (no compact slices); slot_begin/slot_count as above, rb/pw
+// at the row-level's first slot.
+cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int64_t *rb, const uint64_t *pw,
+                                 int64_t pw_stride, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                 int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
+                                 int sm_count, cudaStream_t st);
 // a-4 level-ordered row index: for every row slot t (row-levels concatenated,
 // lexicographic within a level) its row base index rb[t] and packed leading
 // digits pw[w * rows + t].

@@ -188,9 +188,12 @@ def test_dp_fill_invalid(P):
     assert ei.value.rc == -2
 
 
-def test_dp_fill_scalar_kernel(P, monkeypatch):
-    # the scalar fill kernel (fallback for rows > 1 KiB) on the same random cases
-    monkeypatch.setenv("PTAS_FORCE_SCALAR", "1")
+@pytest.mark.parametrize("mode", ["1", "2"])
+def test_dp_fill_scalar_kernel(P, monkeypatch, mode):
+    # 1: the full-relaxation scalar kernel (fallback of the sharded compact path);
+    # 2: the long-row two-launch path (row_cross + row_chain, rows > 1 KiB), forced
+    # on every level, on the same random cases
+    monkeypatch.setenv("PTAS_FORCE_SCALAR", mode)
     rng = np.random.default_rng(31)
     for K in (1, 2, 3, 5, 7):
         for _ in range(4):
@@ -228,10 +231,23 @@ def test_dp_fill_lane_layouts(P, monkeypatch, ch):
 
 
 def test_dp_fill_very_long_rows(P):
-    # rows longer than 1 KiB (uint16, W = 701) use the scalar kernel; W*e = 1024 B exactly uses 8 chunks
+    # rows longer than 1 KiB (uint16, W = 701) use the long-row path; W*e = 1024 B exactly uses 8 chunks
     _check_table(P, np.array([2, 700], np.int32), np.array([60, 13], np.int64), 120)
     _check_table(P, np.array([3, 511], np.int32), np.array([60, 13], np.int64), 120)
     _check_table(P, np.array([1, 1, 300], np.int32), np.array([50, 40, 7], np.int64), 120)
+    # long rows with ragged chunk tails, J0 > 32 (in-row source in an earlier chunk) and J0 = 1
+    _check_table(P, np.array([4, 3, 1200], np.int32), np.array([300, 170, 3], np.int64), 310)
+    _check_table(P, np.array([6, 1500], np.int32), np.array([100, 99], np.int64), 250)
+    _check_table(P, np.array([2, 2, 2, 900], np.int32), np.array([40, 35, 33, 5], np.int64), 100)
+
+
+def test_dp_fill_long_rows_solve(P):
+    # a full solve whose DPs have rows > 1 KiB (N = [32, 1200], uint16 rows of 2402 B):
+    # probe log, T*, makespan, assignment
+    p = np.array([100] * 30 + [110] * 2 + [130] * 1200, np.int64)
+    np.random.default_rng(0).shuffle(p)
+    got = _cmp_solve(P, p, 420, 0.25, 1)
+    assert max(x[5] for x in got["probes"]) == 39633
 
 
 def test_dp_fill_padding_pitches(P, fillmode):

@@ -30,6 +30,8 @@ cases = [
     ([2, 300], [60, 13], 120),                # uint16, 151 words: CH = 8
     ([1, 1, 1, 1, 1, 1, 40], [30, 31, 32, 33, 34, 35, 9], 120),
     ([6, 260], [40, 7], 100),                 # uint16, J0 > 2
+    ([2, 700], [60, 13], 120),                # rows > 1 KiB: long-row path (row_cross + row_chain)
+    ([6, 1500], [100, 99], 250),              # long rows, J0 = 2, ragged last chunk
 ]
 for N, r, T in cases:
     P.dp_fill(np.array(N, np.int32), np.array(r, np.int64), T)
@@ -88,3 +90,10 @@ def test_memcheck_dataflow(env):
 @pytest.mark.timeout(1800)
 def test_racecheck_dataflow_split():
     _run("racecheck", {"PTAS_DF": "3", "PTAS_DF_SPLIT_ROWS": "1000000000"})
+
+
+@pytest.mark.timeout(1200)
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck"])
+def test_sanitizer_long_row_path_forced(tool):
+    # the long-row two-launch path on every level of every case (PTAS_FORCE_SCALAR=2)
+    _run(tool, {"PTAS_FORCE_SCALAR": "2"})
