@@ -447,8 +447,8 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
 //    every finite acc is an OPT of a smaller state, <= sum N - 1).
 //  row_chain_kernel: one warp per row, chunks in order; in-row term of D5
 //    OPT(p, x) = 1 + min(acc(x), OPT(p, x - min(x, J0))), x >= 1, resolved
-//    inside a chunk by Bellman-Ford over shuffles (<= 32 / J0 + 1 rounds),
-//    from earlier chunks by a plain read of the stored final value.
+//    inside a chunk by min-plus doubling over the lanes (log2(32 / J0) rounds),
+//    from the previous chunk through registers, from older ones by a read.
 // Executed relaxations equal the collapsed count of the packed kernel.
 template <typename E, int NW>
 __global__ void __launch_bounds__(256)
@@ -516,6 +516,8 @@ row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
     }
 }
 
+constexpr int CHAIN_BATCH = 8;
+
 template <typename E>
 __global__ void __launch_bounds__(256)
 row_chain_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const DpMeta *__restrict__ meta,
@@ -528,30 +530,45 @@ row_chain_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
     const E SENT = (E)~(E)0;
     for (int64_t slot = gw; slot < slot_count; slot += nw) {
         E *out = table + rb[slot];
-        for (int64_t x0 = 0; x0 < g.W; x0 += 32) {
-            const int64_t x = x0 + lane;
-            const bool act = x < g.W;
-            int opt = INF;
-            if (act) {
-                const int a = out[x];
-                opt = (rho == 0 && x == 0) ? 0 : (a == (int)SENT ? INF : a + 1);
+        int prev = INF;                                   // previous chunk's final values
+        for (int64_t xb = 0; xb < g.W; xb += 32 * CHAIN_BATCH) {
+            // provisional acc of CHAIN_BATCH chunks loaded together (one latency per batch)
+            int av[CHAIN_BATCH];
+#pragma unroll
+            for (int c = 0; c < CHAIN_BATCH; ++c) {
+                const int64_t xi = xb + 32 * c + lane;
+                av[c] = xi < g.W ? (int)out[xi] : 0;
             }
-            const int64_t src = act && x > 0 ? x - (J0 < x ? J0 : x) : -1;
-            if (src >= 0 && src < x0) {          // earlier chunk: already final
-                const int v = out[src] + 1;
-                opt = v < opt ? v : opt;
+#pragma unroll
+            for (int c = 0; c < CHAIN_BATCH; ++c) {
+                const int64_t x0 = xb + 32 * c;
+                if (x0 >= g.W) break;
+                const int64_t x = x0 + lane;
+                const bool act = x < g.W;
+                const int a = av[c];
+                int opt = !act ? INF : ((rho == 0 && x == 0) ? 0 : (a == (int)SENT ? INF : a + 1));
+                // in-row source x - min(x, J0) before this chunk: previous chunk from registers, older from memory
+                const int64_t src = act && x > 0 ? x - (J0 < x ? J0 : x) : x;
+                const int64_t pl = src - (x0 - 32);
+                const int t = __shfl_sync(FULL, prev, (int)(pl >= 0 && pl < 32 ? pl : 0));
+                if (act && x > 0 && src < x0) {
+                    const int v = (pl >= 0 ? t : (int)out[src]) + 1;
+                    opt = v < opt ? v : opt;
+                }
+                if (x0 == 0) {                            // x < J0 reaches back to x = 0 directly
+                    const int t0 = __shfl_sync(FULL, opt, 0);
+                    if (x >= 1 && x < J0 && t0 + 1 < opt) opt = t0 + 1;
+                }
+                // in-chunk chain x -> x - J0 -> ... : min-plus doubling over the lanes
+                for (int sft = 1; sft * J0 < 32; sft <<= 1) {
+                    const int d = sft * J0;
+                    const int u = __shfl_up_sync(FULL, opt, d);
+                    if (lane >= d && x >= J0 && u + sft < opt) opt = u + sft;
+                }
+                if (act) out[x] = (E)opt;
+                prev = opt;
+                __syncwarp();
             }
-            const bool inchunk = src >= x0;
-            const int sl = inchunk ? (int)(src - x0) : lane;
-            bool changed = true;
-            while (__any_sync(FULL, changed)) {
-                const int t = __shfl_sync(FULL, opt, sl);
-                const int nopt = inchunk && t + 1 < opt ? t + 1 : opt;
-                changed = nopt < opt;
-                opt = nopt;
-            }
-            if (act) out[x] = (E)opt;
-            __syncwarp();
         }
     }
 }

@@ -22,11 +22,12 @@ from synth import dstar  # noqa: E402
 peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
 targets = [float(x) for x in os.environ.get("DSWEEP_SIGMA", "1e6,1e7,1e8,1e9,4e9").split(",")]
 reps = int(os.environ.get("DSWEEP_REPS", "3"))
+Ks = [int(x) for x in os.environ.get("DSWEEP_K", "3,4,5,6,7,8").split(",")]
 torch.cuda.set_device(0)
 stream = torch.cuda.Stream()
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for k in (4, 5, 7):
-    for K in range(3, 9):
+    for K in Ks:
         for st in targets:
             N, r, T = dstar(K, st, k)
             sigma, e = P.dp_table_shape(N)
