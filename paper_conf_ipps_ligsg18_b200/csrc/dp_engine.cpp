@@ -23,6 +23,18 @@
 
 namespace ptas {
 
+// Rows per shard of a sharded row-level: ceil(R / G) rounded up so that every
+// shard's compact slice starts 16-byte aligned (the packed fill kernel writes
+// compact rows with vector stores and rejects unaligned slices, which would
+// send the level to the scalar kernel).  Trailing shards may be short or empty.
+static int64_t shard_chunk(int64_t R, int G, int64_t row_bytes)
+{
+    const int64_t c = (R + G - 1) / G;
+    int64_t q = 1;
+    while ((q * row_bytes) % 16 != 0) ++q;      // smallest q with q * row_bytes = 0 (mod 16), q <= 16
+    return (c + q - 1) / q * q;
+}
+
 // PTAS_SLOW_CALLS=<ms> (diagnostics): report every checked call slower than
 // <ms> milliseconds of host time, with its source line.
 static double slow_call_ms()
@@ -542,7 +554,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         for (int rho = 0; rho <= g.rho_max; ++rho) {
             int64_t R = cnt[rho];
             if (!sharded(R)) continue;
-            int64_t chunk = (R + G - 1) / G;
+            const int64_t chunk = shard_chunk(R, G, g.Wp * e);
             mx = std::max(mx, (size_t)(chunk * G * g.Wp * e));
         }
         PT_CK(stage_.ensure(mx));
@@ -728,7 +740,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             ++o.fill_launches;
             continue;
         }
-        const int64_t chunk = (R + G - 1) / G;
+        const int64_t chunk = shard_chunk(R, G, g.Wp * e);
         unsigned char *stage = (unsigned char *)stage_.p;
         if (virt) {
             for (int v = 0; v < G; ++v) {

@@ -618,3 +618,17 @@ def test_dstar_shapes_full_table(P, k):
     for K in range(3, 9):
         N, r, T = dstar(K, 3.0e4 if k < 7 else 1.2e4, k)
         _check_table(P, N, r, T)
+
+
+@pytest.mark.parametrize("vs", [2, 3, 8])
+def test_virtual_shards_use_packed_kernel(P, vs):
+    # sharded row-levels must keep the packed kernel (16-byte aligned compact slices):
+    # identical results to the single-GPU solve AND the collapsed executed count
+    w = WORKLOADS["M2s"]
+    p = w.p()
+    ref = P.ptas_solve(p, w.m, w.eps, P=1, speculate=0)
+    got = P.ptas_solve(p, w.m, w.eps, P=1, mode=P.MODE_LEVEL_SHARDED, virtual_shards=vs, speculate=0)
+    assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
+    assert (got["assignment"] == ref["assignment"]).all()
+    assert got["stats"]["relaxations"] == ref["stats"]["relaxations"]
+    assert got["stats"]["relax_executed"] == ref["stats"]["relax_executed"] < got["stats"]["relaxations"]
