@@ -374,7 +374,9 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default="M2s", choices=sorted(WORKLOADS))
     ap.add_argument("--P", type=int, default=1, help="probes per round (single GPU)")
-    ap.add_argument("--mode", choices=["sharded", "multiprobe"], default="sharded", help="N>1 mode")
+    ap.add_argument("--mode", choices=["auto", "sharded", "multiprobe"], default="auto",
+                    help="N>1 mode; auto = sharded when the workload's largest table is >= 1 GB "
+                         "(M3g, M4x), else multiprobe (DESIGN.md §9: level sharding only pays on large tables)")
     ap.add_argument("--virtual-shards", type=int, default=1,
                     help="N=1 only: run LEVEL_SHARDED with G logical shards on one GPU (slice fill + "
                          "gather copy + scatter per level, no NCCL) to measure the exchange overhead")
@@ -382,9 +384,13 @@ def main():
     ap.add_argument("--dtype-label", default=None)
     args = ap.parse_args()
     w = WORKLOADS[args.workload]
+    N, _r, _T = _largest_dp(w)
+    e = 1 if int(np.sum(N)) <= 255 else 2
     if args.dtype_label is None:
-        N, _r, _T = _largest_dp(w)
-        args.dtype_label = "u8" if int(np.sum(N)) <= 255 else "u16"
+        args.dtype_label = "u8" if e == 1 else "u16"
+    if args.mode == "auto":
+        table_bytes = float(np.prod(np.asarray(N, np.float64) + 1)) * e if len(N) else 0.0
+        args.mode = "sharded" if table_bytes >= 1e9 else "multiprobe"
     if args.impl == "reference":
         return run_reference(args, w)
     return run_ours(args, w)
