@@ -119,6 +119,16 @@ def _largest_dp(w):
     return N, r, LB
 
 
+def _largest_dp_product(w):
+    """(N, r, T) at T = LB through the library's exported host steps (no oracle)."""
+    import paper_conf_ipps_ligsg18_b200 as P
+    p = w.p()
+    k = P.ptas_k(w.eps)
+    LB, _ = P.ptas_bounds(p, w.m)
+    _u, r, N, _ = P.ptas_classify(p, LB, k)
+    return N, r, LB
+
+
 def _subbox_for(N, r, T, target_relax):
     """Clip counts (largest first) until the closed-form relaxation count of the
     sub-box DP is <= target: the DP restricted to n <= N' is exactly the
@@ -384,7 +394,9 @@ def main():
     ap.add_argument("--dtype-label", default=None)
     args = ap.parse_args()
     w = WORKLOADS[args.workload]
-    N, _r, _T = _largest_dp(w)
+    # geometry of the largest DP: the product's host ABI for our arm, the
+    # oracle only on the reference (oracle) arm
+    N, _r, _T = _largest_dp(w) if args.impl == "reference" else _largest_dp_product(w)
     e = 1 if int(np.sum(N)) <= 255 else 2
     if args.dtype_label is None:
         args.dtype_label = "u8" if e == 1 else "u16"
