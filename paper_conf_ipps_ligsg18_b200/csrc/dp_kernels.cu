@@ -450,11 +450,13 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
 //    inside a chunk by min-plus doubling over the lanes (log2(32 / J0) rounds),
 //    from the previous chunk through registers, from older ones by a read.
 // Executed relaxations equal the collapsed count of the packed kernel.
+constexpr int CHAIN_BATCH = 8;   // chunks whose values a chain warp loads together
+
 template <typename E, int NW>
 __global__ void __launch_bounds__(256)
 row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const uint64_t *__restrict__ pwa,
                  int64_t pw_stride, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
-                 int64_t slot_count, int64_t nch)
+                 int64_t slot_count, int64_t nch, int J0, int local_chain)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     if (meta->ovf) return;
@@ -512,11 +514,76 @@ row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
                 for (int q = 0; q < 4; ++q) acc = v[q] < acc ? v[q] : acc;
             }
         }
-        if (act) table[rowbase + x] = acc >= INF ? SENT : (E)acc;
+        if (!local_chain) {
+            if (act) table[rowbase + x] = acc >= INF ? SENT : (E)acc;
+            continue;
+        }
+        // row-levels >= 1: acc is finite for every state (a unit prefix e_i <= p
+        // always dominates), so the in-row chain inside this chunk is resolved
+        // here (min-plus doubling) and row_carry_kernel only adds what comes
+        // from earlier chunks
+        const int64_t x0 = x - lane;
+        int opt = act ? acc + 1 : INF;
+        if (x0 == 0) {
+            const int t0 = __shfl_sync(FULL, opt, 0);
+            if (x >= 1 && x < J0 && t0 + 1 < opt) opt = t0 + 1;
+        }
+        for (int sft = 1; sft * J0 < 32; sft <<= 1) {
+            const int d = sft * J0;
+            const int u = __shfl_up_sync(FULL, opt, d);
+            if (lane >= d && x >= J0 && u + sft < opt) opt = u + sft;
+        }
+        if (act) table[rowbase + x] = (E)opt;
     }
 }
 
-constexpr int CHAIN_BATCH = 8;
+// Row-levels >= 1 after row_cross_kernel(local_chain = 1): per row, chunks in
+// order, final(x) = min(local(x), final(z - min(z, J0)) + 1 + t) where z is the
+// first element of x's in-row chain inside the chunk (x = z + t * J0).
+template <typename E>
+__global__ void __launch_bounds__(256)
+row_carry_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const DpMeta *__restrict__ meta,
+                 int J0, int64_t slot_count)
+{
+    if (meta->ovf) return;
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int zo = J0 < 32 ? lane % J0 : lane;           // z - x0 (chunk-independent)
+    const int tz = J0 < 32 ? lane / J0 : 0;              // chain steps from z to x
+    for (int64_t slot = gw; slot < slot_count; slot += nw) {
+        E *out = table + rb[slot];
+        int prev = INF;
+        if (lane < g.W) prev = out[lane];                 // chunk 0: local == final
+        for (int64_t xb = 32; xb < g.W; xb += 32 * CHAIN_BATCH) {
+            int av[CHAIN_BATCH];
+#pragma unroll
+            for (int c = 0; c < CHAIN_BATCH; ++c) {
+                const int64_t xi = xb + 32 * c + lane;
+                av[c] = xi < g.W ? (int)out[xi] : INF;
+            }
+#pragma unroll
+            for (int c = 0; c < CHAIN_BATCH; ++c) {
+                const int64_t x0 = xb + 32 * c;
+                if (x0 >= g.W) break;
+                const int64_t x = x0 + lane;
+                const bool act = x < g.W;
+                const int64_t z = x0 + zo;
+                const int64_t src = z - (J0 < z ? J0 : z);
+                const int64_t pl = src - (x0 - 32);
+                const int t = __shfl_sync(FULL, prev, (int)(pl >= 0 && pl < 32 ? pl : 0));
+                int opt = av[c];
+                if (act) {
+                    const int v = (pl >= 0 ? t : (int)out[src]) + 1 + tz;
+                    opt = v < opt ? v : opt;
+                    out[x] = (E)opt;
+                }
+                prev = opt;
+                __syncwarp();
+            }
+        }
+    }
+}
 
 template <typename E>
 __global__ void __launch_bounds__(256)
@@ -910,6 +977,9 @@ cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int
     if (blocks > cap) blocks = cap;
     const int64_t *rbl = rb + slot_begin;
     const uint64_t *pwl = pw + slot_begin;
+    // PTAS_LONG_LOCAL=0: the in-row chain entirely in row_chain_kernel (measurement knob)
+    const char *ll = std::getenv("PTAS_LONG_LOCAL");
+    const int local = (rho >= 1 && !(ll && ll[0] == '0')) ? 1 : 0;
     cudaError_t err;
 #define PTAS_LONG_CASE(E_, NW_)                                                                    \
     do {                                                                                           \
@@ -919,11 +989,15 @@ cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int
             if (err != cudaSuccess) return err;                                                    \
         }                                                                                          \
         kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, rbl, pwl, pw_stride, d_pref, d_meta, \
-                                                slot_count, nch);                                  \
+                                                slot_count, nch, J0, local);                       \
         int64_t b2 = (slot_count + 7) / 8;                                                         \
         if (b2 > cap) b2 = cap;                                                                    \
-        row_chain_kernel<E_><<<(unsigned)b2, bs, 0, st>>>((E_ *)table, g, rbl, d_meta, J0, rho,     \
-                                                          slot_count);                             \
+        if (local)                                                                                 \
+            row_carry_kernel<E_><<<(unsigned)b2, bs, 0, st>>>((E_ *)table, g, rbl, d_meta, J0,      \
+                                                              slot_count);                         \
+        else                                                                                       \
+            row_chain_kernel<E_><<<(unsigned)b2, bs, 0, st>>>((E_ *)table, g, rbl, d_meta, J0, rho, \
+                                                              slot_count);                         \
     } while (0)
     if (e == 1) {
         if (NWk == 1) PTAS_LONG_CASE(uint8_t, 1); else PTAS_LONG_CASE(uint8_t, 2);

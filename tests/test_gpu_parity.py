@@ -632,3 +632,19 @@ def test_virtual_shards_use_packed_kernel(P, vs):
     assert (got["assignment"] == ref["assignment"]).all()
     assert got["stats"]["relaxations"] == ref["stats"]["relaxations"]
     assert got["stats"]["relax_executed"] == ref["stats"]["relax_executed"] < got["stats"]["relaxations"]
+
+
+@pytest.mark.parametrize("local", ["0", "1"])
+def test_long_row_chain_variants(P, monkeypatch, local):
+    # long-row path with the in-chunk chain in the cross kernel (1, default) or
+    # entirely in the chain kernel (0), forced on every level; J0 from 1 to > 32
+    monkeypatch.setenv("PTAS_FORCE_SCALAR", "2")
+    monkeypatch.setenv("PTAS_LONG_LOCAL", local)
+    _check_table(P, np.array([4, 3, 1200], np.int32), np.array([300, 170, 3], np.int64), 310)
+    _check_table(P, np.array([6, 1500], np.int32), np.array([100, 99], np.int64), 250)
+    _check_table(P, np.array([3, 3, 200], np.int32), np.array([50, 45, 1], np.int64), 60)
+    rng = np.random.default_rng(77)
+    for K in (2, 3, 4):
+        for _ in range(3):
+            N, r, T = _rand_case(rng, K, {2: 120, 3: 30, 4: 10}[K])
+            _check_table(P, N, r, T)
