@@ -451,6 +451,8 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
 //    from the previous chunk through registers, from older ones by a read.
 // Executed relaxations equal the collapsed count of the packed kernel.
 constexpr int CHAIN_BATCH = 8;   // chunks whose values a chain warp loads together
+constexpr int CARRY_BATCH = 16;  // same for row_carry_kernel
+constexpr int CROSS_CPT = 4;     // 32-entry chunks of one row per row_cross_kernel task
 
 template <typename E, int NW>
 __global__ void __launch_bounds__(256)
@@ -477,63 +479,70 @@ row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
 #pragma unroll
     for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
     const E SENT = (E)~(E)0;
-    for (int64_t task = gw; task < slot_count * nch; task += nw) {
-        const int64_t slot = task / nch;
-        const int64_t x = (task - slot * nch) * 32 + lane;
-        const bool act = x < g.W;
+    const int64_t ngrp = (nch + CROSS_CPT - 1) / CROSS_CPT;   // CROSS_CPT chunks of one row per task
+    for (int64_t task = gw; task < slot_count * ngrp; task += nw) {
+        const int64_t slot = task / ngrp;
+        const int64_t xg = (task - slot * ngrp) * (32 * CROSS_CPT);
         uint64_t pw[NW];
 #pragma unroll
         for (int w = 0; w < NW; ++w) pw[w] = pwa[(int64_t)w * pw_stride + slot];
         const int64_t rowbase = rb[slot];
-        const E *rowp = table + rowbase + x;
-        int acc = INF;
+        const E *rowp = table + rowbase + xg + lane;
+        int acc[CROSS_CPT];
+#pragma unroll
+        for (int c = 0; c < CROSS_CPT; ++c) acc[c] = INF;
         for (int base = 0; base < np; base += 32) {
-            const int c = base + lane;
-            bool dom = c < np;
+            const int cc = base + lane;
+            bool dom = cc < np;
             if (dom) {
 #pragma unroll
                 for (int w = 0; w < NW; ++w)
-                    dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + c]) & guard[w]) == guard[w];
+                    dom &= (((pw[w] | guard[w]) - s_w[(size_t)w * np + cc]) & guard[w]) == guard[w];
             }
             unsigned m = __ballot_sync(FULL, dom);
             while (m) {
-                int v[4];
+                const int b = __ffs(m) - 1;
+                m &= m - 1;
+                const uint64_t oj = s_oj[base + b];
+                const int64_t jm = (int64_t)(oj >> 48);
+                const int64_t off = (int64_t)(oj & 0xffffffffffffull);
+                int v[CROSS_CPT];
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    v[q] = INF;
-                    if (m) {
-                        const int b = __ffs(m) - 1;
-                        m &= m - 1;
-                        const uint64_t oj = s_oj[base + b];
-                        const int64_t jm = (int64_t)(oj >> 48);
-                        const int64_t J = jm < x ? jm : x;
-                        if (act) v[q] = rowp[-(int64_t)(oj & 0xffffffffffffull) - J];
-                    }
+                for (int c = 0; c < CROSS_CPT; ++c) {
+                    const int64_t x = xg + 32 * c + lane;
+                    const int64_t J = jm < x ? jm : x;
+                    v[c] = x < g.W ? (int)rowp[32 * c - off - J] : INF;
                 }
 #pragma unroll
-                for (int q = 0; q < 4; ++q) acc = v[q] < acc ? v[q] : acc;
+                for (int c = 0; c < CROSS_CPT; ++c) acc[c] = v[c] < acc[c] ? v[c] : acc[c];
             }
         }
-        if (!local_chain) {
-            if (act) table[rowbase + x] = acc >= INF ? SENT : (E)acc;
-            continue;
+#pragma unroll
+        for (int c = 0; c < CROSS_CPT; ++c) {
+            const int64_t x0 = xg + 32 * c;
+            if (x0 >= g.W) break;
+            const int64_t x = x0 + lane;
+            const bool act = x < g.W;
+            if (!local_chain) {
+                if (act) table[rowbase + x] = acc[c] >= INF ? SENT : (E)acc[c];
+                continue;
+            }
+            // row-levels >= 1: acc is finite for every state (a unit prefix e_i <= p
+            // always dominates), so the in-row chain inside this chunk is resolved
+            // here (min-plus doubling) and row_carry_kernel only adds what comes
+            // from earlier chunks
+            int opt = act ? acc[c] + 1 : INF;
+            if (x0 == 0) {
+                const int t0 = __shfl_sync(FULL, opt, 0);
+                if (x >= 1 && x < J0 && t0 + 1 < opt) opt = t0 + 1;
+            }
+            for (int sft = 1; sft * J0 < 32; sft <<= 1) {
+                const int d = sft * J0;
+                const int u = __shfl_up_sync(FULL, opt, d);
+                if (lane >= d && x >= J0 && u + sft < opt) opt = u + sft;
+            }
+            if (act) table[rowbase + x] = (E)opt;
         }
-        // row-levels >= 1: acc is finite for every state (a unit prefix e_i <= p
-        // always dominates), so the in-row chain inside this chunk is resolved
-        // here (min-plus doubling) and row_carry_kernel only adds what comes
-        // from earlier chunks
-        const int64_t x0 = x - lane;
-        int opt = act ? acc + 1 : INF;
-        if (x0 == 0) {
-            const int t0 = __shfl_sync(FULL, opt, 0);
-            if (x >= 1 && x < J0 && t0 + 1 < opt) opt = t0 + 1;
-        }
-        for (int sft = 1; sft * J0 < 32; sft <<= 1) {
-            const int d = sft * J0;
-            const int u = __shfl_up_sync(FULL, opt, d);
-            if (lane >= d && x >= J0 && u + sft < opt) opt = u + sft;
-        }
-        if (act) table[rowbase + x] = (E)opt;
     }
 }
 
@@ -555,15 +564,15 @@ row_carry_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
         E *out = table + rb[slot];
         int prev = INF;
         if (lane < g.W) prev = out[lane];                 // chunk 0: local == final
-        for (int64_t xb = 32; xb < g.W; xb += 32 * CHAIN_BATCH) {
-            int av[CHAIN_BATCH];
+        for (int64_t xb = 32; xb < g.W; xb += 32 * CARRY_BATCH) {
+            int av[CARRY_BATCH];
 #pragma unroll
-            for (int c = 0; c < CHAIN_BATCH; ++c) {
+            for (int c = 0; c < CARRY_BATCH; ++c) {
                 const int64_t xi = xb + 32 * c + lane;
                 av[c] = xi < g.W ? (int)out[xi] : INF;
             }
 #pragma unroll
-            for (int c = 0; c < CHAIN_BATCH; ++c) {
+            for (int c = 0; c < CARRY_BATCH; ++c) {
                 const int64_t x0 = xb + 32 * c;
                 if (x0 >= g.W) break;
                 const int64_t x = x0 + lane;
@@ -973,7 +982,7 @@ cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int
     const int64_t nch = (g.W + 31) / 32;
     const int bs = 256;
     const int64_t cap = (int64_t)sm_count * 8;
-    int64_t blocks = (slot_count * nch + 7) / 8;
+    int64_t blocks = (slot_count * ((nch + CROSS_CPT - 1) / CROSS_CPT) + 7) / 8;
     if (blocks > cap) blocks = cap;
     const int64_t *rbl = rb + slot_begin;
     const uint64_t *pwl = pw + slot_begin;
