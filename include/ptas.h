@@ -243,7 +243,9 @@ int ptas_probe_targets(int64_t LB, int64_t UB, int32_t P, int64_t *out,
 int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T,
                          const int32_t *feasible, int32_t count);
 /* Contiguous slice [begin, end) of `count` items owned by `rank` of
- * `world` (ceil split; trailing ranks may be empty). */
+ * `world` (ceil split; trailing ranks may be empty).  The level-sharded DP
+ * splits each sharded row-level the same way, except that the per-rank row
+ * count is rounded up so every slice starts 16-byte aligned. */
 int ptas_shard_range(int64_t count, int32_t rank, int32_t world,
                      int64_t *begin, int64_t *end);
 
