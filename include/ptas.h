@@ -249,6 +249,19 @@ int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T,
 int ptas_shard_range(int64_t count, int32_t rank, int32_t world,
                      int64_t *begin, int64_t *end);
 
+/* Internal class order of the DP table (D2,
+ * D13): order_out[i] = the caller class laid out at position i (the
+ * non-empty classes only, *K_out of them; position K_out - 1 is the
+ * contiguous row dimension).  layout 0 (ptas_solve's default, options.layout):
+ * the largest-count class last, the others by descending size; layout 1: the
+ * given order.  ptas_solve lays out every probe's table this way, so
+ * dp_fill(counts[order], sizes[order]) computes the solve's own layout.
+ *   counts[K], sizes[K] host; order_out host int32[K] (room for K).
+ * EINVAL: K < 0 or > 64, counts < 0, null pointers, layout not 0/1.
+ * Pure host function (no CUDA). */
+int ptas_table_order(const int32_t *counts, const int64_t *sizes, int32_t K,
+                     int32_t layout, int32_t *order_out, int32_t *K_out);
+
 /* ---------------------------------------------------------------- inspection
  * Device steps exposed for parity tests (need a GPU). */
 

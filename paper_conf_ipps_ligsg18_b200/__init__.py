@@ -15,7 +15,7 @@ from ._native import (MODE_LEVEL_SHARDED, MODE_MULTI_PROBE, MODE_SINGLE, EXPORTS
 
 __all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
            "dp_row_index", "ptas_k", "ptas_bounds", "ptas_classify", "ptas_probe_targets",
-           "ptas_interval_update", "ptas_shard_range", "Comm", "init_comm", "options", "lib", "strerror",
+           "ptas_interval_update", "ptas_shard_range", "ptas_table_order", "Comm", "init_comm", "options", "lib", "strerror",
            "PtasError", "EXPORTS", "MODE_SINGLE", "MODE_LEVEL_SHARDED", "MODE_MULTI_PROBE"]
 
 
@@ -197,6 +197,17 @@ def ptas_interval_update(LB: int, UB: int, T, feasible):
     _chk("ptas_interval_update", lib().ptas_interval_update(ctypes.byref(lb), ctypes.byref(ub),
                                                             _ptr(T, ctypes.c_int64), _ptr(f, ctypes.c_int32), len(T)))
     return lb.value, ub.value
+
+
+def ptas_table_order(counts, sizes, layout: int = 0):
+    """Internal class order of the DP table (list of caller class indices, non-empty classes)."""
+    c = _a(counts, np.int32)
+    s = _a(sizes, np.int64)
+    out = np.zeros(max(len(c), 1), np.int32)
+    k = ctypes.c_int32()
+    _chk("ptas_table_order", lib().ptas_table_order(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), len(c),
+                                                    int(layout), _ptr(out, ctypes.c_int32), ctypes.byref(k)))
+    return [int(x) for x in out[: k.value]]
 
 
 def ptas_shard_range(count: int, rank: int, world: int):

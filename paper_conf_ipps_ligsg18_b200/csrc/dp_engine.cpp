@@ -343,6 +343,8 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     std::vector<int64_t> cnt, stride;
     rc = build_geom(N, e, true, &g, &cnt, &stride);
     if (rc) return rc;
+    PT_CK(blk_.ensure(sizeof(int32_t) * 2 * MAXK));
+    g.blk = (int32_t *)blk_.p;   // pivot blocks, written by build_prefix_kernel (D13)
     const int64_t rows = sigma / g.W;
     const int64_t ibytes = rows * g.Wp * e;  // padded internal table
     // compute in the caller's buffer when its layout is the padded one
@@ -578,7 +580,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         size_t plan_off;       // int32 offset into dfplan_
     };
     std::vector<DfRun> runs;
-    {
+    // narrow K = 3 DPs: the whole fill on one thread-block cluster, recent levels
+    // in distributed shared memory (row_ring.cu, D14); PTAS_RING=0: off
+    const bool ring = G == 1 && !force_scalar && K == 3 &&
+                      launch_row_fill_ring(e, table, g, N.data(), r.data(), rq.T, J0, (const PrefixEntry *)pref_.p,
+                                           d_meta_, nP_bound, st, true) == cudaSuccess;
+    cudaGetLastError();
+    if (!ring) {
         const char *dfs = std::getenv("PTAS_DF");
         const int df_mode = dfs && dfs[0] ? std::atoi(dfs) : 3;
         const char *dfr = std::getenv("PTAS_DF_ROWS");
@@ -672,7 +680,12 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         for (auto &ev : lev) PT_CK(cudaEventCreate(&ev));
         PT_CK(cudaEventRecord(lev[0], st));
     }
-    for (int rho = 0; rho <= g.rho_max; ++rho) {
+    if (ring) {
+        PT_CK(launch_row_fill_ring(e, table, g, N.data(), r.data(), rq.T, J0, (const PrefixEntry *)pref_.p, d_meta_,
+                                   nP_bound, st, false));
+        ++o.fill_launches;
+    }
+    for (int rho = 0; rho <= (ring ? -1 : g.rho_max); ++rho) {
         const int64_t R = cnt[rho];
         if (lvl_times && rho > 0) PT_CK(cudaEventRecord(lev[rho], st));
         if (R <= 0) continue;
@@ -764,7 +777,9 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         ++o.launches;
     }
     PT_CK(cudaEventRecord(ev_[2], st));
-    if (lvl_times) {
+    if (lvl_times && ring) {
+        for (auto &ev : lev) cudaEventDestroy(ev);
+    } else if (lvl_times) {
         PT_CK(cudaEventRecord(lev[g.rho_max + 1], st));
         PT_CK(cudaEventSynchronize(lev[g.rho_max + 1]));
         std::fprintf(stderr, "[ptas] level times (us, rows) sigma=%lld:", (long long)sigma);

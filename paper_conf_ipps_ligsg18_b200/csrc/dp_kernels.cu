@@ -3,9 +3,10 @@
 //  enum_configs_kernel   §8(a) a-3: C(T) (Alg 2 l.17), once per T
 //  exclusive_scan_kernel compaction offsets for a-3
 //  build_prefix_kernel   a-3: group C by leading digits, packed words, off(s'),
-//                        closed-form relaxation count
-//  row_fill_kernel       a-5: Eq. 1 for one row-level
-//  row_cross_kernel / row_chain_kernel  a-5 for rows longer than 1 KiB (D5, two launches)
+//                        pivot blocks (D13), closed-form relaxation counts
+//  row_fill_kernel       a-5: Eq. 1 for one row-level (scalar
+//                        fallback: full relaxation incl. the in-row terms)
+//  row_cross_kernel      a-5 for rows longer than 1 KiB (D5, D12, D13; one launch)
 //  row_scatter_kernel    §8(e): gathered compact rows -> mixed-radix table
 //  build_row_index_kernel a-4: level-ordered row index (row base + packed digits)
 //  traceback_kernel      a-8: schedule of the rounded long jobs from DP(T*)
@@ -153,9 +154,11 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
     __shared__ int64_t warp_sums[32];
     __shared__ int64_t carry;
     __shared__ unsigned long long relax_acc, exec_acc;
+    __shared__ int32_t blo[MAXK], bhi[MAXK];   // pivot blocks (D13), nonzero-prefix indices
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int K1 = K - 1;
     if (tid == 0) { carry = 0; relax_acc = 0ull; exec_acc = 0ull; }
+    if (tid < MAXK) { blo[tid] = INT32_MAX; bhi[tid] = -1; }
     __syncthreads();
     unsigned long long my_relax = 0, my_exec = 0;
     for (int64_t base = 0; base < nC; base += blockDim.x) {
@@ -195,16 +198,19 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
                 e.jmax = 0;
                 e.pad = 0;
                 pref[id] = e;
-                // collapsed relaxations (D5): one per (row dominating s', x) for s' != 0,
-                // one per state with x >= 1 for the in-row term s' = 0
-                unsigned long long rows_dom = 1;
-                bool zero = true;
-                for (int i = 0; i < K1; ++i) {
-                    rows_dom *= (unsigned long long)(Nall.v[i] - dc[i] + 1);
-                    zero &= dc[i] == 0;
+                // executed window gathers (D5, D12, D13): one per (row p >= s' whose first
+                // nonzero digit is q = fnz(s'), x) for s' != 0; none for s' = 0 (the
+                // in-row configurations never win for p != 0; row 0 is a closed form)
+                int q = 0;
+                while (q < K1 && dc[q] == 0) ++q;
+                if (q < K1) {
+                    unsigned long long rows_piv = 1;
+                    for (int i = q; i < K1; ++i) rows_piv *= (unsigned long long)(Nall.v[i] - dc[i] + 1);
+                    const unsigned long long Wl = (unsigned long long)Nall.v[K - 1] + 1;
+                    my_exec += rows_piv * Wl;
+                    atomicMin(&blo[q], (int32_t)(id - 1));   // index in the nonzero-prefix list
+                    atomicMax(&bhi[q], (int32_t)(id - 1));
                 }
-                const unsigned long long Wl = (unsigned long long)Nall.v[K - 1] + 1;
-                my_exec += zero ? rows_dom * (Wl - 1) : rows_dom * Wl;
             }
             // closed-form relaxation count: prod_i (N_i - s_i + 1) states dominate s
             unsigned long long pr = 1;
@@ -228,6 +234,12 @@ __global__ void build_prefix_kernel(int K, const uint16_t *__restrict__ digits,
         meta->relax = relax_acc;
         meta->relax_exec = exec_acc;
         meta->ovf = carry - 1 > np_cap ? 1 : 0;
+    }
+    // pivot blocks: [first, last + 1) per first-nonzero digit, empty = [0, 0)
+    if (tid < MAXK && g.blk) {
+        const bool ne = tid < K1 && bhi[tid] >= 0;
+        g.blk[2 * tid] = ne ? blo[tid] : 0;
+        g.blk[2 * tid + 1] = ne ? bhi[tid] + 1 : 0;
     }
 }
 
@@ -438,27 +450,38 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
 }
 
 // Long rows (W > 1 KiB, beyond the packed kernel's one-row-per-group layout):
-// the row-level is filled in two launches so that a long row is spread over
-// many warps instead of one.
-//  row_cross_kernel: one warp per (row, 32-entry chunk); for each state
-//    acc(x) = min over prefixes s' != 0, s' <= p of OPT(p - s', x - min(x, Jmax(s')))
-//    (the window min of reading D5: OPT is monotone in x), written to the
-//    state's own entry as a provisional value (sentinel = the all-ones E value:
-//    every finite acc is an OPT of a smaller state, <= sum N - 1).
-//  row_chain_kernel: one warp per row, chunks in order; in-row term of D5
-//    OPT(p, x) = 1 + min(acc(x), OPT(p, x - min(x, J0))), x >= 1, resolved
-//    inside a chunk by min-plus doubling over the lanes (log2(32 / J0) rounds),
-//    from the previous chunk through registers, from older ones by a read.
-// Executed relaxations equal the collapsed count of the packed kernel.
-constexpr int CHAIN_BATCH = 8;   // chunks whose values a chain warp loads together
-constexpr int CARRY_BATCH = 16;  // same for row_carry_kernel
-constexpr int CROSS_CPT = 4;     // 32-entry chunks of one row per row_cross_kernel task
+// one launch per row-level, one warp per (row, CROSS_CPT chunks of 32 entries),
+// so a long row is spread over many warps.  For a row p != 0
+//   OPT(p, x) = 1 + min over prefixes s' <= p of the row's pivot block of
+//               OPT(p - s', x - min(x, Jmax(s')))
+// (window minimum of reading D5: OPT is monotone in x; pivot block and no
+// in-row term by readings D12/D13); row p = 0 is the closed form
+// OPT(0, x) = ceil(x / J0).  Executed relaxations equal the packed kernel's.
+constexpr int CROSS_CPT = 4;     // 32-entry chunks of one row per task
+
+// first nonzero leading digit of a row from its packed digits (-1: p = 0)
+template <int NW>
+__device__ __forceinline__ int pivot_digit(const RowGeom &g, const uint64_t *pw)
+{
+    int wd = -1, bit = 0;
+#pragma unroll
+    for (int w = NW - 1; w >= 0; --w)
+        if (pw[w]) {
+            wd = w;
+            bit = __ffsll((long long)pw[w]) - 1;
+        }
+    if (wd < 0) return -1;
+    int q = -1;
+    for (int i = 0; i < g.K1; ++i)
+        if (g.word[i] == wd && g.shift[i] <= bit) q = i;
+    return q;
+}
 
 template <typename E, int NW>
 __global__ void __launch_bounds__(256)
 row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const uint64_t *__restrict__ pwa,
                  int64_t pw_stride, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta,
-                 int64_t slot_count, int64_t nch, int J0, int local_chain)
+                 int64_t slot_count, int64_t nch, int J0)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     if (meta->ovf) return;
@@ -478,7 +501,6 @@ row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
     uint64_t guard[NW];
 #pragma unroll
     for (int w = 0; w < NW; ++w) guard[w] = g.guard[w];
-    const E SENT = (E)~(E)0;
     const int64_t ngrp = (nch + CROSS_CPT - 1) / CROSS_CPT;   // CROSS_CPT chunks of one row per task
     for (int64_t task = gw; task < slot_count * ngrp; task += nw) {
         const int64_t slot = task / ngrp;
@@ -487,13 +509,23 @@ row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
 #pragma unroll
         for (int w = 0; w < NW; ++w) pw[w] = pwa[(int64_t)w * pw_stride + slot];
         const int64_t rowbase = rb[slot];
+        const int q = pivot_digit<NW>(g, pw);
+        if (q < 0) {   // row p = 0
+#pragma unroll
+            for (int c = 0; c < CROSS_CPT; ++c) {
+                const int64_t x = xg + 32 * c + lane;
+                if (x < g.W) table[rowbase + x] = (E)((x + J0 - 1) / J0);
+            }
+            continue;
+        }
+        const int plo = g.blk[2 * q], phi = g.blk[2 * q + 1];
         const E *rowp = table + rowbase + xg + lane;
         int acc[CROSS_CPT];
 #pragma unroll
         for (int c = 0; c < CROSS_CPT; ++c) acc[c] = INF;
-        for (int base = 0; base < np; base += 32) {
+        for (int base = plo & ~31; base < phi; base += 32) {
             const int cc = base + lane;
-            bool dom = cc < np;
+            bool dom = cc >= plo && cc < phi;
             if (dom) {
 #pragma unroll
                 for (int w = 0; w < NW; ++w)
@@ -519,132 +551,8 @@ row_cross_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, cons
         }
 #pragma unroll
         for (int c = 0; c < CROSS_CPT; ++c) {
-            const int64_t x0 = xg + 32 * c;
-            if (x0 >= g.W) break;
-            const int64_t x = x0 + lane;
-            const bool act = x < g.W;
-            if (!local_chain) {
-                if (act) table[rowbase + x] = acc[c] >= INF ? SENT : (E)acc[c];
-                continue;
-            }
-            // row-levels >= 1: acc is finite for every state (a unit prefix e_i <= p
-            // always dominates), so the in-row chain inside this chunk is resolved
-            // here (min-plus doubling) and row_carry_kernel only adds what comes
-            // from earlier chunks
-            int opt = act ? acc[c] + 1 : INF;
-            if (x0 == 0) {
-                const int t0 = __shfl_sync(FULL, opt, 0);
-                if (x >= 1 && x < J0 && t0 + 1 < opt) opt = t0 + 1;
-            }
-            for (int sft = 1; sft * J0 < 32; sft <<= 1) {
-                const int d = sft * J0;
-                const int u = __shfl_up_sync(FULL, opt, d);
-                if (lane >= d && x >= J0 && u + sft < opt) opt = u + sft;
-            }
-            if (act) table[rowbase + x] = (E)opt;
-        }
-    }
-}
-
-// Row-levels >= 1 after row_cross_kernel(local_chain = 1): per row, chunks in
-// order, final(x) = min(local(x), final(z - min(z, J0)) + 1 + t) where z is the
-// first element of x's in-row chain inside the chunk (x = z + t * J0).
-template <typename E>
-__global__ void __launch_bounds__(256)
-row_carry_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const DpMeta *__restrict__ meta,
-                 int J0, int64_t slot_count)
-{
-    if (meta->ovf) return;
-    const int lane = threadIdx.x & 31;
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int zo = J0 < 32 ? lane % J0 : lane;           // z - x0 (chunk-independent)
-    const int tz = J0 < 32 ? lane / J0 : 0;              // chain steps from z to x
-    for (int64_t slot = gw; slot < slot_count; slot += nw) {
-        E *out = table + rb[slot];
-        int prev = INF;
-        if (lane < g.W) prev = out[lane];                 // chunk 0: local == final
-        for (int64_t xb = 32; xb < g.W; xb += 32 * CARRY_BATCH) {
-            int av[CARRY_BATCH];
-#pragma unroll
-            for (int c = 0; c < CARRY_BATCH; ++c) {
-                const int64_t xi = xb + 32 * c + lane;
-                av[c] = xi < g.W ? (int)out[xi] : INF;
-            }
-#pragma unroll
-            for (int c = 0; c < CARRY_BATCH; ++c) {
-                const int64_t x0 = xb + 32 * c;
-                if (x0 >= g.W) break;
-                const int64_t x = x0 + lane;
-                const bool act = x < g.W;
-                const int64_t z = x0 + zo;
-                const int64_t src = z - (J0 < z ? J0 : z);
-                const int64_t pl = src - (x0 - 32);
-                const int t = __shfl_sync(FULL, prev, (int)(pl >= 0 && pl < 32 ? pl : 0));
-                int opt = av[c];
-                if (act) {
-                    const int v = (pl >= 0 ? t : (int)out[src]) + 1 + tz;
-                    opt = v < opt ? v : opt;
-                    out[x] = (E)opt;
-                }
-                prev = opt;
-                __syncwarp();
-            }
-        }
-    }
-}
-
-template <typename E>
-__global__ void __launch_bounds__(256)
-row_chain_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const DpMeta *__restrict__ meta,
-                 int J0, int rho, int64_t slot_count)
-{
-    if (meta->ovf) return;
-    const int lane = threadIdx.x & 31;
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const E SENT = (E)~(E)0;
-    for (int64_t slot = gw; slot < slot_count; slot += nw) {
-        E *out = table + rb[slot];
-        int prev = INF;                                   // previous chunk's final values
-        for (int64_t xb = 0; xb < g.W; xb += 32 * CHAIN_BATCH) {
-            // provisional acc of CHAIN_BATCH chunks loaded together (one latency per batch)
-            int av[CHAIN_BATCH];
-#pragma unroll
-            for (int c = 0; c < CHAIN_BATCH; ++c) {
-                const int64_t xi = xb + 32 * c + lane;
-                av[c] = xi < g.W ? (int)out[xi] : 0;
-            }
-#pragma unroll
-            for (int c = 0; c < CHAIN_BATCH; ++c) {
-                const int64_t x0 = xb + 32 * c;
-                if (x0 >= g.W) break;
-                const int64_t x = x0 + lane;
-                const bool act = x < g.W;
-                const int a = av[c];
-                int opt = !act ? INF : ((rho == 0 && x == 0) ? 0 : (a == (int)SENT ? INF : a + 1));
-                // in-row source x - min(x, J0) before this chunk: previous chunk from registers, older from memory
-                const int64_t src = act && x > 0 ? x - (J0 < x ? J0 : x) : x;
-                const int64_t pl = src - (x0 - 32);
-                const int t = __shfl_sync(FULL, prev, (int)(pl >= 0 && pl < 32 ? pl : 0));
-                if (act && x > 0 && src < x0) {
-                    const int v = (pl >= 0 ? t : (int)out[src]) + 1;
-                    opt = v < opt ? v : opt;
-                }
-                if (x0 == 0) {                            // x < J0 reaches back to x = 0 directly
-                    const int t0 = __shfl_sync(FULL, opt, 0);
-                    if (x >= 1 && x < J0 && t0 + 1 < opt) opt = t0 + 1;
-                }
-                // in-chunk chain x -> x - J0 -> ... : min-plus doubling over the lanes
-                for (int sft = 1; sft * J0 < 32; sft <<= 1) {
-                    const int d = sft * J0;
-                    const int u = __shfl_up_sync(FULL, opt, d);
-                    if (lane >= d && x >= J0 && u + sft < opt) opt = u + sft;
-                }
-                if (act) out[x] = (E)opt;
-                prev = opt;
-                __syncwarp();
-            }
+            const int64_t x = xg + 32 * c + lane;
+            if (x < g.W) table[rowbase + x] = (E)(acc[c] + 1);
         }
     }
 }
@@ -974,6 +882,7 @@ cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int
                                  int64_t nP_bound, int J0, int rho, int64_t slot_begin, int64_t slot_count,
                                  int sm_count, cudaStream_t st)
 {
+    (void)rho;
     if (slot_count <= 0) return cudaSuccess;
     const int NWk = g.nwords <= 1 ? 1 : 2;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
@@ -986,9 +895,6 @@ cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int
     if (blocks > cap) blocks = cap;
     const int64_t *rbl = rb + slot_begin;
     const uint64_t *pwl = pw + slot_begin;
-    // PTAS_LONG_LOCAL=0: the in-row chain entirely in row_chain_kernel (measurement knob)
-    const char *ll = std::getenv("PTAS_LONG_LOCAL");
-    const int local = (rho >= 1 && !(ll && ll[0] == '0')) ? 1 : 0;
     cudaError_t err;
 #define PTAS_LONG_CASE(E_, NW_)                                                                    \
     do {                                                                                           \
@@ -998,15 +904,7 @@ cudaError_t launch_row_fill_long(int e, void *table, const RowGeom &g, const int
             if (err != cudaSuccess) return err;                                                    \
         }                                                                                          \
         kfn<<<(unsigned)blocks, bs, smem, st>>>((E_ *)table, g, rbl, pwl, pw_stride, d_pref, d_meta, \
-                                                slot_count, nch, J0, local);                       \
-        int64_t b2 = (slot_count + 7) / 8;                                                         \
-        if (b2 > cap) b2 = cap;                                                                    \
-        if (local)                                                                                 \
-            row_carry_kernel<E_><<<(unsigned)b2, bs, 0, st>>>((E_ *)table, g, rbl, d_meta, J0,      \
-                                                              slot_count);                         \
-        else                                                                                       \
-            row_chain_kernel<E_><<<(unsigned)b2, bs, 0, st>>>((E_ *)table, g, rbl, d_meta, J0, rho, \
-                                                              slot_count);                         \
+                                                slot_count, nch, J0);                              \
     } while (0)
     if (e == 1) {
         if (NWk == 1) PTAS_LONG_CASE(uint8_t, 1); else PTAS_LONG_CASE(uint8_t, 2);

@@ -54,6 +54,12 @@ struct RowGeom {
     int32_t hi[MAXK];
     int32_t dbase[MAXK];
     const uint32_t *domtab;     // device table (TS > 0)
+    // pivot blocks (D13): blk[2q], blk[2q+1] = [first, end) of the
+    // prefixes (indices into the nonzero-prefix list, entry 1 of the prefix
+    // table = index 0) whose first nonzero leading digit is q; written by
+    // build_prefix_kernel.  A row p != 0 walks only the block of its own first
+    // nonzero digit.  Empty block: first == end.
+    int32_t *blk;               // device [2 * MAXK]
 };
 constexpr int64_t DOMTAB_MAX_BYTES = 16384;
 
@@ -87,13 +93,27 @@ struct DfArgs {
     uint64_t dmask[MAXK];         // bits of leading digit i inside its packed word g.word[i]
 };
 
+// Narrow K = 3 DPs on one thread-block cluster (row_ring.cu, D14).
+struct RingArgs {
+    int32_t N0, N1;       // the two leading counts (row (a, b), level a + b)
+    int64_t stride0;      // elements between rows (a, b) and (a + 1, b)
+    int32_t Wp;           // row pitch (elements)
+    int32_t Lw, Lg;       // words per row, lanes per row (Lw / CH)
+    int32_t J0;           // min(N_last, floor(T / r_last))
+    int32_t R;            // ring depth in row-levels
+    int32_t A;            // ring rows per level per CTA: ceil((N0 + 1) / cluster size)
+    int32_t rho_max;      // N0 + N1
+};
+
 // Device-side summary written by the planning kernels and read back once.
 struct DpMeta {
     int64_t nC;            // |C|
     int64_t nP;            // number of prefix entries (incl. the zero prefix)
     unsigned long long relax;  // closed-form relaxations sum_{s in C} prod(N_i - s_i + 1)
-    unsigned long long relax_exec;  // (n, s') pairs the packed kernel evaluates (reading D5):
-                                    // sum_{s' != 0} prod_{i<K-1}(N_i - s'_i + 1) * W + rows * (W - 1)
+    unsigned long long relax_exec;  // (n, s') window gathers of the fill kernels (readings D5, D12,
+                                    // D13): sum over prefixes s' != 0 with first nonzero digit q of
+                                    // prod_{q<=i<K-1}(N_i - s'_i + 1) * W  (rows p >= s' whose own
+                                    // first nonzero digit is q); row p = 0 is a closed form
     int32_t opt;           // OPT(N)
     int32_t err;           // device-detected error (traceback)
     int32_t ovf;           // enumeration without a host round trip: |C| or the prefix
@@ -168,6 +188,13 @@ cudaError_t launch_row_fill_swar_df(int e, void *table, const RowGeom &g, const 
                                     int64_t nP_bound, int J0, int64_t max_level_rows, const DfArgs &df,
                                     unsigned long long *ticket_base, int sm_count, cudaStream_t st, int pdl,
                                     int cslot);
+// Whole level fill of a K = 3 DP on one thread-block cluster with the recent
+// row-levels in distributed shared memory (row_ring.cu); N, r internal order.
+// cudaErrorNotSupported: the DP does not qualify (use the other launchers);
+// dry = true: only the check, no launch.
+cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int32_t *N, const int64_t *r,
+                                 int64_t T, int J0, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                 int64_t nP_bound, cudaStream_t st, bool dry);
 // Rows per row set the dataflow kernel will use for this geometry (0 = unsupported).
 int swar_df_rows_per_set(int e, const RowGeom &g, int J0, int64_t max_level_rows, int sm_count);
 // Copies the DP's prefix offsets/Jmax into the fill kernel's constant bank

@@ -134,14 +134,28 @@ std::vector<int64_t> memo_key(const Classified &c, int64_t T)
     return key;
 }
 
-// internal class order for the table (layout 0): ascending count, ties by
-// class index, so the largest class is the contiguous (row) dimension.
-std::vector<int> choose_order(const std::vector<int32_t> &N, int layout)
+// internal class order for the table (layout 0, D2/D13): the
+// non-empty class with the largest count (ties: the highest index) is the
+// contiguous row dimension; the leading classes follow by descending size r
+// (ties by index), so that the first nonzero leading digit of most rows -- the
+// row's pivot, D13 -- is a large class whose block of configurations is short.
+// layout 1: the non-empty classes in the given (classify) order.
+std::vector<int> choose_order(const std::vector<int32_t> &N, const std::vector<int64_t> &r, int layout)
 {
-    std::vector<int> o(N.size());
-    for (size_t i = 0; i < N.size(); ++i) o[i] = (int)i;
-    if (layout == 0)
-        std::stable_sort(o.begin(), o.end(), [&](int a, int b) { return N[a] < N[b]; });
+    std::vector<int> o;
+    for (size_t i = 0; i < N.size(); ++i)
+        if (N[i] > 0) o.push_back((int)i);
+    if (layout == 0 && !o.empty()) {
+        int last = o[0];
+        for (int i : o)
+            if (N[i] >= N[last]) last = i;
+        std::vector<int> lead;
+        for (int i : o)
+            if (i != last) lead.push_back(i);
+        std::stable_sort(lead.begin(), lead.end(), [&](int a, int b) { return r[a] > r[b]; });
+        lead.push_back(last);
+        o.swap(lead);
+    }
     return o;
 }
 
@@ -289,7 +303,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         return rq;
     };
     auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
-        std::vector<int> order = choose_order(c.N, opt.layout);
+        std::vector<int> order = choose_order(c.N, c.r, opt.layout);
         DpRequest rq = make_rq(c, T, s, order, (cudaStream_t)opt.stream);
         DpOutcome o;
         int r2 = eng->run_dp(rq, &o);
@@ -321,7 +335,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             }
             std::vector<int> rcs(nb, PTAS_OK);
             std::vector<std::vector<int>> orders(nb);
-            for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, opt.layout);
+            for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, cls_v[j0 + b].r, opt.layout);
             auto work = [&](int b) {
                 if (cudaSetDevice(dev) != cudaSuccess) {
                     rcs[b] = PTAS_ECUDA;
@@ -361,7 +375,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             std::vector<DpOutcome> outs(nb);
             std::vector<int> rcs(nb, PTAS_OK);
             std::vector<std::vector<int>> orders(nb);
-            for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, opt.layout);
+            for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, cls_v[j0 + b].r, opt.layout);
             auto work = [&](int b) {
                 if (cudaSetDevice(dev) != cudaSuccess) {
                     rcs[b] = PTAS_ECUDA;
@@ -777,6 +791,20 @@ int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T, const int32
     return PTAS_OK;
 }
 
+int ptas_table_order(const int32_t *counts, const int64_t *sizes, int32_t K, int32_t layout, int32_t *order_out,
+                     int32_t *K_out)
+{
+    if (K < 0 || K > 64 || (K > 0 && (!counts || !sizes || !order_out)) || !K_out || layout < 0 || layout > 1)
+        return PTAS_EINVAL;
+    for (int32_t i = 0; i < K; ++i)
+        if (counts[i] < 0) return PTAS_EINVAL;
+    const std::vector<int> o = choose_order(std::vector<int32_t>(counts, counts + K),
+                                            std::vector<int64_t>(sizes, sizes + K), layout);
+    for (size_t i = 0; i < o.size(); ++i) order_out[i] = o[i];
+    *K_out = (int32_t)o.size();
+    return PTAS_OK;
+}
+
 int ptas_shard_range(int64_t count, int32_t rank, int32_t world, int64_t *begin, int64_t *end)
 {
     if (count < 0 || world < 1 || rank < 0 || rank >= world || !begin || !end) return PTAS_EINVAL;
@@ -934,11 +962,8 @@ int hmbp_solve(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t c
     rc = Engine::get(dev, &eng);
     if (rc) return rc;
     std::lock_guard<std::mutex> lk(eng->mu);
-    // internal layout: the non-empty classes by ascending count (D2)
-    std::vector<int> order;
-    for (int i = 0; i < K; ++i)
-        if (N[i] > 0) order.push_back(i);
-    std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return N[a] < N[b]; });
+    // internal layout of the solve (D2, D13)
+    std::vector<int> order = choose_order(N, std::vector<int64_t>(sizes, sizes + K), 0);
     DpRequest rq;
     rq.K = K;
     rq.N = counts;

@@ -10,10 +10,16 @@
 //
 //     min_{0 <= j <= min(x, Jmax(s'))} OPT(p - s', x - j) = OPT(p - s', x - min(x, Jmax(s')))
 //
-// and the in-row configurations (0, j), 1 <= j <= J0, reduce to the single
-// term OPT(p, x - min(x, J0)).  Per (row, prefix) the kernel therefore takes
-// ONE shifted window of the source row instead of Jmax(s') + 1 of them; the
-// value is bit-identical to the plain recurrence (pinned by the parity tests).
+// Per (row, prefix) the kernel therefore takes ONE shifted window of the
+// source row instead of Jmax(s') + 1 of them.  Two more result-identical
+// restrictions follow from the bins of a packing being unordered (DESIGN.md
+// D12, D13): for a row p != 0 some bin of an optimal packing holds an item
+// of the row's first nonzero leading class q, so only the prefixes with
+// s'_q >= 1 (one contiguous block of the lexicographic prefix list) are
+// walked, and the in-row configurations (0, j) never win; row p = 0 is the
+// closed form OPT(0, x) = ceil(x / J0).  OPT(p, x) = 1 + the window minimum:
+// no in-row closure, no chain.  Values are bit-identical to the plain
+// recurrence (pinned by the parity tests).
 //
 // Lane layout: a row of Lw 32-bit words (pitch padded by the driver to a
 // multiple of CH words) is owned by a group of Lg = Lw / CH lanes; lane xl of
@@ -35,230 +41,11 @@
 
 #include "device_common.cuh"
 #include "internal.h"
+#include "swar_common.cuh"
 
 namespace ptas {
 namespace swar {
 
-namespace {
-
-__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel)
-{
-    uint32_t r;
-    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
-    return r;
-}
-
-__device__ __forceinline__ uint32_t vmin2(uint32_t a, uint32_t b) { return __vminu2(a, b); }
-
-template <int CH>
-struct Words {
-    uint32_t v[CH];
-};
-
-template <int CH>
-__device__ __forceinline__ void fill_words(Words<CH> &w, uint32_t x)
-{
-#pragma unroll
-    for (int t = 0; t < CH; ++t) w.v[t] = x;
-}
-
-#ifndef PTAS_DF_NOACQ
-#define PTAS_DF_NOACQ 0
-#endif
-#ifndef PTAS_DF_PROFILE
-#define PTAS_DF_PROFILE 0
-#endif
-#ifndef PTAS_DF_LD_CG
-#define PTAS_DF_LD_CG 0
-#endif
-// Coherent 32-bit loads of table words for the dataflow kernel (the table is
-// written during the launch, so the read-only path is not allowed): ordinary
-// weak loads, kept after the flag acquire by `volatile` (the acquire
-// invalidates L1); PTAS_DF_LD_CG=1 reads through L2 only.
-__device__ __forceinline__ uint32_t ld_co(const uint32_t *p)
-{
-    uint32_t v;
-    if (PTAS_DF_LD_CG) asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p));
-    else asm volatile("ld.global.u32 %0, [%1];" : "=r"(v) : "l"(p));
-    return v;
-}
-__device__ __forceinline__ uint2 ld_co2(const uint32_t *p)
-{
-    uint2 v;
-    if (PTAS_DF_LD_CG) asm volatile("ld.global.cg.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
-    else asm volatile("ld.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
-    return v;
-}
-__device__ __forceinline__ uint4 ld_co4(const uint32_t *p)
-{
-    uint4 v;
-    if (PTAS_DF_LD_CG)
-        asm volatile("ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
-    else
-        asm volatile("ld.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
-    return v;
-}
-__device__ __forceinline__ uint32_t ld_acquire(const uint32_t *p)
-{
-    uint32_t v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_relaxed(uint32_t *p, uint32_t v)
-{
-    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// CH consecutive words at p (4*CH-byte aligned: the pitch is a multiple of CH words)
-template <int CH, bool CO = false>
-__device__ __forceinline__ Words<CH> load_words(const uint32_t *p)
-{
-    Words<CH> w;
-    if constexpr (CO) {
-        if constexpr (CH == 1) {
-            w.v[0] = ld_co(p);
-        } else if constexpr (CH == 2) {
-            const uint2 a = ld_co2(p);
-            w.v[0] = a.x;
-            w.v[1] = a.y;
-        } else {
-#pragma unroll
-            for (int c = 0; c < CH; c += 4) {
-                const uint4 a = ld_co4(p + c);
-                w.v[c] = a.x;
-                w.v[c + 1] = a.y;
-                w.v[c + 2] = a.z;
-                w.v[c + 3] = a.w;
-            }
-        }
-    } else if constexpr (CH == 1) {
-        w.v[0] = __ldg(p);
-    } else if constexpr (CH == 2) {
-        const uint2 a = __ldg(reinterpret_cast<const uint2 *>(p));
-        w.v[0] = a.x;
-        w.v[1] = a.y;
-    } else {
-#pragma unroll
-        for (int c = 0; c < CH; c += 4) {
-            const uint4 a = __ldg(reinterpret_cast<const uint4 *>(p + c));
-            w.v[c] = a.x;
-            w.v[c + 1] = a.y;
-            w.v[c + 2] = a.z;
-            w.v[c + 3] = a.w;
-        }
-    }
-    return w;
-}
-
-template <int CH>
-__device__ __forceinline__ void store_words(uint32_t *p, const Words<CH> &w)
-{
-    if constexpr (CH == 1) {
-        p[0] = w.v[0];
-    } else if constexpr (CH == 2) {
-        *reinterpret_cast<uint2 *>(p) = make_uint2(w.v[0], w.v[1]);
-    } else {
-#pragma unroll
-        for (int c = 0; c < CH; c += 4)
-            *reinterpret_cast<uint4 *>(p + c) = make_uint4(w.v[c], w.v[c + 1], w.v[c + 2], w.v[c + 3]);
-    }
-}
-
-// Word w - k of the row for the lane's slot t (w = xl*CH + t), k >= 0 warp-uniform;
-// `fill` for w - k < 0.  Every lane of the warp must call it (shuffle).
-template <int CH>
-__device__ __forceinline__ uint32_t word_back(const Words<CH> &a, int t, int k, int xl, uint32_t fill)
-{
-    const int d = k - t;  // > 0: the word lives in a lane to the left
-    if (d <= 0) {
-        uint32_t r = a.v[0];
-#pragma unroll
-        for (int c = 1; c < CH; ++c)
-            if (c == t - k) r = a.v[c];
-        return r;
-    }
-    const int dl = (d + CH - 1) / CH;
-    const int slot = dl * CH - d;
-    uint32_t send = a.v[0];
-#pragma unroll
-    for (int c = 1; c < CH; ++c)
-        if (c == slot) send = a.v[c];
-    const uint32_t got = __shfl_up_sync(FULL, send, dl > 31 ? 31 : dl);
-    return xl >= dl ? got : fill;
-}
-
-// Operands of the 4-byte window that starts db bytes left of each of the
-// lane's words: PRMT(lo, hi) at byte offset o = (4 - db % 4) % 4, with
-// lo = word w - k1, hi = word w - k1 + 1, k1 = ceil(db / 4) (db > 0; the
-// caller uses the word itself for db = 0).  db <= 4: the only word needed
-// from another lane is the left neighbour's last one (one shuffle); db <= 8:
-// two shuffles; longer shifts: word_back.  WIN = the largest db the caller
-// can pass (4, 8, or 0 = any), so the unneeded forms are not compiled.  Words before
-// the row read `fill`.
-template <int CH, int WIN>
-__device__ __forceinline__ void windows(const Words<CH> &a, int db, int xl, uint32_t fill, Words<CH> &lo,
-                                        Words<CH> &hi)
-{
-    const uint32_t left = __shfl_up_sync(FULL, a.v[CH - 1], 1);
-    const uint32_t l1 = xl >= 1 ? left : fill;   // word w - 1 of slot 0
-    if (WIN == 4 || db <= 4) {
-#pragma unroll
-        for (int t = 0; t < CH; ++t) {
-            lo.v[t] = t == 0 ? l1 : a.v[t - 1];
-            hi.v[t] = a.v[t];
-        }
-    } else if (WIN == 8 || db <= 8) {
-        // word w - 2 of slot 0: lane xl-1's slot CH-2 (CH >= 2) or lane xl-2 (CH = 1)
-        const uint32_t left2 = __shfl_up_sync(FULL, a.v[CH >= 2 ? CH - 2 : 0], CH >= 2 ? 1 : 2);
-        const uint32_t l2 = xl >= (CH >= 2 ? 1 : 2) ? left2 : fill;
-        const bool two = db > 4;   // k1 = 2
-#pragma unroll
-        for (int t = 0; t < CH; ++t) {
-            const uint32_t w1 = t == 0 ? l1 : a.v[t - 1];
-            const uint32_t w2 = t >= 2 ? a.v[t - 2] : (t == 1 ? l1 : l2);
-            lo.v[t] = two ? w2 : w1;
-            hi.v[t] = two ? w1 : a.v[t];
-        }
-    } else {
-        const int k1 = (db + 3) >> 2;
-#pragma unroll
-        for (int t = 0; t < CH; ++t) {
-            lo.v[t] = word_back(a, t, k1, xl, fill);
-            hi.v[t] = word_back(a, t, k1 - 1, xl, fill);
-        }
-    }
-}
-
-// Same operands from a copy of the group's row in shared memory (row word r
-// at srow[r]), any db > 0: used by the in-row closure's long shifts.
-template <int CH>
-__device__ __forceinline__ void windows_smem(const uint32_t *srow, int db, int xl, uint32_t fill, Words<CH> &lo,
-                                             Words<CH> &hi)
-{
-    const int k1 = (db + 3) >> 2;
-#pragma unroll
-    for (int t = 0; t < CH; ++t) {
-        const int w = xl * CH + t - k1;
-        lo.v[t] = w >= 0 ? srow[w] : fill;
-        hi.v[t] = w + 1 >= 0 ? srow[w + 1] : fill;
-    }
-}
-
-// Kernel-side prefix entry: x = -off(s') in words, y = PRMT selector of the
-// window (low 16 bits; the odd-byte selector is y + 0x1111) | db << 16, where
-// db = Jmax(s') * e is the window's byte shift.  db = 0 (the word itself)
-// takes byte offset 4, i.e. the selector reads the high operand (the word)
-// only, so every prefix runs the same branch-free window code.
-constexpr int SEL_U8 = 0xA280, SEL_U16 = 0x3210, SEL_SELF = 0x4444;
-__device__ __forceinline__ int2 oj_entry(const PrefixEntry &pe, int eb)
-{
-    const int db = pe.jmax * eb;
-    const int o = db == 0 ? 4 : (4 - (db & 3)) & 3;
-    const int sel = (eb == 1 ? SEL_U8 : SEL_U16) + 0x1111 * o;
-    return make_int2(-(int)((uint64_t)pe.off * eb / 4), sel | (db << 16));
-}
-
-}  // namespace
 
 // Prefix offsets/Jmax in constant memory: indexed by a warp-uniform loop
 // counter they load into uniform registers.  One slot per DP slot of the engine.
@@ -418,8 +205,11 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     // dominance table (g.TS > 0, D10): per-digit selectors, then the
     // chunk words (copied from the DP's table built after the prefix list)
     // (offset arithmetic from smem_raw keeps the shared state space: LDS, not generic loads)
+    // pivot blocks (D13) and the packed-bit -> leading-digit map
+    int32_t *s_blk = reinterpret_cast<int32_t *>(s_tk + 1);
+    int8_t *s_b2d = reinterpret_cast<int8_t *>(s_blk + 2 * MAXK);
     int4 *s_dsel = reinterpret_cast<int4 *>(
-        smem_raw + ((reinterpret_cast<unsigned char *>(s_tk + 1) - smem_raw + 15) & ~(ptrdiff_t)15));
+        smem_raw + ((reinterpret_cast<unsigned char *>(s_b2d + NW * 64) - smem_raw + 15) & ~(ptrdiff_t)15));
     uint32_t *s_tab = reinterpret_cast<uint32_t *>(s_dsel + g.K1);
     // (uint8 kernels only: in the 64-register uint16 kernels the extra code
     // costs more than it saves, measured)
@@ -433,10 +223,21 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         for (int e = threadIdx.x; e < n; e += blockDim.x) s_tab[e] = g.domtab[e];
         __syncthreads();
     }
+    for (int i = threadIdx.x; i < 2 * MAXK + NW * 64; i += blockDim.x) {
+        if (i < 2 * MAXK) {
+            s_blk[i] = i < 2 * g.K1 ? g.blk[i] : 0;
+        } else {
+            const int b = i - 2 * MAXK, wd = b >> 6, bit = b & 63;
+            int d = -1;
+            for (int q = 0; q < g.K1; ++q)
+                if (g.word[q] == wd && g.shift[q] <= bit) d = q;
+            s_b2d[b] = (int8_t)d;
+        }
+    }
     if constexpr (RUN) {
         for (int i = threadIdx.x; i < 2 * (df.nlev + 1); i += blockDim.x) s_set[i] = df.plan[i];
-        __syncthreads();
     }
+    __syncthreads();
     // first row set's index entries, loaded before waiting on the previous level
     int64_t nrb = 0;
     uint64_t npw[NW];
@@ -598,15 +399,31 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         unsigned long long pf_g1 = 0;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(pf_g1));
 #endif
-        // ---- cross-row relaxations: acc = min over s' <= p of OPT(p - s', x - min(x, Jmax(s')))
+        // ---- pivot block of the row (D13): prefixes whose first nonzero digit is
+        // the row's first nonzero digit; row 0 and idle lanes: empty
+        int plo = 0, phi = 0;
+        if (rowok) {
+            const int b0 = NW == 1 || pw[0] ? __ffsll((long long)pw[0]) - 1 : (NW > 1 && pw[NW - 1] ? 63 + __ffsll((long long)pw[NW - 1]) : -1);
+            if (b0 >= 0) {
+                const int q = s_b2d[b0];
+                plo = s_blk[2 * q];
+                phi = s_blk[2 * q + 1];
+            }
+        }
+        const int wlo = __reduce_min_sync(FULL, plo < phi ? plo : INT32_MAX);
+        const int whi = __reduce_max_sync(FULL, phi);
+        // ---- cross-row relaxations: acc = min over s' <= p in the block of OPT(p - s', x - min(x, Jmax(s')))
         Words<CH> ae, ao;
         fill_words(ae, 0xffffffffu);
         fill_words(ao, 0xffffffffu);
-        for (int base = pbase0; base < np; base += pstep) {
-            const int cnt = np - base < 32 ? np - base : 32;
+        for (int base = (whi > 0 ? (wlo & ~31) : np) + pbase0; base < whi; base += pstep) {
+            const int cnt = whi - base < 32 ? whi - base : 32;
+            // the row's block within this chunk
+            const int rl = min(max(plo - base, 0), 32), rh = min(max(phi - base, 0), 32);
+            const unsigned rmask = (rh >= 32 ? FULL : ((1u << rh) - 1u)) & ~(rl >= 32 ? FULL : ((1u << rl) - 1u));
             unsigned m;
             if (allint) {
-                m = !rowok ? 0u : (cnt == 32 ? FULL : ((1u << cnt) - 1u));  // idle lanes load nothing
+                m = !rowok ? 0u : rmask;  // idle lanes load nothing
             } else {
                 // lane xl tests prefixes base + xl + k*Lg for its group's row (uniform
                 // trip count), then an OR all-reduce over the group by rotations
@@ -644,11 +461,13 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     const int xs = xl + d >= Lg ? xl + d - Lg : xl + d;
                     bits |= __shfl_sync(FULL, bits, lane - xl + xs);
                 }
-                m = rowok ? bits : 0u;  // idle lanes (past 32 / Lg groups) may have read foreign bits
+                m = rowok ? bits & rmask : 0u;  // idle lanes (past 32 / Lg groups) may have read foreign bits
             }
             const int cend = PB_POW2 ? ((cnt + PB - 1) & ~(PB - 1)) : (cnt + PB - 1) / PB * PB;
+            // first batch holding a prefix of the warp's blocks (the chunk may start below them)
+            const int qlo = wlo > base ? (PB_POW2 ? ((wlo - base) & ~(PB - 1)) : (wlo - base) / PB * PB) : 0;
             // PB prefixes per step: their gathers are issued before any is consumed
-            for (int q0 = qbase0; q0 < cend; q0 += qstep) {
+            for (int q0 = qlo + qbase0; q0 < cend; q0 += qstep) {
                 Words<CH> cur[PB];
                 int sj[PB];
 #pragma unroll
@@ -719,8 +538,10 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
             }
         }
         if (!SPLIT || wid == 0) {
-            // ---- in-row term on plain uint16 lanes: opt(x) = min(1 + acc(x), 1 + opt(x - min(x, J0)))
-            // uint8: E holds x = 4w, 4w+2; O holds x = 4w+1, 4w+3.  uint16: E holds 2w, 2w+1.
+            // ---- OPT(p, x) = 1 + acc(x) for p != 0 (D12); row p = 0: ceil(x / J0)
+            // uint8: E holds x = 4w, 4w+2; O holds x = 4w+1, 4w+3 (uint16 lanes).
+            // uint16: E holds 2w, 2w+1.  Every row p != 0 dominates a unit prefix of
+            // its pivot block, so acc is finite there.
             Words<CH> oe, oo;
 #pragma unroll
             for (int t = 0; t < CH; ++t) {
@@ -732,78 +553,18 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     oo.v[t] = 0;
                 }
             }
-            if ((RUN ? rowbase == 0 : rho == 0) && xl == 0) oe.v[0] &= 0xffff0000u;  // OPT(0) = 0
-            // opt(p, 0) is final (no in-row term at x = 0): the clamp value
-            uint32_t f0 = __shfl_sync(FULL, oe.v[0], lane - xl);
-            f0 = prmt(f0, 0u, 0x1010u);
-            // Closure of opt(x) = min(v(x), 1 + opt(max(0, x - J0))) by doubling:
-            // round k relaxes opt(x) against opt(x - S) + 2^k with S = 2^k * J0,
-            // positions before the row holding opt(p, 0).  After round k every x
-            // has the minimum over paths of fewer than 2^(k+1) in-row steps; a
-            // round without change means the closure is complete (a later round
-            // can only repeat a path already covered), and S >= W ends it.
-            // u16-lane shifts: uint8, S even: E <- E >> S/2, O <- O >> S/2;
-            // S odd: E <- O >> (S+1)/2, O <- E >> (S-1)/2; uint16: E <- E >> S.
-            int S = J0;
-            uint32_t inc = 1;
-            for (;;) {
-                const bool odd = EB == 1 && (S & 1);
-                const int dbe = EB == 1 ? 2 * (odd ? (S + 1) >> 1 : S >> 1) : 2 * S;
-                const int dbo = EB == 1 ? 2 * (odd ? (S - 1) >> 1 : S >> 1) : 0;
-                const uint32_t oe_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbe & 3)) & 3u);
-                const uint32_t oo_sel = 0x3210u + 0x1111u * ((uint32_t)(4 - (dbo & 3)) & 3u);
-                Words<CH> le, he, lo2, ho2;
-                if (dbe <= 8 && dbo <= 8) {
-                    Words<CH> se, so;   // sources of the even / odd destinations (registers, no aliasing)
-#pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        se.v[t] = odd ? oo.v[t] : oe.v[t];
-                        so.v[t] = odd ? oe.v[t] : oo.v[t];
-                    }
-                    windows<CH, 8>(se, dbe, xl, f0, le, he);
-                    if (dbe == 0) le = se;
-                    if constexpr (EB == 1) {
-                        windows<CH, 8>(so, dbo, xl, f0, lo2, ho2);
-                        if (dbo == 0) lo2 = so;
-                    }
-                } else {
-                    // long shift: through this warp's slice of s_red ([2][CH * 32] words)
-                    uint32_t *sE = s_red + (size_t)wid * 2 * CH * 32 + grp * Lg * CH;
-                    uint32_t *sO = sE + CH * 32;
-                    __syncwarp();
-#pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        sE[xl * CH + t] = oe.v[t];
-                        if (EB == 1) sO[xl * CH + t] = oo.v[t];
-                    }
-                    __syncwarp();
-                    windows_smem<CH>(odd ? sO : sE, dbe, xl, f0, le, he);
-                    if constexpr (EB == 1) {
-                        if (dbo == 0) lo2 = odd ? oe : oo;
-                        else windows_smem<CH>(odd ? sE : sO, dbo, xl, f0, lo2, ho2);
-                    }
-                }
-                const uint32_t incw = inc * ONES;
-                const uint32_t capw = (0xffffu - inc) * ONES;   // saturating + inc on uint16 lanes
-                bool changed = false;
+            if (rowok && rowbase == 0) {   // row p = 0 (once per DP): OPT(0, x) = ceil(x / J0)
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
-                    const uint32_t ve = prmt(le.v[t], he.v[t], oe_sel);
-                    uint32_t ne, no = 0;
+                    const uint32_t x0 = (uint32_t)(xl * CH + t) * (4 / EB);
+                    auto cf = [&](uint32_t x) { return (x + (uint32_t)J0 - 1u) / (uint32_t)J0; };
                     if constexpr (EB == 1) {
-                        const uint32_t vo = prmt(lo2.v[t], ho2.v[t], oo_sel);
-                        ne = vmin2(oe.v[t], ve + incw);   // uint8 values stay below 0x200
-                        no = vmin2(oo.v[t], vo + incw);
+                        oe.v[t] = cf(x0) | (cf(x0 + 2) << 16);
+                        oo.v[t] = cf(x0 + 1) | (cf(x0 + 3) << 16);
                     } else {
-                        ne = vmin2(oe.v[t], vmin2(ve, capw) + incw);
+                        oe.v[t] = cf(x0) | (cf(x0 + 1) << 16);
                     }
-                    if (rowok && (ne != oe.v[t] || (EB == 1 && no != oo.v[t]))) changed = true;
-                    oe.v[t] = ne;
-                    oo.v[t] = no;
                 }
-                if (!__any_sync(FULL, changed) || (int64_t)S >= g.W) break;
-                S *= 2;
-                inc *= 2;
             }
             // ---- store the packed row (padding bytes receive don't-care values)
             if (rowok) {
@@ -910,7 +671,7 @@ static size_t swar_smem(int64_t np, int NW, int nlev_df, const RowGeom &g, int C
     // s_oj | s_w | pad | s_red | DF plan | ticket (16 B) | dominance selectors + table
     // (s_red sized for the kernel's lane chunk: smem left over is L1 for the gathers)
     return (size_t)((np + 31) & ~31) * 8 + 16 * 8 + (size_t)np * 8 * NW + 16 + (size_t)(256 / 32) * 2 * CH * 32 * 4 +
-           (size_t)8 * (nlev_df + 1) + 32 +
+           (size_t)8 * (nlev_df + 1) + 32 + (size_t)8 * MAXK + (size_t)64 * NW + 16 +
            (g.TS > 0 ? (size_t)16 * g.K1 + (size_t)((np + 31) / 32) * g.TS * 4 : 0);
 }
 

@@ -1,0 +1,371 @@
+// row_ring.cu — level fill of narrow DPs on ONE thread-block cluster with the
+// recent row-levels resident in distributed shared memory (§8(a) a-5; DESIGN.md
+// D14).
+//
+// For K = 3 classes the rows are (a, b) (two leading digits, last class in the
+// row) and row-level L = a + b holds at most min(N0, N1) + 1 rows, while the
+// dependency chain is N0 + N1 + 1 levels long (M5s: 541 levels of <= 251
+// rows).  Such a DP is bound by the latency of one level, not by bandwidth:
+// through L2 with ready flags a level costs ~3.5 us (flag acquire, gathers,
+// release fence, per-row tickets).  Here the C CTAs of one cluster (C = 16,
+// or 8 when 16 cannot be co-scheduled) fill the DP in lockstep:
+//
+//   * CTA c owns the rows with a in [c A, (c + 1) A) (A = ceil((N0 + 1) / C)
+//     <= 16, one row of a level per warp); the last R row-levels of its rows
+//     live in a ring in its shared memory (R = 1 + the largest leading-digit
+//     sum of a configuration, so every source row p - s' of level L is one of
+//     levels L - R + 1 .. L - 1).  A source row (a - s0, .) is in the same CTA
+//     unless a - s0 crosses the block boundary (~s0 / A of the reads): DSMEM is
+//     ~20 B/cycle per SM, local shared memory ~128;
+//   * a warp computes one row (a, b) of level L: for every prefix s' = (s0, s1)
+//     of the row's pivot block (D13) with s' <= (a, b) it reads the source row
+//     (a - s0, b - s1) from the owner CTA's ring through DSMEM
+//     (local shared memory or ld.shared::cluster, ~40 / ~200 cycles instead of an L2 round trip), takes the
+//     shifted window of reading D5 (shuffles + PRMT, swar_common.cuh), and
+//     OPT(a, b, x) = 1 + the minimum (D12); row (0, 0) is ceil(x / J0);
+//   * the row goes to the own ring slot (shared memory) and to the table in HBM
+//     (the table is written once and never read back by this kernel);
+//   * one cluster barrier (arrive.release / wait.acquire) per level orders the
+//     ring writes of level L before the reads of level L + 1.
+//
+// Same recurrence, same windows, same executed relaxations as the packed
+// kernel; the values are bit-identical (parity tests, PTAS_RING=0 for the A/B).
+#include <algorithm>
+#include <cstdint>
+#include <cstdlib>
+#include <cuda_runtime.h>
+
+#include "internal.h"
+#include "swar_common.cuh"
+
+namespace ptas {
+namespace swar {
+namespace {
+
+// prefixes whose DSMEM loads are issued together (CH = 8: 4, so 32 words in flight per lane)
+constexpr int RING_PB_MAX = 8;
+
+__device__ __forceinline__ uint32_t dsm_map(uint32_t local_addr, uint32_t rank)
+{
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(local_addr), "r"(rank));
+    return r;
+}
+
+template <int CH>
+__device__ __forceinline__ Words<CH> ld_dsm(uint32_t addr)
+{
+    Words<CH> w;
+    if constexpr (CH == 1) {
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(w.v[0]) : "r"(addr) : "memory");
+    } else if constexpr (CH == 2) {
+        asm volatile("ld.shared::cluster.v2.u32 {%0, %1}, [%2];" : "=r"(w.v[0]), "=r"(w.v[1]) : "r"(addr) : "memory");
+    } else {
+#pragma unroll
+        for (int c = 0; c < CH; c += 4)
+            asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];"
+                         : "=r"(w.v[c]), "=r"(w.v[c + 1]), "=r"(w.v[c + 2]), "=r"(w.v[c + 3])
+                         : "r"(addr + 4 * c)
+                         : "memory");
+    }
+    return w;
+}
+
+// CH consecutive words of the own CTA's ring (shared memory, 4*CH-byte aligned)
+template <int CH>
+__device__ __forceinline__ Words<CH> lds_words(const uint32_t *p)
+{
+    Words<CH> w;
+    if constexpr (CH == 1) {
+        w.v[0] = p[0];
+    } else if constexpr (CH == 2) {
+        const uint2 a = *reinterpret_cast<const uint2 *>(p);
+        w.v[0] = a.x;
+        w.v[1] = a.y;
+    } else {
+#pragma unroll
+        for (int c = 0; c < CH; c += 4) {
+            const uint4 a = *reinterpret_cast<const uint4 *>(p + c);
+            w.v[c] = a.x;
+            w.v[c + 1] = a.y;
+            w.v[c + 2] = a.z;
+            w.v[c + 3] = a.w;
+        }
+    }
+    return w;
+}
+
+__device__ __forceinline__ void cluster_sync_all()
+{
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <typename E, int CH, int WIN>
+__global__ void __launch_bounds__(1024, 1)
+row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta)
+{
+    constexpr int EB = (int)sizeof(E);
+    constexpr uint32_t ONES = 0x00010001u;
+    constexpr int PB = 4;   // prefixes whose loads are issued together
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    if (meta->ovf) return;   // grid-uniform: every CTA exits before any barrier
+    uint32_t crank, csize;
+    asm("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+    asm("mov.u32 %0, %%cluster_nctarank;" : "=r"(csize));
+    const int np = (int)(meta->nP - 1);
+    const int Lw = ra.Lw, Lg = ra.Lg;
+    const uint32_t row_bytes = (uint32_t)Lw * 4;
+    // smem: ring [R][A][Lw] words | prefix table int4 [np + PB] | cluster addresses of the rings [16]
+    uint32_t *ring = reinterpret_cast<uint32_t *>(smem_raw);
+    int4 *s_pf = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * ra.A * row_bytes + 15) & ~(size_t)15));
+    uint32_t *s_base = reinterpret_cast<uint32_t *>(s_pf + np + RING_PB_MAX);
+    __shared__ int s_nb1;
+    if (threadIdx.x == 0) s_nb1 = 0;
+    __syncthreads();
+    // prefixes (lexicographic, s0 major): s0, s1 from off(s') = s0 * stride0 + s1 * Wp,
+    // window selector | byte shift (oj_entry), |s'|; pivot block B1 = {s0 = 0} first, then B0
+    int nb1 = 0;
+    for (int i = threadIdx.x; i < np + RING_PB_MAX; i += blockDim.x) {
+        int4 v = make_int4(1 << 20, 1 << 20, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF, 0);
+        if (i < np) {
+            const PrefixEntry pe = gpref[1 + i];
+            const int s0 = (int)(pe.off / ra.stride0);
+            const int s1 = (int)((pe.off - (int64_t)s0 * ra.stride0) / ra.Wp);
+            v = make_int4(s0, s1, oj_entry(pe, EB).y, s0 + s1);
+            nb1 += s0 == 0;
+        }
+        s_pf[i] = v;
+    }
+    atomicAdd(&s_nb1, nb1);
+    if (threadIdx.x < csize) s_base[threadIdx.x] = dsm_map((uint32_t)__cvta_generic_to_shared(ring), threadIdx.x);
+    __syncthreads();
+    nb1 = s_nb1;
+    cluster_sync_all();   // every CTA of the cluster runs before any DSMEM access
+
+    const int a0 = (int)crank * ra.A;          // first row digit a of this CTA
+    uint32_t *tab32 = reinterpret_cast<uint32_t *>(table);
+    int slot = 0;                              // L mod R
+    for (int L = 0; L <= ra.rho_max; ++L) {
+        // this CTA's rows of level L: a in [lo, hi] (contiguous), b = L - a
+        const int lo = max(max(L - ra.N1, 0), a0);
+        const int hi = min(min(L, ra.N0), a0 + ra.A - 1);
+        const int ntask = hi >= lo ? (hi - lo + 1) * Lg : 0;
+        for (int task = threadIdx.x; task < ntask; task += blockDim.x) {
+            const int a = lo + task / Lg;       // (Lg is small: one IMAD.HI)
+            const int c = task - (a - lo) * Lg; // lane chunk: words c*CH .. c*CH+CH-1 of the row
+            const int b = L - a;
+            const int ia = a - a0;
+            // pivot block (D13): a >= 1 -> prefixes with s0 >= 1, else s0 = 0 (and s1 >= 1)
+            const int plo = a >= 1 ? nb1 : 0, phi = a >= 1 ? np : nb1;
+            Words<CH> ae, ao;
+            fill_words(ae, 0xffffffffu);
+            fill_words(ao, 0xffffffffu);
+            for (int q0 = plo; q0 < phi; q0 += PB) {
+                Words<CH> cur[PB];
+                uint32_t l1[PB], l2[PB];
+                int sj[PB];
+#pragma unroll
+                for (int u = 0; u < PB; ++u) {
+                    const int q = q0 + u;
+                    const int4 pf = s_pf[q];   // padded past np: never dominated
+                    sj[u] = pf.z;
+                    if (q < phi && pf.x <= a && pf.y <= b) {
+                        int ss = slot - pf.w;
+                        ss += ss < 0 ? ra.R : 0;
+                        int li = ia - pf.x, ow = (int)crank;   // owner CTA and its local row
+                        while (li < 0) {
+                            li += ra.A;
+                            --ow;
+                        }
+                        const uint32_t row = s_base[ow] + ((uint32_t)ss * (uint32_t)ra.A + (uint32_t)li) * row_bytes;
+                        cur[u] = ld_dsm<CH>(row + (uint32_t)c * (CH * 4));
+                        // the two words left of the chunk (positions before the row: its
+                        // first entry, the clamp x - min(x, J))
+                        if (WIN == 8 && c >= 1 && CH >= 2) {
+                            const Words<2> w2 = ld_dsm<2>(row + (uint32_t)c * (CH * 4) - 8);
+                            l2[u] = w2.v[0];
+                            l1[u] = w2.v[1];
+                        } else {
+                            l1[u] = c >= 1 ? ld_dsm<1>(row + (uint32_t)c * (CH * 4) - 4).v[0] : 0u;
+                            l2[u] = (WIN == 8 && c * CH >= 2) ? ld_dsm<1>(row + (uint32_t)c * (CH * 4) - 8).v[0] : 0u;
+                        }
+                    } else {
+                        fill_words(cur[u], 0xffffffffu);
+                        l1[u] = l2[u] = 0xffffffffu;
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < PB; ++u) {
+                    const uint32_t sel = (uint32_t)sj[u];
+                    const int db = (int)(sel >> 16);
+                    // positions before the row: its first entry replicated (word 0 of the
+                    // row is the chunk's own word for c = 0, the left word for c = 1, CH = 1)
+                    uint32_t f = c == 0 ? cur[u].v[0] : l1[u];
+                    f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
+                    const uint32_t w1 = c >= 1 ? l1[u] : f;              // word w0 - 1
+                    const uint32_t w2 = c * CH >= 2 ? l2[u] : f;         // word w0 - 2
+#pragma unroll
+                    for (int t = 0; t < CH; ++t) {
+                        uint32_t lo_, hi_;
+                        if (WIN == 4 || db <= 4) {
+                            lo_ = t == 0 ? w1 : cur[u].v[t - 1];
+                            hi_ = cur[u].v[t];
+                        } else {   // 4 < db <= 8: words w - 2, w - 1
+                            lo_ = t >= 2 ? cur[u].v[t - 2] : (t == 1 ? w1 : w2);
+                            hi_ = t >= 1 ? cur[u].v[t - 1] : w1;
+                        }
+                        if constexpr (EB == 1) {
+                            ae.v[t] = vmin2(ae.v[t], prmt(lo_, hi_, sel));
+                            ao.v[t] = vmin2(ao.v[t], prmt(lo_, hi_, sel + 0x1111u));
+                        } else {
+                            ae.v[t] = vmin2(ae.v[t], prmt(lo_, hi_, sel));
+                        }
+                    }
+                }
+            }
+            Words<CH> wv;
+#pragma unroll
+            for (int t = 0; t < CH; ++t) {
+                uint32_t oe, oo = 0;
+                if constexpr (EB == 1) {
+                    oe = (ae.v[t] & 0x00ff00ffu) + ONES;
+                    oo = (ao.v[t] & 0x00ff00ffu) + ONES;
+                } else {
+                    oe = vmin2(ae.v[t], 0xfffefffeu) + ONES;
+                }
+                if (L == 0) {   // row (0, 0): OPT(0, x) = ceil(x / J0)
+                    const uint32_t x0 = (uint32_t)(c * CH + t) * (4 / EB);
+                    auto cf = [&](uint32_t x) { return (x + (uint32_t)ra.J0 - 1u) / (uint32_t)ra.J0; };
+                    if constexpr (EB == 1) {
+                        oe = cf(x0) | (cf(x0 + 2) << 16);
+                        oo = cf(x0 + 1) | (cf(x0 + 3) << 16);
+                    } else {
+                        oe = cf(x0) | (cf(x0 + 1) << 16);
+                    }
+                }
+                wv.v[t] = EB == 1 ? prmt(oe, oo, 0x6240u) : oe;
+            }
+            store_words<CH>(ring + ((size_t)slot * ra.A + ia) * Lw + c * CH, wv);
+            const int64_t rowbase = (int64_t)a * ra.stride0 + (int64_t)b * ra.Wp;   // elements
+            store_words<CH>(tab32 + rowbase * EB / 4 + c * CH, wv);
+        }
+        cluster_sync_all();   // level L complete in every CTA's ring
+        slot = slot + 1 == ra.R ? 0 : slot + 1;
+    }
+}
+
+template <typename E, int CH, int WIN>
+cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                          int64_t nP_bound, int csize, cudaStream_t st, bool dry)
+{
+    auto kfn = row_ring_kernel<E, CH, WIN>;
+    const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
+    const size_t smem = (((size_t)ra.R * ra.A * ra.Lw * 4 + 15) & ~(size_t)15) + (size_t)(np + RING_PB_MAX) * 16 + 16 * 4;
+    cudaError_t err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (err != cudaSuccess) return err;
+    if (csize > 8) {
+        err = cudaFuncSetAttribute(kfn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (err != cudaSuccess) return err;
+    }
+    const int lanes = ra.A * ra.Lg;
+    const int warps = std::min(32, (lanes + 31) / 32);
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)csize;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.gridDim = dim3((unsigned)csize);
+    cfg.blockDim = dim3((unsigned)(32 * warps));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int ncl = 0;
+    err = cudaOccupancyMaxActiveClusters(&ncl, kfn, &cfg);
+    if (err != cudaSuccess || ncl < 1) {
+        cudaGetLastError();
+        return cudaErrorNotSupported;
+    }
+    if (dry) return cudaSuccess;
+    return cudaLaunchKernelEx(&cfg, kfn, (E *)table, ra, d_pref, d_meta);
+}
+
+template <typename E, int CH>
+cudaError_t launch_ring_ch(void *table, const RingArgs &ra, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                           int64_t nP_bound, int csize, int win, cudaStream_t st, bool dry)
+{
+    if (win == 4) return launch_ring_t<E, CH, 4>(table, ra, d_pref, d_meta, nP_bound, csize, st, dry);
+    return launch_ring_t<E, CH, 8>(table, ra, d_pref, d_meta, nP_bound, csize, st, dry);
+}
+
+template <typename E>
+cudaError_t launch_ring_e(void *table, const RingArgs &ra, int CH, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                          int64_t nP_bound, int csize, int win, cudaStream_t st, bool dry)
+{
+    switch (CH) {
+    case 1: return launch_ring_ch<E, 1>(table, ra, d_pref, d_meta, nP_bound, csize, win, st, dry);
+    case 2: return launch_ring_ch<E, 2>(table, ra, d_pref, d_meta, nP_bound, csize, win, st, dry);
+    case 4: return launch_ring_ch<E, 4>(table, ra, d_pref, d_meta, nP_bound, csize, win, st, dry);
+    default: return launch_ring_ch<E, 8>(table, ra, d_pref, d_meta, nP_bound, csize, win, st, dry);
+    }
+}
+
+}  // namespace
+}  // namespace swar
+
+// Host planning (D14): K = 3 only (two leading digits), a row of at
+// most 256 words (one warp), window shifts J0 * e <= 124 bytes, and the ring of
+// R levels x A rows per CTA within the shared memory of one CTA.  Returns
+// cudaErrorNotSupported when the DP does not qualify (the caller then uses the
+// dataflow / per-level launches).  dry: only check (no launch).
+cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int32_t *N, const int64_t *r,
+                                 int64_t T, int J0, const PrefixEntry *d_pref, const DpMeta *d_meta,
+                                 int64_t nP_bound, cudaStream_t st, bool dry)
+{
+    if (g.K1 != 2 || (g.Wp * e) % 4 != 0) return cudaErrorNotSupported;
+    const int Lw = (int)(g.Wp * e / 4);
+    // windows up to two words left (J0 * e <= 8 bytes: the M5s shapes have 6)
+    if (J0 * e > 8 || nP_bound > 4096) return cudaErrorNotSupported;
+    const char *en = std::getenv("PTAS_RING");
+    if (en && en[0] == '0') return cudaErrorNotSupported;
+    RingArgs ra;
+    ra.N0 = N[0];
+    ra.N1 = N[1];
+    ra.Wp = (int32_t)g.Wp;
+    ra.stride0 = g.stride[0];
+    ra.Lw = Lw;
+    ra.J0 = J0;
+    // ring depth: 1 + the largest leading-digit sum of a configuration, bounded by
+    // min(hi0 + hi1, floor(T / min(r0, r1)))
+    const int64_t hi0 = std::min<int64_t>(N[0], T / r[0]), hi1 = std::min<int64_t>(N[1], T / r[1]);
+    ra.R = (int)std::min<int64_t>(hi0 + hi1, T / std::min(r[0], r[1])) + 1;
+    ra.rho_max = N[0] + N[1];
+    const int win = J0 * e <= 4 ? 4 : 8;
+    const size_t smem_cap = 220 * 1024;
+    const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
+    const char *cs_env = std::getenv("PTAS_RING_CS");   // experiment: force the cluster size
+    const int cs_force = cs_env && cs_env[0] ? std::atoi(cs_env) : 0;
+    for (int csize : {16, 8, 4, 2}) {
+        if (cs_force ? csize != cs_force : csize < 8) continue;
+        ra.A = (N[0] + csize) / csize;   // ceil((N0 + 1) / C) rows of each level per CTA
+        const size_t smem = (((size_t)ra.R * ra.A * Lw * 4 + 15) & ~(size_t)15) + (size_t)(np + 8) * 16 + 64;
+        if (smem > smem_cap) continue;
+        // words per lane: the smallest chunk with one pass over the CTA's rows of a level
+        int CH = 8;
+        for (int c : {1, 2, 4})
+            if (Lw % c == 0 && (int64_t)ra.A * (Lw / c) <= 1024) {
+                CH = c;
+                break;
+            }
+        if (Lw % CH != 0) continue;
+        ra.Lg = Lw / CH;
+        cudaError_t err = e == 1 ? swar::launch_ring_e<uint8_t>(table, ra, CH, d_pref, d_meta, nP_bound, csize, win, st, dry)
+                                 : swar::launch_ring_e<uint16_t>(table, ra, CH, d_pref, d_meta, nP_bound, csize, win, st, dry);
+        if (err == cudaSuccess) return err;
+        cudaGetLastError();
+    }
+    return cudaErrorNotSupported;
+}
+
+}  // namespace ptas

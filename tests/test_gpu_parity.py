@@ -85,18 +85,24 @@ def test_row_index_complete(P):
 
 # ------------------------------------------------------------------ a-5
 def _collapsed_relax(N, r, T):
-    """Closed form of the (n, s') pairs the packed kernel evaluates (DESIGN.md
-    D5): one window per (row dominating s' != 0, x), plus the in-row term for
-    every state with x >= 1.  Internal order = the non-empty classes."""
+    """Closed form of the (n, s') window gathers the packed kernel evaluates
+    (D5, D12, D13): one window per (row p, x) for every prefix s' != 0
+    with s' <= p whose first nonzero digit q is also the first nonzero digit of
+    p, i.e. prod_{i >= q} (N_i - s'_i + 1) rows; no in-row term; row 0 is a
+    closed form.  Internal order = the non-empty classes."""
     nz = np.asarray(N) > 0
     Nn, rn = np.asarray(N)[nz].astype(np.int64), np.asarray(r)[nz]
     if len(Nn) == 0:
         return 0.0
     W = float(Nn[-1] + 1)
-    rows = float(np.prod((Nn[:-1] + 1).astype(np.float64)))
     C = oracle.configs(Nn.astype(np.int32), rn, T)
     pre = {tuple(int(x) for x in c[:-1]) for c in C} - {tuple([0] * (len(Nn) - 1))}
-    return sum(float(np.prod((Nn[:-1] - np.array(s) + 1).astype(np.float64))) * W for s in pre) + rows * (W - 1)
+    tot = 0.0
+    for s in pre:
+        s = np.array(s, np.int64)
+        q = int(np.argmax(s > 0))
+        tot += float(np.prod((Nn[q:-1] - s[q:] + 1).astype(np.float64))) * W
+    return tot
 
 
 def _check_table(P, N, r, T):
@@ -634,12 +640,10 @@ def test_virtual_shards_use_packed_kernel(P, vs):
     assert got["stats"]["relax_executed"] == ref["stats"]["relax_executed"] < got["stats"]["relaxations"]
 
 
-@pytest.mark.parametrize("local", ["0", "1"])
-def test_long_row_chain_variants(P, monkeypatch, local):
-    # long-row path with the in-chunk chain in the cross kernel (1, default) or
-    # entirely in the chain kernel (0), forced on every level; J0 from 1 to > 32
+def test_long_row_path(P, monkeypatch):
+    # long-row path (one warp per 4 chunks of 32 entries, pivot blocks, row 0 in
+    # closed form) forced on every level; J0 from 1 to > 32
     monkeypatch.setenv("PTAS_FORCE_SCALAR", "2")
-    monkeypatch.setenv("PTAS_LONG_LOCAL", local)
     _check_table(P, np.array([4, 3, 1200], np.int32), np.array([300, 170, 3], np.int64), 310)
     _check_table(P, np.array([6, 1500], np.int32), np.array([100, 99], np.int64), 250)
     _check_table(P, np.array([3, 3, 200], np.int32), np.array([50, 45, 1], np.int64), 60)
