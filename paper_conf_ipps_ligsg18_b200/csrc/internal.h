@@ -195,6 +195,8 @@ cudaError_t launch_row_fill_swar_df(int e, void *table, const RowGeom &g, const 
 cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int32_t *N, const int64_t *r,
                                  int64_t T, int J0, const PrefixEntry *d_pref, const DpMeta *d_meta,
                                  int64_t nP_bound, cudaStream_t st, bool dry);
+// Host-only geometry test of launch_row_fill_ring (internal class order).
+bool ring_fits(const int32_t *N, const int64_t *r, int K, int64_t T);
 // Rows per row set the dataflow kernel will use for this geometry (0 = unsupported).
 int swar_df_rows_per_set(int e, const RowGeom &g, int J0, int64_t max_level_rows, int sm_count);
 // Copies the DP's prefix offsets/Jmax into the fill kernel's constant bank

@@ -413,6 +413,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     std::map<std::vector<int64_t>, SpecRes> spec;
     int spec_depth = opt.speculate < 0 ? 3 : opt.speculate;
     int64_t spec_sigma = (int64_t)1 << 24;
+    const char *sr = std::getenv("PTAS_SPEC_RING");   // 0: ring DPs only below spec_sigma (A/B)
+    const bool spec_ring = !(sr && sr[0] == '0');
     {
         const char *sd = std::getenv("PTAS_SPEC_DEPTH");
         if (sd && sd[0] && opt.speculate < 0) spec_depth = std::atoi(sd);
@@ -441,6 +443,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         std::vector<Classified> cls_v;
         std::vector<int64_t> T_v;
         std::vector<std::vector<int64_t>> key_v;
+        int depth_lim = spec_depth;
         for (size_t h = 0; h < q.size(); ++h) {
             const Node nd = q[h];
             if (nd.lb >= nd.ub) continue;
@@ -449,7 +452,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             const int64_t T = t1[0];
             Classified c;
             classify(p, n, T, k, &c);
-            bool take = false;
+            bool take = false, lat = false;
             std::vector<int64_t> key;
             if (!c.N.empty()) {
                 key = memo_key(c, T);
@@ -460,16 +463,30 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 }
                 const bool known = memo.count(key) || spec.count(key) ||
                                    std::find(key_v.begin(), key_v.end(), key) != key_v.end();
+                // latency-bound DPs (the K = 3 cluster ring kernel fills them on 16 SMs,
+                // DESIGN.md D14) overlap whatever their size
+                if (spec_ring) {
+                    const std::vector<int> o = choose_order(c.N, c.r, opt.layout);
+                    std::vector<int32_t> No;
+                    std::vector<int64_t> ro;
+                    for (int i : o) {
+                        No.push_back(c.N[i]);
+                        ro.push_back(c.r[i]);
+                    }
+                    lat = ring_fits(No.data(), ro.data(), (int)No.size(), T);
+                }
                 // a large next probe runs alone (throughput-bound: nothing to overlap)
-                if (nd.d == 0 && sg > (__int128)spec_sigma) return PTAS_OK;
-                take = !known && sg <= (__int128)spec_sigma;
+                if (nd.d == 0 && sg > (__int128)spec_sigma && !lat) return PTAS_OK;
+                take = !known && (sg <= (__int128)spec_sigma || lat);
             }
             if (take) {
                 cls_v.push_back(c);
                 T_v.push_back(T);
                 key_v.push_back(key);
             }
-            if (nd.d + 1 < spec_depth && (int)cls_v.size() < MAX_SLOTS) {
+            // a chain of latency-bound ring DPs runs up to MAX_SLOTS deep (16 SMs each)
+            if (lat && spec_chain) depth_lim = MAX_SLOTS;
+            if (nd.d + 1 < depth_lim && (int)cls_v.size() < MAX_SLOTS) {
                 q.push_back({nd.lb, T, nd.d + 1});        // T feasible
                 if (!spec_chain) q.push_back({T + 1, nd.ub, nd.d + 1});    // T infeasible
             }

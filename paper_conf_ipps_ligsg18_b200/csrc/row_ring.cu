@@ -32,6 +32,7 @@
 // kernel; the values are bit-identical (parity tests, PTAS_RING=0 for the A/B).
 #include <algorithm>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <cuda_runtime.h>
 
@@ -44,6 +45,12 @@ namespace {
 
 // prefixes whose DSMEM loads are issued together (CH = 8: 4, so 32 words in flight per lane)
 constexpr int RING_PB_MAX = 8;
+#ifndef PTAS_RING_PROFILE
+#define PTAS_RING_PROFILE 0
+#endif
+// diagnostics build (-DPTAS_RING_PROFILE=1): per level, clock64 of CTA `prof_cta`
+// thread 0 at level start, after its rows, after arrive, after wait
+__device__ long long g_ring_prof[4][2048];
 
 __device__ __forceinline__ uint32_t dsm_map(uint32_t local_addr, uint32_t rank)
 {
@@ -100,6 +107,26 @@ __device__ __forceinline__ void cluster_sync_all()
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// Windows of one prefix for the lane's CH words: class 1 = shift of at most one
+// word (db <= 4 bytes: words w - 1, w), class 2 = at most two (4 < db <= 8:
+// words w - 2, w - 1); w1 / w2 = the words left of the chunk.
+template <typename E, int CH, int CLS>
+__device__ __forceinline__ void ring_windows(const Words<CH> &cur, uint32_t w1, uint32_t w2, uint32_t sel,
+                                             Words<CH> &ae, Words<CH> &ao)
+{
+#pragma unroll
+    for (int t = 0; t < CH; ++t) {
+        const uint32_t lo = CLS == 1 ? (t == 0 ? w1 : cur.v[t - 1]) : (t >= 2 ? cur.v[t - 2] : (t == 1 ? w1 : w2));
+        const uint32_t hi = CLS == 1 ? cur.v[t] : (t >= 1 ? cur.v[t - 1] : w1);
+        if constexpr (sizeof(E) == 1) {
+            ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, sel));
+            ao.v[t] = vmin2(ao.v[t], prmt(lo, hi, sel + 0x1111u));
+        } else {
+            ae.v[t] = vmin2(ae.v[t], prmt(lo, hi, sel));
+        }
+    }
+}
+
 template <typename E, int CH, int WIN>
 __global__ void __launch_bounds__(1024, 1)
 row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta)
@@ -109,117 +136,108 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
     constexpr int PB = 4;   // prefixes whose loads are issued together
     extern __shared__ __align__(16) unsigned char smem_raw[];
     if (meta->ovf) return;   // grid-uniform: every CTA exits before any barrier
-    uint32_t crank, csize;
+    uint32_t crank;
     asm("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
-    asm("mov.u32 %0, %%cluster_nctarank;" : "=r"(csize));
     const int np = (int)(meta->nP - 1);
     const int Lw = ra.Lw, Lg = ra.Lg;
     const uint32_t row_bytes = (uint32_t)Lw * 4;
-    // smem: ring [R][A][Lw] words | prefix table int4 [np + PB] | cluster addresses of the rings [16]
+    // smem: ring [R][A][Lw] words | 4 prefix lists int4 [np + PB] each
     uint32_t *ring = reinterpret_cast<uint32_t *>(smem_raw);
-    int4 *s_pf = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * ra.A * row_bytes + 15) & ~(size_t)15));
-    uint32_t *s_base = reinterpret_cast<uint32_t *>(s_pf + np + RING_PB_MAX);
-    __shared__ int s_nb1;
-    if (threadIdx.x == 0) s_nb1 = 0;
+    int4 *s_pl = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * ra.A * row_bytes + 15) & ~(size_t)15));
+    const int lcap = np + PB;
+    __shared__ int s_cnt[4];
+    if (threadIdx.x < 4) s_cnt[threadIdx.x] = 0;
     __syncthreads();
-    // prefixes (lexicographic, s0 major): s0, s1 from off(s') = s0 * stride0 + s1 * Wp,
-    // window selector | byte shift (oj_entry), |s'|; pivot block B1 = {s0 = 0} first, then B0
-    int nb1 = 0;
-    for (int i = threadIdx.x; i < np + RING_PB_MAX; i += blockDim.x) {
-        int4 v = make_int4(1 << 20, 1 << 20, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF, 0);
-        if (i < np) {
-            const PrefixEntry pe = gpref[1 + i];
-            const int s0 = (int)(pe.off / ra.stride0);
-            const int s1 = (int)((pe.off - (int64_t)s0 * ra.stride0) / ra.Wp);
-            v = make_int4(s0, s1, oj_entry(pe, EB).y, s0 + s1);
-            nb1 += s0 == 0;
-        }
-        s_pf[i] = v;
+    // prefix lists by (pivot block, window class): list 2*blk + cls - 1, blk 0 = {s0 = 0}
+    // (rows a = 0), blk 1 = {s0 >= 1} (rows a >= 1); entries (s0, s1, selector | db << 16,
+    // |s'|).  The order inside a list does not matter (min is commutative).
+    for (int i = threadIdx.x; i < np; i += blockDim.x) {
+        const PrefixEntry pe = gpref[1 + i];
+        const int s0 = (int)(pe.off / ra.stride0);
+        const int s1 = (int)((pe.off - (int64_t)s0 * ra.stride0) / ra.Wp);
+        const int sel = oj_entry(pe, EB).y;
+        const int li = 2 * (s0 >= 1) + ((sel >> 16) > 4 ? 1 : 0);
+        s_pl[li * lcap + atomicAdd(&s_cnt[li], 1)] = make_int4(s0, s1, sel, s0 + s1);
     }
-    atomicAdd(&s_nb1, nb1);
-    if (threadIdx.x < csize) s_base[threadIdx.x] = dsm_map((uint32_t)__cvta_generic_to_shared(ring), threadIdx.x);
     __syncthreads();
-    nb1 = s_nb1;
+    for (int i = threadIdx.x; i < 4 * PB; i += blockDim.x)   // padding: never dominated
+        s_pl[(i / PB) * lcap + s_cnt[i / PB] + i % PB] =
+            make_int4(1 << 20, 1 << 20, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF, 0);
+    const uint32_t rem = dsm_map((uint32_t)__cvta_generic_to_shared(ring), crank > 0 ? crank - 1 : 0);
+    __syncthreads();
     cluster_sync_all();   // every CTA of the cluster runs before any DSMEM access
 
     const int a0 = (int)crank * ra.A;          // first row digit a of this CTA
     uint32_t *tab32 = reinterpret_cast<uint32_t *>(table);
     int slot = 0;                              // L mod R
+    Words<CH> last;
+    int64_t last_off = -1;                     // word offset of the thread's last row chunk of the level
     for (int L = 0; L <= ra.rho_max; ++L) {
+#if PTAS_RING_PROFILE
+        const bool pr = threadIdx.x == 0 && crank == 8 && L < 2048;
+        if (pr) g_ring_prof[0][L] = clock64();
+#endif
         // this CTA's rows of level L: a in [lo, hi] (contiguous), b = L - a
         const int lo = max(max(L - ra.N1, 0), a0);
         const int hi = min(min(L, ra.N0), a0 + ra.A - 1);
         const int ntask = hi >= lo ? (hi - lo + 1) * Lg : 0;
         for (int task = threadIdx.x; task < ntask; task += blockDim.x) {
-            const int a = lo + task / Lg;       // (Lg is small: one IMAD.HI)
-            const int c = task - (a - lo) * Lg; // lane chunk: words c*CH .. c*CH+CH-1 of the row
+            const int r_ = task / Lg;
+            const int a = lo + r_;
+            const int c = task - r_ * Lg;       // lane chunk: words c*CH .. c*CH+CH-1 of the row
             const int b = L - a;
             const int ia = a - a0;
-            // pivot block (D13): a >= 1 -> prefixes with s0 >= 1, else s0 = 0 (and s1 >= 1)
-            const int plo = a >= 1 ? nb1 : 0, phi = a >= 1 ? np : nb1;
+            const int pos0 = ia * Lw + c * CH;  // the lane's words within a ring slot
             Words<CH> ae, ao;
             fill_words(ae, 0xffffffffu);
             fill_words(ao, 0xffffffffu);
-            for (int q0 = plo; q0 < phi; q0 += PB) {
-                Words<CH> cur[PB];
-                uint32_t l1[PB], l2[PB];
-                int sj[PB];
+            const int blk = a >= 1 ? 1 : 0;    // pivot block (D13)
 #pragma unroll
-                for (int u = 0; u < PB; ++u) {
-                    const int q = q0 + u;
-                    const int4 pf = s_pf[q];   // padded past np: never dominated
-                    sj[u] = pf.z;
-                    if (q < phi && pf.x <= a && pf.y <= b) {
+            for (int cls = 1; cls <= (WIN == 8 ? 2 : 1); ++cls) {
+                const int4 *pl = s_pl + (2 * blk + cls - 1) * lcap;
+                const int n = s_cnt[2 * blk + cls - 1];
+                for (int q0 = 0; q0 < n; q0 += PB) {
+                    Words<CH> cur[PB];
+                    uint32_t l1[PB], l2[PB];
+                    int sj[PB];
+#pragma unroll
+                    for (int u = 0; u < PB; ++u) {
+                        const int4 pf = pl[q0 + u];
+                        sj[u] = pf.z;
+                        // source row (a - s0, b - s1) of level L - |s'|: in this CTA's ring, or
+                        // (first s0 rows of the block) the previous CTA's: A >= every s0
                         int ss = slot - pf.w;
                         ss += ss < 0 ? ra.R : 0;
-                        int li = ia - pf.x, ow = (int)crank;   // owner CTA and its local row
-                        while (li < 0) {
-                            li += ra.A;
-                            --ow;
-                        }
-                        const uint32_t row = s_base[ow] + ((uint32_t)ss * (uint32_t)ra.A + (uint32_t)li) * row_bytes;
-                        cur[u] = ld_dsm<CH>(row + (uint32_t)c * (CH * 4));
-                        // the two words left of the chunk (positions before the row: its
-                        // first entry, the clamp x - min(x, J))
-                        if (WIN == 8 && c >= 1 && CH >= 2) {
-                            const Words<2> w2 = ld_dsm<2>(row + (uint32_t)c * (CH * 4) - 8);
-                            l2[u] = w2.v[0];
-                            l1[u] = w2.v[1];
+                        const int pos = pos0 + (ss * ra.A - pf.x) * Lw;   // word index in the ring
+                        if (pf.x <= a && pf.y <= b) {
+                            // own rows through plain shared-memory loads (~128 B/cycle); the few
+                            // rows of the previous CTA through DSMEM (~20 B/cycle per SM)
+                            if (ia >= pf.x) {
+                                const uint32_t *p = ring + pos;
+                                cur[u] = lds_words<CH>(p);
+                                l1[u] = c >= 1 ? p[-1] : 0u;
+                                l2[u] = (cls == 2 && c * CH >= 2) ? p[-2] : 0u;
+                            } else {
+                                const uint32_t src = rem + 4u * (uint32_t)(pos + ra.A * Lw);
+                                cur[u] = ld_dsm<CH>(src);
+                                l1[u] = c >= 1 ? ld_dsm<1>(src - 4).v[0] : 0u;
+                                l2[u] = (cls == 2 && c * CH >= 2) ? ld_dsm<1>(src - 8).v[0] : 0u;
+                            }
                         } else {
-                            l1[u] = c >= 1 ? ld_dsm<1>(row + (uint32_t)c * (CH * 4) - 4).v[0] : 0u;
-                            l2[u] = (WIN == 8 && c * CH >= 2) ? ld_dsm<1>(row + (uint32_t)c * (CH * 4) - 8).v[0] : 0u;
+                            fill_words(cur[u], 0xffffffffu);
+                            l1[u] = l2[u] = 0xffffffffu;
                         }
-                    } else {
-                        fill_words(cur[u], 0xffffffffu);
-                        l1[u] = l2[u] = 0xffffffffu;
                     }
-                }
 #pragma unroll
-                for (int u = 0; u < PB; ++u) {
-                    const uint32_t sel = (uint32_t)sj[u];
-                    const int db = (int)(sel >> 16);
-                    // positions before the row: its first entry replicated (word 0 of the
-                    // row is the chunk's own word for c = 0, the left word for c = 1, CH = 1)
-                    uint32_t f = c == 0 ? cur[u].v[0] : l1[u];
-                    f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
-                    const uint32_t w1 = c >= 1 ? l1[u] : f;              // word w0 - 1
-                    const uint32_t w2 = c * CH >= 2 ? l2[u] : f;         // word w0 - 2
-#pragma unroll
-                    for (int t = 0; t < CH; ++t) {
-                        uint32_t lo_, hi_;
-                        if (WIN == 4 || db <= 4) {
-                            lo_ = t == 0 ? w1 : cur[u].v[t - 1];
-                            hi_ = cur[u].v[t];
-                        } else {   // 4 < db <= 8: words w - 2, w - 1
-                            lo_ = t >= 2 ? cur[u].v[t - 2] : (t == 1 ? w1 : w2);
-                            hi_ = t >= 1 ? cur[u].v[t - 1] : w1;
-                        }
-                        if constexpr (EB == 1) {
-                            ae.v[t] = vmin2(ae.v[t], prmt(lo_, hi_, sel));
-                            ao.v[t] = vmin2(ao.v[t], prmt(lo_, hi_, sel + 0x1111u));
-                        } else {
-                            ae.v[t] = vmin2(ae.v[t], prmt(lo_, hi_, sel));
-                        }
+                    for (int u = 0; u < PB; ++u) {
+                        // positions before the row: its first entry replicated (row word 0 is
+                        // the chunk's own word for c = 0, the left word for c = 1 with CH = 1)
+                        uint32_t f = c == 0 ? cur[u].v[0] : l1[u];
+                        f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
+                        const uint32_t w1 = c >= 1 ? l1[u] : f;
+                        const uint32_t w2 = c * CH >= 2 ? l2[u] : f;
+                        if (cls == 1) ring_windows<E, CH, 1>(cur[u], w1, w2, (uint32_t)sj[u], ae, ao);
+                        else ring_windows<E, CH, 2>(cur[u], w1, w2, (uint32_t)sj[u], ae, ao);
                     }
                 }
             }
@@ -246,10 +264,31 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
                 wv.v[t] = EB == 1 ? prmt(oe, oo, 0x6240u) : oe;
             }
             store_words<CH>(ring + ((size_t)slot * ra.A + ia) * Lw + c * CH, wv);
-            const int64_t rowbase = (int64_t)a * ra.stride0 + (int64_t)b * ra.Wp;   // elements
-            store_words<CH>(tab32 + rowbase * EB / 4 + c * CH, wv);
+            if (task + (int)blockDim.x < ntask) {   // (not the thread's last row of the level)
+                const int64_t rowbase = (int64_t)a * ra.stride0 + (int64_t)b * ra.Wp;   // elements
+                store_words<CH>(tab32 + rowbase * EB / 4 + c * CH, wv);
+            } else {
+                last = wv;
+                last_off = ((int64_t)a * ra.stride0 + (int64_t)b * ra.Wp) * EB / 4 + c * CH;
+            }
         }
-        cluster_sync_all();   // level L complete in every CTA's ring
+        // level L complete in every CTA's ring: the release covers the ring stores; the
+        // thread's last row goes to HBM between arrive and wait, off the critical path
+#if PTAS_RING_PROFILE
+        if (pr) g_ring_prof[1][L] = clock64();
+#endif
+        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+#if PTAS_RING_PROFILE
+        if (pr) g_ring_prof[2][L] = clock64();
+#endif
+#ifndef PTAS_RING_NOSTORE
+        if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
+#endif
+        last_off = -1;
+        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+#if PTAS_RING_PROFILE
+        if (pr) g_ring_prof[3][L] = clock64();
+#endif
         slot = slot + 1 == ra.R ? 0 : slot + 1;
     }
 }
@@ -260,7 +299,7 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
 {
     auto kfn = row_ring_kernel<E, CH, WIN>;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (((size_t)ra.R * ra.A * ra.Lw * 4 + 15) & ~(size_t)15) + (size_t)(np + RING_PB_MAX) * 16 + 16 * 4;
+    const size_t smem = (((size_t)ra.R * ra.A * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
     cudaError_t err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     if (csize > 8) {
@@ -288,7 +327,26 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
         return cudaErrorNotSupported;
     }
     if (dry) return cudaSuccess;
-    return cudaLaunchKernelEx(&cfg, kfn, (E *)table, ra, d_pref, d_meta);
+    err = cudaLaunchKernelEx(&cfg, kfn, (E *)table, ra, d_pref, d_meta);
+#if PTAS_RING_PROFILE
+    if (err == cudaSuccess) {
+        static long long h[4][2048];
+        cudaStreamSynchronize(st);
+        cudaMemcpyFromSymbol(h, g_ring_prof, sizeof(h));
+        double s0 = 0, s1 = 0, s2 = 0;
+        const int nl = std::min(ra.rho_max + 1, 2048);
+        for (int L = 1; L < nl; ++L) {
+            s0 += h[1][L] - h[0][L];
+            s1 += h[2][L] - h[1][L];
+            s2 += h[3][L] - h[2][L];
+        }
+        std::fprintf(stderr, "[ring] CTA 8 thread 0, cycles per level: rows %.0f arrive %.0f wait %.0f (levels %d, CH %d, threads %d)\n",
+                     s0 / (nl - 1), s1 / (nl - 1), s2 / (nl - 1), nl, CH, 32 * warps);
+        for (int L = 300; L < nl && L < 306; ++L)
+            std::fprintf(stderr, "  L=%d rows %lld arrive %lld wait %lld\n", L, h[1][L] - h[0][L], h[2][L] - h[1][L], h[3][L] - h[2][L]);
+    }
+#endif
+    return err;
 }
 
 template <typename E, int CH>
@@ -313,6 +371,30 @@ cudaError_t launch_ring_e(void *table, const RingArgs &ra, int CH, const PrefixE
 
 }  // namespace
 }  // namespace swar
+
+// Host-side test of the ring kernel's geometry for a DP with internal counts N,
+// sizes r (K classes) at T: true when launch_row_fill_ring would take it (the
+// shared-memory fit for one of the cluster sizes; occupancy is not queried).
+// The solve driver evaluates such latency-bound DPs concurrently (D8, D14).
+bool ring_fits(const int32_t *N, const int64_t *r, int K, int64_t T)
+{
+    if (K != 3) return false;
+    int64_t sumN = 0;
+    for (int i = 0; i < K; ++i) sumN += N[i];
+    const int e = sumN <= 255 ? 1 : 2;
+    const int64_t W = (int64_t)N[2] + 1;
+    const int Lw = (int)row_pitch_words(W * e);
+    const int J0 = (int)std::min<int64_t>(N[2], T / r[2]);
+    if (J0 * e > 8) return false;
+    const int64_t hi0 = std::min<int64_t>(N[0], T / r[0]), hi1 = std::min<int64_t>(N[1], T / r[1]);
+    const int64_t R = std::min<int64_t>(hi0 + hi1, T / std::min(r[0], r[1])) + 1;
+    for (int csize : {16, 8}) {
+        const int64_t A = (N[0] + csize) / csize;
+        if (A < hi0) continue;
+        if (((R * A * Lw * 4 + 15) & ~(int64_t)15) + 4 * (int64_t)(hi0 + 1) * (hi1 + 1) * 16 <= 220 * 1024) return true;
+    }
+    return false;
+}
 
 // Host planning (D14): K = 3 only (two leading digits), a row of at
 // most 256 words (one warp), window shifts J0 * e <= 124 bytes, and the ring of
@@ -349,7 +431,8 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     for (int csize : {16, 8, 4, 2}) {
         if (cs_force ? csize != cs_force : csize < 8) continue;
         ra.A = (N[0] + csize) / csize;   // ceil((N0 + 1) / C) rows of each level per CTA
-        const size_t smem = (((size_t)ra.R * ra.A * Lw * 4 + 15) & ~(size_t)15) + (size_t)(np + 8) * 16 + 64;
+        if (ra.A < hi0) continue;         // every source row is in this CTA's block or the previous one
+        const size_t smem = (((size_t)ra.R * ra.A * Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
         if (smem > smem_cap) continue;
         // words per lane: the smallest chunk with one pass over the CTA's rows of a level
         int CH = 8;
