@@ -415,6 +415,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     int64_t spec_sigma = (int64_t)1 << 24;
     const char *sr = std::getenv("PTAS_SPEC_RING");   // 0: ring DPs only below spec_sigma (A/B)
     const bool spec_ring = !(sr && sr[0] == '0');
+    const char *sl = std::getenv("PTAS_SPEC_LEVELS");
+    const int64_t spec_levels = sl && sl[0] ? std::atoll(sl) : 160;
     {
         const char *sd = std::getenv("PTAS_SPEC_DEPTH");
         if (sd && sd[0] && opt.speculate < 0) spec_depth = std::atoi(sd);
@@ -463,8 +465,11 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 }
                 const bool known = memo.count(key) || spec.count(key) ||
                                    std::find(key_v.begin(), key_v.end(), key) != key_v.end();
-                // latency-bound DPs (the K = 3 cluster ring kernel fills them on 16 SMs,
-                // DESIGN.md D14) overlap whatever their size
+                // latency-bound DPs overlap whatever their size: the K = 3 cluster ring
+                // kernel fills them on 16 SMs (D14), and DPs with few wide
+                // row-levels (<= spec_levels: the u8 K = 6..8 shapes) leave the GPU idle at
+                // every level boundary (measured: M2s -28%, M4s -12%; DPs with hundreds of
+                // levels lose by sharing the GPU, M3s +50%)
                 if (spec_ring) {
                     const std::vector<int> o = choose_order(c.N, c.r, opt.layout);
                     std::vector<int32_t> No;
@@ -474,6 +479,9 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                         ro.push_back(c.r[i]);
                     }
                     lat = ring_fits(No.data(), ro.data(), (int)No.size(), T);
+                    int64_t levels = 1;
+                    for (size_t i = 0; i + 1 < No.size(); ++i) levels += No[i];
+                    lat = lat || (No.size() >= 2 && levels <= spec_levels);
                 }
                 // a large next probe runs alone (throughput-bound: nothing to overlap)
                 if (nd.d == 0 && sg > (__int128)spec_sigma && !lat) return PTAS_OK;
@@ -484,7 +492,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 T_v.push_back(T);
                 key_v.push_back(key);
             }
-            // a chain of latency-bound ring DPs runs up to MAX_SLOTS deep (16 SMs each)
+            // a chain of latency-bound DPs runs up to MAX_SLOTS deep
             if (lat && spec_chain) depth_lim = MAX_SLOTS;
             if (nd.d + 1 < depth_lim && (int)cls_v.size() < MAX_SLOTS) {
                 q.push_back({nd.lb, T, nd.d + 1});        // T feasible
