@@ -6,17 +6,33 @@ One step = one full ptas_solve of the workload (every §8(a) row: classify,
 configuration enumeration, row-level index, level fill per probe, readout,
 search, traceback + greedy schedule).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload M2s] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload W] [--impl ours|reference]
 
-value  : executed relaxations (closed form, summed over the DPs the solve ran)
-         / device-timed step, with p resident in HBM (ptas_solve_device)
+Workloads: N = 1 -> M2s (the shaped twin of configs[1], the
+single-GPU level-fill baseline); N > 1 -> M4x level-sharded (north_star's
+largest-dimension instance, configs[3]'s role), with a multi-section block on
+M5s-0.3 at P = N (configs[4]).  The N = 1 line carries the single-GPU M4x
+number in `scaling_ref` so every N of a scaling run has the same instance.
+
+value  : Eq. 1 relaxations (closed form, summed over the DPs the search used;
+         speculative DPs the search never probed are not counted) / device-timed
+         step, with p resident in HBM (ptas_solve_device)
 e2e    : the same through ptas_solve with pinned host p / host assignment
-roofline: level-fill kernel, algorithmic bytes (relax + sigma) * e per DP over
-         its event-timed duration, against MEASURED_PEAKS.json hbm_gbs
-cpu_baseline: the oracle (plain sequential C) on a bounded sub-box sample of
-         the same workload's largest DP, one host core; cpu_baseline.omp: the
-         paper's Alg 2 comparator shape (OpenMP level-parallel) on all host cores,
-         same sub-box
+roofline: level fill, SURVEY.md §8(d) algorithmic bytes (relax + sigma) * e over
+         the fill time (CUDA events: union of the DPs' fill intervals) against
+         N x MEASURED_PEAKS.json hbm_gbs.  The kernels gather fewer bytes than
+         Eq. 1 (one window per prefix, pivot blocks, D5/D13), so
+         frac > 1 is possible; `frac_executed` uses the bytes actually gathered
+         and `dram` the ncu DRAM bytes of the profiled launch (profiles/).
+parity : asserted on every run, outside the timed region: the solve (T*,
+         makespan, assignment, probe log) against the oracle's golden
+         (tests/golden/shaped, written by scripts/make_shaped_goldens.py from
+         oracle/ only) and the SHA-256 of the largest DP table (T = LB) in the
+         solve's layout against the oracle's.  A mismatch exits non-zero.
+cpu_baseline: the oracle (plain sequential C) on the workload's largest DP (the
+         whole table when it is at most 6e9 relaxations, else a sub-box), one
+         host core; cpu_baseline.omp: the paper's Alg 2 comparator shape (OpenMP
+         level-parallel) on all host cores, same table
 """
 from __future__ import annotations
 
@@ -147,20 +163,35 @@ def _subbox_for(N, r, T, target_relax):
     return Nc.astype(np.int32), relax(Nc)
 
 
-def cpu_oracle_sample(w, target_relax=2.0e9):
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
+def cpu_oracle_sample(w, target_relax=6.0e9):
+    """The oracle on the workload's largest DP (T = LB): the whole table when its
+    closed-form relaxation count is at most target_relax, else a sub-box."""
     import oracle
     N, r, T = _largest_dp(w)
     if len(N) == 0:
         return None
     Nc, rel = _subbox_for(N, r, T, target_relax)
+    whole = bool((np.asarray(Nc) == np.asarray(N)).all())
     t0 = time.perf_counter()
     _tab, relax = oracle.dp(Nc, r, T)
     dt = time.perf_counter() - t0
-    out = {"value": relax / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-           "sample": f"oracle_dp on the sub-box N'={Nc.tolist()} of the {w.name} DP at T=LB={T} "
-                     f"(full N={list(map(int, N))}); {relax:.3g} relaxations in {dt:.2f} s, 1 core"}
+    what = (f"oracle_dp on the WHOLE {w.name} DP at T=LB={T} (N={list(map(int, N))})" if whole else
+            f"oracle_dp on the sub-box N'={Nc.tolist()} of the {w.name} DP at T=LB={T} (full N={list(map(int, N))})")
+    out = {"value": relax / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "cpu_model": _cpu_model(),
+           "nproc": os.cpu_count(), "whole_table": whole,
+           "sample": f"{what}; {relax:.3g} relaxations in {dt:.2f} s, 1 core"}
     # The paper's comparator shape (Alg 2, OpenMP level-parallel) on all host
-    # cores, same sub-box; its table must equal the sequential oracle's.
+    # cores, same table; its table must equal the sequential oracle's.
     try:
         t0 = time.perf_counter()
         tab2, relax2 = oracle.dp_omp(Nc, r, T)
@@ -168,10 +199,58 @@ def cpu_oracle_sample(w, target_relax=2.0e9):
         cores = oracle.omp_threads()
         out["omp"] = {"value": relax2 / dt2, "unit": UNIT, "cores": cores, "kind": "oracle_alg2_openmp",
                       "tables_equal": bool(np.array_equal(_tab, tab2)),
-                      "sample": f"oracle_dp_omp (Alg 2 level-parallel) on the same sub-box; "
+                      "sample": f"oracle_dp_omp (Alg 2 level-parallel) on the same table; "
                                 f"{relax2:.3g} relaxations in {dt2:.2f} s, {cores} threads"}
     except Exception as e:  # noqa: BLE001 — the comparator is optional context
         out["omp"] = {"unavailable": str(e)}
+    return out
+
+
+GOLD = os.path.join(ROOT, "tests", "golden", "shaped")
+
+
+def parity_check(P, w, opts, Pp, table=True):
+    """Bit-exact parity of this run's configuration against the oracle's goldens
+    (tests/golden/shaped): the solve, and the largest DP table in the solve's
+    layout.  Returns a dict; raises SystemExit on a mismatch."""
+    import hashlib
+    import torch
+    out = {}
+    p = w.p()
+    gs = os.path.join(GOLD, f"solve_{w.name}_P{Pp}.json")
+    if os.path.exists(gs):
+        g = json.load(open(gs))
+        got = P.ptas_solve(p, w.m, w.eps, opts=opts, log=True)
+        ok = (got["T_star"] == g["T_star"] and got["makespan"] == g["makespan"] and
+              [int(x) for x in got["assignment"]] == g["assignment"] and
+              [list(x[:6]) for x in got["probes"]] == g["probes"])
+        out["solve"] = {"match": ok, "T_star": got["T_star"], "makespan": got["makespan"],
+                        "probes": len(got["probes"]), "golden": os.path.relpath(gs, ROOT)}
+    else:
+        out["solve"] = {"match": None, "note": f"no oracle golden for {w.name} at P={Pp}"}
+    gt = os.path.join(GOLD, f"table_{w.name}.json")
+    if table and os.path.exists(gt):
+        g = json.load(open(gt))
+        N = np.asarray(g["N"], np.int32)
+        r = np.asarray(g["r"], np.int64)
+        order = P.ptas_table_order(N, r, 0)
+        No, ro = N[order], r[order]
+        sg, e = P.dp_table_shape(No)
+        t = torch.empty(sg, dtype=torch.uint8 if e == 1 else torch.int16, device=torch.cuda.current_device())
+        opt = P.dp_fill_device(No, ro, g["T"], t)
+        torch.cuda.synchronize()
+        tv = t.view(tuple(int(x) + 1 for x in No)).permute(*[int(i) for i in np.argsort(order)])
+        h = hashlib.sha256()
+        step = max(1, int((256 << 20) // max(1, tv[0].numel() * tv.element_size())))
+        for a in range(0, tv.shape[0], step):
+            h.update(tv[a:a + step].contiguous().cpu().numpy().tobytes())
+        ok = h.hexdigest() == g["sha256"] and opt == g["opt"]
+        out["table_sha256"] = {"match": ok, "sigma": sg, "T": g["T"], "golden": os.path.relpath(gt, ROOT)}
+        del t, tv
+        torch.cuda.empty_cache()
+    if any(v.get("match") is False for v in out.values()):
+        print(json.dumps({"parity_failure": out}), flush=True)
+        raise SystemExit(3)
     return out
 
 
@@ -214,6 +293,64 @@ def run_reference(args, w):
     return 0
 
 
+def _measure(P, w, opts, lib_stream, flush, local, world, steps, warmup, barrier, clk=None):
+    """Warm-up + timed steps of one configuration: device-resident and end-to-end.
+    Returns (dev_ms, stats, e2e_ms, e2e_stats)."""
+    import torch
+    p = w.p()
+    n = len(p)
+    p_pin = torch.from_numpy(p).pin_memory()
+    p_dev = p_pin.to(f"cuda:{local}")
+    a_dev = torch.zeros(n, dtype=torch.int32, device=f"cuda:{local}")
+    s_ev = torch.cuda.Event(enable_timing=True)
+    e_ev = torch.cuda.Event(enable_timing=True)
+
+    def step_device():
+        return P.ptas_solve_device(p_dev, w.m, w.eps, a_dev, opts=opts)
+
+    def step_e2e():
+        # pinned host p in, host assignment out (the public ABI call a user makes)
+        return P.ptas_solve(p_pin.numpy(), w.m, w.eps, opts=opts, log=False)
+
+    def timed(fn, out_ms, out_stats):
+        flush.zero_()                       # L2 flush between steps (outside the events)
+        torch.cuda.synchronize()
+        s_ev.record(lib_stream)
+        r = fn()
+        e_ev.record(lib_stream)
+        torch.cuda.synchronize()
+        if out_ms is not None:
+            out_ms.append(s_ev.elapsed_time(e_ev))
+            out_stats.append(r["stats"])
+
+    dev_ms, stats, e2e_ms, e2e_stats = [], [], [], []
+    for _ in range(warmup):        # warm-up steps are identical to the timed ones
+        timed(step_device, None, None)
+        timed(step_e2e, None, None)
+    barrier()
+    for _ in range(steps):
+        timed(step_device, dev_ms, stats)
+    barrier()
+    for _ in range(steps):
+        timed(step_e2e, e2e_ms, e2e_stats)
+    barrier()
+    return dev_ms, stats, e2e_ms, e2e_stats
+
+
+def _reduce(dist, torch, local, world, mode_multi, vals_max, vals_sum):
+    """Max over ranks of times, sum over ranks of per-rank work (multi-probe: each
+    rank counts only the DPs it ran; level-sharded: every rank counts the same
+    DPs, so no sum)."""
+    if world == 1:
+        return vals_max, vals_sum
+    t = torch.tensor(vals_max, dtype=torch.float64, device=f"cuda:{local}")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    u = torch.tensor(vals_sum, dtype=torch.float64, device=f"cuda:{local}")
+    if mode_multi:
+        dist.all_reduce(u, op=dist.ReduceOp.SUM)
+    return t.tolist(), u.tolist()
+
+
 def run_ours(args, w):
     import torch
     import torch.distributed as dist
@@ -235,12 +372,6 @@ def run_ours(args, w):
     lib_stream = torch.cuda.Stream(device=local)
     opts = P.options(P=Pp, mode=mode, device=local, comm=comm, stream=lib_stream,
                      virtual_shards=args.virtual_shards if world == 1 else 1)
-
-    p = w.p()
-    n = len(p)
-    p_pin = torch.from_numpy(p).pin_memory()
-    p_dev = p_pin.to(f"cuda:{local}")
-    a_dev = torch.zeros(n, dtype=torch.int32, device=f"cuda:{local}")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{local}")
 
     def barrier():
@@ -248,75 +379,47 @@ def run_ours(args, w):
             dist.barrier()
         torch.cuda.synchronize()
 
-    def step_device():
-        return P.ptas_solve_device(p_dev, w.m, w.eps, a_dev, opts=opts)
-
-    def step_e2e():
-        # pinned host p in, host assignment out (the public ABI call a user makes)
-        r = P.ptas_solve(p_pin.numpy(), w.m, w.eps, opts=opts, log=False)
-        return r
-
-    dev_ms, stats = [], []
-    e2e_ms, e2e_stats = [], []
-    s_ev = torch.cuda.Event(enable_timing=True)
-    e_ev = torch.cuda.Event(enable_timing=True)
-
-    def timed(fn, out_ms, out_stats):
-        flush.zero_()                       # L2 flush between steps (outside the events)
-        torch.cuda.synchronize()
-        s_ev.record(lib_stream)
-        r = fn()
-        e_ev.record(lib_stream)
-        torch.cuda.synchronize()
-        if out_ms is not None:
-            out_ms.append(s_ev.elapsed_time(e_ev))
-            out_stats.append(r["stats"])
+    # parity against the oracle's goldens, before anything is timed (rank 0's GPU;
+    # the configuration's results do not depend on the rank)
+    parity = None
+    if not args.no_parity:
+        # the solve runs collectively at N > 1 (every rank takes part); rank 0 alone
+        # hashes the table
+        parity = parity_check(P, w, opts, Pp, table=rank == 0)
+        barrier()
 
     with ClockSampler(local) as clk:
-        for _ in range(args.warmup):        # warm-up steps are identical to the timed ones
-            timed(step_device, None, None)
-            timed(step_e2e, None, None)
-        barrier()
-        for _ in range(args.steps):
-            timed(step_device, dev_ms, stats)
-        barrier()
-        for _ in range(args.steps):
-            timed(step_e2e, e2e_ms, e2e_stats)
-        barrier()
+        dev_ms, stats, e2e_ms, e2e_stats = _measure(P, w, opts, lib_stream, flush, local, world, args.steps,
+                                                    args.warmup, barrier)
     clocks = clk.summary()
-
-    relax_total = sum(s["relaxations"] for s in stats)
-    t_total = sum(dev_ms) / 1e3
-    # device time during which level-fill loops ran (union of the DPs' fill
-    # intervals: speculative DPs overlap); the per-DP sum is reported beside it
-    fill_s = sum(s["fill_wall_seconds"] for s in stats)
+    multi = mode == P.MODE_MULTI_PROBE
+    (t_total, e2e_t, fill_s), (relax_total, e2e_relax, alg_bytes, exec_bytes) = _reduce(
+        dist, torch, local, world, multi,
+        [sum(dev_ms) / 1e3, sum(e2e_ms) / 1e3, sum(s["fill_wall_seconds"] for s in stats)],
+        [sum(s["relaxations"] for s in stats), sum(s["relaxations"] for s in e2e_stats),
+         sum(s["alg_bytes"] for s in stats), sum(s["exec_bytes"] for s in stats)])
     fill_sum_s = sum(s["fill_seconds"] for s in stats)
-    alg_bytes = sum(s["alg_bytes"] for s in stats)
-    exec_bytes = sum(s["exec_bytes"] for s in stats)
     relax_exec = sum(s["relax_executed"] for s in stats)
     fill_launches = sum(s["fill_launches"] for s in stats)
     launches = sum(s["kernel_launches"] for s in stats)
-    e2e_relax = sum(s["relaxations"] for s in e2e_stats)
-    e2e_t = sum(e2e_ms) / 1e3
-    if world > 1:
-        t = torch.tensor([t_total, e2e_t, fill_s], dtype=torch.float64, device=f"cuda:{local}")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        t_total, e2e_t, fill_s = t.tolist()
-        rl = torch.tensor([relax_total, e2e_relax, alg_bytes], dtype=torch.float64, device=f"cuda:{local}")
-        if mode == P.MODE_MULTI_PROBE:
-            dist.all_reduce(rl, op=dist.ReduceOp.SUM)   # distinct probes per rank
-        relax_total, e2e_relax, alg_bytes = rl.tolist()
-    peak, peak_kind = _peaks()
+    peak1, peak_kind = _peaks()
+    # level-sharded: every rank fills its slice, so the aggregate bandwidth of the
+    # job is compared with N GPUs' peak; multi-probe: the ranks' DPs run side by side
+    peak = peak1 * world
+    # job-wide algorithmic bytes (level-sharded: the one DP every rank fills a slice
+    # of; multi-probe: the sum of the ranks' DPs) over the job's fill time (max over ranks)
     achieved = alg_bytes / fill_s / 1e9 if fill_s > 0 else 0.0
-    traffic, traffic_note = None, None
+    traffic, traffic_note, dram = None, None, None
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
             t = json.load(open(tf)).get(w.name)
             if t:
                 traffic = t["dram_bytes_per_launch"]
-                traffic_note = {"alg_bytes_per_launch": t["alg_bytes_per_launch"],
-                                "traffic_over_alg": t["traffic_over_alg"], "source": t["source"]}
+                traffic_note = {k: t[k] for k in t if k != "dram_bytes_per_launch"}
+                if t.get("dram_gbs"):
+                    dram = {"achieved": t["dram_gbs"], "peak": peak1, "unit": "GB/s",
+                            "frac": t["dram_gbs"] / peak1, "source": t["source"]}
         except Exception:
             traffic = None
     st0 = stats[0]
@@ -344,20 +447,26 @@ def run_ours(args, w):
                 "solve_ms": 1e3 * e2e_t / args.steps},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "traffic_note": traffic_note,
-                     "kernel": "row_fill_swar_kernel (level fill, §8(a) a-5; dataflow launches, DESIGN.md D7)",
-                     "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)" if peak_kind == "measured" else "fallback",
+                     "bytes": "SURVEY.md §8(d) algorithmic bytes of Eq. 1: (relaxations + states) * e per DP",
+                     "kernel": "level fill (row_fill_swar_kernel dataflow / per-level launches, "
+                               "row_ring_kernel for K = 3; §8(a) a-5)",
+                     "peak_kind": (peak_kind + " (MEASURED_PEAKS.json hbm_gbs)" if peak_kind == "measured" else "fallback")
+                                  + (f" x {world} GPUs" if world > 1 else ""),
                      "fill_ms_per_step": 1e3 * fill_s / args.steps,
                      "fill_time": "union of the DPs' fill intervals (CUDA events, one time axis); "
                                   "alg bytes count only the DPs the search used",
                      "fill_ms_sum_per_step": 1e3 * fill_sum_s / args.steps,
                      "fill_launches_per_step": fill_launches / args.steps,
                      "alg_bytes_per_step": alg_bytes / args.steps,
-                     # the kernel takes one window per (row, prefix) (D5): the
-                     # bytes it actually gathers, and their rate, next to the algorithmic ones
+                     # the kernels take one window per (row, prefix) of the row's pivot block
+                     # (D5, D13): the bytes they actually gather, and their rate
                      "relax_executed_per_step": relax_exec / args.steps,
                      "executed_bytes_per_step": exec_bytes / args.steps,
                      "executed_gbs": exec_bytes / fill_s / 1e9 if fill_s > 0 else None,
+                     "frac_executed": (exec_bytes / fill_s / 1e9 / peak) if fill_s > 0 else None,
+                     "dram": dram,
                      "fill_relax_per_s": relax_total / fill_s if fill_s > 0 else None},
+        "parity": parity,
         "step_ms": [round(x, 3) for x in dev_ms],
         "step_dp_ms": [round(1e3 * st["dp_seconds"], 3) for st in stats],
         "step_lib_wall_ms": [round(1e3 * st["total_seconds"], 3) for st in stats],
@@ -365,6 +474,26 @@ def run_ours(args, w):
         "gpu_launches": int(launches),
         "clocks": clocks,
     }
+    # secondary blocks (same metric, untimed relative to the line above)
+    def block(wb, mode_b, Pb, note):
+        ob = P.options(P=Pb, mode=mode_b, device=local, comm=comm if world > 1 else None, stream=lib_stream)
+        par = parity_check(P, wb, ob, Pb, table=rank == 0) if not args.no_parity else None
+        d, st, e, est = _measure(P, wb, ob, lib_stream, flush, local, world, args.steps, args.warmup, barrier)
+        (tt, et), (rr, er) = _reduce(dist, torch, local, world, mode_b == P.MODE_MULTI_PROBE,
+                                     [sum(d) / 1e3, sum(e) / 1e3],
+                                     [sum(x["relaxations"] for x in st), sum(x["relaxations"] for x in est)])
+        return {"workload": wb.name, "mode": {0: "single", 1: "level_sharded", 2: "multi_probe"}[mode_b],
+                "probes_per_round": Pb, "n_gpus": world, "value": rr / tt, "unit": UNIT,
+                "ms_per_step": 1e3 * tt / args.steps, "e2e_value": er / et, "T_star": st[0]["T_star"],
+                "unique_dps": st[0]["unique_dps"], "parity": par, "note": note}
+    if not args.no_blocks:
+        if world == 1 and w.name != "M4x":
+            line["scaling_ref"] = block(WORKLOADS["M4x"], P.MODE_SINGLE, 1,
+                                        "north_star's scaling instance on this single GPU: the N = 1 point of the "
+                                        "level-sharded 1/2/4/8-GPU curve (bench.py --gpus N defaults to it)")
+        if world > 1:
+            line["multi_probe"] = block(WORKLOADS["M5s-0.3"], P.MODE_MULTI_PROBE, world,
+                                        "multi-section search (Alg 3 generalised, one probe per GPU per round)")
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_oracle_sample(w)
     if comm is not None:
@@ -382,7 +511,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", default="M2s", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default=None, choices=sorted(WORKLOADS),
+                    help="default: M2s at N = 1, M4x (level-sharded) at N > 1")
     ap.add_argument("--P", type=int, default=1, help="probes per round (single GPU)")
     ap.add_argument("--mode", choices=["auto", "sharded", "multiprobe"], default="auto",
                     help="N>1 mode; auto = sharded when the workload's largest table is >= 1 GB "
@@ -391,8 +521,13 @@ def main():
                     help="N=1 only: run LEVEL_SHARDED with G logical shards on one GPU (slice fill + "
                          "gather copy + scatter per level, no NCCL) to measure the exchange overhead")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-parity", action="store_true", help="skip the oracle-golden parity assertion")
+    ap.add_argument("--no-blocks", action="store_true", help="skip the scaling_ref / multi_probe blocks")
     ap.add_argument("--dtype-label", default=None)
     args = ap.parse_args()
+    _rank, _local, world = _dist_env()
+    if args.workload is None:
+        args.workload = "M2s" if world == 1 else "M4x"
     w = WORKLOADS[args.workload]
     # geometry of the largest DP: the product's host ABI for our arm, the
     # oracle only on the reference (oracle) arm

@@ -80,6 +80,11 @@ typedef struct {
                                    2^d - 1 probes in flight).  The probe
                                    sequence, T* and the schedule are those of
                                    Alg 1 (D8); only time changes.      */
+    int64_t shard_min_rows;     /* LEVEL_SHARDED with comm: row-levels with fewer
+                                   rows are computed redundantly on every rank
+                                   (-1 = library default 2048); 0 = shard every
+                                   row-level, also at world size 1 (the slice /
+                                   ncclAllGather / scatter path on one GPU)      */
 } ptas_options;
 
 typedef struct {
@@ -151,7 +156,10 @@ int ptas_solve_ex(const int64_t *p, int32_t n, int32_t m, double eps,
 
 /* Device-resident variant: d_p (int64[n]) and d_assignment (int32[n]) are
  * device pointers on the chosen device; makespan_out is host.  The host
- * driver stages p to host memory internally (counted in stats->d2h_bytes). */
+ * driver stages p to host memory internally (counted in stats->d2h_bytes).
+ * d_p is read and d_assignment written on options->stream, or on the legacy
+ * default stream when it is NULL, so both are ordered with the caller's work
+ * on that stream; the call returns when d_assignment is written. */
 int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps,
                       const ptas_options *opt, int64_t *makespan_out,
                       int32_t *d_assignment, ptas_stats *stats);
@@ -243,11 +251,19 @@ int ptas_probe_targets(int64_t LB, int64_t UB, int32_t P, int64_t *out,
 int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T,
                          const int32_t *feasible, int32_t count);
 /* Contiguous slice [begin, end) of `count` items owned by `rank` of
- * `world` (ceil split; trailing ranks may be empty).  The level-sharded DP
- * splits each sharded row-level the same way, except that the per-rank row
- * count is rounded up so every slice starts 16-byte aligned. */
+ * `world` (ceil split; trailing ranks may be empty). */
 int ptas_shard_range(int64_t count, int32_t rank, int32_t world,
                      int64_t *begin, int64_t *end);
+/* The split the level-sharded DP uses for one row-level of `rows` rows of
+ * `row_bytes` bytes each (rows of a level are independent,
+ * PAPER.md:215): ceil(rows / world) rounded up to the smallest multiple q with
+ * q * row_bytes = 0 (mod 16), so every rank's compact slice starts 16-byte
+ * aligned; rank r owns [min(rows, r*chunk), min(rows, (r+1)*chunk)), trailing
+ * ranks may be empty.  *chunk_out (nullable) = the per-rank slice length every
+ * rank contributes to the ncclAllGather (padded).  EINVAL: rows < 0,
+ * world < 1, rank outside [0, world), row_bytes < 1, null begin/end. */
+int ptas_level_shard(int64_t rows, int32_t rank, int32_t world, int64_t row_bytes,
+                     int64_t *begin, int64_t *end, int64_t *chunk_out);
 
 /* Internal class order of the DP table (D2,
  * D13): order_out[i] = the caller class laid out at position i (the

@@ -15,13 +15,13 @@ from ._native import (MODE_LEVEL_SHARDED, MODE_MULTI_PROBE, MODE_SINGLE, EXPORTS
 
 __all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
            "dp_row_index", "ptas_k", "ptas_bounds", "ptas_classify", "ptas_probe_targets",
-           "ptas_interval_update", "ptas_shard_range", "ptas_table_order", "Comm", "init_comm", "options", "lib", "strerror",
+           "ptas_interval_update", "ptas_shard_range", "ptas_level_shard", "ptas_table_order", "Comm", "init_comm", "options", "lib", "strerror",
            "PtasError", "EXPORTS", "MODE_SINGLE", "MODE_LEVEL_SHARDED", "MODE_MULTI_PROBE"]
 
 
 def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, budget: int = 0,
             memoize: bool = True, virtual_shards: int = 1, layout: int = 0, stream=None,
-            speculate: int = -1) -> PtasOptions:
+            speculate: int = -1, shard_min_rows: int = -1) -> PtasOptions:
     o = PtasOptions()
     lib().ptas_default_options(ctypes.byref(o))
     o.probes_per_round = int(P)
@@ -33,6 +33,7 @@ def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, bu
     o.virtual_shards = int(virtual_shards)
     o.layout = int(layout)
     o.speculate = int(speculate)
+    o.shard_min_rows = int(shard_min_rows)
     o.stream = None if stream is None else ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
     return o
 
@@ -62,6 +63,9 @@ def ptas_solve_device(p_dev, m: int, eps: float, assignment_dev, P: int = 1, opt
     import torch
     assert p_dev.is_cuda and p_dev.dtype == torch.int64 and p_dev.is_contiguous()
     assert assignment_dev.is_cuda and assignment_dev.dtype == torch.int32 and assignment_dev.numel() == p_dev.numel()
+    if opts is None and "stream" not in kw:
+        # the caller's current stream: p_dev is read after the work that produced it
+        kw["stream"] = torch.cuda.current_stream(p_dev.device)
     o = opts if opts is not None else options(P=P, device=p_dev.device.index, **kw)
     ms = ctypes.c_int64()
     st = PtasStats()
@@ -208,6 +212,14 @@ def ptas_table_order(counts, sizes, layout: int = 0):
     _chk("ptas_table_order", lib().ptas_table_order(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), len(c),
                                                     int(layout), _ptr(out, ctypes.c_int32), ctypes.byref(k)))
     return [int(x) for x in out[: k.value]]
+
+
+def ptas_level_shard(rows: int, rank: int, world: int, row_bytes: int):
+    """(begin, end, chunk) of the level-sharded DP's aligned split of one row-level."""
+    b, e, c = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+    _chk("ptas_level_shard", lib().ptas_level_shard(int(rows), int(rank), int(world), int(row_bytes), ctypes.byref(b),
+                                                    ctypes.byref(e), ctypes.byref(c)))
+    return b.value, e.value, c.value
 
 
 def ptas_shard_range(count: int, rank: int, world: int):

@@ -27,7 +27,7 @@ class PtasOptions(ctypes.Structure):
     _fields_ = [("probes_per_round", ctypes.c_int32), ("mode", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("comm", vp), ("table_budget_bytes", ctypes.c_int64), ("memoize", ctypes.c_int32),
                 ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32), ("stream", vp),
-                ("speculate", ctypes.c_int32)]
+                ("speculate", ctypes.c_int32), ("shard_min_rows", ctypes.c_int64)]
 
 
 class PtasStats(ctypes.Structure):
@@ -55,7 +55,7 @@ EXPORTS = [
     "ptas_default_options", "ptas_solve", "ptas_solve_ex", "ptas_solve_device", "dp_table_shape", "dp_fill",
     "dp_fill_device", "ptas_get_unique_id", "ptas_comm_init", "ptas_comm_destroy", "ptas_strerror", "ptas_k",
     "ptas_bounds", "ptas_classify", "ptas_probe_targets", "ptas_interval_update", "ptas_shard_range",
-    "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order",
+    "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order", "ptas_level_shard",
 ]
 
 _lib = None
@@ -98,6 +98,7 @@ def lib():
     L.ptas_probe_targets.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, i64p, i32p]
     L.ptas_interval_update.argtypes = [i64p, i64p, i64p, i32p, ctypes.c_int32]
     L.ptas_shard_range.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, i64p, i64p]
+    L.ptas_level_shard.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, i64p, i64p, i64p]
     L.dp_configs.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, ctypes.c_int64, i64p]
     L.hmbp_solve.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, i32p, ctypes.c_int32,
                              ctypes.POINTER(PtasStats)]

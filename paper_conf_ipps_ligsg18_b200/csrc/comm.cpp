@@ -26,6 +26,8 @@ struct NcclApi {
     decltype(&ncclGetUniqueId) getUniqueId = nullptr;
     decltype(&ncclCommInitRank) commInitRank = nullptr;
     decltype(&ncclAllGather) allGather = nullptr;
+    decltype(&ncclAllReduce) allReduce = nullptr;
+    decltype(&ncclBroadcast) broadcast = nullptr;
     decltype(&ncclCommDestroy) commDestroy = nullptr;
 };
 
@@ -40,8 +42,11 @@ NcclApi *nccl()
         api.getUniqueId = (decltype(api.getUniqueId))dlsym(h, "ncclGetUniqueId");
         api.commInitRank = (decltype(api.commInitRank))dlsym(h, "ncclCommInitRank");
         api.allGather = (decltype(api.allGather))dlsym(h, "ncclAllGather");
+        api.allReduce = (decltype(api.allReduce))dlsym(h, "ncclAllReduce");
+        api.broadcast = (decltype(api.broadcast))dlsym(h, "ncclBroadcast");
         api.commDestroy = (decltype(api.commDestroy))dlsym(h, "ncclCommDestroy");
-        api.ok = api.getUniqueId && api.commInitRank && api.allGather && api.commDestroy;
+        api.ok = api.getUniqueId && api.commInitRank && api.allGather && api.allReduce && api.broadcast &&
+                 api.commDestroy;
     });
     return &api;
 }
@@ -107,6 +112,24 @@ int comm_allgather(ptas_comm *c, const void *send, void *recv, size_t bytes_per_
     if (!a->ok || !c) return PTAS_ENCCL;
     if (a->allGather(send, recv, bytes_per_rank, ncclUint8, c->comm, st) != ncclSuccess)
         return PTAS_ENCCL;
+    return PTAS_OK;
+}
+
+// In-place min over the ranks of `count` int32 values (status agreement).
+int comm_allreduce_min_i32(ptas_comm *c, int32_t *d_buf, size_t count, cudaStream_t st)
+{
+    NcclApi *a = nccl();
+    if (!a->ok || !c) return PTAS_ENCCL;
+    if (a->allReduce(d_buf, d_buf, count, ncclInt32, ncclMin, c->comm, st) != ncclSuccess) return PTAS_ENCCL;
+    return PTAS_OK;
+}
+
+// In-place broadcast of `bytes` bytes from `root`.
+int comm_broadcast(ptas_comm *c, void *d_buf, size_t bytes, int root, cudaStream_t st)
+{
+    NcclApi *a = nccl();
+    if (!a->ok || !c) return PTAS_ENCCL;
+    if (a->broadcast(d_buf, d_buf, bytes, ncclUint8, root, c->comm, st) != ncclSuccess) return PTAS_ENCCL;
     return PTAS_OK;
 }
 

@@ -23,18 +23,6 @@
 
 namespace ptas {
 
-// Rows per shard of a sharded row-level: ceil(R / G) rounded up so that every
-// shard's compact slice starts 16-byte aligned (the packed fill kernel writes
-// compact rows with vector stores and rejects unaligned slices, which would
-// send the level to the scalar kernel).  Trailing shards may be short or empty.
-static int64_t shard_chunk(int64_t R, int G, int64_t row_bytes)
-{
-    const int64_t c = (R + G - 1) / G;
-    int64_t q = 1;
-    while ((q * row_bytes) % 16 != 0) ++q;      // smallest q with q * row_bytes = 0 (mod 16), q <= 16
-    return (c + q - 1) / q * q;
-}
-
 // PTAS_SLOW_CALLS=<ms> (diagnostics): report every checked call slower than
 // <ms> milliseconds of host time, with its source line.
 static double slow_call_ms()
@@ -347,21 +335,59 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     g.blk = (int32_t *)blk_.p;   // pivot blocks, written by build_prefix_kernel (D13)
     const int64_t rows = sigma / g.W;
     const int64_t ibytes = rows * g.Wp * e;  // padded internal table
+    // level sharding over the ranks of a communicator
+    int G = 1, myrank = 0;
+    bool virt = false;
+    const ShardCtx *sh = rq.shard;
+    if (sh) {
+        if (sh->comm) {
+            G = sh->world;
+            myrank = sh->rank;
+        } else if (sh->virtual_shards > 1) {
+            G = sh->virtual_shards;
+            virt = true;
+        }
+    }
+    const bool comm_dp = sh && sh->comm && (G > 1 || sh->force);   // collectives in this DP
+    auto sharded = [&](int64_t R) { return (G > 1 || comm_dp) && R >= std::max<int64_t>(sh->min_rows, 1); };
+    size_t stage_bytes = 0;
+    for (int rho = 0; rho <= g.rho_max && (G > 1 || comm_dp); ++rho) {
+        const int64_t R = cnt[rho];
+        if (!sharded(R)) continue;
+        stage_bytes = std::max(stage_bytes, (size_t)(shard_chunk(R, G, g.Wp * e) * G * g.Wp * e));
+    }
     // compute in the caller's buffer when its layout is the padded one
     void *table = nullptr;
     const bool in_place = rq.ext_table && g.Wp == g.W && ((uintptr_t)rq.ext_table & 15) == 0;
-    if (in_place) {
-        table = rq.ext_table;
-    } else {
+    // admission: the budget and every large allocation first; a comm-backed DP then
+    // agrees on the outcome over all ranks (min of the status words) before any
+    // collective, so no rank returns while its peers wait in an all-gather
+    int adm = PTAS_OK;
+    if (!in_place) {
         // auto budget: query free HBM only when the table has to grow
         // (cudaMemGetInfo costs ~0.1 ms per call)
         if (rq.budget > 0 || (size_t)ibytes > table_.cap) {
             const int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
-            if (ibytes > budget) return PTAS_ETOOBIG;
+            if (ibytes > budget) adm = PTAS_ETOOBIG;
         }
-        PT_CK(table_.ensure((size_t)ibytes));
-        table = table_.p;
+        if (!adm && table_.ensure((size_t)ibytes) != cudaSuccess) adm = PTAS_ENOMEM;
     }
+    const int NWk = g.nwords <= 1 ? 1 : 2;
+    if (!adm && rowidx_.ensure((size_t)rows * 8 * (1 + NWk)) != cudaSuccess) adm = PTAS_ENOMEM;
+    if (!adm && stage_bytes && stage_.ensure(stage_bytes) != cudaSuccess) adm = PTAS_ENOMEM;
+    if (comm_dp) {
+        if (xch_.ensure(64) != cudaSuccess) return PTAS_ENOMEM;   // (64 B: never fails after the first DP)
+        int32_t *dx = (int32_t *)xch_.p;
+        h_scalar_[0] = adm;
+        PT_CK(cudaMemcpyAsync(dx, h_scalar_, 4, cudaMemcpyHostToDevice, st));
+        const int crc = comm_allreduce_min_i32(sh->comm, dx, 1, st);
+        if (crc) return crc;
+        PT_CK(cudaMemcpyAsync(h_scalar_, dx, 4, cudaMemcpyDeviceToHost, st));
+        PT_CK(sync_spin(st));
+        adm = (int32_t)h_scalar_[0];
+    }
+    if (adm) return adm;
+    table = in_place ? rq.ext_table : table_.p;
     PT_CK(cudaEventRecord(ev_[0], st));
     int64_t idxN = N[K - 1];
     for (int i = 0; i < K - 1; ++i) idxN += (int64_t)N[i] * stride[i];
@@ -395,8 +421,6 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     void *const d_small = cnt_.p;
     const int64_t *d_cnt = (const int64_t *)((unsigned char *)cnt_.p + small_pad);
     // ---- a-4 level-ordered row index (row base + packed leading digits per row)
-    const int NWk = g.nwords <= 1 ? 1 : 2;
-    PT_CK(rowidx_.ensure((size_t)rows * 8 * (1 + NWk)));
     int64_t *d_rb = (int64_t *)rowidx_.p;
     uint64_t *d_pw = (uint64_t *)(d_rb + rows);
     // on the side stream: overlaps the enumeration below and its host round trip
@@ -436,7 +460,9 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // kernels exit and the DP is redone synchronously if a bound is exceeded
     // (meta->ovf), which then grows the bounds.
     const char *es = std::getenv("PTAS_ENUM_SYNC");
-    const bool nosync = np_hint_ >= 0 && nc_cap_ > 0 && !force_sync_enum_ && !(es && es[0] == '1');
+    // (a comm-backed DP always reads |C| back: every rank then takes the same path,
+    // no rank can redo the DP alone while its peers wait in a collective)
+    const bool nosync = np_hint_ >= 0 && nc_cap_ > 0 && !force_sync_enum_ && !(es && es[0] == '1') && !comm_dp;
     int64_t nC;        // |C| (synchronous) or its bound
     int64_t nP_bound;  // bound of the prefix list incl. the zero prefix (smem sizing)
     // test knobs: PTAS_NC_CAP / PTAS_NP_CAP lower the bounds (exercise the redo path)
@@ -537,30 +563,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     };
 
     // ---- a-5 level fill, one launch per row-level
-    int G = 1, myrank = 0;
-    bool virt = false;
-    const ShardCtx *sh = rq.shard;
-    if (sh) {
-        if (sh->comm) {
-            G = sh->world;
-            myrank = sh->rank;
-        } else if (sh->virtual_shards > 1) {
-            G = sh->virtual_shards;
-            virt = true;
-        }
-    }
     const int ld = g.rho_max + 1;
-    auto sharded = [&](int64_t R) { return G > 1 && R >= std::max<int64_t>(sh->min_rows, 1); };
-    if (G > 1) {
-        size_t mx = 0;
-        for (int rho = 0; rho <= g.rho_max; ++rho) {
-            int64_t R = cnt[rho];
-            if (!sharded(R)) continue;
-            const int64_t chunk = shard_chunk(R, G, g.Wp * e);
-            mx = std::max(mx, (size_t)(chunk * G * g.Wp * e));
-        }
-        PT_CK(stage_.ensure(mx));
-    }
     // ---- dataflow runs (D7): runs of row-levels filled by ONE
     // launch each.  PTAS_DF = 0: off (one launch per row-level); 1: the whole
     // DP in one launch, one row set per warp; 2: maximal runs of row-levels
@@ -582,7 +585,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     std::vector<DfRun> runs;
     // narrow K = 3 DPs: the whole fill on one thread-block cluster, recent levels
     // in distributed shared memory (row_ring.cu, D14); PTAS_RING=0: off
-    const bool ring = G == 1 && !force_scalar && K == 3 &&
+    const bool ring = G == 1 && !comm_dp && !force_scalar && K == 3 &&
                       launch_row_fill_ring(e, table, g, N.data(), r.data(), rq.T, J0, (const PrefixEntry *)pref_.p,
                                            d_meta_, nP_bound, st, true) == cudaSuccess;
     cudaGetLastError();
@@ -595,7 +598,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                              : (dfr && dfr[0] ? std::atoll(dfr) : (int64_t)2 * 32 * sm_count_);
         // (measured on M2s/M3s/M4s/M5s: 600..8000 within a few %, 2000 best overall)
         const int64_t split_rows = dsr && dsr[0] ? std::atoll(dsr) : 2000;
-        if (df_mode > 0 && G == 1 && !force_scalar && g.rho_max >= 1) {
+        if (df_mode > 0 && G == 1 && !comm_dp && !force_scalar && g.rho_max >= 1) {
             if (df_mode == 3 || df_mode == 4) {
                 // levels wider than df_rows get a launch of their own (enough rows to fill
                 // the GPU: the flag protocol costs more than the launch boundary saves,

@@ -1,5 +1,6 @@
 // engine.h — per-device DP engine (host orchestration of the kernels).
 #pragma once
+#include <algorithm>
 #include <cstdint>
 #include <mutex>
 #include <vector>
@@ -18,6 +19,7 @@ struct ShardCtx {
     int world = 1;
     int virtual_shards = 1;     // >1: logical shards on this GPU (testing)
     int64_t min_rows = 0;       // row-levels with fewer rows are computed redundantly
+    bool force = false;         // shard (slice, all-gather, scatter) also at world size 1
 };
 
 struct DpRequest {
@@ -110,7 +112,7 @@ class DpSlot {
     size_t pin_cap_ = 0, pin_used_ = 0;
     Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_, rowidx_, cpstage_;
     // dataflow fill (D7): per-row ready flags, ticket counter, run plans
-    Buf flags_, ticket_, dfplan_, dfprof_, domtab_, blk_;
+    Buf flags_, ticket_, dfplan_, dfprof_, domtab_, blk_, xch_;
     uint32_t df_epoch_ = 0;
     unsigned long long ticket_base_ = 0;
 
@@ -156,8 +158,27 @@ class Engine {
     // DPs' fill intervals (events on any stream) can be placed on one axis
     int mark_reference(cudaStream_t st, cudaEvent_t *out);
     cudaError_t sync_spin(cudaStream_t st) { return slots_[0]->sync_spin(st); }
+    // device buffer for the multi-GPU exchanges of a solve (grown, never freed)
+    int exchange_buffer(size_t bytes, void **out)
+    {
+        if (bytes > xcap_) {
+            if (xbuf_) cudaFree(xbuf_);
+            xbuf_ = nullptr;
+            xcap_ = 0;
+            const size_t want = std::max<size_t>(bytes, 4096);
+            if (cudaMalloc(&xbuf_, want) != cudaSuccess) {
+                cudaGetLastError();
+                return PTAS_ENOMEM;
+            }
+            xcap_ = want;
+        }
+        *out = xbuf_;
+        return PTAS_OK;
+    }
 
   private:
+    void *xbuf_ = nullptr;
+    size_t xcap_ = 0;
     int init(int device);
     int device_ = -1;
     int sm_count_ = 148;
@@ -170,5 +191,7 @@ int comm_rank(const ptas_comm *c);
 int comm_world(const ptas_comm *c);
 int comm_allgather(ptas_comm *c, const void *send, void *recv, size_t bytes_per_rank,
                    cudaStream_t st);
+int comm_allreduce_min_i32(ptas_comm *c, int32_t *d_buf, size_t count, cudaStream_t st);
+int comm_broadcast(ptas_comm *c, void *d_buf, size_t bytes, int root, cudaStream_t st);
 
 }  // namespace ptas

@@ -63,6 +63,19 @@ struct RowGeom {
 };
 constexpr int64_t DOMTAB_MAX_BYTES = 16384;
 
+// Rows per shard of a sharded row-level: ceil(R / G)
+// rounded up so that every shard's compact slice (rows of row_bytes bytes)
+// starts 16-byte aligned -- the packed fill kernel writes compact rows with
+// vector stores.  Rank g owns rows [g * chunk, min(R, (g + 1) * chunk)); trailing
+// ranks may be empty.  Exported as ptas_level_shard.
+inline int64_t shard_chunk(int64_t R, int G, int64_t row_bytes)
+{
+    const int64_t c = (R + G - 1) / G;
+    int64_t q = 1;
+    while ((q * row_bytes) % 16 != 0) ++q;      // smallest q with q * row_bytes = 0 (mod 16), q <= 16
+    return (c + q - 1) / q * q;
+}
+
 // Padded row pitch in 32-bit words for a row of `bytes` bytes: a multiple of
 // the packed fill kernel's words per lane (2 up to 64 words, 4 up to 128, 8
 // beyond), so each lane's chunk is one aligned vector load.

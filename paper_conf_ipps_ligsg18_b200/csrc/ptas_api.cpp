@@ -269,7 +269,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         sh.rank = rank;
         sh.world = world;
         sh.virtual_shards = opt.comm ? 1 : std::max(1, opt.virtual_shards);
-        sh.min_rows = opt.comm ? 2048 : 0;
+        sh.min_rows = opt.comm ? (opt.shard_min_rows >= 0 ? opt.shard_min_rows : 2048) : 0;
+        sh.force = opt.comm && opt.shard_min_rows == 0;
         shp = &sh;
     }
 
@@ -283,6 +284,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     }
     std::map<std::vector<int64_t>, int32_t> memo;
     std::vector<ptas_probe> plog;
+    constexpr int32_t XERR = -1000;                          // MULTI_PROBE: exchanged error codes
+    std::vector<std::vector<int64_t>> last_key_of(world);  // MULTI_PROBE: the last DP of each rank
     int round = 0;
     Classified cl;
 
@@ -523,7 +526,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             }
         }
         const int np = (int)Tj.size();
-        std::vector<int32_t> optj(np, 0), hit(np, 0), who(np, 0), Kj(np, 0);
+        std::vector<int32_t> optj(np, 0), hit(np, 0), who(np, 0), Kj(np, 0), xsrc(np, -1);
         std::vector<int64_t> sgj(np, 1);
         std::vector<std::vector<int64_t>> keys(np);
         std::vector<int> pend_q;
@@ -561,8 +564,18 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 spec.erase(sp);
                 continue;
             }
-            const bool mine = opt.mode != PTAS_MODE_MULTI_PROBE || q == rank;
-            who[q] = opt.mode == PTAS_MODE_MULTI_PROBE ? q : rank;
+            // MULTI_PROBE: rank q evaluates probe q, unless an earlier probe of the round
+            // has the same DP key (then that rank's result serves both: one DP per key)
+            int src = q;
+            if (opt.mode == PTAS_MODE_MULTI_PROBE)
+                for (int q2 = 0; q2 < q; ++q2)
+                    if (keys[q2] == keys[q]) {
+                        src = q2;
+                        break;
+                    }
+            xsrc[q] = src;
+            const bool mine = opt.mode != PTAS_MODE_MULTI_PROBE || (q == rank && src == q);
+            who[q] = opt.mode == PTAS_MODE_MULTI_PROBE ? src : rank;
             if (!mine) {
                 optj[q] = -1;  // filled by the exchange
                 continue;
@@ -586,6 +599,12 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 continue;
             }
             rc = run(cl, Tj[q], opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, &optj[q]);
+            if (rc && opt.mode == PTAS_MODE_MULTI_PROBE) {
+                // every rank must still reach the exchange: the error travels with it
+                optj[q] = XERR + rc;
+                slot_key[0].clear();
+                continue;
+            }
             if (rc) return rc;
             slot_key[0] = keys[q];
             if (opt.memoize) memo[keys[q]] = optj[q];
@@ -599,27 +618,33 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 for (size_t jj = 0; jj < pend_key.size(); ++jj) memo[pend_key[jj]] = pend_opt[jj];
         }
         if (opt.mode == PTAS_MODE_MULTI_PROBE) {
-            // exchange OPT(N) of every rank's probe (int32 per rank) over NCCL
-            std::vector<int32_t> mine(1, -1), all(world, -1);
-            if (rank < np) mine[0] = optj[rank];
+            // exchange OPT(N) of every rank's probe (int32 per rank) over NCCL; a
+            // failed DP contributes XERR + its status, and then every rank returns it
+            std::vector<int32_t> all(world, -1);
+            const int32_t mine = rank < np ? optj[rank] : -1;
             int32_t *dbuf = nullptr;
-            if (cudaMalloc(&dbuf, sizeof(int32_t) * world) != cudaSuccess) return PTAS_ENOMEM;
+            int xrc = eng->exchange_buffer(sizeof(int32_t) * world, (void **)&dbuf);
+            if (xrc) return xrc;
             cudaStream_t st = opt.stream ? (cudaStream_t)opt.stream : eng->stream();
-            cudaMemcpyAsync(dbuf + rank, mine.data(), 4, cudaMemcpyHostToDevice, st);
-            int crc = comm_allgather(opt.comm, dbuf + rank, dbuf, 4, st);
-            cudaMemcpyAsync(all.data(), dbuf, 4 * world, cudaMemcpyDeviceToHost, st);
-            cudaError_t ce = eng->sync_spin(st);
-            cudaFree(dbuf);
-            if (crc) return crc;
-            if (ce != cudaSuccess) return PTAS_ECUDA;
+            xrc = eng->s0()->h2d(dbuf + rank, &mine, 4, st) == cudaSuccess ? PTAS_OK : PTAS_ECUDA;
+            if (!xrc) xrc = comm_allgather(opt.comm, dbuf + rank, dbuf, 4, st);
+            if (!xrc && (cudaMemcpyAsync(all.data(), dbuf, 4 * world, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+                         eng->sync_spin(st) != cudaSuccess))
+                xrc = PTAS_ECUDA;
+            if (xrc) return xrc;
             acc.s.h2d_bytes += 4;
             acc.s.d2h_bytes += 4 * world;
-            for (int q = 0; q < np; ++q)
+            for (int q = 0; q < np && q < world; ++q)
+                if (all[q] <= XERR) return all[q] - XERR;
+            for (int q = 0; q < np; ++q) {
                 if (optj[q] < 0) {
-                    optj[q] = all[q];
+                    if (xsrc[q] < 0 || xsrc[q] >= world) return PTAS_EINTERNAL;
+                    optj[q] = all[xsrc[q]];
                     if (optj[q] < 0) return PTAS_EINTERNAL;
                     if (opt.memoize && !keys[q].empty()) memo[keys[q]] = optj[q];
                 }
+                if (xsrc[q] == q && q < world) last_key_of[q] = keys[q];   // rank q holds DP(T_q)
+            }
         }
         std::vector<int32_t> f(np);
         for (int q = 0; q < np; ++q) {
@@ -647,25 +672,71 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     int32_t opt_star = 0;
     if (!cl.N.empty()) {
         std::vector<int64_t> key = memo_key(cl, Ts);
-        int tslot = -1;
-        for (int b = 0; b < MAX_SLOTS; ++b)
-            if (slot_key[b] == key) {
-                tslot = b;
-                break;
-            }
-        if (tslot < 0) {
-            rc = run(cl, Ts, opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, &opt_star);
-            if (rc) return rc;
-            tslot = 0;
-        }
-        DpSlot *tsl = nullptr;
-        rc = eng->slot(tslot, &tsl);
-        if (rc) return rc;
         std::vector<MachineCfg> machines;
         DpOutcome tb;
         const double ttb0 = now_s();
-        rc = tsl->traceback(&machines, &tb);
-        if (rc) return rc;
+        int tslot = -1;
+        // MULTI_PROBE: the traceback runs on ONE rank -- the lowest rank whose last DP
+        // is DP(T*) (every rank knows which rank computed which probe), else rank 0
+        // recomputes it -- and its machine configurations are broadcast
+        const bool mp = opt.mode == PTAS_MODE_MULTI_PROBE;
+        int owner = 0;
+        if (mp)
+            for (int r2 = world - 1; r2 >= 0; --r2)
+                if (last_key_of[r2] == key) owner = r2;
+        if (!mp || rank == owner) {
+            for (int b = 0; b < MAX_SLOTS; ++b)
+                if (slot_key[b] == key) {
+                    tslot = b;
+                    break;
+                }
+            int trc = PTAS_OK;
+            if (tslot < 0) {
+                DpOutcome ro;
+                std::vector<int> order = choose_order(cl.N, cl.r, opt.layout);
+                DpRequest rq = make_rq(cl, Ts, opt.mode == PTAS_MODE_LEVEL_SHARDED ? shp : nullptr, order,
+                                       (cudaStream_t)opt.stream);
+                trc = eng->run_dp(rq, &ro);
+                // a recomputation of a DP the search already ran: time, not new work
+                acc.s.kernel_launches += ro.launches;
+                acc.s.h2d_bytes += ro.h2d;
+                acc.s.d2h_bytes += ro.d2h;
+                tslot = 0;
+            }
+            DpSlot *tsl = nullptr;
+            if (!trc) trc = eng->slot(tslot, &tsl);
+            if (!trc) trc = tsl->traceback(&machines, &tb);
+            if (trc && !mp) return trc;
+            if (trc) machines.clear(), opt_star = XERR + trc;
+            else opt_star = (int32_t)machines.size();
+        }
+        if (mp) {
+            const int Kc = (int)cl.N.size();
+            std::vector<int32_t> buf(1 + (size_t)m * Kc, 0);
+            buf[0] = opt_star;
+            for (size_t mu = 0; mu < machines.size() && (int)mu < m; ++mu)
+                std::copy(machines[mu].begin(), machines[mu].end(), buf.begin() + 1 + mu * Kc);
+            int32_t *dbuf = nullptr;
+            int xrc = eng->exchange_buffer(buf.size() * 4, (void **)&dbuf);
+            if (xrc) return xrc;
+            cudaStream_t st = opt.stream ? (cudaStream_t)opt.stream : eng->stream();
+            if (cudaMemcpyAsync(dbuf, buf.data(), buf.size() * 4, cudaMemcpyHostToDevice, st) != cudaSuccess)
+                return PTAS_ECUDA;
+            xrc = comm_broadcast(opt.comm, dbuf, buf.size() * 4, owner, st);
+            if (xrc) return xrc;
+            if (cudaMemcpyAsync(buf.data(), dbuf, buf.size() * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+                eng->sync_spin(st) != cudaSuccess)
+                return PTAS_ECUDA;
+            if (buf[0] <= XERR) return buf[0] - XERR;
+            if (buf[0] < 0 || buf[0] > m) return PTAS_EINTERNAL;
+            machines.assign((size_t)buf[0], MachineCfg(Kc));
+            for (int32_t mu = 0; mu < buf[0]; ++mu)
+                std::copy(buf.begin() + 1 + (size_t)mu * Kc, buf.begin() + 1 + (size_t)(mu + 1) * Kc, machines[mu].begin());
+            if (rank != owner) {
+                acc.s.h2d_bytes += (int64_t)buf.size() * 4;
+                acc.s.d2h_bytes += (int64_t)buf.size() * 4;
+            }
+        }
         if (std::getenv("PTAS_TRACE"))
             std::fprintf(stderr, "[ptas] traceback at T*=%lld: %zu machines, %.3f ms (slot %d)\n", (long long)Ts,
                          machines.size(), 1e3 * (now_s() - ttb0), tslot);
@@ -756,6 +827,7 @@ void ptas_default_options(ptas_options *o)
     o->layout = 0;
     o->stream = nullptr;
     o->speculate = -1;
+    o->shard_min_rows = -1;
 }
 
 const char *ptas_strerror(int s)
@@ -830,6 +902,17 @@ int ptas_table_order(const int32_t *counts, const int64_t *sizes, int32_t K, int
     return PTAS_OK;
 }
 
+int ptas_level_shard(int64_t rows, int32_t rank, int32_t world, int64_t row_bytes, int64_t *begin, int64_t *end,
+                     int64_t *chunk_out)
+{
+    if (rows < 0 || world < 1 || rank < 0 || rank >= world || row_bytes < 1 || !begin || !end) return PTAS_EINVAL;
+    const int64_t chunk = shard_chunk(rows, world, row_bytes);
+    *begin = std::min<int64_t>(rows, (int64_t)rank * chunk);
+    *end = std::min<int64_t>(rows, *begin + chunk);
+    if (chunk_out) *chunk_out = chunk;
+    return PTAS_OK;
+}
+
 int ptas_shard_range(int64_t count, int32_t rank, int32_t world, int64_t *begin, int64_t *end)
 {
     if (count < 0 || world < 1 || rank < 0 || rank >= world || !begin || !end) return PTAS_EINVAL;
@@ -865,9 +948,12 @@ int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps, cons
     if (rc) return rc;
     std::vector<int64_t> hp(n);
     std::vector<int32_t> ha(n);
+    // d_p / d_assignment are read / written on options.stream, or on the legacy
+    // default stream when it is NULL (ptas.h): ordered after the work that made p
+    // and before the caller's later work on that stream
     {
         std::lock_guard<std::mutex> lk(eng->mu);
-        cudaStream_t st = (opt && opt->stream) ? (cudaStream_t)opt->stream : eng->stream();
+        cudaStream_t st = (opt && opt->stream) ? (cudaStream_t)opt->stream : cudaStreamLegacy;
         if (cudaMemcpyAsync(hp.data(), d_p, (size_t)n * 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
             eng->sync_spin(st) != cudaSuccess) {
             cudaGetLastError();
@@ -878,7 +964,7 @@ int ptas_solve_device(const int64_t *d_p, int32_t n, int32_t m, double eps, cons
                     (int64_t)n * 4, (int64_t)n * 8);
     if (rc) return rc;
     std::lock_guard<std::mutex> lk(eng->mu);
-    cudaStream_t st = (opt && opt->stream) ? (cudaStream_t)opt->stream : eng->stream();
+    cudaStream_t st = (opt && opt->stream) ? (cudaStream_t)opt->stream : cudaStreamLegacy;
     if (cudaMemcpyAsync(d_assignment, ha.data(), (size_t)n * 4, cudaMemcpyHostToDevice, st) != cudaSuccess ||
         eng->sync_spin(st) != cudaSuccess) {
         cudaGetLastError();
@@ -1032,8 +1118,10 @@ int dp_fill_device(const int32_t *counts, const int64_t *sizes, int32_t K, int64
                    int64_t table_bytes, void *cuda_stream, int32_t *opt_N_out)
 {
     if (!d_table) return PTAS_EINVAL;
-    return dp_fill_common(counts, sizes, K, T, d_table, table_bytes, (cudaStream_t)cuda_stream,
-                          nullptr, 0, opt_N_out, nullptr);
+    // NULL = the legacy default stream (ptas.h): ordered after the caller's work on it
+    return dp_fill_common(counts, sizes, K, T, d_table, table_bytes,
+                          cuda_stream ? (cudaStream_t)cuda_stream : cudaStreamLegacy, nullptr, 0, opt_N_out,
+                          nullptr);
 }
 
 int dp_configs(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int32_t *out_digits,

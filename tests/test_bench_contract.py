@@ -33,4 +33,4 @@ def test_reference_arm_torchrun_world2():
         assert key in d
     assert d["value"] > 0 and d["cpu_baseline"]["value"] == d["value"]
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["gpu_launches"] == 0
-    assert d["config"]["workload"] == "M2s"
+    assert d["config"]["workload"] == "M4x"   # N > 1: north_star's scaling instance

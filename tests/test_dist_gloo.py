@@ -8,10 +8,10 @@ the protocol each rank executes around it, with the library's own host steps:
   only probe j == rank (here with the oracle's DP: test infrastructure),
   exchanges OPT(N) with an all-gather, and applies ptas_interval_update.  The
   result must equal the single-process oracle run with P = world.
-* level sharding (LEVEL_SHARDED): each rank takes its
-  ptas_shard_range slice of every row-level, "computes" it (row ids), the
-  slices are all-gathered with the equal-count padding the engine uses, and
-  the scattered result must cover every row exactly once.
+* level sharding (LEVEL_SHARDED): each rank takes the
+  engine's aligned slice (ptas_level_shard) of every row-level, "computes" it
+  (row ids), the slices are all-gathered with the equal-count padding the
+  engine uses, and the scattered result must cover every row exactly once.
 """
 from __future__ import annotations
 
@@ -89,24 +89,28 @@ def multisection_rank(rank, world):
 
 
 def sharding_rank(rank, world):
+    """The engine's own split of a row-level (ptas_level_shard, dp_engine.cpp): rank
+    g fills rows [b, e) of the level into its compact slice of `chunk` rows of
+    row_bytes bytes (16-byte aligned, padded to equal counts), the slices are
+    all-gathered in rank order, and the scatter reads slot s at s * row_bytes:
+    every row must arrive exactly once, from its owner."""
     import paper_conf_ipps_ligsg18_b200 as P
     rng = np.random.default_rng(3)
     ok = True
-    for _ in range(20):
+    for _ in range(40):
         R = int(rng.integers(1, 500))
-        W = int(rng.integers(1, 40))
-        b, e = P.ptas_shard_range(R, rank, world)
-        chunk = -(-R // world)
-        # the engine computes rows [b, e) into a compact slice of `chunk` rows (padded)
-        mine = torch.full((chunk * W,), -1, dtype=torch.int64)
+        row_bytes = int(rng.integers(1, 80))
+        b, e, chunk = P.ptas_level_shard(R, rank, world, row_bytes)
+        ok &= (chunk * row_bytes) % 16 == 0 and chunk >= -(-R // world)
+        ok &= b == min(R, rank * chunk) and e == min(R, b + chunk)
+        mine = torch.full((chunk * row_bytes,), -1, dtype=torch.int64)
         for s in range(b, e):
-            mine[(s - b) * W:(s - b + 1) * W] = s
-        gathered = [torch.empty(chunk * W, dtype=torch.int64) for _ in range(world)]
+            mine[(s - b) * row_bytes:(s - b + 1) * row_bytes] = s
+        gathered = [torch.empty(chunk * row_bytes, dtype=torch.int64) for _ in range(world)]
         dist.all_gather(gathered, mine)
         flat = torch.cat(gathered)
-        # scatter: slot s lives at flat[s * W : (s + 1) * W] when ranks own contiguous equal chunks
         for s in range(R):
-            ok &= bool((flat[s * W:(s + 1) * W] == s).all())
+            ok &= bool((flat[s * row_bytes:(s + 1) * row_bytes] == s).all())
     return ok
 
 

@@ -1,18 +1,30 @@
 """The real NCCL code path on the one GPU a round has: a world-size-1 NCCL
 communicator created through torch.distributed (unique-id broadcast) drives
-the LEVEL_SHARDED mode (per-row-level compact slice -> ncclAllGather ->
-scatter) and the MULTI_PROBE mode (per-round OPT(N) exchange).  Results must
-equal the single-GPU solve bit for bit (determinism across modes, §8(b))."""
+
+* LEVEL_SHARDED with shard_min_rows = 0: EVERY row-level goes through the
+  sharded path -- fill of the rank's aligned slice (ptas_level_shard) into the
+  compact stage buffer, ncclAllGather, row_scatter into the table -- plus the
+  admission agreement (ncclAllReduce of the status word) before the first
+  collective;
+* MULTI_PROBE: per-round OPT(N) exchange (ncclAllGather) and the traceback on
+  the owning rank with its machine configurations broadcast (ncclBroadcast).
+
+Results are compared with the ORACLE (goldens written by
+scripts/make_shaped_goldens.py from oracle/ only, and live oracle runs), not
+with the single-GPU solve."""
 from __future__ import annotations
 
+import json
 import os
 import socket
 
 import pytest
 
-from synth import jobs
+import oracle
+from synth import WORKLOADS, jobs
 
 pytestmark = pytest.mark.gpu
+GOLD = os.path.join(os.path.dirname(__file__), "golden", "shaped")
 
 
 def _port():
@@ -36,22 +48,51 @@ def comm():
     dist.destroy_process_group()
 
 
-def test_level_sharded_nccl_world1(comm):
+def _cmp(got, want):
+    assert got["T_star"] == want["T_star"]
+    assert got["makespan"] == want["makespan"]
+    assert [int(x) for x in got["assignment"]] == [int(x) for x in want["assignment"]]
+    assert [list(x[:6]) for x in got["probes"]] == [list(x) for x in want["probes"]]
+
+
+def test_level_sharded_every_level_nccl_vs_oracle(comm):
     P, c = comm
-    for seed, (n, m, eps) in enumerate([(60, 14, 0.3), (40, 8, 0.25), (200, 60, 0.3)]):
+    for seed, (n, m, eps) in enumerate([(60, 14, 0.3), (40, 8, 0.25), (50, 10, 0.2)]):
         p = jobs(n, 1000, seed + 2)
-        ref = P.ptas_solve(p, m, eps, P=1)
-        got = P.ptas_solve(p, m, eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c)
-        assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
-        assert (got["assignment"] == ref["assignment"]).all()
-        assert [x[:5] for x in got["probes"]] == [x[:5] for x in ref["probes"]]
+        got = P.ptas_solve(p, m, eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c, shard_min_rows=0)
+        _cmp(got, oracle.ptas(p, m, eps, 1))
+        assert got["stats"]["fill_launches"] > 0
 
 
-def test_multi_probe_nccl_world1(comm):
+@pytest.mark.parametrize("name", ["M2s", "M5s-0.3"])
+def test_level_sharded_shaped_nccl_vs_golden(comm, name):
+    P, c = comm
+    w = WORKLOADS[name]
+    g = json.load(open(os.path.join(GOLD, f"solve_{name}_P1.json")))
+    _cmp(P.ptas_solve(w.p(), w.m, w.eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c, shard_min_rows=0), g)
+
+
+def test_level_sharded_default_threshold_nccl(comm):
+    # default threshold (2048 rows): small levels redundant, large ones sharded
+    P, c = comm
+    w = WORKLOADS["M2s"]
+    g = json.load(open(os.path.join(GOLD, "solve_M2s_P1.json")))
+    _cmp(P.ptas_solve(w.p(), w.m, w.eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c), g)
+
+
+def test_multi_probe_nccl_vs_oracle(comm):
     P, c = comm
     for seed in range(4):
         p = jobs(40, 1000, seed)
-        ref = P.ptas_solve(p, 8, 0.3, P=1)
-        got = P.ptas_solve(p, 8, 0.3, P=1, mode=P.MODE_MULTI_PROBE, comm=c)
-        assert got["T_star"] == ref["T_star"] and got["makespan"] == ref["makespan"]
-        assert (got["assignment"] == ref["assignment"]).all()
+        _cmp(P.ptas_solve(p, 8, 0.3, P=1, mode=P.MODE_MULTI_PROBE, comm=c), oracle.ptas(p, 8, 0.3, 1))
+    w = WORKLOADS["M5s-0.2"]
+    g = json.load(open(os.path.join(GOLD, "solve_M5s-0.2_P1.json")))
+    _cmp(P.ptas_solve(w.p(), w.m, w.eps, P=1, mode=P.MODE_MULTI_PROBE, comm=c), g)
+
+
+def test_level_shard_split_exported(comm):
+    # the exported split is the one the engine uses: aligned, covering, rank 0 owns all at world 1
+    P, _ = comm
+    for R, rb in [(1, 1), (7, 31), (2048, 17), (12345, 612)]:
+        b, e, ch = P.ptas_level_shard(R, 0, 1, rb)
+        assert (b, e) == (0, R) and (ch * rb) % 16 == 0 and ch >= R

@@ -271,6 +271,7 @@ def test_dp_fill_device_torch(P):
     sg, e = P.dp_table_shape(N)
     t = torch.full((sg,), 255, dtype=torch.uint8, device="cuda:0")
     s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())   # the fill above is ordered before the DP
     opt = P.dp_fill_device(N, r, 150, t, stream=s)
     want, _ = oracle.dp(N, r, 150)
     torch.cuda.synchronize()
@@ -377,6 +378,8 @@ def test_solve_device_variant(P):
     import torch
     p = jobs(60, 1000, 9)
     pd = torch.from_numpy(p).cuda()
+    # default stream: p produced by a kernel just before the call (legacy default stream order)
+    pd = (pd * 2) // 2
     ad = torch.zeros(60, dtype=torch.int32, device="cuda")
     got = P.ptas_solve_device(pd, 14, 0.3, ad)
     want = oracle.ptas(p, 14, 0.3, 1)
