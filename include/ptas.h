@@ -80,6 +80,13 @@ typedef struct {
                                    2^d - 1 probes in flight).  The probe
                                    sequence, T* and the schedule are those of
                                    Alg 1 (D8); only time changes.      */
+    int32_t window;             /* level window for feasibility probes (DESIGN.md
+                                   D15): 0 = when a probe's full
+                                   table exceeds the budget (default), 1 = for
+                                   every probe DP, -1 = never.  Only OPT(N) of a
+                                   windowed DP is kept; the schedule's DP at T* is
+                                   always a full table (ETOOBIG if it does not fit) */
+    int32_t pad0_;
     int64_t shard_min_rows;     /* LEVEL_SHARDED with comm: row-levels with fewer
                                    rows are computed redundantly on every rank
                                    (-1 = library default 2048); 0 = shard every
@@ -113,6 +120,10 @@ typedef struct {
                                (CUDA events on one time axis).  Equals
                                fill_seconds when DPs run one at a time; below it
                                when speculative / concurrent DPs overlap       */
+    int32_t window_dps;     /* DPs run in level-window mode (D15)     */
+    int32_t pad_;
+    int64_t dev_bytes_max;  /* largest device memory of one DP: table (or the
+                               window's resident slabs) + row index            */
 } ptas_stats;
 
 typedef struct {
@@ -186,6 +197,28 @@ int dp_table_shape(const int32_t *counts, int32_t K, int64_t *sigma_out,
 int dp_fill(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T,
             void *table_out, int64_t table_bytes, int32_t *opt_N_out,
             ptas_stats *stats);
+
+/* OPT(N) of Eq. 1 only (no table), with the level window of SURVEY.md
+ * §8(f)-2i / DESIGN.md D15 when the full table does not fit: rows whose first
+ * internal class count p0 is >= 1 depend only on the slabs p0 - s0 (1 <= s0 <=
+ * min(N0, T / r0)), so only those slabs are resident (a ring mapped twice in
+ * virtual memory) and the table can exceed the device memory by the factor
+ * (N0 + 1) / (min(N0, T / r0) + 1) ("only the values of the
+ * subproblems in these blocks are needed on the GPU").
+ *   counts, sizes, K, T : as dp_fill (caller order; the library picks the
+ *                         internal order, the result does not depend on it)
+ *   table_budget_bytes  : device bytes the DP may use (0 = free HBM - 2 GiB)
+ *   window              : 0 = only when the full table exceeds the budget,
+ *                         1 = always (when it saves memory), -1 = never
+ *   opt_N_out           : host int32, OPT(counts)
+ *   stats               : nullable (window_dps = 1 when windowed,
+ *                         dev_bytes_max = device bytes used)
+ * EINVAL as dp_fill; ETOOBIG when even the window exceeds the budget, or the
+ * window saves nothing (min(N0, T / r0) >= N0 for every class) and the full
+ * table does not fit. */
+int dp_fill_opt(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T,
+                int64_t table_budget_bytes, int32_t window, int32_t *opt_N_out,
+                ptas_stats *stats);
 
 /* High-multiplicity bin packing on the same level-fill engine (SURVEY.md
  * §8(f)-4; the paper's future work on other higher-dimensional DPs,

@@ -13,7 +13,7 @@ import numpy as np
 from ._native import (MODE_LEVEL_SHARDED, MODE_MULTI_PROBE, MODE_SINGLE, EXPORTS, PtasError, PtasOptions,
                       PtasProbe, PtasStats, _a, _chk, _ptr, lib, strerror)
 
-__all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
+__all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_opt", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
            "dp_row_index", "ptas_k", "ptas_bounds", "ptas_classify", "ptas_probe_targets",
            "ptas_interval_update", "ptas_shard_range", "ptas_level_shard", "ptas_table_order", "Comm", "init_comm", "options", "lib", "strerror",
            "PtasError", "EXPORTS", "MODE_SINGLE", "MODE_LEVEL_SHARDED", "MODE_MULTI_PROBE"]
@@ -21,7 +21,7 @@ __all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_device", "hmbp
 
 def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, budget: int = 0,
             memoize: bool = True, virtual_shards: int = 1, layout: int = 0, stream=None,
-            speculate: int = -1, shard_min_rows: int = -1) -> PtasOptions:
+            speculate: int = -1, shard_min_rows: int = -1, window: int = 0) -> PtasOptions:
     o = PtasOptions()
     lib().ptas_default_options(ctypes.byref(o))
     o.probes_per_round = int(P)
@@ -34,6 +34,7 @@ def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, bu
     o.layout = int(layout)
     o.speculate = int(speculate)
     o.shard_min_rows = int(shard_min_rows)
+    o.window = int(window)
     o.stream = None if stream is None else ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
     return o
 
@@ -98,6 +99,18 @@ def dp_fill(counts, sizes, T: int, table: bool = True):
     if table:
         out = out.reshape(tuple(int(x) + 1 for x in c)) if len(c) else out.reshape(())
     return opt.value, out, st.to_dict()
+
+
+def dp_fill_opt(counts, sizes, T: int, budget: int = 0, window: int = 0):
+    """OPT(N) only, with the level window when the table exceeds `budget` bytes
+    (window=1: always, -1: never).  Returns (opt, stats)."""
+    c = _a(counts, np.int32)
+    s = _a(sizes, np.int64)
+    opt = ctypes.c_int32()
+    st = PtasStats()
+    _chk("dp_fill_opt", lib().dp_fill_opt(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), len(c), int(T),
+                                          int(budget), int(window), ctypes.byref(opt), ctypes.byref(st)))
+    return opt.value, st.to_dict()
 
 
 def hmbp_solve(counts, sizes, capacity: int, packing: bool = True):

@@ -27,7 +27,8 @@ class PtasOptions(ctypes.Structure):
     _fields_ = [("probes_per_round", ctypes.c_int32), ("mode", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("comm", vp), ("table_budget_bytes", ctypes.c_int64), ("memoize", ctypes.c_int32),
                 ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32), ("stream", vp),
-                ("speculate", ctypes.c_int32), ("shard_min_rows", ctypes.c_int64)]
+                ("speculate", ctypes.c_int32), ("window", ctypes.c_int32), ("pad0_", ctypes.c_int32),
+                ("shard_min_rows", ctypes.c_int64)]
 
 
 class PtasStats(ctypes.Structure):
@@ -39,7 +40,8 @@ class PtasStats(ctypes.Structure):
                 ("kernel_launches", ctypes.c_int32), ("fill_launches", ctypes.c_int32),
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64), ("relax_executed", ctypes.c_double),
                 ("exec_bytes", ctypes.c_double), ("spec_dps", ctypes.c_int32), ("spec_wasted", ctypes.c_int32),
-                ("fill_wall_seconds", ctypes.c_double)]
+                ("fill_wall_seconds", ctypes.c_double), ("window_dps", ctypes.c_int32), ("pad_", ctypes.c_int32),
+                ("dev_bytes_max", ctypes.c_int64)]
 
     def to_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -55,7 +57,7 @@ EXPORTS = [
     "ptas_default_options", "ptas_solve", "ptas_solve_ex", "ptas_solve_device", "dp_table_shape", "dp_fill",
     "dp_fill_device", "ptas_get_unique_id", "ptas_comm_init", "ptas_comm_destroy", "ptas_strerror", "ptas_k",
     "ptas_bounds", "ptas_classify", "ptas_probe_targets", "ptas_interval_update", "ptas_shard_range",
-    "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order", "ptas_level_shard",
+    "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order", "ptas_level_shard", "dp_fill_opt",
 ]
 
 _lib = None
@@ -100,6 +102,8 @@ def lib():
     L.ptas_shard_range.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, i64p, i64p]
     L.ptas_level_shard.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, i64p, i64p, i64p]
     L.dp_configs.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, ctypes.c_int64, i64p]
+    L.dp_fill_opt.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, i32p,
+                              ctypes.POINTER(PtasStats)]
     L.hmbp_solve.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, i32p, ctypes.c_int32,
                              ctypes.POINTER(PtasStats)]
     L.ptas_table_order.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int32, i32p, i32p]

@@ -19,6 +19,8 @@
 #include <map>
 #include <numeric>
 
+#include <cuda.h>
+
 #include "engine.h"
 
 namespace ptas {
@@ -179,6 +181,85 @@ int64_t DpSlot::free_budget()
     return b > 0 ? b : 0;
 }
 
+// ---- level-window ring (D15): `phys` bytes of device memory mapped
+// twice, back to back, into one 2 * phys virtual range (CUDA virtual memory
+// management, driver entry points fetched through the runtime), so a slab at
+// ring position Rw + (p0 mod Rw) sees the slabs p0 - s0 (s0 <= hi0 < Rw) at plain
+// negative offsets -- the fill kernels address the window as an ordinary table.
+namespace {
+struct VmmApi {
+    bool ok = false;
+    decltype(&cuMemGetAllocationGranularity) gran = nullptr;
+    decltype(&cuMemCreate) create = nullptr;
+    decltype(&cuMemRelease) release = nullptr;
+    decltype(&cuMemAddressReserve) reserve = nullptr;
+    decltype(&cuMemAddressFree) addr_free = nullptr;
+    decltype(&cuMemMap) map = nullptr;
+    decltype(&cuMemUnmap) unmap = nullptr;
+    decltype(&cuMemSetAccess) access = nullptr;
+};
+VmmApi *vmm()
+{
+    static VmmApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        auto get = [](const char *n, void **f) {
+            cudaDriverEntryPointQueryResult q;
+            return cudaGetDriverEntryPoint(n, f, cudaEnableDefault, &q) == cudaSuccess &&
+                   q == cudaDriverEntryPointSuccess && *f;
+        };
+        api.ok = get("cuMemGetAllocationGranularity", (void **)&api.gran) && get("cuMemCreate", (void **)&api.create) &&
+                 get("cuMemRelease", (void **)&api.release) && get("cuMemAddressReserve", (void **)&api.reserve) &&
+                 get("cuMemAddressFree", (void **)&api.addr_free) && get("cuMemMap", (void **)&api.map) &&
+                 get("cuMemUnmap", (void **)&api.unmap) && get("cuMemSetAccess", (void **)&api.access);
+        cudaGetLastError();
+    });
+    return &api;
+}
+}  // namespace
+
+int DpSlot::ring_ensure(size_t phys_bytes, size_t *granularity)
+{
+    VmmApi *a = vmm();
+    if (!a->ok) return PTAS_ECUDA;
+    CUmemAllocationProp prop = {};
+    prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+    prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    prop.location.id = device_;
+    size_t gran = 0;
+    if (a->gran(&gran, &prop, CU_MEM_ALLOC_GRANULARITY_MINIMUM) != CUDA_SUCCESS || gran == 0) return PTAS_ECUDA;
+    *granularity = gran;
+    if (phys_bytes == 0) return PTAS_OK;   // granularity query only
+    if (ring_.va && ring_.phys == phys_bytes) return PTAS_OK;
+    if (ring_.va) {   // release the previous ring (different size)
+        a->unmap((CUdeviceptr)ring_.va, 2 * ring_.phys);
+        a->addr_free((CUdeviceptr)ring_.va, 2 * ring_.phys);
+        a->release((CUmemGenericAllocationHandle)ring_.handle);
+        ring_ = Ring();
+    }
+    CUmemGenericAllocationHandle h;
+    if (a->create(&h, phys_bytes, &prop, 0) != CUDA_SUCCESS) return PTAS_ENOMEM;
+    CUdeviceptr va = 0;
+    if (a->reserve(&va, 2 * phys_bytes, gran, 0, 0) != CUDA_SUCCESS) {
+        a->release(h);
+        return PTAS_ENOMEM;
+    }
+    CUmemAccessDesc acc = {};
+    acc.location = prop.location;
+    acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+    if (a->map(va, phys_bytes, 0, h, 0) != CUDA_SUCCESS || a->map(va + phys_bytes, phys_bytes, 0, h, 0) != CUDA_SUCCESS ||
+        a->access(va, 2 * phys_bytes, &acc, 1) != CUDA_SUCCESS) {
+        a->unmap(va, 2 * phys_bytes);
+        a->addr_free(va, 2 * phys_bytes);
+        a->release(h);
+        return PTAS_ENOMEM;
+    }
+    ring_.va = (unsigned long long)va;
+    ring_.phys = phys_bytes;
+    ring_.handle = (unsigned long long)h;
+    return PTAS_OK;
+}
+
 static int bits_of(int32_t x)
 {
     int b = 0;
@@ -335,6 +416,44 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     g.blk = (int32_t *)blk_.p;   // pivot blocks, written by build_prefix_kernel (D13)
     const int64_t rows = sigma / g.W;
     const int64_t ibytes = rows * g.Wp * e;  // padded internal table
+    // ---- level window (D15): rows with p0 >= 1 depend only on slabs
+    // p0 - s0, 1 <= s0 <= hi0 (their pivot is digit 0, D13), so slab p0 = 1 .. N0 is
+    // ONE launch over all its rows and only Rw = hi0 + 1 slabs are resident: a ring
+    // of Rw slabs mapped twice in virtual memory; slab 0 (p0 = 0) is the DP of the
+    // other classes, filled level by level from its own row index
+    const int32_t hi0w = K >= 2 ? (int32_t)std::min<int64_t>(N[0], rq.T / r[0]) : 0;
+    const bool window = rq.window && K >= 2 && !rq.ext_table && !rq.shard && hi0w < N[0];
+    if (rq.window && !window) return PTAS_ETOOBIG;   // no saving possible: the caller falls back
+    RowGeom gidx;                                     // row index geometry (window: slab 0's rows)
+    std::vector<int64_t> cnt_sub, stride_sub;
+    int64_t rows_idx = rows, slab_bytes = 0, Rw = 0;
+    size_t gran = 0;
+    if (window) {
+        std::vector<int32_t> Nsub(N.begin() + 1, N.end());
+        if (Nsub.size() == 1) {   // K = 2: slab 0 is one row
+            cnt_sub.assign(1, 1);
+            std::memset(&gidx, 0, sizeof(gidx));
+        } else {
+            rc = build_geom(Nsub, e, true, &gidx, &cnt_sub, &stride_sub);
+            if (rc) return rc;
+        }
+        rows_idx = sigma / (N[0] + 1) / g.W;
+        // the row index of slab 0 in the FULL layout: digits 1 .. K-2 with the full
+        // strides and the full digit packing (digit 0 = 0)
+        for (int i = 0; i + 1 < K - 1; ++i) {
+            gidx.stride[i] = g.stride[i + 1];
+            gidx.word[i] = g.word[i + 1];
+            gidx.shift[i] = g.shift[i + 1];
+        }
+        gidx.nwords = g.nwords;
+        Rw = hi0w + 1;
+        rc = ring_ensure(0, &gran);
+        if (rc) return rc;
+        slab_bytes = (rows_idx * g.Wp * e + (int64_t)gran - 1) / (int64_t)gran * (int64_t)gran;
+        stride[0] = slab_bytes / e;
+        g.stride[0] = stride[0];
+        g.span_words = 2 * Rw * slab_bytes / 4;
+    }
     // level sharding over the ranks of a communicator
     int G = 1, myrank = 0;
     bool virt = false;
@@ -363,7 +482,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // agrees on the outcome over all ranks (min of the status words) before any
     // collective, so no rank returns while its peers wait in an all-gather
     int adm = PTAS_OK;
-    if (!in_place) {
+    if (window) {
+        const int64_t need = Rw * slab_bytes + rows_idx * 8 * (1 + (g.nwords <= 1 ? 1 : 2));
+        const int64_t budget = rq.budget > 0 ? rq.budget : free_budget() + (int64_t)ring_.phys;
+        if (need > budget) adm = PTAS_ETOOBIG;
+        else adm = ring_ensure((size_t)(Rw * slab_bytes), &gran);
+        o.dev_bytes = need;
+    } else if (!in_place) {
         // auto budget: query free HBM only when the table has to grow
         // (cudaMemGetInfo costs ~0.1 ms per call)
         if (rq.budget > 0 || (size_t)ibytes > table_.cap) {
@@ -373,7 +498,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         if (!adm && table_.ensure((size_t)ibytes) != cudaSuccess) adm = PTAS_ENOMEM;
     }
     const int NWk = g.nwords <= 1 ? 1 : 2;
-    if (!adm && rowidx_.ensure((size_t)rows * 8 * (1 + NWk)) != cudaSuccess) adm = PTAS_ENOMEM;
+    if (!adm && rowidx_.ensure((size_t)rows_idx * 8 * (1 + NWk)) != cudaSuccess) adm = PTAS_ENOMEM;
     if (!adm && stage_bytes && stage_.ensure(stage_bytes) != cudaSuccess) adm = PTAS_ENOMEM;
     if (comm_dp) {
         if (xch_.ensure(64) != cudaSuccess) return PTAS_ENOMEM;   // (64 B: never fails after the first DP)
@@ -388,9 +513,18 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     }
     if (adm) return adm;
     table = in_place ? rq.ext_table : table_.p;
+    if (!window) o.dev_bytes = ibytes + rows * 8 * (1 + NWk);
     PT_CK(cudaEventRecord(ev_[0], st));
     int64_t idxN = N[K - 1];
     for (int i = 0; i < K - 1; ++i) idxN += (int64_t)N[i] * stride[i];
+    // window: ring position of slab p0 is Rw + (p0 mod Rw) (slabs), relative to the ring
+    auto slab_ptr = [&](int64_t p0) {
+        return (void *)((unsigned char *)(uintptr_t)ring_.va + (Rw + p0 % Rw) * slab_bytes);
+    };
+    if (window) {
+        table = slab_ptr(0);
+        idxN = (Rw + N[0] % Rw) * stride[0] + (idxN - (int64_t)N[0] * stride[0]);   // relative to the ring
+    }
 
     // ---- uploads: r[K] int64 | stride[K] int64 | hi[K] int32, then cnt table
     std::vector<int32_t> hi(K);
@@ -407,13 +541,16 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     std::memcpy(small.data() + K * 16, hi.data(), (size_t)K * 4);
     // one upload (one API call): [r | stride | hi] (8-byte padded), then the
     // cnt table and level_start[rho_max + 2] (prefix sums of the row counts)
-    std::vector<int64_t> lstart((size_t)g.rho_max + 2, 0);
-    for (int rho = 0; rho <= g.rho_max; ++rho) lstart[rho + 1] = lstart[rho] + cnt[rho];
-    const size_t cnt_words = cnt.size() + lstart.size();
+    // (window: the row index covers slab 0's rows, i.e. the levels of the other classes)
+    const std::vector<int64_t> &cntU = window ? cnt_sub : cnt;
+    const int rho_maxU = window ? (K >= 3 ? gidx.rho_max : 0) : g.rho_max;
+    std::vector<int64_t> lstart((size_t)rho_maxU + 2, 0);
+    for (int rho = 0; rho <= rho_maxU; ++rho) lstart[rho + 1] = lstart[rho] + cntU[rho];
+    const size_t cnt_words = cntU.size() + lstart.size();
     const size_t small_pad = (small_bytes + 7) & ~(size_t)7;
     small.resize(small_pad + cnt_words * 8, 0);
-    std::memcpy(small.data() + small_pad, cnt.data(), cnt.size() * 8);
-    std::memcpy(small.data() + small_pad + cnt.size() * 8, lstart.data(), lstart.size() * 8);
+    std::memcpy(small.data() + small_pad, cntU.data(), cntU.size() * 8);
+    std::memcpy(small.data() + small_pad + cntU.size() * 8, lstart.data(), lstart.size() * 8);
     PT_CK(cnt_.ensure(small.size()));
     pin_reset();
     PT_CK(h2d(cnt_.p, small.data(), small.size(), st));
@@ -422,7 +559,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     const int64_t *d_cnt = (const int64_t *)((unsigned char *)cnt_.p + small_pad);
     // ---- a-4 level-ordered row index (row base + packed leading digits per row)
     int64_t *d_rb = (int64_t *)rowidx_.p;
-    uint64_t *d_pw = (uint64_t *)(d_rb + rows);
+    uint64_t *d_pw = (uint64_t *)(d_rb + rows_idx);
     // on the side stream: overlaps the enumeration below and its host round trip
     // (PTAS_ROWIDX_MAIN=1: on the DP's own stream, three API calls fewer)
     const char *rim = std::getenv("PTAS_ROWIDX_MAIN");
@@ -431,7 +568,8 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         PT_CK(cudaEventRecord(ev_fork_, st));
         PT_CK(cudaStreamWaitEvent(side_, ev_fork_, 0));
     }
-    PT_CK(launch_build_row_index(g, d_cnt, d_cnt + cnt.size(), rows, d_rb, d_pw, ri_main ? st : side_));
+    PT_CK(launch_build_row_index(window ? gidx : g, d_cnt, d_cnt + cntU.size(), rows_idx, d_rb, d_pw,
+                                 ri_main ? st : side_));
     if (!ri_main) PT_CK(cudaEventRecord(ev_join_, side_));
     ++o.launches;
     const int64_t *d_r = (const int64_t *)d_small;
@@ -539,13 +677,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         const uint64_t *pwl = d_pw + lstart[rho_];
         cudaError_t err = cudaErrorNotSupported;
         if (!force_scalar) {
-            err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
+            err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows_idx, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
                                        j0, rho_, b, c, compact, sm_count_, st, (use_pdl && prev_fill) ? 1 : 0,
                                        cpref_ok ? index_ : -1);
             if (err == cudaSuccess) prev_fill = true;
         }
         if (err == cudaErrorNotSupported && compact == nullptr && (force_long || !force_scalar)) {
-            err = launch_row_fill_long(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
+            err = launch_row_fill_long(e, tab, gg, rbl, pwl, rows_idx, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
                                        j0, rho_, b, c, sm_count_, st);
             if (err == cudaSuccess) {
                 prev_fill = false;
@@ -554,7 +692,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             if (err == cudaErrorInvalidValue) err = cudaErrorNotSupported;
         }
         if (err == cudaErrorNotSupported) {
-            err = launch_row_fill(e, tab, gg, rbl, pwl, rows, (const PrefixEntry *)pref_.p, d_meta_, nP_bound, j0,
+            err = launch_row_fill(e, tab, gg, rbl, pwl, rows_idx, (const PrefixEntry *)pref_.p, d_meta_, nP_bound, j0,
                                   rho_, b, c, compact, sm_count_, st);
             prev_fill = false;
             used_scalar = true;
@@ -585,7 +723,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     std::vector<DfRun> runs;
     // narrow K = 3 DPs: the whole fill on one thread-block cluster, recent levels
     // in distributed shared memory (row_ring.cu, D14); PTAS_RING=0: off
-    const bool ring = G == 1 && !comm_dp && !force_scalar && K == 3 &&
+    const bool ring = G == 1 && !comm_dp && !window && !force_scalar && K == 3 &&
                       launch_row_fill_ring(e, table, g, N.data(), r.data(), rq.T, J0, (const PrefixEntry *)pref_.p,
                                            d_meta_, nP_bound, st, true) == cudaSuccess;
     cudaGetLastError();
@@ -598,7 +736,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                              : (dfr && dfr[0] ? std::atoll(dfr) : (int64_t)2 * 32 * sm_count_);
         // (measured on M2s/M3s/M4s/M5s: 600..8000 within a few %, 2000 best overall)
         const int64_t split_rows = dsr && dsr[0] ? std::atoll(dsr) : 2000;
-        if (df_mode > 0 && G == 1 && !comm_dp && !force_scalar && g.rho_max >= 1) {
+        if (df_mode > 0 && G == 1 && !comm_dp && !window && !force_scalar && g.rho_max >= 1) {
             if (df_mode == 3 || df_mode == 4) {
                 // levels wider than df_rows get a launch of their own (enough rows to fill
                 // the GPU: the flag protocol costs more than the launch boundary saves,
@@ -692,7 +830,26 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                    nP_bound, st, false));
         ++o.fill_launches;
     }
-    for (int rho = 0; rho <= (ring ? -1 : g.rho_max); ++rho) {
+    if (window) {
+        // slab 0: the DP of the other classes, level by level (its rows dominate only
+        // prefixes with s0 = 0); then slabs 1 .. N0, one launch each over all rows
+        for (int rho = 0; rho <= rho_maxU; ++rho) {
+            PT_CK(fill(table, g, J0, rho, 0, cntU[rho], nullptr));
+            ++o.fill_launches;
+        }
+        for (int64_t p0 = 1; p0 <= N[0]; ++p0) {
+            RowGeom gs = g;
+            gs.pw_or[g.word[0]] |= (uint64_t)p0 << g.shift[0];
+            const cudaError_t err = launch_row_fill_swar(e, slab_ptr(p0), gs, d_rb, d_pw, rows_idx,
+                                                         (const PrefixEntry *)pref_.p, d_meta_, nP_bound, J0, 0, 0,
+                                                         rows_idx, nullptr, sm_count_, st, use_pdl ? 1 : 0,
+                                                         cpref_ok ? index_ : -1);
+            if (err == cudaErrorNotSupported) return PTAS_ETOOBIG;   // (rows > 1 KiB: no window)
+            PT_CK(err);
+            ++o.fill_launches;
+        }
+    }
+    for (int rho = 0; rho <= ((ring || window) ? -1 : g.rho_max); ++rho) {
         const int64_t R = cnt[rho];
         if (lvl_times && rho > 0) PT_CK(cudaEventRecord(lev[rho], st));
         if (R <= 0) continue;
@@ -726,7 +883,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                 PT_CK(cudaMemcpyAsync(dfprof_.p, prof_h.data(), prof_h.size() * 8, cudaMemcpyHostToDevice, st));
                 dfa.prof = (unsigned long long *)dfprof_.p;
             }
-            cudaError_t err = launch_row_fill_swar_df(e, table, g, d_rb, d_pw, rows, (const PrefixEntry *)pref_.p,
+            cudaError_t err = launch_row_fill_swar_df(e, table, g, d_rb, d_pw, rows_idx, (const PrefixEntry *)pref_.p,
                                                       d_meta_, nP_bound, J0, rn.max_rows, dfa, &ticket_base_, sm_count_,
                                                       st, (use_pdl && prev_fill) ? 1 : 0, cpref_ok ? index_ : -1);
             if (err == cudaSuccess && df_prof) {
@@ -803,7 +960,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     (void)ld;
 
     // ---- a-6 readout
-    PT_CK(launch_read_opt(e, table, idxN, d_meta_, st));
+    PT_CK(launch_read_opt(e, window ? (void *)(uintptr_t)ring_.va : table, idxN, d_meta_, st));
     ++o.launches;
     if (rq.ext_table && !in_place) {
         PT_CK(launch_compact_rows(e, table, rq.ext_table, rows, g.W, g.Wp, st));
@@ -857,7 +1014,8 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     o.nC = h_meta_->nC;
     o.nP = h_meta_->nP;
 
-    last_valid_ = true;
+    o.windowed = window ? 1 : 0;
+    last_valid_ = !window;   // a window keeps no table for a traceback
     last_table_ = table;
     last_stream_ = st;
     last_K_ = K;

@@ -34,6 +34,9 @@ struct DpRequest {
     cudaStream_t stream = nullptr;  // nullptr = engine stream
     const ShardCtx *shard = nullptr;
     int64_t budget = 0;           // bytes allowed for the table (0 = auto)
+    int window = 0;               // 1: level window (D15): only hi0 + 1 slabs of the
+                                  // first internal digit are resident (a ring mapped twice in
+                                  // virtual memory); OPT(N) only, no table for a traceback
     int grid_div = 1;             // >1: this many DPs run concurrently; persistent grids take 1/grid_div of the GPU
     cudaEvent_t ref_event = nullptr;  // completed timing event: fill interval reported relative to it
 };
@@ -50,6 +53,8 @@ struct DpOutcome {
     double fill_t0 = -1, fill_t1 = -1;   // fill interval in seconds after rq.ref_event (-1: none)
     int launches = 0, fill_launches = 0;
     int64_t h2d = 0, d2h = 0;
+    int windowed = 0;              // the DP ran in level-window mode
+    int64_t dev_bytes = 0;         // device memory of its table (ring) and row index
 };
 
 // one machine of the traceback: canonical digit vector s (length K canonical)
@@ -113,6 +118,13 @@ class DpSlot {
     Buf table_, digits_, off_, counts_, offsets_, pref_, cnt_, stage_, small_, rank_, tb_, rowidx_, cpstage_;
     // dataflow fill (D7): per-row ready flags, ticket counter, run plans
     Buf flags_, ticket_, dfplan_, dfprof_, domtab_, blk_, xch_;
+    // level-window ring (D15): physical slabs mapped twice back to back
+    struct Ring {
+        unsigned long long va = 0;   // CUdeviceptr of the 2 * phys virtual range
+        size_t phys = 0;             // bytes of physical memory (= one mapping)
+        unsigned long long handle = 0;
+    } ring_;
+    int ring_ensure(size_t phys_bytes, size_t *granularity);
     uint32_t df_epoch_ = 0;
     unsigned long long ticket_base_ = 0;
 

@@ -60,6 +60,12 @@ struct RowGeom {
     // build_prefix_kernel.  A row p != 0 walks only the block of its own first
     // nonzero digit.  Empty block: first == end.
     int32_t *blk;               // device [2 * MAXK]
+    // level window (D15): OR-ed into every row's packed digits (the
+    // slab digit p0 of a slab launch whose row index holds the p0 = 0 rows), and
+    // the word span the kernel may address relative to the table pointer
+    // (int32 word offsets; 0 = the whole table)
+    uint64_t pw_or[MAXW];
+    int64_t span_words;
 };
 constexpr int64_t DOMTAB_MAX_BYTES = 16384;
 

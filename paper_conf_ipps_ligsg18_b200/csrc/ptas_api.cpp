@@ -159,6 +159,27 @@ std::vector<int> choose_order(const std::vector<int32_t> &N, const std::vector<i
     return o;
 }
 
+// internal order for a level-window DP (D15): the row class as in
+// layout 0, digit 0 = the class with the most slabs per resident slab,
+// (N + 1) / (min(N, T / r) + 1), the other leading classes by descending size
+std::vector<int> window_order(const std::vector<int32_t> &N, const std::vector<int64_t> &r, int64_t T)
+{
+    std::vector<int> o = choose_order(N, r, 0);
+    if (o.size() < 3) return o;
+    size_t best = 0;
+    double bv = -1;
+    for (size_t i = 0; i + 1 < o.size(); ++i) {
+        const double hi = (double)std::min<int64_t>(N[o[i]], T / r[o[i]]);
+        const double v = (N[o[i]] + 1.0) / (hi + 1.0);
+        if (v > bv) {
+            bv = v;
+            best = i;
+        }
+    }
+    std::rotate(o.begin(), o.begin() + best, o.begin() + best + 1);
+    return o;
+}
+
 double now_s()
 {
     return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
@@ -204,6 +225,8 @@ struct Acc {
         s.h2d_bytes += o.h2d;
         s.d2h_bytes += o.d2h;
         s.sigma_max = std::max(s.sigma_max, o.sigma);
+        s.window_dps += o.windowed;
+        s.dev_bytes_max = std::max(s.dev_bytes_max, o.dev_bytes);
     }
 };
 
@@ -291,6 +314,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
 
     // which slot holds the table of which DP key (for the traceback at T*)
     std::vector<std::vector<int64_t>> slot_key(MAX_SLOTS);
+    int last_windowed = 0;
     auto make_rq = [&](const Classified &c, int64_t T, const ShardCtx *s, const std::vector<int> &order,
                        cudaStream_t st) {
         DpRequest rq;
@@ -305,15 +329,34 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         rq.ref_event = ref_ev;
         return rq;
     };
-    auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
+    // One probe DP on a slot; the level window (D15) when options.window
+    // asks for it or when the full table does not fit (window = 0), single GPU only
+    auto probe_dp = [&](DpSlot *sl, const Classified &c, int64_t T, const ShardCtx *s, cudaStream_t st,
+                        int grid_div, DpOutcome *o) -> int {
+        const bool can_win = opt.window >= 0 && !s && opt.mode == PTAS_MODE_SINGLE;
         std::vector<int> order = choose_order(c.N, c.r, opt.layout);
-        DpRequest rq = make_rq(c, T, s, order, (cudaStream_t)opt.stream);
+        DpRequest rq = make_rq(c, T, s, order, st);
+        rq.grid_div = grid_div;
+        int r2 = PTAS_ETOOBIG;
+        if (!(can_win && opt.window == 1)) r2 = sl->run_dp(rq, o);
+        if (r2 == PTAS_ETOOBIG && can_win) {
+            std::vector<int> worder = window_order(c.N, c.r, T);
+            DpRequest rw = make_rq(c, T, s, worder, st);
+            rw.grid_div = grid_div;
+            rw.window = 1;
+            r2 = sl->run_dp(rw, o);
+            if (r2 == PTAS_ETOOBIG && opt.window == 1) r2 = sl->run_dp(rq, o);   // no saving possible
+        }
+        return r2;
+    };
+    auto run = [&](const Classified &c, int64_t T, const ShardCtx *s, int32_t *opt_out) -> int {
         DpOutcome o;
-        int r2 = eng->run_dp(rq, &o);
+        int r2 = probe_dp(eng->s0(), c, T, s, (cudaStream_t)opt.stream, 1, &o);
         if (r2) return r2;
         acc.add(o);
         acc.s.unique_dps++;
         *opt_out = o.opt;
+        last_windowed = o.windowed;
         return PTAS_OK;
     };
     // Concurrent evaluation of several probes of one round (SINGLE mode): one
@@ -344,15 +387,14 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                     rcs[b] = PTAS_ECUDA;
                     return;
                 }
-                DpRequest rq = make_rq(cls_v[j0 + b], T_v[j0 + b], nullptr, orders[b],
-                                       b == 0 ? (cudaStream_t)opt.stream : nullptr);
                 // PTAS_GRID_DIV (experiment knob): 0 = every launch may take the whole GPU
                 static const int gd_env = [] {
                     const char *t = std::getenv("PTAS_GRID_DIV");
                     return t && t[0] ? std::atoi(t) : -1;
                 }();
-                rq.grid_div = gd_env == 0 ? 1 : (share_grid ? nb : 1);
-                rcs[b] = sl[b]->run_dp(rq, &outs_all[j0 + b]);
+                rcs[b] = probe_dp(sl[b], cls_v[j0 + b], T_v[j0 + b], nullptr,
+                                  b == 0 ? (cudaStream_t)opt.stream : nullptr,
+                                  gd_env == 0 ? 1 : (share_grid ? nb : 1), &outs_all[j0 + b]);
             };
             std::vector<std::thread> th;
             for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
@@ -360,7 +402,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             for (auto &t : th) t.join();
             for (int b = 0; b < nb; ++b) {
                 if (rcs[b]) return rcs[b];
-                slot_key[b] = key_v[j0 + b];
+                slot_key[b] = outs_all[j0 + b].windowed ? std::vector<int64_t>() : key_v[j0 + b];
             }
         }
         return PTAS_OK;
@@ -384,9 +426,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                     rcs[b] = PTAS_ECUDA;
                     return;
                 }
-                DpRequest rq = make_rq(cls_v[j0 + b], T_v[j0 + b], nullptr, orders[b],
-                                       b == 0 ? (cudaStream_t)opt.stream : nullptr);
-                rcs[b] = sl[b]->run_dp(rq, &outs[b]);
+                rcs[b] = probe_dp(sl[b], cls_v[j0 + b], T_v[j0 + b], nullptr,
+                                  b == 0 ? (cudaStream_t)opt.stream : nullptr, 1, &outs[b]);
             };
             std::vector<std::thread> th;
             for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
@@ -397,7 +438,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 acc.add(outs[b]);
                 acc.s.unique_dps++;
                 opt_v[j0 + b] = outs[b].opt;
-                slot_key[b] = key_v[j0 + b];
+                slot_key[b] = outs[b].windowed ? std::vector<int64_t>() : key_v[j0 + b];
             }
         }
         return PTAS_OK;
@@ -606,7 +647,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 continue;
             }
             if (rc) return rc;
-            slot_key[0] = keys[q];
+            slot_key[0] = last_windowed ? std::vector<int64_t>() : keys[q];
             if (opt.memoize) memo[keys[q]] = optj[q];
         }
         if (!pend_q.empty()) {
@@ -828,6 +869,7 @@ void ptas_default_options(ptas_options *o)
     o->stream = nullptr;
     o->speculate = -1;
     o->shard_min_rows = -1;
+    o->window = 0;
 }
 
 const char *ptas_strerror(int s)
@@ -1033,6 +1075,62 @@ static int dp_fill_common(const int32_t *counts, const int64_t *sizes, int32_t K
         if (rc) return rc;
         acc.s.d2h_bytes += sigma * e;
     }
+    *opt_N_out = o.opt;
+    if (stats) {
+        acc.s.unique_dps = 1;
+        acc.s.total_seconds = now_s() - t0;
+        *stats = acc.s;
+    }
+    return PTAS_OK;
+}
+
+int dp_fill_opt(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int64_t table_budget_bytes,
+                int32_t window, int32_t *opt_N_out, ptas_stats *stats)
+{
+    const double t0 = now_s();
+    int rc = validate_dp(counts, sizes, K, T);
+    if (rc) return rc;
+    if (!opt_N_out || window < -1 || window > 1 || table_budget_bytes < 0) return PTAS_EINVAL;
+    int64_t sigma;
+    int32_t e;
+    rc = dp_table_shape(counts, K, &sigma, &e);
+    if (rc) return rc;
+    int dev;
+    rc = resolve_device(-1, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+    const std::vector<int32_t> N(counts, counts + K);
+    const std::vector<int64_t> r(sizes, sizes + K);
+    const std::vector<int> full = choose_order(N, r, 0), win = window_order(N, r, T);
+    DpRequest rq;
+    rq.K = K;
+    rq.N = counts;
+    rq.r = sizes;
+    rq.T = T;
+    rq.budget = table_budget_bytes;
+    DpOutcome o;
+    rc = PTAS_ETOOBIG;
+    if (window <= 0) {
+        rq.order = full.data();
+        rc = eng->run_dp(rq, &o);
+    }
+    if (rc == PTAS_ETOOBIG && window >= 0) {
+        rq.order = win.data();
+        rq.window = 1;
+        rc = eng->run_dp(rq, &o);
+        if (rc == PTAS_ETOOBIG && window == 1) {   // the window saves nothing: full table
+            rq.order = full.data();
+            rq.window = 0;
+            rc = eng->run_dp(rq, &o);
+        }
+    }
+    if (rc) return rc;
+    Acc acc;
+    acc.add(o);
+    acc.s.fill_wall_seconds = o.fill_s;
     *opt_N_out = o.opt;
     if (stats) {
         acc.s.unique_dps = 1;

@@ -322,8 +322,12 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
         const bool rowok = CL ? (grp < rpw && slot < s_sl[CL ? c_lv + 1 : 0]) : (DF ? cur_ok : (grp < rpw && slot < slot_count));
         const int64_t rowbase = nrb;
         uint64_t pw[NW];
+        bool row0 = rowok;   // p = 0 (all leading digits zero)
 #pragma unroll
-        for (int w = 0; w < NW; ++w) pw[w] = npw[w];
+        for (int w = 0; w < NW; ++w) {
+            pw[w] = npw[w] | (rowok ? g.pw_or[w] : 0ull);
+            row0 &= pw[w] == 0;
+        }
         unsigned long long tnext = 0;
         if constexpr (CL) {
             // next set of this warp (possibly levels ahead) and its index entries
@@ -553,7 +557,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
                     oo.v[t] = 0;
                 }
             }
-            if (rowok && rowbase == 0) {   // row p = 0 (once per DP): OPT(0, x) = ceil(x / J0)
+            if (row0) {   // row p = 0 (once per DP): OPT(0, x) = ceil(x / J0)
 #pragma unroll
                 for (int t = 0; t < CH; ++t) {
                     const uint32_t x0 = (uint32_t)(xl * CH + t) * (4 / EB);
@@ -648,7 +652,7 @@ static int plan_ch(int e, const RowGeom &g, int J0, int64_t rows, int sm_count, 
     // int32 word offsets: the table (incl. padding) must stay below 2^31 words
     int64_t rows_all = 1;
     for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
-    if (rows_all * (int64_t)Lw >= ((int64_t)1 << 31)) return 0;
+    if ((g.span_words > 0 ? g.span_words : rows_all * (int64_t)Lw) >= ((int64_t)1 << 31)) return 0;
     int CH;
     const char *chs = std::getenv(df ? "PTAS_DF_CH" : "PTAS_SWAR_CH");
     const char *cht = std::getenv("PTAS_SMALL_LEVEL_ROWS");
