@@ -422,7 +422,10 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // of Rw slabs mapped twice in virtual memory; slab 0 (p0 = 0) is the DP of the
     // other classes, filled level by level from its own row index
     const int32_t hi0w = K >= 2 ? (int32_t)std::min<int64_t>(N[0], rq.T / r[0]) : 0;
-    const bool window = rq.window && K >= 2 && !rq.ext_table && !rq.shard && hi0w < N[0];
+    // (the slabs p0 >= 1 need the packed kernel: rows of at most 1 KiB, window shifts <= 124 B)
+    const int64_t J0w = std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
+    const bool window = rq.window && K >= 2 && !rq.ext_table && (!rq.shard || rq.shard->comm) && hi0w < N[0] &&
+                        g.Wp * e / 4 <= 256 && J0w * e <= 124;
     if (rq.window && !window) return PTAS_ETOOBIG;   // no saving possible: the caller falls back
     RowGeom gidx;                                     // row index geometry (window: slab 0's rows)
     std::vector<int64_t> cnt_sub, stride_sub;
@@ -470,10 +473,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     const bool comm_dp = sh && sh->comm && (G > 1 || sh->force);   // collectives in this DP
     auto sharded = [&](int64_t R) { return (G > 1 || comm_dp) && R >= std::max<int64_t>(sh->min_rows, 1); };
     size_t stage_bytes = 0;
-    for (int rho = 0; rho <= g.rho_max && (G > 1 || comm_dp); ++rho) {
-        const int64_t R = cnt[rho];
-        if (!sharded(R)) continue;
-        stage_bytes = std::max(stage_bytes, (size_t)(shard_chunk(R, G, g.Wp * e) * G * g.Wp * e));
+    {   // the sharded units: row-levels, or (window) slab 0's levels and whole slabs
+        std::vector<int64_t> units = window ? cnt_sub : cnt;
+        if (window) units.push_back(rows_idx);
+        for (int64_t R : units) {
+            if (!(G > 1 || comm_dp) || !sharded(R)) continue;
+            stage_bytes = std::max(stage_bytes, (size_t)(shard_chunk(R, G, g.Wp * e) * G * g.Wp * e));
+        }
     }
     // compute in the caller's buffer when its layout is the padded one
     void *table = nullptr;
@@ -671,10 +677,13 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     bool prev_fill = false;  // the previous launch on st was a packed fill (PDL-safe)
     bool used_scalar = false;  // some level ran on the scalar (uncollapsed) kernel
     // one row-level (or slice of it): packed-word kernel, scalar kernel as fallback
-    auto fill = [&](void *tab, const RowGeom &gg, int j0, int rho_, int64_t b, int64_t c,
+    // one row-level (or slab, or a slice of either): rows [b, b + c) of the row
+    // index from slot idx_off
+    auto fill = [&](void *tab, const RowGeom &gg, int j0, int64_t idx_off, int64_t b, int64_t c,
                     void *compact) -> cudaError_t {
-        const int64_t *rbl = d_rb + lstart[rho_];
-        const uint64_t *pwl = d_pw + lstart[rho_];
+        const int rho_ = 0;   // (unused by the kernels)
+        const int64_t *rbl = d_rb + idx_off;
+        const uint64_t *pwl = d_pw + idx_off;
         cudaError_t err = cudaErrorNotSupported;
         if (!force_scalar) {
             err = launch_row_fill_swar(e, tab, gg, rbl, pwl, rows_idx, (const PrefixEntry *)pref_.p, d_meta_, nP_bound,
@@ -830,23 +839,52 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                    nP_bound, st, false));
         ++o.fill_launches;
     }
+    // one unit (a row-level, or a window slab) of R rows from index slot idx_off into
+    // `tab`: directly, or sharded -- the rank's aligned slice into the compact stage
+    // buffer, ncclAllGather (in place), row_scatter into every rank's table
+    auto fill_unit = [&](void *tab, const RowGeom &gg, int64_t idx_off, int64_t R) -> int {
+        if (!sharded(R)) {
+            PT_CK(fill(tab, gg, J0, idx_off, 0, R, nullptr));
+            ++o.fill_launches;
+            return PTAS_OK;
+        }
+        const int64_t chunk = shard_chunk(R, G, g.Wp * e);
+        unsigned char *stage = (unsigned char *)stage_.p;
+        if (virt) {
+            for (int v = 0; v < G; ++v) {
+                int64_t b = v * chunk, c = std::min(R, b + chunk) - b;
+                if (c <= 0) continue;
+                PT_CK(fill(tab, gg, J0, idx_off, b, c, stage + b * g.Wp * e));
+                ++o.fill_launches;
+            }
+        } else {
+            int64_t b = myrank * chunk, c = std::min(R, b + chunk) - b;
+            if (c > 0) {
+                PT_CK(fill(tab, gg, J0, idx_off, b, c, stage + b * g.Wp * e));
+                ++o.fill_launches;
+            }
+            int crc = comm_allgather(sh->comm, stage + (size_t)myrank * chunk * g.Wp * e, stage,
+                                     (size_t)(chunk * g.Wp * e), st);
+            if (crc) return crc;
+        }
+        PT_CK(launch_row_scatter(e, tab, g, d_rb + idx_off, R, stage, sm_count_, st));
+        prev_fill = false;
+        ++o.launches;
+        return PTAS_OK;
+    };
     if (window) {
         // slab 0: the DP of the other classes, level by level (its rows dominate only
-        // prefixes with s0 = 0); then slabs 1 .. N0, one launch each over all rows
+        // prefixes with s0 = 0); then slabs 1 .. N0, one unit each over all rows
+        // (sharded over the ranks of a communicator: SURVEY.md §8(f)-2ii)
         for (int rho = 0; rho <= rho_maxU; ++rho) {
-            PT_CK(fill(table, g, J0, rho, 0, cntU[rho], nullptr));
-            ++o.fill_launches;
+            const int urc = fill_unit(table, g, lstart[rho], cntU[rho]);
+            if (urc) return urc;
         }
         for (int64_t p0 = 1; p0 <= N[0]; ++p0) {
             RowGeom gs = g;
             gs.pw_or[g.word[0]] |= (uint64_t)p0 << g.shift[0];
-            const cudaError_t err = launch_row_fill_swar(e, slab_ptr(p0), gs, d_rb, d_pw, rows_idx,
-                                                         (const PrefixEntry *)pref_.p, d_meta_, nP_bound, J0, 0, 0,
-                                                         rows_idx, nullptr, sm_count_, st, use_pdl ? 1 : 0,
-                                                         cpref_ok ? index_ : -1);
-            if (err == cudaErrorNotSupported) return PTAS_ETOOBIG;   // (rows > 1 KiB: no window)
-            PT_CK(err);
-            ++o.fill_launches;
+            const int urc = fill_unit(slab_ptr(p0), gs, 0, rows_idx);
+            if (urc) return urc;
         }
     }
     for (int rho = 0; rho <= ((ring || window) ? -1 : g.rho_max); ++rho) {
@@ -912,33 +950,8 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             if (err != cudaErrorNotSupported) PT_CK(err);
             // unsupported geometry: fill the run level by level
         }
-        if (!sharded(R)) {
-            PT_CK(fill(table, g, J0, rho, 0, R, nullptr));
-            ++o.fill_launches;
-            continue;
-        }
-        const int64_t chunk = shard_chunk(R, G, g.Wp * e);
-        unsigned char *stage = (unsigned char *)stage_.p;
-        if (virt) {
-            for (int v = 0; v < G; ++v) {
-                int64_t b = v * chunk, c = std::min(R, b + chunk) - b;
-                if (c <= 0) continue;
-                PT_CK(fill(table, g, J0, rho, b, c, stage + b * g.Wp * e));
-                ++o.fill_launches;
-            }
-        } else {
-            int64_t b = myrank * chunk, c = std::min(R, b + chunk) - b;
-            if (c > 0) {
-                PT_CK(fill(table, g, J0, rho, b, c, stage + b * g.Wp * e));
-                ++o.fill_launches;
-            }
-            int crc = comm_allgather(sh->comm, stage + (size_t)myrank * chunk * g.Wp * e, stage,
-                                     (size_t)(chunk * g.Wp * e), st);
-            if (crc) return crc;
-        }
-        PT_CK(launch_row_scatter(e, table, g, d_rb + lstart[rho], R, stage, sm_count_, st));
-        prev_fill = false;
-        ++o.launches;
+        const int urc = fill_unit(table, g, lstart[rho], R);
+        if (urc) return urc;
     }
     PT_CK(cudaEventRecord(ev_[2], st));
     if (lvl_times && ring) {

@@ -333,7 +333,10 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     // asks for it or when the full table does not fit (window = 0), single GPU only
     auto probe_dp = [&](DpSlot *sl, const Classified &c, int64_t T, const ShardCtx *s, cudaStream_t st,
                         int grid_div, DpOutcome *o) -> int {
-        const bool can_win = opt.window >= 0 && !s && opt.mode == PTAS_MODE_SINGLE;
+        // (level-sharded over a communicator too: the slabs are then the sharded units,
+        // SURVEY.md §8(f)-2ii; every rank takes the same decision: window = 1, or the
+        // ETOOBIG the ranks agreed on at admission)
+        const bool can_win = opt.window >= 0 && (!s || s->comm) && opt.mode != PTAS_MODE_MULTI_PROBE;
         std::vector<int> order = choose_order(c.N, c.r, opt.layout);
         DpRequest rq = make_rq(c, T, s, order, st);
         rq.grid_div = grid_div;

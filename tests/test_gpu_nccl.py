@@ -96,3 +96,16 @@ def test_level_shard_split_exported(comm):
     for R, rb in [(1, 1), (7, 31), (2048, 17), (12345, 612)]:
         b, e, ch = P.ptas_level_shard(R, 0, 1, rb)
         assert (b, e) == (0, R) and (ch * rb) % 16 == 0 and ch >= R
+
+
+@pytest.mark.parametrize("name", ["M2s", "M5s-0.3"])
+def test_window_slabs_sharded_nccl_vs_golden(comm, name):
+    """Level window + level sharding: every probe DP keeps only
+    min(N0, T/r0) + 1 slabs, and every slab (and every level of slab 0) goes through
+    the rank slice -> ncclAllGather -> scatter path; the schedule's DP at T* is full."""
+    P, c = comm
+    w = WORKLOADS[name]
+    g = json.load(open(os.path.join(GOLD, f"solve_{name}_P1.json")))
+    got = P.ptas_solve(w.p(), w.m, w.eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c, shard_min_rows=0, window=1)
+    _cmp(got, g)
+    assert got["stats"]["window_dps"] > 0
