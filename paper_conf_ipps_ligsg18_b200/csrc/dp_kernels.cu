@@ -369,6 +369,9 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
 #pragma unroll
         for (int w = 0; w < NW; ++w) pw[w] = rowok ? pwa[(int64_t)w * pw_stride + slot_begin + slot] : 0;
         if (rowok) rowbase = rb[slot_begin + slot];
+        bool row0 = rowok;   // p = 0 (all leading digits zero): OPT(0) = 0
+#pragma unroll
+        for (int w = 0; w < NW; ++w) row0 &= pw[w] == 0;
         E *out = compact ? compact + slot * g.Wp : table + rowbase;
         for (int64_t x0 = 0; x0 < W; x0 += Wg) {
             const int64_t x = x0 + xl;
@@ -430,7 +433,7 @@ row_fill_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb, const
                     acc = v < acc ? v : acc;
                 }
             }
-            int opt = (rho == 0 && x == 0) ? 0 : acc + 1;
+            int opt = (row0 && x == 0) ? 0 : acc + 1;
             // in-chunk chain: Bellman-Ford over shuffles
             const int jin = J0 < Wg - 1 ? J0 : Wg - 1;
             bool changed = jin > 0;
