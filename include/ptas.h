@@ -220,6 +220,26 @@ int dp_fill_opt(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t 
                 int64_t table_budget_bytes, int32_t window, int32_t *opt_N_out,
                 ptas_stats *stats);
 
+/* The paper's own DP design as an A/B baseline: the
+ * data-partitioning scheme of Alg 4 / Alg 5 --
+ * divisor per dimension (floor(sqrt(n_i + 1)) lowered until it divides n_i + 1,
+ * only the `dim` largest kept), the table reorganised into blocks stored
+ * consecutively, block-levels in order with the blocks of a level
+ * concurrently (one CTA each), in-block anti-diagonal levels in order, every
+ * entry relaxed over every configuration s <= v.  Same values as dp_fill.
+ *   counts, sizes, K (1..16), T : as dp_fill;  dim >= 1 (the paper used 3..9)
+ *   table_out   : host, nullable; row-major in the caller's order (converted
+ *                 back from the blocked layout), table_bytes >= sigma * e
+ *   opt_N_out   : host int32, OPT(counts)
+ *   divisor_out : host int32[K], nullable: the divisor used
+ *   stats       : nullable (fill_seconds = device time of the block-levels,
+ *                 fill_launches = block-levels, relaxations = Eq. 1 count)
+ * Errors as dp_fill; ETOOBIG when a block exceeds 2^31 entries or the
+ * per-CTA tables exceed shared memory. */
+int dp_fill_alg4(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int32_t dim,
+                 void *table_out, int64_t table_bytes, int32_t *opt_N_out, int32_t *divisor_out,
+                 ptas_stats *stats);
+
 /* High-multiplicity bin packing on the same level-fill engine (SURVEY.md
  * §8(f)-4; the paper's future work on other higher-dimensional DPs,
  * PAPER.md:472).  Eq. 1 with T = capacity and r = sizes is

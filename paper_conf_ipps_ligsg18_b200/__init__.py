@@ -13,7 +13,7 @@ import numpy as np
 from ._native import (MODE_LEVEL_SHARDED, MODE_MULTI_PROBE, MODE_SINGLE, EXPORTS, PtasError, PtasOptions,
                       PtasProbe, PtasStats, _a, _chk, _ptr, lib, strerror)
 
-__all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_opt", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
+__all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_opt", "dp_fill_alg4", "dp_fill_device", "hmbp_solve", "dp_table_shape", "dp_configs",
            "dp_row_index", "ptas_k", "ptas_bounds", "ptas_classify", "ptas_probe_targets",
            "ptas_interval_update", "ptas_shard_range", "ptas_level_shard", "ptas_table_order", "Comm", "init_comm", "options", "lib", "strerror",
            "PtasError", "EXPORTS", "MODE_SINGLE", "MODE_LEVEL_SHARDED", "MODE_MULTI_PROBE"]
@@ -111,6 +111,24 @@ def dp_fill_opt(counts, sizes, T: int, budget: int = 0, window: int = 0):
     _chk("dp_fill_opt", lib().dp_fill_opt(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), len(c), int(T),
                                           int(budget), int(window), ctypes.byref(opt), ctypes.byref(st)))
     return opt.value, st.to_dict()
+
+
+def dp_fill_alg4(counts, sizes, T: int, dim: int = 6, table: bool = True):
+    """The paper's Alg 4 partitioned DP (A/B baseline): (opt, table or None, divisor, stats)."""
+    c = _a(counts, np.int32)
+    s = _a(sizes, np.int64)
+    sg, e = dp_table_shape(c)
+    out = np.zeros(sg, np.uint8 if e == 1 else np.uint16) if table else None
+    opt = ctypes.c_int32()
+    dv = np.zeros(max(len(c), 1), np.int32)
+    st = PtasStats()
+    _chk("dp_fill_alg4", lib().dp_fill_alg4(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), len(c), int(T), int(dim),
+                                            out.ctypes.data_as(ctypes.c_void_p) if table else None,
+                                            sg * e if table else 0, ctypes.byref(opt), _ptr(dv, ctypes.c_int32),
+                                            ctypes.byref(st)))
+    if table:
+        out = out.reshape(tuple(int(x) + 1 for x in c))
+    return opt.value, out, dv[: len(c)].tolist(), st.to_dict()
 
 
 def hmbp_solve(counts, sizes, capacity: int, packing: bool = True):

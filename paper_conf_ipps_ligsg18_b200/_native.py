@@ -57,7 +57,7 @@ EXPORTS = [
     "ptas_default_options", "ptas_solve", "ptas_solve_ex", "ptas_solve_device", "dp_table_shape", "dp_fill",
     "dp_fill_device", "ptas_get_unique_id", "ptas_comm_init", "ptas_comm_destroy", "ptas_strerror", "ptas_k",
     "ptas_bounds", "ptas_classify", "ptas_probe_targets", "ptas_interval_update", "ptas_shard_range",
-    "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order", "ptas_level_shard", "dp_fill_opt",
+    "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order", "ptas_level_shard", "dp_fill_opt", "dp_fill_alg4",
 ]
 
 _lib = None
@@ -104,6 +104,8 @@ def lib():
     L.dp_configs.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, ctypes.c_int64, i64p]
     L.dp_fill_opt.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, i32p,
                               ctypes.POINTER(PtasStats)]
+    L.dp_fill_alg4.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, vp, ctypes.c_int64, i32p,
+                               i32p, ctypes.POINTER(PtasStats)]
     L.hmbp_solve.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, i32p, ctypes.c_int32,
                              ctypes.POINTER(PtasStats)]
     L.ptas_table_order.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int32, i32p, i32p]

@@ -214,6 +214,10 @@ cudaError_t launch_row_fill_swar_df(int e, void *table, const RowGeom &g, const 
 cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int32_t *N, const int64_t *r,
                                  int64_t T, int J0, const PrefixEntry *d_pref, const DpMeta *d_meta,
                                  int64_t nP_bound, cudaStream_t st, bool dry);
+// The paper's Alg 4 / Alg 5 partitioned DP as an A/B baseline (alg4.cu):
+// blocked layout, block-levels, in-block levels, full Eq. 1 relaxation per entry.
+int alg4_fill(int e, const int32_t *N, int K, const int32_t *cfg_digits, int64_t nC, int dim, void *host_out,
+              int32_t *opt_out, double *fill_s, int64_t *nblocks_out, int32_t *block_levels_out, int32_t *div_out);
 // Host-only geometry test of launch_row_fill_ring (internal class order).
 bool ring_fits(const int32_t *N, const int64_t *r, int K, int64_t T);
 // Rows per row set the dataflow kernel will use for this geometry (0 = unsupported).

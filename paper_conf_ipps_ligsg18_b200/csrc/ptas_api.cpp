@@ -1143,6 +1143,67 @@ int dp_fill_opt(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t 
     return PTAS_OK;
 }
 
+int dp_fill_alg4(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int32_t dim, void *table_out,
+                 int64_t table_bytes, int32_t *opt_N_out, int32_t *divisor_out, ptas_stats *stats)
+{
+    const double t0 = now_s();
+    int rc = validate_dp(counts, sizes, K, T);
+    if (rc) return rc;
+    if (!opt_N_out || K < 1 || K > 16 || dim < 1) return PTAS_EINVAL;
+    int64_t sigma;
+    int32_t e;
+    rc = dp_table_shape(counts, K, &sigma, &e);
+    if (rc) return rc;
+    if (table_out && table_bytes < sigma * e) return PTAS_EINVAL;
+    int dev;
+    rc = resolve_device(-1, &dev);
+    if (rc) return rc;
+    Engine *eng;
+    rc = Engine::get(dev, &eng);
+    if (rc) return rc;
+    std::lock_guard<std::mutex> lk(eng->mu);
+    DpRequest rq;
+    rq.K = K;
+    rq.N = counts;
+    rq.r = sizes;
+    rq.T = T;
+    std::vector<int32_t> dig;
+    int64_t nC = 0;
+    rc = eng->configs_canonical(rq, &dig, &nC);   // C(T), caller order (enumerated on the device)
+    if (rc) return rc;
+    ptas_stats st;
+    std::memset(&st, 0, sizeof(st));
+    for (int64_t c = 0; c < nC; ++c) {   // closed-form relaxation count
+        double pr = 1;
+        for (int i = 0; i < K; ++i) pr *= (double)(counts[i] - dig[(size_t)c * K + i] + 1);
+        st.relaxations += pr;
+    }
+    double fs = 0;
+    int64_t nb = 0;
+    int32_t bl = 0;
+    int32_t divs[16];
+    if (nC == 0) {   // no long class: OPT(0) = 0 only
+        *opt_N_out = 0;
+    } else {
+        rc = alg4_fill(e, counts, K, dig.data(), nC, dim, table_out, opt_N_out, &fs, &nb, &bl, divs);
+        if (rc) return rc;
+    }
+    if (divisor_out) std::memcpy(divisor_out, divs, sizeof(int32_t) * K);
+    if (stats) {
+        st.unique_dps = 1;
+        st.fill_seconds = st.fill_wall_seconds = fs;
+        st.states = sigma;
+        st.sigma_max = sigma;
+        st.relax_executed = st.relaxations;
+        st.alg_bytes = st.exec_bytes = (st.relaxations + (double)sigma) * e;
+        st.fill_launches = bl;
+        st.total_seconds = now_s() - t0;
+        st.opt_at_Tstar = *opt_N_out;
+        *stats = st;
+    }
+    return PTAS_OK;
+}
+
 int hmbp_solve(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t capacity, int32_t *bins_out,
                int32_t *packing_out, int32_t max_bins, ptas_stats *stats)
 {

@@ -44,13 +44,14 @@ namespace swar {
 namespace {
 
 // prefixes whose DSMEM loads are issued together (CH = 8: 4, so 32 words in flight per lane)
-constexpr int RING_PB_MAX = 8;
 #ifndef PTAS_RING_PROFILE
 #define PTAS_RING_PROFILE 0
 #endif
 // diagnostics build (-DPTAS_RING_PROFILE=1): per level, clock64 of CTA `prof_cta`
 // thread 0 at level start, after its rows, after arrive, after wait
+#if PTAS_RING_PROFILE
 __device__ long long g_ring_prof[4][2048];
+#endif
 
 __device__ __forceinline__ uint32_t dsm_map(uint32_t local_addr, uint32_t rank)
 {
