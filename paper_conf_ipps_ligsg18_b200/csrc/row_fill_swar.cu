@@ -1,25 +1,19 @@
-// row_fill_swar.cu — packed-word level fill, the production kernel of §8(a) a-5.
+// row_fill_swar.cu — packed-word level fill, the production kernel of §8(a) a-5
+// (dispatch by entry type and digit words; the kernel template is in
+// row_fill_swar.cuh, its instantiations in row_fill_swar_<E>_nw<NW>.cu).
 //
-// Same recurrence and row-wavefront as row_fill_kernel (dp_kernels.cu), Eq. 1
-// of PAPER.md:74-79, but every lane owns one 32-bit word of a row: 4 uint8
-// states or 2 uint16 states.  Rows are padded to a multiple of 4 bytes
-// (RowGeom::Wp), so every row and every off(s') is word aligned:
-//
-//   * the source row p - s' of a prefix is read with ONE coalesced 32-bit
-//     load per lane;
-//   * the j-shifted windows (s = (s', j), j = 0..Jmax(s')) come from the
-//     lane's word and its left neighbours (warp shuffles) through one PRMT
-//     each; uint8 windows are split into even/odd uint16 lanes with the
-//     sign-replicating PRMT mode (v < 128 -> v, v >= 128 -> 0xFF00|v, a
-//     monotone encoding), so VIMNMX.U16x2 takes two minima per instruction;
-//   * all row groups of a warp walk the prefix list in lockstep (uniform
-//     loop, uniform Jmax), each with its own dominance predicate s' <= p.
-//
-// The in-row term (s' = 0, j = 1..J0) is then resolved on packed uint16
-// lanes by Bellman-Ford rounds (shift, +1, min) until no lane changes.
-// Every (n, s) with s in C, s <= n is relaxed exactly once, so the closed
-// form relaxation count still holds.  Entries in the row padding and in
-// lanes past the row end are computed but never read as sources.
+// Eq. 1 of PAPER.md:74-79 on the row wavefront (D1): a lane group
+// owns a row p, each lane CH 32-bit words of it (4 uint8 or 2 uint16 states
+// per word; rows padded to a multiple of CH words, D3).  For every prefix s'
+// of the row's pivot block (D13) with s' <= p the lanes take ONE vector load
+// of the source row p - s' and ONE shifted window of it (the clamp
+// x - min(x, Jmax(s')) of D5, built from the left neighbour's words by shuffles
+// and a PRMT; uint8 as even/odd uint16 lanes with the sign-replicating PRMT, a
+// monotone encoding), and keep the minimum with VIMNMX.U16x2.  The row is then
+// 1 + that minimum (D12: the in-row configurations never win for p != 0; row 0
+// is ceil(x / J0)); there is no in-row closure and no chain.  Each (row,
+// prefix, x) is evaluated once; the executed count is stats.relax_executed.
+// Entries in the row padding are computed but never read as sources.
 #include <cstdint>
 #include <cuda_runtime.h>
 
