@@ -121,6 +121,7 @@ struct RingArgs {
     int32_t J0;           // min(N_last, floor(T / r_last))
     int32_t R;            // ring depth in row-levels
     int32_t A;            // ring rows per level per CTA: ceil((N0 + 1) / cluster size)
+    int32_t H;            // halo rows: copies of the previous CTA's top H rows (H = max s0 <= A)
     int32_t rho_max;      // N0 + N1
 };
 

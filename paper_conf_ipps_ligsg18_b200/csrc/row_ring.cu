@@ -79,6 +79,22 @@ __device__ __forceinline__ Words<CH> ld_dsm(uint32_t addr)
     return w;
 }
 
+template <int CH>
+__device__ __forceinline__ void st_dsm(uint32_t addr, const Words<CH> &w)
+{
+    if constexpr (CH == 1) {
+        asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(w.v[0]) : "memory");
+    } else if constexpr (CH == 2) {
+        asm volatile("st.shared::cluster.v2.u32 [%0], {%1, %2};" ::"r"(addr), "r"(w.v[0]), "r"(w.v[1]) : "memory");
+    } else {
+#pragma unroll
+        for (int c = 0; c < CH; c += 4)
+            asm volatile("st.shared::cluster.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(addr + 4 * c), "r"(w.v[c]),
+                         "r"(w.v[c + 1]), "r"(w.v[c + 2]), "r"(w.v[c + 3])
+                         : "memory");
+    }
+}
+
 // CH consecutive words of the own CTA's ring (shared memory, 4*CH-byte aligned)
 template <int CH>
 __device__ __forceinline__ Words<CH> lds_words(const uint32_t *p)
@@ -144,7 +160,8 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
     const uint32_t row_bytes = (uint32_t)Lw * 4;
     // smem: ring [R][A][Lw] words | 4 prefix lists int4 [np + PB] each
     uint32_t *ring = reinterpret_cast<uint32_t *>(smem_raw);
-    int4 *s_pl = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * ra.A * row_bytes + 15) & ~(size_t)15));
+    const int AH = ra.A + ra.H;                  // ring rows per level: H halo rows, then A own rows
+    int4 *s_pl = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * AH * row_bytes + 15) & ~(size_t)15));
     const int lcap = np + PB;
     __shared__ int s_cnt[4];
     if (threadIdx.x < 4) s_cnt[threadIdx.x] = 0;
@@ -164,7 +181,11 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
     for (int i = threadIdx.x; i < 4 * PB; i += blockDim.x)   // padding: never dominated
         s_pl[(i / PB) * lcap + s_cnt[i / PB] + i % PB] =
             make_int4(1 << 20, 1 << 20, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF, 0);
-    const uint32_t rem = dsm_map((uint32_t)__cvta_generic_to_shared(ring), crank > 0 ? crank - 1 : 0);
+    uint32_t csize;
+    asm("mov.u32 %0, %%cluster_nctarank;" : "=r"(csize));
+    // the next CTA's ring: this CTA's top H rows of every level are pushed into its halo
+    const bool has_next = crank + 1 < csize;
+    const uint32_t nxt = dsm_map((uint32_t)__cvta_generic_to_shared(ring), has_next ? crank + 1 : crank);
     __syncthreads();
     cluster_sync_all();   // every CTA of the cluster runs before any DSMEM access
 
@@ -188,7 +209,7 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
             const int c = task - r_ * Lg;       // lane chunk: words c*CH .. c*CH+CH-1 of the row
             const int b = L - a;
             const int ia = a - a0;
-            const int pos0 = ia * Lw + c * CH;  // the lane's words within a ring slot
+            const int pos0 = (ra.H + ia) * Lw + c * CH;  // the lane's words within a ring slot
             Words<CH> ae, ao;
             fill_words(ae, 0xffffffffu);
             fill_words(ao, 0xffffffffu);
@@ -205,25 +226,16 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
                     for (int u = 0; u < PB; ++u) {
                         const int4 pf = pl[q0 + u];
                         sj[u] = pf.z;
-                        // source row (a - s0, b - s1) of level L - |s'|: in this CTA's ring, or
-                        // (first s0 rows of the block) the previous CTA's: A >= every s0
+                        // source row (a - s0, b - s1) of level L - |s'|: always in this CTA's ring
+                        // (own rows, or the halo copy of the previous CTA's top rows, s0 <= H)
                         int ss = slot - pf.w;
                         ss += ss < 0 ? ra.R : 0;
-                        const int pos = pos0 + (ss * ra.A - pf.x) * Lw;   // word index in the ring
+                        const int pos = pos0 + (ss * AH - pf.x) * Lw;   // word index in the ring
                         if (pf.x <= a && pf.y <= b) {
-                            // own rows through plain shared-memory loads (~128 B/cycle); the few
-                            // rows of the previous CTA through DSMEM (~20 B/cycle per SM)
-                            if (ia >= pf.x) {
-                                const uint32_t *p = ring + pos;
-                                cur[u] = lds_words<CH>(p);
-                                l1[u] = c >= 1 ? p[-1] : 0u;
-                                l2[u] = (cls == 2 && c * CH >= 2) ? p[-2] : 0u;
-                            } else {
-                                const uint32_t src = rem + 4u * (uint32_t)(pos + ra.A * Lw);
-                                cur[u] = ld_dsm<CH>(src);
-                                l1[u] = c >= 1 ? ld_dsm<1>(src - 4).v[0] : 0u;
-                                l2[u] = (cls == 2 && c * CH >= 2) ? ld_dsm<1>(src - 8).v[0] : 0u;
-                            }
+                            const uint32_t *p = ring + pos;
+                            cur[u] = lds_words<CH>(p);
+                            l1[u] = c >= 1 ? p[-1] : 0u;
+                            l2[u] = (cls == 2 && c * CH >= 2) ? p[-2] : 0u;
                         } else {
                             fill_words(cur[u], 0xffffffffu);
                             l1[u] = l2[u] = 0xffffffffu;
@@ -264,7 +276,9 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
                 }
                 wv.v[t] = EB == 1 ? prmt(oe, oo, 0x6240u) : oe;
             }
-            store_words<CH>(ring + ((size_t)slot * ra.A + ia) * Lw + c * CH, wv);
+            store_words<CH>(ring + ((size_t)slot * AH + ra.H + ia) * Lw + c * CH, wv);
+            if (has_next && ia >= ra.A - ra.H)   // halo of the next CTA (one DSMEM store per word)
+                st_dsm<CH>(nxt + 4u * (uint32_t)(((slot * AH + ia - (ra.A - ra.H)) * Lw + c * CH)), wv);
             if (task + (int)blockDim.x < ntask) {   // (not the thread's last row of the level)
                 const int64_t rowbase = (int64_t)a * ra.stride0 + (int64_t)b * ra.Wp;   // elements
                 store_words<CH>(tab32 + rowbase * EB / 4 + c * CH, wv);
@@ -300,7 +314,7 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
 {
     auto kfn = row_ring_kernel<E, CH, WIN>;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (((size_t)ra.R * ra.A * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
+    const size_t smem = (((size_t)ra.R * (ra.A + ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
     cudaError_t err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     if (csize > 8) {
@@ -392,7 +406,8 @@ bool ring_fits(const int32_t *N, const int64_t *r, int K, int64_t T)
     for (int csize : {16, 8}) {
         const int64_t A = (N[0] + csize) / csize;
         if (A < hi0) continue;
-        if (((R * A * Lw * 4 + 15) & ~(int64_t)15) + 4 * (int64_t)(hi0 + 1) * (hi1 + 1) * 16 <= 220 * 1024) return true;
+        if (((R * (A + hi0) * Lw * 4 + 15) & ~(int64_t)15) + 4 * (int64_t)(hi0 + 1) * (hi1 + 1) * 16 <= 220 * 1024)
+            return true;
     }
     return false;
 }
@@ -432,16 +447,27 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     for (int csize : {16, 8, 4, 2}) {
         if (cs_force ? csize != cs_force : csize < 8) continue;
         ra.A = (N[0] + csize) / csize;   // ceil((N0 + 1) / C) rows of each level per CTA
+        ra.H = (int32_t)hi0;              // halo rows (s0 <= hi0)
         if (ra.A < hi0) continue;         // every source row is in this CTA's block or the previous one
-        const size_t smem = (((size_t)ra.R * ra.A * Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
+        const size_t smem = (((size_t)ra.R * (ra.A + ra.H) * Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
         if (smem > smem_cap) continue;
         // words per lane: the smallest chunk with one pass over the CTA's rows of a level
+        // words per lane: 4 when the CTA's rows of a level fit one pass (measured best on
+        // M5s: 2 words 1.82 / 1.69 ms, 4 words 1.39 / 1.48 ms, 8 words 1.94 / 1.96 ms per DP),
+        // else the smallest chunk that fits, else 8
         int CH = 8;
-        for (int c : {1, 2, 4})
-            if (Lw % c == 0 && (int64_t)ra.A * (Lw / c) <= 1024) {
-                CH = c;
-                break;
-            }
+        if (Lw % 4 == 0 && (int64_t)ra.A * (Lw / 4) <= 1024) CH = 4;
+        else
+            for (int c : {1, 2, 4})
+                if (Lw % c == 0 && (int64_t)ra.A * (Lw / c) <= 1024) {
+                    CH = c;
+                    break;
+                }
+        static const int ch_env = [] {   // experiment knob: words per lane
+            const char *t = std::getenv("PTAS_RING_CH");
+            return t && t[0] ? std::atoi(t) : 0;
+        }();
+        if (ch_env == 1 || ch_env == 2 || ch_env == 4 || ch_env == 8) CH = ch_env;
         if (Lw % CH != 0) continue;
         ra.Lg = Lw / CH;
         cudaError_t err = e == 1 ? swar::launch_ring_e<uint8_t>(table, ra, CH, d_pref, d_meta, nP_bound, csize, win, st, dry)
