@@ -71,7 +71,7 @@ class ClockSampler:
     """SM clock and throttle reasons sampled in-process through NVML during the
     timed region (no nvidia-smi subprocesses, which stall the driver)."""
 
-    def __init__(self, index: int, period: float = float(os.environ.get("BENCH_CLOCK_PERIOD", "0.25"))):
+    def __init__(self, index: int, period: float = float(os.environ.get("BENCH_CLOCK_PERIOD", "0.01"))):
         self.index = index
         self.period = period
         self.rows = []
@@ -508,7 +508,7 @@ def run_ours(args, w):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default=None, choices=sorted(WORKLOADS),
