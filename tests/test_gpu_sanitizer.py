@@ -1,5 +1,6 @@
 """compute-sanitizer over the fill kernels (memcheck; racecheck on the split
-mode's shared-memory reduction and the dataflow kernel's block ticket).  Small geometries that exercise every lane
+mode's shared-memory reduction, the dataflow kernel's block ticket, and the
+K = 3 cluster ring kernel's shared-memory ring with its DSMEM halo stores).  Small geometries that exercise every lane
 layout: group widths that do not divide 32 (idle lanes), multi-word shifts
 (GEN path), vector chunks CH = 1/2/4/8, uint8 and uint16 tables, split mode.
 Parity of the same cases is checked in test_gpu_parity.py; here only memory
@@ -37,6 +38,12 @@ for N, r, T in cases:
     P.dp_fill(np.array(N, np.int32), np.array(r, np.int64), T)
 p = np.random.default_rng(0).integers(1, 100, 12)
 P.ptas_solve(p, 3, 0.3)
+# level window (VMM ring, slab launches), the K = 3 cluster ring kernel on a
+# multi-CTA block, and the paper's Alg 4 partitioned A/B
+for N, r, T in [([5, 4, 18], [35, 50, 21], 110), ([3, 3, 3, 30], [40, 50, 60, 9], 150), ([4, 300], [60, 13], 120)]:
+    P.dp_fill_opt(np.array(N, np.int32), np.array(r, np.int64), T, window=1)
+P.dp_fill(np.array([40, 30, 25], np.int32), np.array([700, 600, 500], np.int64), 1900)
+P.dp_fill_alg4(np.array([5, 5, 5], np.int32), np.array([30, 40, 50], np.int64), 120, dim=3)
 print("ok")
 """
 
@@ -90,6 +97,12 @@ def test_memcheck_dataflow(env):
 @pytest.mark.timeout(1800)
 def test_racecheck_dataflow_split():
     _run("racecheck", {"PTAS_DF": "3", "PTAS_DF_SPLIT_ROWS": "1000000000"})
+
+
+@pytest.mark.timeout(1800)
+def test_racecheck_default_paths():
+    # default schedule: dataflow runs, per-level launches, the ring kernel (K = 3)
+    _run("racecheck")
 
 
 @pytest.mark.timeout(1200)
