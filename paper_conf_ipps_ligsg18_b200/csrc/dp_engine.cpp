@@ -296,8 +296,7 @@ static int build_geom(const std::vector<int32_t> &N, int e, bool pad, RowGeom *g
     int word = 0, bit = 0;
     // PTAS_FORCE_TWO_WORDS=1 (tests only): split the leading digits over two
     // words even when they fit in one, to exercise the two-word kernels.
-    const char *force2 = std::getenv("PTAS_FORCE_TWO_WORDS");
-    const int split = (force2 && force2[0] == '1' && K - 1 >= 2) ? (K - 1) / 2 : -1;
+    const int split = (PTAS_KNOB("PTAS_FORCE_TWO_WORDS", 0) == 1 && K - 1 >= 2) ? (K - 1) / 2 : -1;
     for (int i = 0; i < K - 1; ++i) {
         int w = bits_of(N[i]) + 1;
         if (bit + w > 64 || i == split) {
@@ -568,8 +567,7 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     uint64_t *d_pw = (uint64_t *)(d_rb + rows_idx);
     // on the side stream: overlaps the enumeration below and its host round trip
     // (PTAS_ROWIDX_MAIN=1: on the DP's own stream, three API calls fewer)
-    const char *rim = std::getenv("PTAS_ROWIDX_MAIN");
-    const bool ri_main = rim && rim[0] == '1';
+    const bool ri_main = PTAS_KNOB("PTAS_ROWIDX_MAIN", 0) == 1;
     if (!ri_main) {
         PT_CK(cudaEventRecord(ev_fork_, st));
         PT_CK(cudaStreamWaitEvent(side_, ev_fork_, 0));
@@ -603,18 +601,17 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // NP_CAP, launch heuristics from the previous DP's prefix count; the
     // kernels exit and the DP is redone synchronously if a bound is exceeded
     // (meta->ovf), which then grows the bounds.
-    const char *es = std::getenv("PTAS_ENUM_SYNC");
+    const bool es_sync = PTAS_KNOB("PTAS_ENUM_SYNC", 0) == 1;
     // (a comm-backed DP always reads |C| back: every rank then takes the same path,
     // no rank can redo the DP alone while its peers wait in a collective)
-    const bool nosync = np_hint_ >= 0 && nc_cap_ > 0 && !force_sync_enum_ && !(es && es[0] == '1') && !comm_dp;
+    const bool nosync = np_hint_ >= 0 && nc_cap_ > 0 && !force_sync_enum_ && !es_sync && !comm_dp;
     int64_t nC;        // |C| (synchronous) or its bound
     int64_t nP_bound;  // bound of the prefix list incl. the zero prefix (smem sizing)
     // test knobs: PTAS_NC_CAP / PTAS_NP_CAP lower the bounds (exercise the redo path)
-    const char *ncc = std::getenv("PTAS_NC_CAP");
-    const char *npc = std::getenv("PTAS_NP_CAP");
-    const int64_t np_cap = npc && npc[0] ? std::min<int64_t>(NP_CAP, std::atoll(npc)) : NP_CAP;
+    const int64_t ncc = PTAS_KNOB("PTAS_NC_CAP", 0);
+    const int64_t np_cap = std::min<int64_t>(NP_CAP, PTAS_KNOB("PTAS_NP_CAP", NP_CAP));
     if (nosync) {
-        nC = ncc && ncc[0] ? std::min<int64_t>(nc_cap_, std::max<int64_t>(1, std::atoll(ncc))) : nc_cap_;
+        nC = ncc > 0 ? std::min<int64_t>(nc_cap_, ncc) : nc_cap_;
         nP_bound = NP_CAP + 1;
     } else {
         PT_CK(cudaMemcpyAsync(h_scalar_, d_offsets + nprefix, 8, cudaMemcpyDeviceToHost, st));
@@ -645,10 +642,10 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             ts += hi[i] + 1;
         }
         const int64_t nch = (std::max<int64_t>(nP_bound - 1, 0) + 31) / 32;
-        const char *dt = std::getenv("PTAS_DOMTAB");
+        const int64_t dt = PTAS_KNOB("PTAS_DOMTAB", -1);
         // (K - 1 >= 4: many leading digits, so few interior rows and long per-row
         // dominance tests; with 1-3 digits the lane-parallel test is as fast)
-        const bool want = e == 1 && (dt && dt[0] ? dt[0] != '0' : K - 1 >= 4);   // (uint8 kernels only)
+        const bool want = e == 1 && (dt >= 0 ? dt != 0 : K - 1 >= 4);   // (uint8 kernels only)
         if (K > 1 && want && (int64_t)ts * nch * 4 <= DOMTAB_MAX_BYTES) {
             PT_CK(domtab_.ensure((size_t)DOMTAB_MAX_BYTES));
             g.TS = ts;
@@ -662,18 +659,16 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     cudaError_t cpe = index_ < 4 ? prepare_const_prefix((const PrefixEntry *)pref_.p, d_meta_, nP_bound, e, g.nwords, index_,
                                                    cpstage_.p, st)
                                 : cudaErrorNotSupported;
-    const char *ncp = std::getenv("PTAS_NO_CPREF");
-    const int cpref_ok = (cpe == cudaSuccess && !(ncp && ncp[0] == '1')) ? 1 : 0;
+    const int cpref_ok = (cpe == cudaSuccess && PTAS_KNOB("PTAS_NO_CPREF", 0) != 1) ? 1 : 0;
     if (cpe != cudaSuccess && cpe != cudaErrorNotSupported) PT_CK(cpe);
     ++o.launches;
     const int J0 = (int)std::min<int64_t>(N[K - 1], rq.T / r[K - 1]);
-    const char *fs = std::getenv("PTAS_FORCE_SCALAR");
     // PTAS_FORCE_SCALAR=1: the full-relaxation scalar kernel for every level;
-    // =2: the long-row two-launch path for every level (test coverage)
-    const bool force_scalar = fs && (fs[0] == '1' || fs[0] == '2');
-    const bool force_long = fs && fs[0] == '2';
-    const char *pdls = std::getenv("PTAS_PDL");
-    const bool use_pdl = !(pdls && pdls[0] == '0');
+    // =2: the long-row path for every level (test coverage)
+    const int64_t fs = PTAS_KNOB("PTAS_FORCE_SCALAR", 0);
+    const bool force_scalar = fs == 1 || fs == 2;
+    const bool force_long = fs == 2;
+    const bool use_pdl = PTAS_KNOB("PTAS_PDL", 1) != 0;
     bool prev_fill = false;  // the previous launch on st was a packed fill (PDL-safe)
     bool used_scalar = false;  // some level ran on the scalar (uncollapsed) kernel
     // one row-level (or slice of it): packed-word kernel, scalar kernel as fallback
@@ -737,14 +732,11 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                            d_meta_, nP_bound, st, true) == cudaSuccess;
     cudaGetLastError();
     if (!ring) {
-        const char *dfs = std::getenv("PTAS_DF");
-        const int df_mode = dfs && dfs[0] ? std::atoi(dfs) : 3;
-        const char *dfr = std::getenv("PTAS_DF_ROWS");
-        const char *dsr = std::getenv("PTAS_DF_SPLIT_ROWS");
-        const int64_t df_rows = df_mode == 1 ? INT64_MAX
-                                             : (dfr && dfr[0] ? std::atoll(dfr) : (int64_t)2 * 32 * sm_count_);
+        const int df_mode = (int)PTAS_KNOB("PTAS_DF", 3);
+        const int64_t dfr = PTAS_KNOB("PTAS_DF_ROWS", -1);
+        const int64_t df_rows = df_mode == 1 ? INT64_MAX : (dfr >= 0 ? dfr : (int64_t)2 * 32 * sm_count_);
         // (measured on M2s/M3s/M4s/M5s: 600..8000 within a few %, 2000 best overall)
-        const int64_t split_rows = dsr && dsr[0] ? std::atoll(dsr) : 2000;
+        const int64_t split_rows = PTAS_KNOB("PTAS_DF_SPLIT_ROWS", 2000);
         if (df_mode > 0 && G == 1 && !comm_dp && !window && !force_scalar && g.rho_max >= 1) {
             if (df_mode == 3 || df_mode == 4) {
                 // levels wider than df_rows get a launch of their own (enough rows to fill
@@ -899,14 +891,9 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             dfa.base = ticket_base_;
             dfa.epoch = ++df_epoch_;
             dfa.nsplit = rn.nsplit;
-            // PTAS_DF_SLEEP=a:b: poll backoff from a ns doubling up to b ns
-            {
-                const char *sl = std::getenv("PTAS_DF_SLEEP");
-                int a = 64, b = 64;
-                if (sl && sl[0]) std::sscanf(sl, "%d:%d", &a, &b);
-                dfa.sleep0 = std::max(0, a);
-                dfa.sleep_max = std::max(dfa.sleep0, b);
-            }
+            // PTAS_DF_SLEEP0 / PTAS_DF_SLEEP_MAX: poll backoff (ns), doubling
+            dfa.sleep0 = (int32_t)std::max<int64_t>(0, PTAS_KNOB("PTAS_DF_SLEEP0", 64));
+            dfa.sleep_max = (int32_t)std::max<int64_t>(dfa.sleep0, PTAS_KNOB("PTAS_DF_SLEEP_MAX", 64));
             dfa.grid_div = rq.grid_div > 1 ? rq.grid_div : 1;
             // PTAS_DF_PROF=1 (with a PTAS_DF_PROFILE=1 build): per-level set timings of the run
             static const bool df_prof = [] {

@@ -24,6 +24,10 @@ namespace ptas {
 
 thread_local int64_t tl_np_hint = -1;
 
+static std::atomic<uint64_t> g_knob_gen{1};
+uint64_t knob_generation() { return g_knob_gen.load(std::memory_order_acquire); }
+void knobs_refresh() { g_knob_gen.fetch_add(1, std::memory_order_acq_rel); }
+
 
 namespace {
 
@@ -946,8 +950,8 @@ cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N
 {
     // one warp with the configurations in shared memory when they fit (48 KB)
     const size_t smem = (size_t)nC * (8 + 4) + (size_t)K * 4 + (size_t)nC * K * 2 + 16;
-    const char *tbb = std::getenv("PTAS_TB_BLOCK");   // tests: force the block kernel
-    if (smem <= 48 * 1024 && !(tbb && tbb[0] == '1')) {
+    const int64_t tbb = PTAS_KNOB("PTAS_TB_BLOCK", 0);   // tests: 1 forces the block kernel
+    if (smem <= 48 * 1024 && tbb != 1) {
         if (e == 1)
             traceback_warp_kernel<uint8_t><<<1, 32, smem, st>>>((const uint8_t *)table, K, d_N, d_digits, d_off, d_rank,
                                                                 (int)nC, idx_start, d_out, max_out, d_len, d_meta);
@@ -970,8 +974,7 @@ cudaError_t launch_traceback_canon(int e, const void *table, int K, const int32_
                                    int32_t *d_len, DpMeta *d_meta, cudaStream_t st)
 {
     const size_t smem = (size_t)nC * (8 + 4) + (size_t)K * 4 + (size_t)nC * K * 2 + 16;
-    const char *tbb = std::getenv("PTAS_TB_BLOCK");
-    if (smem > 48 * 1024 || nC > (1 << 20) || (tbb && tbb[0] == '1')) return cudaErrorNotSupported;
+    if (smem > 48 * 1024 || nC > (1 << 20) || PTAS_KNOB("PTAS_TB_BLOCK", 0) == 1) return cudaErrorNotSupported;
     rank_configs_kernel<<<(unsigned)((nC + 127) / 128), 128, 0, st>>>(d_digits, (int)nC, K, d_inv, Kc, d_rank);
     if (e == 1)
         traceback_warp_kernel<uint8_t><<<1, 32, smem, st>>>((const uint8_t *)table, K, d_N, d_digits, d_off, d_rank,

@@ -17,10 +17,32 @@
 //            lexicographic order): packed digits, off(s'), Jmax(s') = largest
 //            last digit with (s', j) in C.  Entry 0 is s' = 0 (j = 1..J0).
 #pragma once
+#include <atomic>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 namespace ptas {
+
+// Tuning / test knobs (PTAS_* environment variables; the defaults are the
+// measured best).  Every C-ABI entry point calls knobs_refresh(), and
+// each PTAS_KNOB call site re-reads its variable only when the generation has
+// changed: no getenv per launch or per level, while tests can still change a
+// knob between calls.  Unset or empty -> DFLT.
+uint64_t knob_generation();
+void knobs_refresh();
+#define PTAS_KNOB(NAME, DFLT)                                                                    \
+    ([]() -> int64_t {                                                                             \
+        static std::atomic<uint64_t> g_{~0ull};                                                    \
+        static std::atomic<int64_t> v_{0};                                                          \
+        const uint64_t cur_ = ::ptas::knob_generation();                                           \
+        if (g_.load(std::memory_order_acquire) != cur_) {                                          \
+            const char *t_ = std::getenv(NAME);                                                    \
+            v_.store(t_ && t_[0] ? (int64_t)std::atoll(t_) : (int64_t)(DFLT), std::memory_order_relaxed); \
+            g_.store(cur_, std::memory_order_release);                                             \
+        }                                                                                          \
+        return v_.load(std::memory_order_relaxed);                                                 \
+    }())
 
 constexpr int MAXK = 40;   // internal (non-empty) classes
 constexpr int MAXW = 2;    // 64-bit words for packed leading digits

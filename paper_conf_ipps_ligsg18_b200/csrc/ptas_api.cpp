@@ -255,6 +255,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                int64_t *makespan_out, int32_t *assignment_out, ptas_stats *stats, ptas_probe *log,
                int32_t log_cap, int32_t *log_len, int64_t extra_h2d, int64_t extra_d2h)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     const double t0 = now_s();
     ptas_options opt;
     ptas_default_options(&opt);
@@ -366,8 +367,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     // host thread and one DP slot (own stream and workspace) per probe -- the
     // quarter split of Alg 3 on one GPU.  With a caller
     // stream, slot 0 uses it; the call is host-synchronous either way.
-    const char *ncs = std::getenv("PTAS_NO_CONCURRENT");
-    const bool concurrent = opt.mode == PTAS_MODE_SINGLE && !(ncs && ncs[0] == '1');
+    const bool concurrent = opt.mode == PTAS_MODE_SINGLE && PTAS_KNOB("PTAS_NO_CONCURRENT", 0) != 1;
     // Runs the jobs concurrently (slots 0..), outcomes in outs; grid_div > 0:
     // persistent fill grids take 1/(jobs in flight) of the GPU each.
     auto run_jobs = [&](std::vector<Classified> &cls_v, std::vector<int64_t> &T_v,
@@ -391,10 +391,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                     return;
                 }
                 // PTAS_GRID_DIV (experiment knob): 0 = every launch may take the whole GPU
-                static const int gd_env = [] {
-                    const char *t = std::getenv("PTAS_GRID_DIV");
-                    return t && t[0] ? std::atoi(t) : -1;
-                }();
+                const int64_t gd_env = PTAS_KNOB("PTAS_GRID_DIV", -1);
                 rcs[b] = probe_dp(sl[b], cls_v[j0 + b], T_v[j0 + b], nullptr,
                                   b == 0 ? (cudaStream_t)opt.stream : nullptr,
                                   gd_env == 0 ? 1 : (share_grid ? nb : 1), &outs_all[j0 + b]);
@@ -460,15 +457,13 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     std::map<std::vector<int64_t>, SpecRes> spec;
     int spec_depth = opt.speculate < 0 ? 3 : opt.speculate;
     int64_t spec_sigma = (int64_t)1 << 24;
-    const char *sr = std::getenv("PTAS_SPEC_RING");   // 0: ring DPs only below spec_sigma (A/B)
-    const bool spec_ring = !(sr && sr[0] == '0');
-    const char *sl = std::getenv("PTAS_SPEC_LEVELS");
-    const int64_t spec_levels = sl && sl[0] ? std::atoll(sl) : 160;
+    const bool spec_ring = PTAS_KNOB("PTAS_SPEC_RING", 1) != 0;   // 0: latency-bound DPs only below spec_sigma (A/B)
+    const int64_t spec_levels = PTAS_KNOB("PTAS_SPEC_LEVELS", 160);
     {
-        const char *sd = std::getenv("PTAS_SPEC_DEPTH");
-        if (sd && sd[0] && opt.speculate < 0) spec_depth = std::atoi(sd);
-        const char *ss = std::getenv("PTAS_SPEC_SIGMA");
-        if (ss && ss[0]) spec_sigma = std::atoll(ss);
+        const int64_t sd = PTAS_KNOB("PTAS_SPEC_DEPTH", -1);
+        if (sd >= 0 && opt.speculate < 0) spec_depth = (int)sd;
+        const int64_t ss = PTAS_KNOB("PTAS_SPEC_SIGMA", -1);
+        if (ss >= 0) spec_sigma = ss;
         if (spec_depth > 3) spec_depth = 3;   // 2^3 - 1 = 7 DPs in flight (MAX_SLOTS slots)
     }
     // Library default (speculate = -1): the feasible-branch chain — the next
@@ -476,12 +471,10 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     // SURVEY §8(d)), 4 deep; all of them are used when the guess holds, none of
     // the tree's other branches occupy the GPU (M2s -5%, M5s-0.2 -44%, measured).
     // speculate = d > 0: the full tree of depth d.  PTAS_SPEC_CHAIN=0 / 1 forces.
-    const char *sch = std::getenv("PTAS_SPEC_CHAIN");
-    const bool spec_chain = sch && sch[0] ? sch[0] == '1' : opt.speculate < 0;
-    if (spec_chain && spec_depth > 0) {   // (PTAS_SPEC_DEPTH=0 still turns speculation off)
-        const char *scd = std::getenv("PTAS_SPEC_CHAIN_DEPTH");
-        spec_depth = scd && scd[0] ? std::max(1, std::min(MAX_SLOTS, std::atoi(scd))) : 4;
-    }
+    const int64_t sch = PTAS_KNOB("PTAS_SPEC_CHAIN", -1);
+    const bool spec_chain = sch >= 0 ? sch == 1 : opt.speculate < 0;
+    if (spec_chain && spec_depth > 0)   // (PTAS_SPEC_DEPTH=0 still turns speculation off)
+        spec_depth = (int)std::max<int64_t>(1, std::min<int64_t>(MAX_SLOTS, PTAS_KNOB("PTAS_SPEC_CHAIN_DEPTH", 4)));
     const bool spec_on = spec_depth >= 1 && P == 1 && concurrent && opt.memoize && opt.mode == PTAS_MODE_SINGLE;
     auto speculate = [&](int64_t lb0, int64_t ub0) -> int {
         struct Node {
@@ -1041,6 +1034,7 @@ static int dp_fill_common(const int32_t *counts, const int64_t *sizes, int32_t K
                           void *d_ext, int64_t ext_bytes, cudaStream_t st, void *host_out,
                           int64_t host_bytes, int32_t *opt_N_out, ptas_stats *stats)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     const double t0 = now_s();
     int rc = validate_dp(counts, sizes, K, T);
     if (rc) return rc;
@@ -1090,6 +1084,7 @@ static int dp_fill_common(const int32_t *counts, const int64_t *sizes, int32_t K
 int dp_fill_opt(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int64_t table_budget_bytes,
                 int32_t window, int32_t *opt_N_out, ptas_stats *stats)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     const double t0 = now_s();
     int rc = validate_dp(counts, sizes, K, T);
     if (rc) return rc;
@@ -1146,6 +1141,7 @@ int dp_fill_opt(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t 
 int dp_fill_alg4(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int32_t dim, void *table_out,
                  int64_t table_bytes, int32_t *opt_N_out, int32_t *divisor_out, ptas_stats *stats)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     const double t0 = now_s();
     int rc = validate_dp(counts, sizes, K, T);
     if (rc) return rc;
@@ -1207,6 +1203,7 @@ int dp_fill_alg4(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t
 int hmbp_solve(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t capacity, int32_t *bins_out,
                int32_t *packing_out, int32_t max_bins, ptas_stats *stats)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     const double t0 = now_s();
     int rc = validate_dp(counts, sizes, K, capacity);
     if (rc) return rc;
@@ -1289,6 +1286,7 @@ int dp_fill_device(const int32_t *counts, const int64_t *sizes, int32_t K, int64
 int dp_configs(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T, int32_t *out_digits,
                int64_t cap, int64_t *count)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     int rc = validate_dp(counts, sizes, K, T);
     if (rc) return rc;
     if (!count || (cap > 0 && !out_digits)) return PTAS_EINVAL;
@@ -1316,6 +1314,7 @@ int dp_configs(const int32_t *counts, const int64_t *sizes, int32_t K, int64_t T
 int dp_row_index(const int32_t *counts, int32_t K, int64_t *level_start, int64_t level_cap,
                  int64_t *out_rowbase, int64_t rows_cap)
 {
+    knobs_refresh();   // PTAS_* knobs: re-read at most once per call
     if (K < 1 || K > 64 || !counts || !level_start) return PTAS_EINVAL;
     int64_t sigma;
     int32_t e;

@@ -654,11 +654,11 @@ static int plan_ch(int e, const RowGeom &g, int J0, int64_t rows, int sm_count, 
     for (int i = 0; i < g.K1; ++i) rows_all *= (int64_t)g.N[i] + 1;
     if ((g.span_words > 0 ? g.span_words : rows_all * (int64_t)Lw) >= ((int64_t)1 << 31)) return 0;
     int CH;
-    const char *chs = std::getenv(df ? "PTAS_DF_CH" : "PTAS_SWAR_CH");
-    const char *cht = std::getenv("PTAS_SMALL_LEVEL_ROWS");
-    const int64_t small_rows = cht ? std::atoll(cht) : (int64_t)sm_count * 32;
+    const int64_t chs = df ? PTAS_KNOB("PTAS_DF_CH", 0) : PTAS_KNOB("PTAS_SWAR_CH", 0);
+    const int64_t cht = PTAS_KNOB("PTAS_SMALL_LEVEL_ROWS", -1);
+    const int64_t small_rows = cht >= 0 ? cht : (int64_t)sm_count * 32;
     if (Lw > 32) CH = Lw <= 64 ? 2 : (Lw <= 128 ? 4 : 8);
-    else if (chs && chs[0]) CH = std::atoi(chs);
+    else if (chs > 0) CH = (int)chs;
     else CH = (Lw >= 8 && rows > small_rows) ? 2 : 1;
     if (CH != 1 && CH != 2 && CH != 4 && CH != 8) CH = 1;
     if (Lw % CH != 0) {
@@ -703,14 +703,14 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // heuristics use the caller's estimate when the exact length is not known on the host
     const int64_t nph = tl_np_hint >= 0 ? std::min<int64_t>(tl_np_hint, np) : np;
     // small row-levels with long prefix lists: split each row set's prefixes over the 8 warps of a block
-    const char *sp = std::getenv("PTAS_SPLIT_ROWS");
+    const int64_t sp = PTAS_KNOB("PTAS_SPLIT_ROWS", -1);
     // (worth it when a row's prefix walk has several batches of gathers in series)
     const int PBh = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);
-    const int64_t split_rows = sp ? std::atoll(sp) : ((nph + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
+    const int64_t split_rows = sp >= 0 ? sp : ((nph + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
     // df->nsplit: 1 = warp row sets, 8 = block row sets, 0 = one cluster in lockstep
     const bool cl = df && df->nsplit == 0;
-    const char *cls = std::getenv("PTAS_CL_SIZE");
-    const int cl_size = cl ? (cls && cls[0] ? std::max(1, std::min(16, std::atoi(cls))) : 16) : 1;
+    const int64_t cls = PTAS_KNOB("PTAS_CL_SIZE", 16);
+    const int cl_size = cl ? (int)std::max<int64_t>(1, std::min<int64_t>(16, cls)) : 1;
     const int nsplit = df ? (df->nsplit > 1 ? bs / 32 : 1) : (slot_count <= split_rows ? bs / 32 : 1);
     const size_t smem = swar_smem(np, NW, df ? df->nlev : 0, g, CH);
     if (smem > 220 * 1024) return cudaErrorNotSupported;
@@ -719,8 +719,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // the in-row closure handles any shift (registers up to 8 bytes, else shared memory)
     const int win = J0 * e <= 4 ? 4 : (J0 * e <= 8 ? 8 : 0);
     const bool cpref = np <= CP_MAX && cslot >= 0 && cslot < CP_SLOTS && nph >= 64;
-    const char *dwv = std::getenv("PTAS_DF_WAVE");
-    const int64_t df_wave = dwv && dwv[0] ? std::max(1, std::atoi(dwv)) : 2;
+    const int64_t df_wave = std::max<int64_t>(1, PTAS_KNOB("PTAS_DF_WAVE", 2));
     DfArgs dfa;
     if (df) dfa = *df;
     else std::memset(&dfa, 0, sizeof(dfa));

@@ -425,8 +425,7 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     const int Lw = (int)(g.Wp * e / 4);
     // windows up to two words left (J0 * e <= 8 bytes: the M5s shapes have 6)
     if (J0 * e > 8 || nP_bound > 4096) return cudaErrorNotSupported;
-    const char *en = std::getenv("PTAS_RING");
-    if (en && en[0] == '0') return cudaErrorNotSupported;
+    if (PTAS_KNOB("PTAS_RING", 1) == 0) return cudaErrorNotSupported;
     RingArgs ra;
     ra.N0 = N[0];
     ra.N1 = N[1];
@@ -442,8 +441,7 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     const int win = J0 * e <= 4 ? 4 : 8;
     const size_t smem_cap = 220 * 1024;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const char *cs_env = std::getenv("PTAS_RING_CS");   // experiment: force the cluster size
-    const int cs_force = cs_env && cs_env[0] ? std::atoi(cs_env) : 0;
+    const int cs_force = (int)PTAS_KNOB("PTAS_RING_CS", 0);   // experiment: force the cluster size
     for (int csize : {16, 8, 4, 2}) {
         if (cs_force ? csize != cs_force : csize < 8) continue;
         ra.A = (N[0] + csize) / csize;   // ceil((N0 + 1) / C) rows of each level per CTA
@@ -463,10 +461,7 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
                     CH = c;
                     break;
                 }
-        static const int ch_env = [] {   // experiment knob: words per lane
-            const char *t = std::getenv("PTAS_RING_CH");
-            return t && t[0] ? std::atoi(t) : 0;
-        }();
+        const int ch_env = (int)PTAS_KNOB("PTAS_RING_CH", 0);   // experiment knob: words per lane
         if (ch_env == 1 || ch_env == 2 || ch_env == 4 || ch_env == 8) CH = ch_env;
         if (Lw % CH != 0) continue;
         ra.Lg = Lw / CH;
