@@ -134,3 +134,44 @@ def test_no_cpu_fallback_in_product():
             if fn.endswith((".py", ".cpp", ".cu", ".h")):
                 src = open(os.path.join(dp, fn)).read()
                 assert "import oracle" not in src and "from oracle" not in src and "ptas_oracle" not in src, fn
+
+
+def test_table_order_rule(P):
+    # layout 0 (D2/D13): non-empty classes only, the largest count last
+    # (ties: the highest index), the others by descending size; layout 1: given order
+    assert P.ptas_table_order([30, 25, 17, 20, 19, 13], [416, 520, 624, 728, 832, 936]) == [5, 4, 3, 2, 1, 0]
+    got = P.ptas_table_order([3, 0, 7, 7], [10, 20, 30, 40])
+    assert got[-1] == 3 and sorted(got) == [0, 2, 3] and got[:2] == [2, 0]
+    assert P.ptas_table_order([3, 0, 7, 7], [10, 20, 30, 40], layout=1) == [0, 2, 3]
+    assert P.ptas_table_order([0, 0], [5, 6]) == []
+    rng = np.random.default_rng(7)
+    for _ in range(50):
+        K = int(rng.integers(1, 9))
+        N = rng.integers(0, 20, K)
+        r = rng.permutation(np.arange(1, K + 1) * 10)
+        o = P.ptas_table_order(N, r)
+        nz = [i for i in range(K) if N[i] > 0]
+        assert sorted(o) == nz
+        if nz:
+            assert N[o[-1]] == max(N[nz])
+            lead = o[:-1]
+            assert all(r[lead[i]] > r[lead[i + 1]] for i in range(len(lead) - 1))
+
+
+def test_level_shard_split(P):
+    # the engine's split of a row-level (ptas_level_shard): aligned slices that tile [0, R)
+    rng = np.random.default_rng(11)
+    for _ in range(200):
+        R = int(rng.integers(0, 5000))
+        W = int(rng.integers(1, 8))
+        rb = int(rng.integers(1, 700))
+        cover = []
+        for g in range(W):
+            b, e, ch = P.ptas_level_shard(R, g, W, rb)
+            assert (ch * rb) % 16 == 0 and ch >= -(-R // W) if R else True
+            assert 0 <= b <= e <= R and (e == b or b == g * ch)
+            cover += list(range(b, e))
+        assert cover == list(range(R))
+    for bad in [(-1, 0, 1, 1), (5, 1, 1, 1), (5, 0, 0, 1), (5, 0, 1, 0)]:
+        with pytest.raises(P.PtasError):
+            P.ptas_level_shard(*bad)
