@@ -989,9 +989,9 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     if (trace) {
         const double t3 = trace_now();
         std::fprintf(stderr, "[ptas] dp sigma=%lld K=%d levels=%d host: setup+enum-sync %.3f ms, fill enqueue %.3f ms, "
-                             "wait %.3f ms | device: dp %.3f ms fill %.3f ms\n",
+                             "wait %.3f ms | device: dp %.3f ms fill %.3f ms | host clock %.3f .. %.3f ms\n",
                      (long long)sigma, K, g.rho_max + 1, 1e3 * (tr_enum - tr0), 1e3 * (tr_fillq - tr_enum),
-                     1e3 * (t3 - tr_fillq), 1e3 * o.dp_s, 1e3 * o.fill_s);
+                     1e3 * (t3 - tr_fillq), 1e3 * o.dp_s, 1e3 * o.fill_s, 1e3 * tr0, 1e3 * t3);
     }
     tl_np_hint = -1;
     if (h_meta_->ovf) {

@@ -141,7 +141,7 @@ class DpSlot {
     std::vector<int64_t> last_stride_; // internal strides
 };
 
-constexpr int MAX_SLOTS = 8;
+constexpr int MAX_SLOTS = 12;
 
 // Per-device engine: a lock serialising API calls on the device and up to
 // MAX_SLOTS DP slots.  Slot 0 serves every single-DP call.

@@ -57,6 +57,48 @@ void classify(const int64_t *p, int32_t n, int64_t T, int32_t k, Classified *c)
     }
 }
 
+// The same classes and counts (no per-job classes) from the distinct processing
+// times and their multiplicities, built once per solve: the search classifies
+// every probe (and the speculative chain ahead of it), and with n = 2000 jobs a
+// per-job pass costs tens of microseconds per probe on the host's critical path.
+struct ValueHistogram {
+    std::vector<int64_t> v;    // distinct p, ascending
+    std::vector<int32_t> c;    // multiplicities
+    ValueHistogram(const int64_t *p, int32_t n)
+    {
+        std::vector<int64_t> s(p, p + n);
+        std::sort(s.begin(), s.end());
+        for (int64_t x : s) {
+            if (!v.empty() && v.back() == x) ++c.back();
+            else {
+                v.push_back(x);
+                c.push_back(1);
+            }
+        }
+    }
+    void classify_counts(int64_t T, int32_t k, Classified *out) const
+    {
+        const int64_t kk = (int64_t)k * k;
+        out->u = std::max<int64_t>(1, T / kk);
+        const int64_t u = out->u;
+        out->r.clear();
+        out->N.clear();
+        out->cls.clear();
+        // long values: k * p > T, a suffix of the ascending list
+        size_t i = (size_t)(std::upper_bound(v.begin(), v.end(), T / k) - v.begin());
+        while (i > 0 && (__int128)k * v[i - 1] > (__int128)T) --i;
+        while (i < v.size() && !((__int128)k * v[i] > (__int128)T)) ++i;
+        for (; i < v.size(); ++i) {
+            const int64_t q = v[i] / u;
+            if (!out->r.empty() && out->r.back() == q * u) out->N.back() += c[i];
+            else {
+                out->r.push_back(q * u);
+                out->N.push_back(c[i]);
+            }
+        }
+    }
+};
+
 int probe_targets(int64_t LB, int64_t UB, int32_t P, std::vector<int64_t> *out)
 {
     out->clear();
@@ -308,6 +350,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     }
     std::map<std::vector<int64_t>, int32_t> memo;
     std::vector<ptas_probe> plog;
+    const ValueHistogram hist(p, n);   // classes and counts of every probe (per-job classes: classify)
     constexpr int32_t XERR = -1000;                          // MULTI_PROBE: exchanged error codes
     std::vector<std::vector<int64_t>> last_key_of(world);  // MULTI_PROBE: the last DP of each rank
     int round = 0;
@@ -385,16 +428,29 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             std::vector<int> rcs(nb, PTAS_OK);
             std::vector<std::vector<int>> orders(nb);
             for (int b = 0; b < nb; ++b) orders[b] = choose_order(cls_v[j0 + b].N, cls_v[j0 + b].r, opt.layout);
+            // persistent fill grids of concurrent DPs: each takes a share of the GPU,
+            // 1/nb (PTAS_GRID_SHARE=0) or proportional to its table size (1: the large
+            // DPs of a speculative chain outlive the small ones)
+            // (PTAS_GRID_DIV=0, experiment: every launch may take the whole GPU)
+            std::vector<int> gdiv(nb, 1);
+            if (share_grid && PTAS_KNOB("PTAS_GRID_DIV", -1) != 0) {
+                const bool prop = PTAS_KNOB("PTAS_GRID_SHARE", 0) == 1;
+                std::vector<double> sz(nb, 1.0);
+                double tot = 0;
+                for (int b = 0; b < nb; ++b) {
+                    if (prop)
+                        for (int32_t x : cls_v[j0 + b].N) sz[b] *= (double)x + 1.0;
+                    tot += sz[b];
+                }
+                for (int b = 0; b < nb; ++b) gdiv[b] = (int)std::max(1.0, std::min(1e6, std::floor(tot / sz[b])));
+            }
             auto work = [&](int b) {
                 if (cudaSetDevice(dev) != cudaSuccess) {
                     rcs[b] = PTAS_ECUDA;
                     return;
                 }
-                // PTAS_GRID_DIV (experiment knob): 0 = every launch may take the whole GPU
-                const int64_t gd_env = PTAS_KNOB("PTAS_GRID_DIV", -1);
                 rcs[b] = probe_dp(sl[b], cls_v[j0 + b], T_v[j0 + b], nullptr,
-                                  b == 0 ? (cudaStream_t)opt.stream : nullptr,
-                                  gd_env == 0 ? 1 : (share_grid ? nb : 1), &outs_all[j0 + b]);
+                                  b == 0 ? (cudaStream_t)opt.stream : nullptr, gdiv[b], &outs_all[j0 + b]);
             };
             std::vector<std::thread> th;
             for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
@@ -493,7 +549,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             probe_targets(nd.lb, nd.ub, 1, &t1);
             const int64_t T = t1[0];
             Classified c;
-            classify(p, n, T, k, &c);
+            hist.classify_counts(T, k, &c);
             bool take = false, lat = false;
             std::vector<int64_t> key;
             if (!c.N.empty()) {
@@ -532,8 +588,10 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 T_v.push_back(T);
                 key_v.push_back(key);
             }
-            // a chain of latency-bound DPs runs up to MAX_SLOTS deep
-            if (lat && spec_chain) depth_lim = MAX_SLOTS;
+            // a chain of latency-bound DPs runs deeper: up to MAX_SLOTS DPs over at most
+            // 16 probes (memo hits in the chain take no slot), so the whole all-feasible
+            // chain of an M5s-shaped search is in flight at once instead of in two batches
+            if (lat && spec_chain) depth_lim = (int)PTAS_KNOB("PTAS_SPEC_LAT_DEPTH", 16);
             if (nd.d + 1 < depth_lim && (int)cls_v.size() < MAX_SLOTS) {
                 q.push_back({nd.lb, T, nd.d + 1});        // T feasible
                 if (!spec_chain) q.push_back({T + 1, nd.ub, nd.d + 1});    // T infeasible
@@ -553,7 +611,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         std::vector<int64_t> Tj;
         probe_targets(LB, UB, P, &Tj);
         if (spec_on) {
-            classify(p, n, Tj[0], k, &cl);
+            hist.classify_counts(Tj[0], k, &cl);
             if (!cl.N.empty()) {
                 const std::vector<int64_t> key = memo_key(cl, Tj[0]);
                 if (!memo.count(key) && !spec.count(key)) {
@@ -572,7 +630,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         std::vector<std::vector<int64_t>> pend_key;
         std::vector<std::pair<int, int>> pend_alias;  // probe -> pending job
         for (int q = 0; q < np; ++q) {
-            classify(p, n, Tj[q], k, &cl);
+            hist.classify_counts(Tj[q], k, &cl);
             Kj[q] = (int32_t)cl.N.size();
             __int128 sg = 1;
             for (int32_t x : cl.N) {
@@ -775,8 +833,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
             }
         }
         if (std::getenv("PTAS_TRACE"))
-            std::fprintf(stderr, "[ptas] traceback at T*=%lld: %zu machines, %.3f ms (slot %d)\n", (long long)Ts,
-                         machines.size(), 1e3 * (now_s() - ttb0), tslot);
+            std::fprintf(stderr, "[ptas] traceback at T*=%lld: %zu machines, %.3f ms (slot %d) | host clock %.3f .. %.3f ms\n",
+                         (long long)Ts, machines.size(), 1e3 * (now_s() - ttb0), tslot, 1e3 * ttb0, 1e3 * now_s());
         acc.s.kernel_launches += tb.launches;
         acc.s.h2d_bytes += tb.h2d;
         acc.s.d2h_bytes += tb.d2h;
@@ -830,6 +888,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         acc.s.opt_at_Tstar = opt_star;
         acc.s.total_seconds = now_s() - t0;
         *stats = acc.s;
+        if (PTAS_KNOB("PTAS_TRACE", 0) == 1)
+            std::fprintf(stderr, "[ptas] solve | host clock %.3f .. %.3f ms\n", 1e3 * t0, 1e3 * now_s());
     }
     return PTAS_OK;
 }

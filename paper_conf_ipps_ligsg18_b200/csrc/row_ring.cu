@@ -26,7 +26,17 @@
 //   * the row goes to the own ring slot (shared memory) and to the table in HBM
 //     (the table is written once and never read back by this kernel);
 //   * one cluster barrier (arrive.release / wait.acquire) per level orders the
-//     ring writes of level L before the reads of level L + 1.
+//     ring writes of level L before the reads of level L + 1 (P2P = false), or
+//     (P2P = true) point-to-point signals instead: a CTA only ever reads the
+//     previous CTA's rows (s0 >= 0), so the halo rows are pushed with
+//     st.async, which completes bytes on an mbarrier of the receiving CTA (one
+//     per ring slot, armed with the level's halo byte count: the receiver
+//     waits for "level L - 1 has landed" with no fence on either side), and a
+//     CTA overwrites a halo slot of CTA c + 1 only after c + 1 has reported
+//     (a relaxed store into this CTA's shared memory) that it finished every
+//     level reading it.  The CTAs then run as a pipeline, up to
+//     Rslots - Rdep levels apart, with two __syncthreads per level instead of
+//     one barrier over the cluster.
 //
 // Same recurrence, same windows, same executed relaxations as the packed
 // kernel; the values are bit-identical (parity tests, PTAS_RING=0 for the A/B).
@@ -35,6 +45,9 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cuda_runtime.h>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 #include "internal.h"
 #include "swar_common.cuh"
@@ -124,6 +137,54 @@ __device__ __forceinline__ void cluster_sync_all()
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// P2P signalling: mbarriers of the ring slots (halo bytes land through st.async
+// complete_tx) and a progress word written by the next CTA
+__device__ __forceinline__ void mbar_init(uint32_t a, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arm(uint32_t a, uint32_t bytes)
+{
+    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(a), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity)
+{
+    asm volatile("{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+                 "@!p bra WAIT_%=;\n\t}" ::"r"(a), "r"(parity)
+                 : "memory");
+}
+// CH words into the next CTA's ring, completing 4 * CH bytes on its slot mbarrier
+template <int CH>
+__device__ __forceinline__ void st_async_words(uint32_t addr, const Words<CH> &w, uint32_t mbar)
+{
+    if constexpr (CH == 1) {
+        asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(addr),
+                     "r"(w.v[0]), "r"(mbar) : "memory");
+    } else if constexpr (CH == 2) {
+        asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.b32 [%0], {%1, %2}, [%3];" ::"r"(addr),
+                     "r"(w.v[0]), "r"(w.v[1]), "r"(mbar) : "memory");
+    } else {
+#pragma unroll
+        for (int c = 0; c < CH; c += 4)
+            asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+                             addr + 4 * c),
+                         "r"(w.v[c]), "r"(w.v[c + 1]), "r"(w.v[c + 2]), "r"(w.v[c + 3]), "r"(mbar)
+                         : "memory");
+    }
+}
+__device__ __forceinline__ int ld_relaxed_cluster(uint32_t addr)
+{
+    int v;
+    asm volatile("ld.relaxed.cluster.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_cluster(uint32_t addr, int v)
+{
+    asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+
 // Windows of one prefix for the lane's CH words: class 1 = shift of at most one
 // word (db <= 4 bytes: words w - 1, w), class 2 = at most two (4 < db <= 8:
 // words w - 2, w - 1); w1 / w2 = the words left of the chunk.
@@ -144,7 +205,7 @@ __device__ __forceinline__ void ring_windows(const Words<CH> &cur, uint32_t w1, 
     }
 }
 
-template <typename E, int CH, int WIN>
+template <typename E, int CH, int WIN, bool P2P>
 __global__ void __launch_bounds__(1024, 1)
 row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta)
 {
@@ -164,7 +225,19 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
     int4 *s_pl = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * AH * row_bytes + 15) & ~(size_t)15));
     const int lcap = np + PB;
     __shared__ int s_cnt[4];
+    // P2P: s_full[slot] = halo bytes of the slot's level have landed; s_dn = last
+    // level CTA c + 1 has finished
+    constexpr int MAXR = 64;
+    __shared__ __align__(8) unsigned long long s_full[P2P ? MAXR : 1];
+    __shared__ int s_dn;
     if (threadIdx.x < 4) s_cnt[threadIdx.x] = 0;
+    if constexpr (P2P) {
+        if (threadIdx.x == 0) {
+            s_dn = -1;
+            for (int i = 0; i < ra.R; ++i) mbar_init((uint32_t)__cvta_generic_to_shared(&s_full[i]), 1);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+    }
     __syncthreads();
     // prefix lists by (pivot block, window class): list 2*blk + cls - 1, blk 0 = {s0 = 0}
     // (rows a = 0), blk 1 = {s0 >= 1} (rows a >= 1); entries (s0, s1, selector | db << 16,
@@ -186,8 +259,21 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
     // the next CTA's ring: this CTA's top H rows of every level are pushed into its halo
     const bool has_next = crank + 1 < csize;
     const uint32_t nxt = dsm_map((uint32_t)__cvta_generic_to_shared(ring), has_next ? crank + 1 : crank);
+    const bool has_prev = crank > 0;
+    const uint32_t full_own = (uint32_t)__cvta_generic_to_shared(&s_full[0]);
+    const uint32_t full_next = dsm_map(full_own, has_next ? crank + 1 : crank);   // CTA c + 1's s_full
+    const uint32_t dn_own = (uint32_t)__cvta_generic_to_shared(&s_dn);
+    const uint32_t dn_prev = dsm_map(dn_own, has_prev ? crank - 1 : crank);       // CTA c - 1's s_dn
+    // a halo slot of CTA c + 1 last held level L - R; c + 1 reads it up to level L - R + Rdep - 1
+    const int dn_lag = ra.R - ra.Rdep + 1;
+    // halo bytes this CTA receives for level L: the previous CTA's top H rows of the level
+    auto halo_bytes = [&](int L) -> uint32_t {
+        const int ap = ((int)crank - 1) * ra.A;
+        const int l = max(max(L - ra.N1, 0), ap + ra.A - ra.H), h = min(min(L, ra.N0), ap + ra.A - 1);
+        return h >= l ? (uint32_t)(h - l + 1) * (uint32_t)Lw * 4u : 0u;
+    };
     __syncthreads();
-    cluster_sync_all();   // every CTA of the cluster runs before any DSMEM access
+    cluster_sync_all();   // every CTA of the cluster runs (and has initialised its words) before any DSMEM access
 
     const int a0 = (int)crank * ra.A;          // first row digit a of this CTA
     uint32_t *tab32 = reinterpret_cast<uint32_t *>(table);
@@ -203,6 +289,15 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
         const int lo = max(max(L - ra.N1, 0), a0);
         const int hi = min(min(L, ra.N0), a0 + ra.A - 1);
         const int ntask = hi >= lo ? (hi - lo + 1) * Lg : 0;
+        if constexpr (P2P) {
+            // arm this level's halo slot (phase L / R) with the bytes the previous CTA
+            // will push into it; its previous phase (level L - R) has landed first
+            if (threadIdx.x == 0 && has_prev) {
+                const int sl = L % ra.R;
+                if (L >= ra.R) mbar_wait(full_own + 8u * (uint32_t)sl, (uint32_t)(((L - ra.R) / ra.R) & 1));
+                mbar_arm(full_own + 8u * (uint32_t)sl, halo_bytes(L));
+            }
+        }
         for (int task = threadIdx.x; task < ntask; task += blockDim.x) {
             const int r_ = task / Lg;
             const int a = lo + r_;
@@ -214,6 +309,22 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
             fill_words(ae, 0xffffffffu);
             fill_words(ao, 0xffffffffu);
             const int blk = a >= 1 ? 1 : 0;    // pivot block (D13)
+            if constexpr (P2P) {
+                // only the bottom H rows read the halo (s0 <= H): they wait until the
+                // previous CTA's rows of the levels they read (L - Rdep + 1 .. L - 1)
+                // have landed; every other row starts at once (the CTAs run skewed)
+                if (has_prev && ia < ra.H) {
+                    for (int j = 1; j < ra.Rdep && j <= L; ++j) {
+                        const int Lj = L - j;
+                        mbar_wait(full_own + 8u * (uint32_t)(Lj % ra.R), (uint32_t)((Lj / ra.R) & 1));
+                    }
+                }
+                // the top H rows are pushed into CTA c + 1's ring: it has finished the
+                // levels that read the slot they overwrite
+                if (has_next && ia >= ra.A - ra.H)
+                    while (ld_relaxed_cluster(dn_own) < L - dn_lag) {
+                    }
+            }
 #pragma unroll
             for (int cls = 1; cls <= (WIN == 8 ? 2 : 1); ++cls) {
                 const int4 *pl = s_pl + (2 * blk + cls - 1) * lcap;
@@ -277,8 +388,11 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
                 wv.v[t] = EB == 1 ? prmt(oe, oo, 0x6240u) : oe;
             }
             store_words<CH>(ring + ((size_t)slot * AH + ra.H + ia) * Lw + c * CH, wv);
-            if (has_next && ia >= ra.A - ra.H)   // halo of the next CTA (one DSMEM store per word)
-                st_dsm<CH>(nxt + 4u * (uint32_t)(((slot * AH + ia - (ra.A - ra.H)) * Lw + c * CH)), wv);
+            if (has_next && ia >= ra.A - ra.H) {   // halo of the next CTA
+                const uint32_t hp = nxt + 4u * (uint32_t)(((slot * AH + ia - (ra.A - ra.H)) * Lw + c * CH));
+                if constexpr (P2P) st_async_words<CH>(hp, wv, full_next + 8u * (uint32_t)slot);
+                else st_dsm<CH>(hp, wv);
+            }
             if (task + (int)blockDim.x < ntask) {   // (not the thread's last row of the level)
                 const int64_t rowbase = (int64_t)a * ra.stride0 + (int64_t)b * ra.Wp;   // elements
                 store_words<CH>(tab32 + rowbase * EB / 4 + c * CH, wv);
@@ -292,19 +406,39 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
 #if PTAS_RING_PROFILE
         if (pr) g_ring_prof[1][L] = clock64();
 #endif
-        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+        if constexpr (P2P) {
+            __syncthreads();   // own ring rows of level L written, halo pushes issued, ring reads done
 #if PTAS_RING_PROFILE
-        if (pr) g_ring_prof[2][L] = clock64();
+            if (pr) g_ring_prof[2][L] = clock64();
+#endif
+            // (every read of the ring for level L has returned: the previous CTA may reuse the slots)
+            if (threadIdx.x == 0 && has_prev) st_relaxed_cluster(dn_prev, L);
+            if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
+            last_off = -1;
+        } else {
+            asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+#if PTAS_RING_PROFILE
+            if (pr) g_ring_prof[2][L] = clock64();
 #endif
 #ifndef PTAS_RING_NOSTORE
-        if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
+            if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
 #endif
-        last_off = -1;
-        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+            last_off = -1;
+            asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+        }
 #if PTAS_RING_PROFILE
         if (pr) g_ring_prof[3][L] = clock64();
 #endif
         slot = slot + 1 == ra.R ? 0 : slot + 1;
+    }
+    // P2P: the last level's halo has landed, and no CTA exits while a neighbour
+    // may still access its shared memory
+    if constexpr (P2P) {
+        if (threadIdx.x == 0 && has_prev)
+            for (int Lj = max(0, ra.rho_max - ra.R + 1); Lj <= ra.rho_max; ++Lj)
+                mbar_wait(full_own + 8u * (uint32_t)(Lj % ra.R), (uint32_t)((Lj / ra.R) & 1));
+        __syncthreads();
+        cluster_sync_all();
     }
 }
 
@@ -312,15 +446,16 @@ template <typename E, int CH, int WIN>
 cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_pref, const DpMeta *d_meta,
                           int64_t nP_bound, int csize, cudaStream_t st, bool dry)
 {
-    auto kfn = row_ring_kernel<E, CH, WIN>;
+    auto kfn = ra.p2p ? row_ring_kernel<E, CH, WIN, true> : row_ring_kernel<E, CH, WIN, false>;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
     const size_t smem = (((size_t)ra.R * (ra.A + ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
-    cudaError_t err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (smem > 220 * 1024) return cudaErrorNotSupported;
+    // function attributes and the co-residency query once per (device, kernel,
+    // smem, cluster size, block): they take the driver lock, and concurrent DP
+    // slots issue from several host threads
+    int dev = 0;
+    cudaError_t err = cudaGetDevice(&dev);
     if (err != cudaSuccess) return err;
-    if (csize > 8) {
-        err = cudaFuncSetAttribute(kfn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-        if (err != cudaSuccess) return err;
-    }
     const int lanes = ra.A * ra.Lg;
     const int warps = std::min(32, (lanes + 31) / 32);
     cudaLaunchConfig_t cfg = {};
@@ -335,12 +470,30 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
     cfg.stream = st;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    int ncl = 0;
-    err = cudaOccupancyMaxActiveClusters(&ncl, kfn, &cfg);
-    if (err != cudaSuccess || ncl < 1) {
-        cudaGetLastError();
-        return cudaErrorNotSupported;
+    static std::mutex mu;
+    static std::map<std::tuple<int, const void *, size_t, int, int>, int> ncl_cache;
+    const auto key = std::make_tuple(dev, (const void *)kfn, smem, csize, warps);
+    int ncl = -1;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = ncl_cache.find(key);
+        if (it != ncl_cache.end()) ncl = it->second;
     }
+    if (ncl < 0) {
+        err = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+        if (err == cudaSuccess && csize > 8) err = cudaFuncSetAttribute(kfn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (err == cudaSuccess) err = cudaOccupancyMaxActiveClusters(&ncl, kfn, &cfg);
+        if (err != cudaSuccess) {
+            cudaGetLastError();
+            ncl = 0;
+        }
+        std::lock_guard<std::mutex> lk(mu);
+        ncl_cache[key] = ncl;
+    }
+    if (ncl < 1) return cudaErrorNotSupported;
+    if (!dry && PTAS_KNOB("PTAS_TRACE", 0) == 1)
+        std::fprintf(stderr, "[ring] cluster %d x %d threads, smem %zu B, slots %d (dep %d), %s: %d clusters co-resident\n",
+                     csize, 32 * warps, smem, ra.R, ra.Rdep, ra.p2p ? "p2p" : "barrier", ncl);
     if (dry) return cudaSuccess;
     err = cudaLaunchKernelEx(&cfg, kfn, (E *)table, ra, d_pref, d_meta);
 #if PTAS_RING_PROFILE
@@ -424,7 +577,7 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     if (g.K1 != 2 || (g.Wp * e) % 4 != 0) return cudaErrorNotSupported;
     const int Lw = (int)(g.Wp * e / 4);
     // windows up to two words left (J0 * e <= 8 bytes: the M5s shapes have 6)
-    if (J0 * e > 8 || nP_bound > 4096) return cudaErrorNotSupported;
+    if (J0 * e > 8) return cudaErrorNotSupported;
     if (PTAS_KNOB("PTAS_RING", 1) == 0) return cudaErrorNotSupported;
     RingArgs ra;
     ra.N0 = N[0];
@@ -436,8 +589,19 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     // ring depth: 1 + the largest leading-digit sum of a configuration, bounded by
     // min(hi0 + hi1, floor(T / min(r0, r1)))
     const int64_t hi0 = std::min<int64_t>(N[0], T / r[0]), hi1 = std::min<int64_t>(N[1], T / r[1]);
-    ra.R = (int)std::min<int64_t>(hi0 + hi1, T / std::min(r[0], r[1])) + 1;
+    // the prefix lists hold the distinct leading parts (s0, s1) <= (hi0, hi1): size the
+    // shared memory by that, not by the engine's generic bound (which is NP_CAP when
+    // the DP is enqueued without reading |C| back): a 16-CTA cluster of 1 CTA per SM
+    // fits 7 times on the GPU, of 2 CTAs per SM 14 times (measured), so concurrent
+    // ring DPs of a speculative chain all co-reside only with the tight size
+    nP_bound = std::min<int64_t>(nP_bound, (hi0 + 1) * (hi1 + 1));
+    if (nP_bound > 4096) return cudaErrorNotSupported;
+    ra.Rdep = (int)std::min<int64_t>(hi0 + hi1, T / std::min(r[0], r[1])) + 1;
     ra.rho_max = N[0] + N[1];
+    // extra ring slots: how many levels a CTA may run ahead of the next one (P2P)
+    // (P2P: one mbarrier per ring slot, at most 64)
+    ra.p2p = PTAS_KNOB("PTAS_RING_P2P", 0) != 0 && ra.Rdep <= 64 ? 1 : 0;
+    const int extra = ra.p2p ? (int)std::min<int64_t>(64 - ra.Rdep, std::max<int64_t>(0, PTAS_KNOB("PTAS_RING_EXTRA", 2))) : 0;
     const int win = J0 * e <= 4 ? 4 : 8;
     const size_t smem_cap = 220 * 1024;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
@@ -447,8 +611,12 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
         ra.A = (N[0] + csize) / csize;   // ceil((N0 + 1) / C) rows of each level per CTA
         ra.H = (int32_t)hi0;              // halo rows (s0 <= hi0)
         if (ra.A < hi0) continue;         // every source row is in this CTA's block or the previous one
-        const size_t smem = (((size_t)ra.R * (ra.A + ra.H) * Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
-        if (smem > smem_cap) continue;
+        auto smem_of = [&](int slots) {
+            return (((size_t)slots * (ra.A + ra.H) * Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
+        };
+        if (smem_of(ra.Rdep) > smem_cap) continue;
+        ra.R = ra.Rdep + extra;
+        while (ra.R > ra.Rdep && smem_of(ra.R) > smem_cap) --ra.R;
         // words per lane: the smallest chunk with one pass over the CTA's rows of a level
         // words per lane: 4 when the CTA's rows of a level fit one pass (measured best on
         // M5s: 2 words 1.82 / 1.69 ms, 4 words 1.39 / 1.48 ms, 8 words 1.94 / 1.96 ms per DP),

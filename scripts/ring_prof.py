@@ -12,8 +12,9 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 p = w.p()
 k = P.ptas_k(w.eps)
 LB, UB = P.ptas_bounds(p, w.m)
-c = P.ptas_classify(p, LB, k)
-N, r = np.asarray(c["N"], np.int32), np.asarray(c["r"], np.int64)
+u, r, N, _ = P.ptas_classify(p, LB, k)
+o = P.ptas_table_order(N, r)            # the solve's internal class order
+N, r = N[o].astype(np.int32), r[o].astype(np.int64)
 print(w.name, "LB", LB, "N", N.tolist(), "r", r.tolist(), flush=True)
 for i in range(reps):
     t0 = time.perf_counter()
