@@ -702,6 +702,91 @@ traceback_warp_kernel(const E *__restrict__ table, int K, const int32_t *__restr
     }
 }
 
+// Same traceback with everything in registers (nC <= 32 G configurations, K <=
+// KM classes): lane l owns configurations l, l + 32 (digits, offset, rank), the
+// state n is replicated in every lane, OPT(n) is tracked instead of re-read
+// (each step lowers it by exactly one), so a step is ONE table load per owned
+// configuration, a min-reduction over the ranks and K shuffles of the chosen
+// digits.  Same choices as the one-step kernels (reading R11).
+template <typename E, int G, int KM>
+__global__ void __launch_bounds__(32)
+traceback_reg_kernel(const E *__restrict__ table, int K, const int32_t *__restrict__ N,
+                     const uint16_t *__restrict__ digits, const int64_t *__restrict__ off,
+                     const int32_t *__restrict__ rank, int nC, int64_t idx_start, int32_t *__restrict__ out,
+                     int32_t max_out, int32_t *__restrict__ len, DpMeta *meta, const int32_t *__restrict__ inv,
+                     int Kc, int32_t *__restrict__ out_dig)
+{
+    const int lane = threadIdx.x;
+    int dg[G][KM];
+    int64_t of[G];
+    uint32_t rk[G];
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+        const int c = lane + 32 * g;
+        const bool ex = c < nC;
+        of[g] = ex ? off[c] : 0;
+        rk[g] = ex ? (uint32_t)rank[c] : 0xffffffffu;
+#pragma unroll
+        for (int i = 0; i < KM; ++i) dg[g][i] = (ex && i < K) ? (int)digits[(size_t)c * K + i] : (1 << 30);
+    }
+    int cur[KM];
+#pragma unroll
+    for (int i = 0; i < KM; ++i) cur[i] = i < K ? N[i] : (1 << 30);
+    int64_t idx = idx_start;
+    int v = (int)table[idx];
+    int32_t mu = 0;
+    bool err = false;
+    while (idx != 0) {
+        int val[G];
+#pragma unroll
+        for (int g = 0; g < G; ++g) {
+            bool dom = true;
+#pragma unroll
+            for (int i = 0; i < KM; ++i) dom &= dg[g][i] <= cur[i];
+            val[g] = dom ? (int)table[idx - of[g]] : -1;
+        }
+        uint32_t br = 0xffffffffu;
+        int bg = 0;
+#pragma unroll
+        for (int g = 0; g < G; ++g)
+            if (val[g] == v - 1 && rk[g] < br) {
+                br = rk[g];
+                bg = g;
+            }
+        const uint32_t m = __reduce_min_sync(FULL, br);
+        if (m == 0xffffffffu || mu >= max_out) {
+            err = true;
+            break;
+        }
+        const int src = __ffs(__ballot_sync(FULL, br == m)) - 1;
+        const int g_ = __shfl_sync(FULL, bg, src);
+        int dd[KM];
+#pragma unroll
+        for (int i = 0; i < KM; ++i) {
+            const int mine = G == 1 ? dg[0][i] : (bg == 1 ? dg[G - 1][i] : dg[0][i]);
+            dd[i] = __shfl_sync(FULL, mine, src);
+            cur[i] -= i < K ? dd[i] : 0;
+        }
+        const int64_t myoff = G == 1 ? of[0] : (bg == 1 ? of[G - 1] : of[0]);
+        idx -= __shfl_sync(FULL, myoff, src);
+        --v;
+        if (lane == 0) out[mu] = src + 32 * g_;
+        if (out_dig)   // the machine's configuration in canonical class order
+            for (int j = lane; j < Kc; j += 32) {
+                const int ij = inv[j];
+                int d = 0;
+#pragma unroll
+                for (int i = 0; i < KM; ++i) d = i == ij ? dd[i] : d;
+                out_dig[(size_t)mu * Kc + j] = d;
+            }
+        ++mu;
+    }
+    if (lane == 0) {
+        *len = mu;
+        if (err) meta->err = 1;
+    }
+}
+
 // Canonical lexicographic rank of every configuration (reading R11): rank(c)
 // = #{c' : key(c') < key(c)}, key = the digits in canonical class order
 // (inv[j] = internal position of canonical class j, -1 = empty class, digit 0).
@@ -976,6 +1061,22 @@ cudaError_t launch_traceback_canon(int e, const void *table, int K, const int32_
     const size_t smem = (size_t)nC * (8 + 4) + (size_t)K * 4 + (size_t)nC * K * 2 + 16;
     if (smem > 48 * 1024 || nC > (1 << 20) || PTAS_KNOB("PTAS_TB_BLOCK", 0) == 1) return cudaErrorNotSupported;
     rank_configs_kernel<<<(unsigned)((nC + 127) / 128), 128, 0, st>>>(d_digits, (int)nC, K, d_inv, Kc, d_rank);
+    // configurations and state in registers when they fit (PTAS_TB_REG=0: shared-memory warp kernel)
+    if (nC <= 64 && K <= 12 && PTAS_KNOB("PTAS_TB_REG", 1) != 0) {
+#define PTAS_TB_REG_GO(E_, G_, KM_)                                                                          \
+    traceback_reg_kernel<E_, G_, KM_><<<1, 32, 0, st>>>((const E_ *)table, K, d_N, d_digits, d_off, d_rank, (int)nC, \
+                                                        idx_start, d_out, max_out, d_len, d_meta, d_inv, Kc, d_out_dig)
+        const bool g1 = nC <= 32, k8 = K <= 8;
+        if (e == 1) {
+            if (g1) { if (k8) PTAS_TB_REG_GO(uint8_t, 1, 8); else PTAS_TB_REG_GO(uint8_t, 1, 12); }
+            else { if (k8) PTAS_TB_REG_GO(uint8_t, 2, 8); else PTAS_TB_REG_GO(uint8_t, 2, 12); }
+        } else {
+            if (g1) { if (k8) PTAS_TB_REG_GO(uint16_t, 1, 8); else PTAS_TB_REG_GO(uint16_t, 1, 12); }
+            else { if (k8) PTAS_TB_REG_GO(uint16_t, 2, 8); else PTAS_TB_REG_GO(uint16_t, 2, 12); }
+        }
+#undef PTAS_TB_REG_GO
+        return cudaGetLastError();
+    }
     if (e == 1)
         traceback_warp_kernel<uint8_t><<<1, 32, smem, st>>>((const uint8_t *)table, K, d_N, d_digits, d_off, d_rank,
                                                             (int)nC, idx_start, d_out, max_out, d_len, d_meta, d_inv,

@@ -1,0 +1,3 @@
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_shaped.py -m gpu -q -x -k "traceback or solve or shaped or hmbp" 2>&1 | tail -2
+bash scripts/r02_tl.sh
+WLS="M5s-0.3 M5s-0.2 M2s" ENVS="NONE=0 PTAS_TB_LA=0" bash scripts/knob_ab.sh

@@ -543,11 +543,15 @@ def test_hmbp_parity(P):
     assert bins == P.dp_fill(N, r, 1674, table=False)[0]
 
 
-@pytest.mark.parametrize("tb", ["0", "1"])
+@pytest.mark.parametrize("tb", ["0", "1", "reg0"])
 def test_traceback_kernels(P, monkeypatch, tb):
-    """Warp traceback (configurations in shared memory) and the block kernel:
+    """Register traceback (default for |C| <= 64, K <= 12), warp traceback
+    (configurations in shared memory, PTAS_TB_REG=0) and the block kernel:
     identical schedules, equal to the oracle's (reading R11)."""
-    monkeypatch.setenv("PTAS_TB_BLOCK", tb)
+    if tb == "reg0":
+        monkeypatch.setenv("PTAS_TB_REG", "0")
+    else:
+        monkeypatch.setenv("PTAS_TB_BLOCK", tb)
     for seed in range(12):
         _cmp_solve(P, jobs(12, 100, seed), 3, 0.3, 1)
     for (n, m, eps, seed) in [(40, 8, 0.3, 1), (60, 14, 0.3, 2), (50, 10, 0.2, 3)]:
