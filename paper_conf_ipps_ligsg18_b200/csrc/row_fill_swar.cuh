@@ -100,10 +100,12 @@ static cudaError_t prepare_const_prefix_tu(const PrefixEntry *d_pref, const DpMe
 // are unused, the row sets come from df).
 // Resident blocks per SM the compiler must allow (register cap 65536 / (256 * MINB)):
 // uint16 tables 4 (64 registers: M3s 8.8 -> 8.1 ms, M5s-0.15 21.8 -> 20.3 ms fill,
-// measured), uint8 tables 3 (80 registers; 64 spills: M2s 3.40 -> 3.59 ms;
-// uncapped, the dominance-table code takes 90-96 and 2 blocks/SM: M4s +13%).
+// measured), uint8 tables 4 (64 registers, round 2: M2s 2.31 -> 2.23 ms, M4x
+// 96.4 -> 94.8 ms, M4s / M3g unchanged, against 3 blocks at 80 registers; in
+// round 1, before the pivot blocks, 64 spilled: M2s 3.40 -> 3.59 ms; uncapped,
+// the dominance-table code takes 90-96 and 2 blocks/SM: M4s +13%).
 #ifndef PTAS_MINB_U8
-#define PTAS_MINB_U8 3
+#define PTAS_MINB_U8 4
 #endif
 #ifndef PTAS_MINB_U16
 #define PTAS_MINB_U16 4

@@ -2,8 +2,8 @@
 mkdir -p gpurun_out
 for W in ${WLS:-M2s}; do
   for E in ${ENVS:-NONE=0}; do
-    env ${E//,/ } timeout 300 python bench.py --workload $W --no-cpu-baseline --no-blocks --steps ${STEPS:-10} --warmup 3 > gpurun_out/kab_${W}_${E//[,=/]/_}.log 2>&1
-    tail -1 gpurun_out/kab_${W}_${E//[,=/]/_}.log | python -c "
+    env ${E//,/ } timeout 300 python bench.py --workload $W --no-cpu-baseline --no-blocks --steps ${STEPS:-10} --warmup 3 > gpurun_out/kab_${W}_${E//[,=\/]/_}.log 2>&1
+    tail -1 gpurun_out/kab_${W}_${E//[,=\/]/_}.log | python -c "
 import json,sys
 try:
   d=json.loads(sys.stdin.read()); r=d['roofline']
