@@ -141,12 +141,12 @@ struct RingArgs {
     int32_t Wp;           // row pitch (elements)
     int32_t Lw, Lg;       // words per row, lanes per row (Lw / CH)
     int32_t J0;           // min(N_last, floor(T / r_last))
-    int32_t R;            // ring slots (row-levels resident); >= Rdep
+    int32_t R;            // ring slots (row-levels resident): Rdep + TB - 1
     int32_t Rdep;         // dependency depth: 1 + the largest leading-digit sum of a configuration
-    int32_t A;            // ring rows per level per CTA: ceil((N0 + 1) / cluster size)
-    int32_t H;            // halo rows: copies of the previous CTA's top H rows (H = max s0 <= A)
+    int32_t A;            // own rows per level per CTA: ceil((N0 + 1) / cluster size)
+    int32_t H;            // rows per level below the block a row can read (H = max s0 <= A)
+    int32_t TB;           // row-levels per cluster barrier; the halo holds TB * H rows per level
     int32_t rho_max;      // N0 + N1
-    int32_t p2p;          // 1: point-to-point halo signals (st.async + mbarriers), 0: cluster barrier per level
 };
 
 // Device-side summary written by the planning kernels and read back once.

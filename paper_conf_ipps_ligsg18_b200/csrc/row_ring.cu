@@ -25,18 +25,13 @@
 //     OPT(a, b, x) = 1 + the minimum (D12); row (0, 0) is ceil(x / J0);
 //   * the row goes to the own ring slot (shared memory) and to the table in HBM
 //     (the table is written once and never read back by this kernel);
-//   * one cluster barrier (arrive.release / wait.acquire) per level orders the
-//     ring writes of level L before the reads of level L + 1 (P2P = false), or
-//     (P2P = true) point-to-point signals instead: a CTA only ever reads the
-//     previous CTA's rows (s0 >= 0), so the halo rows are pushed with
-//     st.async, which completes bytes on an mbarrier of the receiving CTA (one
-//     per ring slot, armed with the level's halo byte count: the receiver
-//     waits for "level L - 1 has landed" with no fence on either side), and a
-//     CTA overwrites a halo slot of CTA c + 1 only after c + 1 has reported
-//     (a relaxed store into this CTA's shared memory) that it finished every
-//     level reading it.  The CTAs then run as a pipeline, up to
-//     Rslots - Rdep levels apart, with two __syncthreads per level instead of
-//     one barrier over the cluster.
+//   * one cluster barrier (arrive.release / wait.acquire) per TB row-levels
+//     (temporal blocking, TB = 2 by default) orders the ring writes of an
+//     interval before the reads of the next: at sub-level t of an interval
+//     each CTA also computes, redundantly, the (TB - 1 - t) * H rows just
+//     below its block (the previous CTA's rows: same inputs, same values), so
+//     every source row of the interval is in its own ring; the halo holds
+//     TB * H rows per level, the ring Rdep + TB - 1 levels.
 //
 // Same recurrence, same windows, same executed relaxations as the packed
 // kernel; the values are bit-identical (parity tests, PTAS_RING=0 for the A/B).
@@ -137,54 +132,6 @@ __device__ __forceinline__ void cluster_sync_all()
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-// P2P signalling: mbarriers of the ring slots (halo bytes land through st.async
-// complete_tx) and a progress word written by the next CTA
-__device__ __forceinline__ void mbar_init(uint32_t a, uint32_t count)
-{
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arm(uint32_t a, uint32_t bytes)
-{
-    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(a), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity)
-{
-    asm volatile("{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
-                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-                 "@!p bra WAIT_%=;\n\t}" ::"r"(a), "r"(parity)
-                 : "memory");
-}
-// CH words into the next CTA's ring, completing 4 * CH bytes on its slot mbarrier
-template <int CH>
-__device__ __forceinline__ void st_async_words(uint32_t addr, const Words<CH> &w, uint32_t mbar)
-{
-    if constexpr (CH == 1) {
-        asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(addr),
-                     "r"(w.v[0]), "r"(mbar) : "memory");
-    } else if constexpr (CH == 2) {
-        asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.b32 [%0], {%1, %2}, [%3];" ::"r"(addr),
-                     "r"(w.v[0]), "r"(w.v[1]), "r"(mbar) : "memory");
-    } else {
-#pragma unroll
-        for (int c = 0; c < CH; c += 4)
-            asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
-                             addr + 4 * c),
-                         "r"(w.v[c]), "r"(w.v[c + 1]), "r"(w.v[c + 2]), "r"(w.v[c + 3]), "r"(mbar)
-                         : "memory");
-    }
-}
-__device__ __forceinline__ int ld_relaxed_cluster(uint32_t addr)
-{
-    int v;
-    asm volatile("ld.relaxed.cluster.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_relaxed_cluster(uint32_t addr, int v)
-{
-    asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
-}
-
 // Windows of one prefix for the lane's CH words: class 1 = shift of at most one
 // word (db <= 4 bytes: words w - 1, w), class 2 = at most two (4 < db <= 8:
 // words w - 2, w - 1); w1 / w2 = the words left of the chunk.
@@ -205,7 +152,7 @@ __device__ __forceinline__ void ring_windows(const Words<CH> &cur, uint32_t w1, 
     }
 }
 
-template <typename E, int CH, int WIN, bool P2P>
+template <typename E, int CH, int WIN>
 __global__ void __launch_bounds__(1024, 1)
 row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpref, const DpMeta *__restrict__ meta)
 {
@@ -219,25 +166,16 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
     const int np = (int)(meta->nP - 1);
     const int Lw = ra.Lw, Lg = ra.Lg;
     const uint32_t row_bytes = (uint32_t)Lw * 4;
-    // smem: ring [R][A][Lw] words | 4 prefix lists int4 [np + PB] each
+    // smem: ring [R][HT + A][Lw] words (per slot: HT halo rows a0 - HT .. a0 - 1,
+    // then the A own rows) | 4 prefix lists int4 [np + PB] each
     uint32_t *ring = reinterpret_cast<uint32_t *>(smem_raw);
-    const int AH = ra.A + ra.H;                  // ring rows per level: H halo rows, then A own rows
+    const int TB = ra.TB;                        // row-levels per cluster barrier
+    const int HT = TB * ra.H;                    // halo rows per slot
+    const int AH = ra.A + HT;
     int4 *s_pl = reinterpret_cast<int4 *>(smem_raw + (((size_t)ra.R * AH * row_bytes + 15) & ~(size_t)15));
     const int lcap = np + PB;
     __shared__ int s_cnt[4];
-    // P2P: s_full[slot] = halo bytes of the slot's level have landed; s_dn = last
-    // level CTA c + 1 has finished
-    constexpr int MAXR = 64;
-    __shared__ __align__(8) unsigned long long s_full[P2P ? MAXR : 1];
-    __shared__ int s_dn;
     if (threadIdx.x < 4) s_cnt[threadIdx.x] = 0;
-    if constexpr (P2P) {
-        if (threadIdx.x == 0) {
-            s_dn = -1;
-            for (int i = 0; i < ra.R; ++i) mbar_init((uint32_t)__cvta_generic_to_shared(&s_full[i]), 1);
-            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        }
-    }
     __syncthreads();
     // prefix lists by (pivot block, window class): list 2*blk + cls - 1, blk 0 = {s0 = 0}
     // (rows a = 0), blk 1 = {s0 >= 1} (rows a >= 1); entries (s0, s1, selector | db << 16,
@@ -256,189 +194,140 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
             make_int4(1 << 20, 1 << 20, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF, 0);
     uint32_t csize;
     asm("mov.u32 %0, %%cluster_nctarank;" : "=r"(csize));
-    // the next CTA's ring: this CTA's top H rows of every level are pushed into its halo
+    // the next CTA's ring: this CTA's top HT rows of every level are pushed into its halo
     const bool has_next = crank + 1 < csize;
     const uint32_t nxt = dsm_map((uint32_t)__cvta_generic_to_shared(ring), has_next ? crank + 1 : crank);
-    const bool has_prev = crank > 0;
-    const uint32_t full_own = (uint32_t)__cvta_generic_to_shared(&s_full[0]);
-    const uint32_t full_next = dsm_map(full_own, has_next ? crank + 1 : crank);   // CTA c + 1's s_full
-    const uint32_t dn_own = (uint32_t)__cvta_generic_to_shared(&s_dn);
-    const uint32_t dn_prev = dsm_map(dn_own, has_prev ? crank - 1 : crank);       // CTA c - 1's s_dn
-    // a halo slot of CTA c + 1 last held level L - R; c + 1 reads it up to level L - R + Rdep - 1
-    const int dn_lag = ra.R - ra.Rdep + 1;
-    // halo bytes this CTA receives for level L: the previous CTA's top H rows of the level
-    auto halo_bytes = [&](int L) -> uint32_t {
-        const int ap = ((int)crank - 1) * ra.A;
-        const int l = max(max(L - ra.N1, 0), ap + ra.A - ra.H), h = min(min(L, ra.N0), ap + ra.A - 1);
-        return h >= l ? (uint32_t)(h - l + 1) * (uint32_t)Lw * 4u : 0u;
-    };
     __syncthreads();
-    cluster_sync_all();   // every CTA of the cluster runs (and has initialised its words) before any DSMEM access
+    cluster_sync_all();   // every CTA of the cluster runs before any DSMEM access
 
     const int a0 = (int)crank * ra.A;          // first row digit a of this CTA
     uint32_t *tab32 = reinterpret_cast<uint32_t *>(table);
     int slot = 0;                              // L mod R
     Words<CH> last;
-    int64_t last_off = -1;                     // word offset of the thread's last row chunk of the level
-    for (int L = 0; L <= ra.rho_max; ++L) {
+    int64_t last_off = -1;                     // word offset of the thread's last row chunk of the interval
+    // TB row-levels per cluster barrier (temporal blocking): at sub-level t of an
+    // interval this CTA also computes, redundantly, the (TB - 1 - t) * H rows below
+    // its block (the previous CTA's rows, same values), so every source of the
+    // interval's levels is either in the halo pushed before the last barrier or
+    // computed here; the previous CTA's pushes of the rows computed here land in
+    // the same ring positions with the same values
+    for (int L0 = 0; L0 <= ra.rho_max; L0 += TB) {
 #if PTAS_RING_PROFILE
-        const bool pr = threadIdx.x == 0 && crank == 8 && L < 2048;
-        if (pr) g_ring_prof[0][L] = clock64();
+        const bool pr = threadIdx.x == 0 && crank == 8 && L0 < 2048;
+        if (pr) g_ring_prof[0][L0] = clock64();
 #endif
-        // this CTA's rows of level L: a in [lo, hi] (contiguous), b = L - a
-        const int lo = max(max(L - ra.N1, 0), a0);
-        const int hi = min(min(L, ra.N0), a0 + ra.A - 1);
-        const int ntask = hi >= lo ? (hi - lo + 1) * Lg : 0;
-        if constexpr (P2P) {
-            // arm this level's halo slot (phase L / R) with the bytes the previous CTA
-            // will push into it; its previous phase (level L - R) has landed first
-            if (threadIdx.x == 0 && has_prev) {
-                const int sl = L % ra.R;
-                if (L >= ra.R) mbar_wait(full_own + 8u * (uint32_t)sl, (uint32_t)(((L - ra.R) / ra.R) & 1));
-                mbar_arm(full_own + 8u * (uint32_t)sl, halo_bytes(L));
-            }
-        }
-        for (int task = threadIdx.x; task < ntask; task += blockDim.x) {
-            const int r_ = task / Lg;
-            const int a = lo + r_;
-            const int c = task - r_ * Lg;       // lane chunk: words c*CH .. c*CH+CH-1 of the row
-            const int b = L - a;
-            const int ia = a - a0;
-            const int pos0 = (ra.H + ia) * Lw + c * CH;  // the lane's words within a ring slot
-            Words<CH> ae, ao;
-            fill_words(ae, 0xffffffffu);
-            fill_words(ao, 0xffffffffu);
-            const int blk = a >= 1 ? 1 : 0;    // pivot block (D13)
-            if constexpr (P2P) {
-                // only the bottom H rows read the halo (s0 <= H): they wait until the
-                // previous CTA's rows of the levels they read (L - Rdep + 1 .. L - 1)
-                // have landed; every other row starts at once (the CTAs run skewed)
-                if (has_prev && ia < ra.H) {
-                    for (int j = 1; j < ra.Rdep && j <= L; ++j) {
-                        const int Lj = L - j;
-                        mbar_wait(full_own + 8u * (uint32_t)(Lj % ra.R), (uint32_t)((Lj / ra.R) & 1));
-                    }
-                }
-                // the top H rows are pushed into CTA c + 1's ring: it has finished the
-                // levels that read the slot they overwrite
-                if (has_next && ia >= ra.A - ra.H)
-                    while (ld_relaxed_cluster(dn_own) < L - dn_lag) {
-                    }
-            }
+        const int tn = min(TB, ra.rho_max - L0 + 1);
+        for (int t = 0; t < tn; ++t) {
+            const int L = L0 + t;
+            const int ext = (TB - 1 - t) * ra.H;     // redundant rows below the block
+            // rows of level L: a in [lo, hi] (contiguous), b = L - a
+            const int lo = max(max(L - ra.N1, 0), a0 - ext);
+            const int hi = min(min(L, ra.N0), a0 + ra.A - 1);
+            const int ntask = hi >= lo ? (hi - lo + 1) * Lg : 0;
+            for (int task = threadIdx.x; task < ntask; task += blockDim.x) {
+                const int r_ = task / Lg;
+                const int a = lo + r_;
+                const int c = task - r_ * Lg;       // lane chunk: words c*CH .. c*CH+CH-1 of the row
+                const int b = L - a;
+                const int ia = a - a0;              // < 0: a redundant row of the previous CTA
+                const int pos0 = (HT + ia) * Lw + c * CH;  // the lane's words within a ring slot
+                Words<CH> ae, ao;
+                fill_words(ae, 0xffffffffu);
+                fill_words(ao, 0xffffffffu);
+                const int blk = a >= 1 ? 1 : 0;    // pivot block (D13)
 #pragma unroll
-            for (int cls = 1; cls <= (WIN == 8 ? 2 : 1); ++cls) {
-                const int4 *pl = s_pl + (2 * blk + cls - 1) * lcap;
-                const int n = s_cnt[2 * blk + cls - 1];
-                for (int q0 = 0; q0 < n; q0 += PB) {
-                    Words<CH> cur[PB];
-                    uint32_t l1[PB], l2[PB];
-                    int sj[PB];
+                for (int cls = 1; cls <= (WIN == 8 ? 2 : 1); ++cls) {
+                    const int4 *pl = s_pl + (2 * blk + cls - 1) * lcap;
+                    const int n = s_cnt[2 * blk + cls - 1];
+                    for (int q0 = 0; q0 < n; q0 += PB) {
+                        Words<CH> cur[PB];
+                        uint32_t l1[PB], l2[PB];
+                        int sj[PB];
 #pragma unroll
-                    for (int u = 0; u < PB; ++u) {
-                        const int4 pf = pl[q0 + u];
-                        sj[u] = pf.z;
-                        // source row (a - s0, b - s1) of level L - |s'|: always in this CTA's ring
-                        // (own rows, or the halo copy of the previous CTA's top rows, s0 <= H)
-                        int ss = slot - pf.w;
-                        ss += ss < 0 ? ra.R : 0;
-                        const int pos = pos0 + (ss * AH - pf.x) * Lw;   // word index in the ring
-                        if (pf.x <= a && pf.y <= b) {
-                            const uint32_t *p = ring + pos;
-                            cur[u] = lds_words<CH>(p);
-                            l1[u] = c >= 1 ? p[-1] : 0u;
-                            l2[u] = (cls == 2 && c * CH >= 2) ? p[-2] : 0u;
-                        } else {
-                            fill_words(cur[u], 0xffffffffu);
-                            l1[u] = l2[u] = 0xffffffffu;
+                        for (int u = 0; u < PB; ++u) {
+                            const int4 pf = pl[q0 + u];
+                            sj[u] = pf.z;
+                            // source row (a - s0, b - s1) of level L - |s'|: always in this CTA's
+                            // ring (own rows, halo rows, or rows computed redundantly this interval)
+                            int ss = slot - pf.w;
+                            ss += ss < 0 ? ra.R : 0;
+                            const int pos = pos0 + (ss * AH - pf.x) * Lw;   // word index in the ring
+                            if (pf.x <= a && pf.y <= b) {
+                                const uint32_t *p = ring + pos;
+                                cur[u] = lds_words<CH>(p);
+                                l1[u] = c >= 1 ? p[-1] : 0u;
+                                l2[u] = (cls == 2 && c * CH >= 2) ? p[-2] : 0u;
+                            } else {
+                                fill_words(cur[u], 0xffffffffu);
+                                l1[u] = l2[u] = 0xffffffffu;
+                            }
+                        }
+#pragma unroll
+                        for (int u = 0; u < PB; ++u) {
+                            // positions before the row: its first entry replicated (row word 0 is
+                            // the chunk's own word for c = 0, the left word for c = 1 with CH = 1)
+                            uint32_t f = c == 0 ? cur[u].v[0] : l1[u];
+                            f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
+                            const uint32_t w1 = c >= 1 ? l1[u] : f;
+                            const uint32_t w2 = c * CH >= 2 ? l2[u] : f;
+                            if (cls == 1) ring_windows<E, CH, 1>(cur[u], w1, w2, (uint32_t)sj[u], ae, ao);
+                            else ring_windows<E, CH, 2>(cur[u], w1, w2, (uint32_t)sj[u], ae, ao);
                         }
                     }
-#pragma unroll
-                    for (int u = 0; u < PB; ++u) {
-                        // positions before the row: its first entry replicated (row word 0 is
-                        // the chunk's own word for c = 0, the left word for c = 1 with CH = 1)
-                        uint32_t f = c == 0 ? cur[u].v[0] : l1[u];
-                        f = EB == 1 ? prmt(f, 0u, 0x0000u) : prmt(f, 0u, 0x1010u);
-                        const uint32_t w1 = c >= 1 ? l1[u] : f;
-                        const uint32_t w2 = c * CH >= 2 ? l2[u] : f;
-                        if (cls == 1) ring_windows<E, CH, 1>(cur[u], w1, w2, (uint32_t)sj[u], ae, ao);
-                        else ring_windows<E, CH, 2>(cur[u], w1, w2, (uint32_t)sj[u], ae, ao);
-                    }
                 }
-            }
-            Words<CH> wv;
+                Words<CH> wv;
 #pragma unroll
-            for (int t = 0; t < CH; ++t) {
-                uint32_t oe, oo = 0;
-                if constexpr (EB == 1) {
-                    oe = (ae.v[t] & 0x00ff00ffu) + ONES;
-                    oo = (ao.v[t] & 0x00ff00ffu) + ONES;
-                } else {
-                    oe = vmin2(ae.v[t], 0xfffefffeu) + ONES;
-                }
-                if (L == 0) {   // row (0, 0): OPT(0, x) = ceil(x / J0)
-                    const uint32_t x0 = (uint32_t)(c * CH + t) * (4 / EB);
-                    auto cf = [&](uint32_t x) { return (x + (uint32_t)ra.J0 - 1u) / (uint32_t)ra.J0; };
+                for (int t2 = 0; t2 < CH; ++t2) {
+                    uint32_t oe, oo = 0;
                     if constexpr (EB == 1) {
-                        oe = cf(x0) | (cf(x0 + 2) << 16);
-                        oo = cf(x0 + 1) | (cf(x0 + 3) << 16);
+                        oe = (ae.v[t2] & 0x00ff00ffu) + ONES;
+                        oo = (ao.v[t2] & 0x00ff00ffu) + ONES;
                     } else {
-                        oe = cf(x0) | (cf(x0 + 1) << 16);
+                        oe = vmin2(ae.v[t2], 0xfffefffeu) + ONES;
+                    }
+                    if (L == 0) {   // row (0, 0): OPT(0, x) = ceil(x / J0)
+                        const uint32_t x0 = (uint32_t)(c * CH + t2) * (4 / EB);
+                        auto cf = [&](uint32_t x) { return (x + (uint32_t)ra.J0 - 1u) / (uint32_t)ra.J0; };
+                        if constexpr (EB == 1) {
+                            oe = cf(x0) | (cf(x0 + 2) << 16);
+                            oo = cf(x0 + 1) | (cf(x0 + 3) << 16);
+                        } else {
+                            oe = cf(x0) | (cf(x0 + 1) << 16);
+                        }
+                    }
+                    wv.v[t2] = EB == 1 ? prmt(oe, oo, 0x6240u) : oe;
+                }
+                store_words<CH>(ring + ((size_t)slot * AH + HT + ia) * Lw + c * CH, wv);
+                if (ia >= 0) {   // own row: the halo of the next CTA, and the table in HBM
+                    if (has_next && ia >= ra.A - HT)
+                        st_dsm<CH>(nxt + 4u * (uint32_t)(((slot * AH + ia - (ra.A - HT)) * Lw + c * CH)), wv);
+                    const int64_t off = ((int64_t)a * ra.stride0 + (int64_t)b * ra.Wp) * EB / 4 + c * CH;
+                    if (t + 1 < tn || task + (int)blockDim.x < ntask) {
+                        store_words<CH>(tab32 + off, wv);
+                    } else {   // (the thread's last row of the interval: stored after the arrive)
+                        last = wv;
+                        last_off = off;
                     }
                 }
-                wv.v[t] = EB == 1 ? prmt(oe, oo, 0x6240u) : oe;
             }
-            store_words<CH>(ring + ((size_t)slot * AH + ra.H + ia) * Lw + c * CH, wv);
-            if (has_next && ia >= ra.A - ra.H) {   // halo of the next CTA
-                const uint32_t hp = nxt + 4u * (uint32_t)(((slot * AH + ia - (ra.A - ra.H)) * Lw + c * CH));
-                if constexpr (P2P) st_async_words<CH>(hp, wv, full_next + 8u * (uint32_t)slot);
-                else st_dsm<CH>(hp, wv);
-            }
-            if (task + (int)blockDim.x < ntask) {   // (not the thread's last row of the level)
-                const int64_t rowbase = (int64_t)a * ra.stride0 + (int64_t)b * ra.Wp;   // elements
-                store_words<CH>(tab32 + rowbase * EB / 4 + c * CH, wv);
-            } else {
-                last = wv;
-                last_off = ((int64_t)a * ra.stride0 + (int64_t)b * ra.Wp) * EB / 4 + c * CH;
-            }
+            slot = slot + 1 == ra.R ? 0 : slot + 1;
+            if (t + 1 < tn) __syncthreads();   // level L complete in this CTA's ring
         }
-        // level L complete in every CTA's ring: the release covers the ring stores; the
-        // thread's last row goes to HBM between arrive and wait, off the critical path
+        // the interval's levels complete in every CTA's ring: the release covers the ring
+        // and halo stores; the thread's last row goes to HBM between arrive and wait
 #if PTAS_RING_PROFILE
-        if (pr) g_ring_prof[1][L] = clock64();
+        if (pr) g_ring_prof[1][L0] = clock64();
 #endif
-        if constexpr (P2P) {
-            __syncthreads();   // own ring rows of level L written, halo pushes issued, ring reads done
+        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
 #if PTAS_RING_PROFILE
-            if (pr) g_ring_prof[2][L] = clock64();
+        if (pr) g_ring_prof[2][L0] = clock64();
 #endif
-            // (every read of the ring for level L has returned: the previous CTA may reuse the slots)
-            if (threadIdx.x == 0 && has_prev) st_relaxed_cluster(dn_prev, L);
-            if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
-            last_off = -1;
-        } else {
-            asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+        if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
+        last_off = -1;
+        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 #if PTAS_RING_PROFILE
-            if (pr) g_ring_prof[2][L] = clock64();
+        if (pr) g_ring_prof[3][L0] = clock64();
 #endif
-#ifndef PTAS_RING_NOSTORE
-            if (last_off >= 0) store_words<CH>(tab32 + last_off, last);
-#endif
-            last_off = -1;
-            asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-        }
-#if PTAS_RING_PROFILE
-        if (pr) g_ring_prof[3][L] = clock64();
-#endif
-        slot = slot + 1 == ra.R ? 0 : slot + 1;
-    }
-    // P2P: the last level's halo has landed, and no CTA exits while a neighbour
-    // may still access its shared memory
-    if constexpr (P2P) {
-        if (threadIdx.x == 0 && has_prev)
-            for (int Lj = max(0, ra.rho_max - ra.R + 1); Lj <= ra.rho_max; ++Lj)
-                mbar_wait(full_own + 8u * (uint32_t)(Lj % ra.R), (uint32_t)((Lj / ra.R) & 1));
-        __syncthreads();
-        cluster_sync_all();
     }
 }
 
@@ -446,9 +335,9 @@ template <typename E, int CH, int WIN>
 cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_pref, const DpMeta *d_meta,
                           int64_t nP_bound, int csize, cudaStream_t st, bool dry)
 {
-    auto kfn = ra.p2p ? row_ring_kernel<E, CH, WIN, true> : row_ring_kernel<E, CH, WIN, false>;
+    auto kfn = row_ring_kernel<E, CH, WIN>;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (((size_t)ra.R * (ra.A + ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
+    const size_t smem = (((size_t)ra.R * (ra.A + ra.TB * ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     // function attributes and the co-residency query once per (device, kernel,
     // smem, cluster size, block): they take the driver lock, and concurrent DP
@@ -456,7 +345,7 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
     int dev = 0;
     cudaError_t err = cudaGetDevice(&dev);
     if (err != cudaSuccess) return err;
-    const int lanes = ra.A * ra.Lg;
+    const int lanes = (ra.A + (ra.TB - 1) * ra.H) * ra.Lg;   // own + redundant rows of a level
     const int warps = std::min(32, (lanes + 31) / 32);
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[1];
@@ -492,8 +381,8 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
     }
     if (ncl < 1) return cudaErrorNotSupported;
     if (!dry && PTAS_KNOB("PTAS_TRACE", 0) == 1)
-        std::fprintf(stderr, "[ring] cluster %d x %d threads, smem %zu B, slots %d (dep %d), %s: %d clusters co-resident\n",
-                     csize, 32 * warps, smem, ra.R, ra.Rdep, ra.p2p ? "p2p" : "barrier", ncl);
+        std::fprintf(stderr, "[ring] cluster %d x %d threads, smem %zu B, slots %d (dep %d), %d levels per barrier: %d clusters co-resident\n",
+                     csize, 32 * warps, smem, ra.R, ra.Rdep, ra.TB, ncl);
     if (dry) return cudaSuccess;
     err = cudaLaunchKernelEx(&cfg, kfn, (E *)table, ra, d_pref, d_meta);
 #if PTAS_RING_PROFILE
@@ -503,15 +392,15 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
         cudaMemcpyFromSymbol(h, g_ring_prof, sizeof(h));
         double s0 = 0, s1 = 0, s2 = 0;
         const int nl = std::min(ra.rho_max + 1, 2048);
-        for (int L = 1; L < nl; ++L) {
+        int ni = 0;
+        for (int L = ra.TB; L < nl; L += ra.TB, ++ni) {   // intervals of TB levels (the first skipped)
             s0 += h[1][L] - h[0][L];
             s1 += h[2][L] - h[1][L];
             s2 += h[3][L] - h[2][L];
         }
-        std::fprintf(stderr, "[ring] CTA 8 thread 0, cycles per level: rows %.0f arrive %.0f wait %.0f (levels %d, CH %d, threads %d)\n",
-                     s0 / (nl - 1), s1 / (nl - 1), s2 / (nl - 1), nl, CH, 32 * warps);
-        for (int L = 300; L < nl && L < 306; ++L)
-            std::fprintf(stderr, "  L=%d rows %lld arrive %lld wait %lld\n", L, h[1][L] - h[0][L], h[2][L] - h[1][L], h[3][L] - h[2][L]);
+        ni = std::max(ni, 1);
+        std::fprintf(stderr, "[ring] CTA 8 thread 0, cycles per interval of %d levels: rows %.0f arrive %.0f wait %.0f (levels %d, CH %d, threads %d)\n",
+                     ra.TB, s0 / ni, s1 / ni, s2 / ni, nl, CH, 32 * warps);
     }
 #endif
     return err;
@@ -598,34 +487,40 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
     if (nP_bound > 4096) return cudaErrorNotSupported;
     ra.Rdep = (int)std::min<int64_t>(hi0 + hi1, T / std::min(r[0], r[1])) + 1;
     ra.rho_max = N[0] + N[1];
-    // extra ring slots: how many levels a CTA may run ahead of the next one (P2P)
-    // (P2P: one mbarrier per ring slot, at most 64)
-    ra.p2p = PTAS_KNOB("PTAS_RING_P2P", 0) != 0 && ra.Rdep <= 64 ? 1 : 0;
-    const int extra = ra.p2p ? (int)std::min<int64_t>(64 - ra.Rdep, std::max<int64_t>(0, PTAS_KNOB("PTAS_RING_EXTRA", 2))) : 0;
     const int win = J0 * e <= 4 ? 4 : 8;
     const size_t smem_cap = 220 * 1024;
+    // row-levels per cluster barrier (temporal blocking): up to PTAS_RING_TB, as long
+    // as two CTAs still fit one SM (14 co-resident clusters, D14) and the halo
+    // (TB * H rows) comes from the previous CTA's block alone
+    const int tb_max = (int)std::max<int64_t>(1, PTAS_KNOB("PTAS_RING_TB", 2));
+    const size_t smem_target = (size_t)PTAS_KNOB("PTAS_RING_SMEM_TARGET", 112 * 1024);
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
     const int cs_force = (int)PTAS_KNOB("PTAS_RING_CS", 0);   // experiment: force the cluster size
     for (int csize : {16, 8, 4, 2}) {
         if (cs_force ? csize != cs_force : csize < 8) continue;
         ra.A = (N[0] + csize) / csize;   // ceil((N0 + 1) / C) rows of each level per CTA
-        ra.H = (int32_t)hi0;              // halo rows (s0 <= hi0)
+        ra.H = (int32_t)hi0;              // halo rows per level (s0 <= hi0)
         if (ra.A < hi0) continue;         // every source row is in this CTA's block or the previous one
-        auto smem_of = [&](int slots) {
-            return (((size_t)slots * (ra.A + ra.H) * Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
+        // ring slots: the Rdep levels a row reads plus the TB - 1 levels of the interval
+        auto smem_of = [&](int tb) {
+            return (((size_t)(ra.Rdep + tb - 1) * (ra.A + tb * ra.H) * Lw * 4 + 15) & ~(size_t)15) +
+                   4 * (size_t)(np + 4) * 16;
         };
-        if (smem_of(ra.Rdep) > smem_cap) continue;
-        ra.R = ra.Rdep + extra;
-        while (ra.R > ra.Rdep && smem_of(ra.R) > smem_cap) --ra.R;
+        int TB = tb_max;
+        while (TB > 1 && (ra.A < TB * ra.H || smem_of(TB) > smem_target)) --TB;
+        if (smem_of(TB) > smem_cap) continue;
+        ra.TB = TB;
+        ra.R = ra.Rdep + TB - 1;
+        const int rows_max = ra.A + (TB - 1) * ra.H;   // own + redundant rows of a level
         // words per lane: the smallest chunk with one pass over the CTA's rows of a level
         // words per lane: 4 when the CTA's rows of a level fit one pass (measured best on
         // M5s: 2 words 1.82 / 1.69 ms, 4 words 1.39 / 1.48 ms, 8 words 1.94 / 1.96 ms per DP),
         // else the smallest chunk that fits, else 8
         int CH = 8;
-        if (Lw % 4 == 0 && (int64_t)ra.A * (Lw / 4) <= 1024) CH = 4;
+        if (Lw % 4 == 0 && (int64_t)rows_max * (Lw / 4) <= 1024) CH = 4;
         else
             for (int c : {1, 2, 4})
-                if (Lw % c == 0 && (int64_t)ra.A * (Lw / c) <= 1024) {
+                if (Lw % c == 0 && (int64_t)rows_max * (Lw / c) <= 1024) {
                     CH = c;
                     break;
                 }

@@ -1,7 +1,6 @@
 """K = 3 cluster ring kernel (row_ring.cu, D14) against the oracle,
-entry by entry: both synchronisation protocols (one cluster barrier per level,
-and the point-to-point progress words with extra ring slots that let the CTAs
-of the cluster run as a pipeline), every cluster size, uint8 and uint16
+entry by entry: 1 to 4 row-levels per cluster barrier (temporal blocking with
+redundant rows below each CTA's block), every cluster size, uint8 and uint16
 tables, one- and two-word windows.  A case counts only when the ring kernel
 actually filled it (one fill launch for the whole DP)."""
 from __future__ import annotations
@@ -42,12 +41,11 @@ def _case(rng, e):
 
 
 @pytest.mark.parametrize("e", [1, 2])
-@pytest.mark.parametrize("proto", [("0", "0"), ("1", "0"), ("1", "1"), ("1", "4")],
-                         ids=["barrier", "p2p-noextra", "p2p-extra1", "p2p-extra4"])
+@pytest.mark.parametrize("tb", ["1", "2", "3", "4"])
 @pytest.mark.parametrize("cs", ["2", "4", "8", "16"])
-def test_ring_protocols_vs_oracle(P, monkeypatch, e, proto, cs):
-    monkeypatch.setenv("PTAS_RING_P2P", proto[0])
-    monkeypatch.setenv("PTAS_RING_EXTRA", proto[1])
+def test_ring_temporal_blocking_vs_oracle(P, monkeypatch, e, tb, cs):
+    monkeypatch.setenv("PTAS_RING_TB", tb)
+    monkeypatch.setenv("PTAS_RING_SMEM_TARGET", str(220 * 1024))   # the requested TB wherever it fits
     monkeypatch.setenv("PTAS_RING_CS", cs)
     rng = np.random.default_rng(7000 + 10 * e + int(cs))
     used = 0
