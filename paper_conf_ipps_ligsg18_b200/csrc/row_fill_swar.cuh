@@ -126,23 +126,30 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
     constexpr bool DF = DFM == 1;
     constexpr bool CL = DFM == 2;
     constexpr bool RUN = DFM != 0;
+// gathers in flight per lane (prefix batch).  The pivot blocks (D13) of the
+// u8 shapes are short (M2s: 3-5 prefixes), so a padded batch computes windows
+// for empty slots; measured round 2 (solve ms, against 16 / 10): uint8 CH = 1
+// 8 and CH = 2 (prefix list in shared memory) 4: M2s 2.24 -> 2.13, M4s 22.6 ->
+// 21.7, M4x unchanged; uint16 CH = 1 stays 16 (M3s, 8 was +3 %).  CH = 2 with
+// the prefix list in shared memory once took 10 (20 prefixes in two batches:
+// M2s -5 % in round 1, before the pivot blocks).
 #ifndef PTAS_PB1
-#define PTAS_PB1 16
+#define PTAS_PB1 8
+#endif
+#ifndef PTAS_PB1U16
+#define PTAS_PB1U16 16
 #endif
 #ifndef PTAS_PB2
 #define PTAS_PB2 8
 #endif
 #ifndef PTAS_PB2S
-#define PTAS_PB2S 10
+#define PTAS_PB2S 4
 #endif
 #ifndef PTAS_PB2U16
 #define PTAS_PB2U16 8
 #endif
-    // gathers in flight per lane (prefix batch); CH = 2 with the prefix list in
-    // shared memory (short lists) takes 10: 20 prefixes in two batches instead
-    // of three (M2s fill -5%, measured; 12 spills at 80 registers)
-    // (uint8 only: the 64-register uint16 kernels lose with it, M3s +3%)
-    constexpr int PB = CH == 1 ? PTAS_PB1 : (CH == 2 ? (EB == 2 ? PTAS_PB2U16 : (CPREF ? PTAS_PB2 : PTAS_PB2S)) : 4);
+    constexpr int PB = CH == 1 ? (EB == 2 ? PTAS_PB1U16 : PTAS_PB1)
+                               : (CH == 2 ? (EB == 2 ? PTAS_PB2U16 : (CPREF ? PTAS_PB2 : PTAS_PB2S)) : 4);
     constexpr bool PB_POW2 = (PB & (PB - 1)) == 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     // Programmatic dependent launch: let the next row-level's grid start its
@@ -707,7 +714,7 @@ static cudaError_t launch_swar_impl(int e, void *table, const RowGeom &g, const 
     // small row-levels with long prefix lists: split each row set's prefixes over the 8 warps of a block
     const int64_t sp = PTAS_KNOB("PTAS_SPLIT_ROWS", -1);
     // (worth it when a row's prefix walk has several batches of gathers in series)
-    const int PBh = CH == 1 ? PTAS_PB1 : (CH == 2 ? PTAS_PB2 : 4);
+    const int PBh = CH == 1 ? (e == 2 ? PTAS_PB1U16 : PTAS_PB1) : (CH == 2 ? PTAS_PB2 : 4);
     const int64_t split_rows = sp >= 0 ? sp : ((nph + PBh - 1) / PBh >= 4 ? (int64_t)sm_count * rpw * 2 : 0);
     // df->nsplit: 1 = warp row sets, 8 = block row sets, 0 = one cluster in lockstep
     const bool cl = df && df->nsplit == 0;
