@@ -130,7 +130,8 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 // u8 shapes are short (M2s: 3-5 prefixes), so a padded batch computes windows
 // for empty slots; measured round 2 (solve ms, against 16 / 10): uint8 CH = 1
 // 8 and CH = 2 (prefix list in shared memory) 4: M2s 2.24 -> 2.13, M4s 22.6 ->
-// 21.7, M4x unchanged; uint16 CH = 1 stays 16 (M3s, 8 was +3 %).  CH = 2 with
+// 21.7, M4x unchanged; uint16 CH = 2 4 (M3s 7.18 -> 6.88, M3g 47.1 -> 44.9);
+// uint16 CH = 1 stays 16 (M3s, 8 was +3 %).  CH = 2 with
 // the prefix list in shared memory once took 10 (20 prefixes in two batches:
 // M2s -5 % in round 1, before the pivot blocks).
 #ifndef PTAS_PB1
@@ -146,7 +147,7 @@ row_fill_swar_kernel(E *table, const RowGeom g, const int64_t *__restrict__ rb,
 #define PTAS_PB2S 4
 #endif
 #ifndef PTAS_PB2U16
-#define PTAS_PB2U16 8
+#define PTAS_PB2U16 4
 #endif
     constexpr int PB = CH == 1 ? (EB == 2 ? PTAS_PB1U16 : PTAS_PB1)
                                : (CH == 2 ? (EB == 2 ? PTAS_PB2U16 : (CPREF ? PTAS_PB2 : PTAS_PB2S)) : 4);
