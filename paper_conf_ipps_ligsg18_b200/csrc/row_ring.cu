@@ -158,7 +158,10 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
 {
     constexpr int EB = (int)sizeof(E);
     constexpr uint32_t ONES = 0x00010001u;
-    constexpr int PB = 4;   // prefixes whose loads are issued together
+#ifndef PTAS_RING_PB
+#define PTAS_RING_PB 4
+#endif
+    constexpr int PB = PTAS_RING_PB;   // prefixes whose loads are issued together
     extern __shared__ __align__(16) unsigned char smem_raw[];
     if (meta->ovf) return;   // grid-uniform: every CTA exits before any barrier
     uint32_t crank;
@@ -189,7 +192,7 @@ row_ring_kernel(E *table, const RingArgs ra, const PrefixEntry *__restrict__ gpr
         s_pl[li * lcap + atomicAdd(&s_cnt[li], 1)] = make_int4(s0, s1, sel, s0 + s1);
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < 4 * PB; i += blockDim.x)   // padding: never dominated
+    for (int i = threadIdx.x; i < 4 * PB; i += blockDim.x)   // padding: never dominated (lists hold np + PB entries)
         s_pl[(i / PB) * lcap + s_cnt[i / PB] + i % PB] =
             make_int4(1 << 20, 1 << 20, (EB == 1 ? SEL_U8 : SEL_U16) + SEL_SELF, 0);
     uint32_t csize;
@@ -337,7 +340,7 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
 {
     auto kfn = row_ring_kernel<E, CH, WIN>;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (((size_t)ra.R * (ra.A + ra.TB * ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + 4) * 16;
+    const size_t smem = (((size_t)ra.R * (ra.A + ra.TB * ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + PTAS_RING_PB) * 16;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
     // function attributes and the co-residency query once per (device, kernel,
     // smem, cluster size, block): they take the driver lock, and concurrent DP
@@ -504,7 +507,7 @@ cudaError_t launch_row_fill_ring(int e, void *table, const RowGeom &g, const int
         // ring slots: the Rdep levels a row reads plus the TB - 1 levels of the interval
         auto smem_of = [&](int tb) {
             return (((size_t)(ra.Rdep + tb - 1) * (ra.A + tb * ra.H) * Lw * 4 + 15) & ~(size_t)15) +
-                   4 * (size_t)(np + 4) * 16;
+                   4 * (size_t)(np + PTAS_RING_PB) * 16;
         };
         int TB = tb_max;
         while (TB > 1 && (ra.A < TB * ra.H || smem_of(TB) > smem_target)) --TB;
