@@ -370,8 +370,12 @@ def run_ours(args, w):
         mode, Pp = P.MODE_SINGLE, args.P
     # all library work on this stream, so the CUDA events below bracket it exactly
     lib_stream = torch.cuda.Stream(device=local)
+    # --slab-pipeline (N > 1, level-sharded): every probe DP windowed and split along
+    # the first class over the ranks, halos by ncclSend/ncclRecv
+    pipe = args.slab_pipeline and world > 1 and mode == P.MODE_LEVEL_SHARDED
     opts = P.options(P=Pp, mode=mode, device=local, comm=comm, stream=lib_stream,
-                     virtual_shards=args.virtual_shards if world == 1 else 1)
+                     virtual_shards=args.virtual_shards if world == 1 else 1,
+                     window=1 if pipe else 0, slab_pipeline=1 if pipe else 0)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{local}")
 
     def barrier():
@@ -432,6 +436,7 @@ def run_ours(args, w):
         "config": _config(w, probes_per_round=Pp,
                           mode={0: "single", 1: "level_sharded", 2: "multi_probe"}[mode],
                           **({"virtual_shards": args.virtual_shards} if world == 1 and args.virtual_shards > 1 else {}),
+                          **({"probe_dps": "windowed, slab/halo pipeline (send/recv)"} if pipe else {}),
                           l2="flushed between steps (256 MiB write)"),
         "solve": {"probes": st0["probes"], "unique_dps": st0["unique_dps"], "T_star": st0["T_star"],
                   "sigma_max": st0["sigma_max"], "K_at_Tstar": st0["K_at_Tstar"],
@@ -520,6 +525,8 @@ def main():
     ap.add_argument("--virtual-shards", type=int, default=1,
                     help="N=1 only: run LEVEL_SHARDED with G logical shards on one GPU (slice fill + "
                          "gather copy + scatter per level, no NCCL) to measure the exchange overhead")
+    ap.add_argument("--slab-pipeline", action="store_true",
+                    help="N > 1 level-sharded: windowed probe DPs on the slab/halo pipeline (send/recv)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-parity", action="store_true", help="skip the oracle-golden parity assertion")
     ap.add_argument("--no-blocks", action="store_true", help="skip the scaling_ref / multi_probe blocks")

@@ -86,7 +86,18 @@ typedef struct {
                                    every probe DP, -1 = never.  Only OPT(N) of a
                                    windowed DP is kept; the schedule's DP at T* is
                                    always a full table (ETOOBIG if it does not fit) */
-    int32_t pad0_;
+    int32_t slab_pipeline;      /* LEVEL_SHARDED with comm, windowed probe DPs
+                                   (window = 1, or a table over the budget):
+                                   0 = the window's slabs split over the ranks and
+                                   all-gathered (default); 1 = the slab/halo
+                                   pipeline of SURVEY.md §8(f)-2ii: rank g holds a
+                                   contiguous range of slabs of the first internal
+                                   class (the table split along that dimension,
+                                   plus min(N0, T/r0) halo slabs), fills them in
+                                   chunks of the other classes' levels, and sends
+                                   the halo of each chunk to rank g + 1 with
+                                   ncclSend / ncclRecv (a wavefront over ranks and
+                                   chunks); OPT(N) is broadcast from the last rank */
     int64_t shard_min_rows;     /* LEVEL_SHARDED with comm: row-levels with fewer
                                    rows are computed redundantly on every rank
                                    (-1 = library default 2048); 0 = shard every
@@ -307,6 +318,16 @@ int ptas_interval_update(int64_t *LB, int64_t *UB, const int64_t *T,
  * `world` (ceil split; trailing ranks may be empty). */
 int ptas_shard_range(int64_t count, int32_t rank, int32_t world,
                      int64_t *begin, int64_t *end);
+/* Slab/halo pipeline plan (ptas_options.slab_pipeline):
+ * S = N0 + 1 slabs of the first internal class over `world` ranks; rank
+ * `rank` owns slabs [*pb, *pe), holds [*pbase, *pe) (its *hin halo slabs are
+ * received per chunk from rank - 1), and sends the chunk rows of its last
+ * *hout slabs to rank + 1 (hin of rank g == hout of rank g - 1).  hi0 =
+ * min(N0, T / r0).  Host only; the engine uses exactly this plan.
+ * EINVAL: S < world, world < 1, rank outside [0, world), hi0 < 0. */
+int ptas_slab_plan(int64_t S, int64_t hi0, int32_t rank, int32_t world, int64_t *pb, int64_t *pe,
+                   int64_t *pbase, int64_t *hin, int64_t *hout);
+
 /* The split the level-sharded DP uses for one row-level of `rows` rows of
  * `row_bytes` bytes each (rows of a level are independent,
  * PAPER.md:215): ceil(rows / world) rounded up to the smallest multiple q with

@@ -21,7 +21,7 @@ __all__ = ["ptas_solve", "ptas_solve_device", "dp_fill", "dp_fill_opt", "dp_fill
 
 def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, budget: int = 0,
             memoize: bool = True, virtual_shards: int = 1, layout: int = 0, stream=None,
-            speculate: int = -1, shard_min_rows: int = -1, window: int = 0) -> PtasOptions:
+            speculate: int = -1, shard_min_rows: int = -1, window: int = 0, slab_pipeline: int = 0) -> PtasOptions:
     o = PtasOptions()
     lib().ptas_default_options(ctypes.byref(o))
     o.probes_per_round = int(P)
@@ -35,6 +35,7 @@ def options(P: int = 1, mode: int = MODE_SINGLE, device: int = -1, comm=None, bu
     o.speculate = int(speculate)
     o.shard_min_rows = int(shard_min_rows)
     o.window = int(window)
+    o.slab_pipeline = int(slab_pipeline)
     o.stream = None if stream is None else ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
     return o
 
@@ -243,6 +244,13 @@ def ptas_table_order(counts, sizes, layout: int = 0):
     _chk("ptas_table_order", lib().ptas_table_order(_ptr(c, ctypes.c_int32), _ptr(s, ctypes.c_int64), len(c),
                                                     int(layout), _ptr(out, ctypes.c_int32), ctypes.byref(k)))
     return [int(x) for x in out[: k.value]]
+
+
+def ptas_slab_plan(S: int, hi0: int, rank: int, world: int):
+    """(pb, pe, pbase, hin, hout) of the slab/halo pipeline (ptas_options.slab_pipeline)."""
+    v = [ctypes.c_int64() for _ in range(5)]
+    _chk("ptas_slab_plan", lib().ptas_slab_plan(int(S), int(hi0), int(rank), int(world), *[ctypes.byref(x) for x in v]))
+    return tuple(x.value for x in v)
 
 
 def ptas_level_shard(rows: int, rank: int, world: int, row_bytes: int):

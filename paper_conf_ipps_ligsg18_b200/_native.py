@@ -27,7 +27,7 @@ class PtasOptions(ctypes.Structure):
     _fields_ = [("probes_per_round", ctypes.c_int32), ("mode", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("comm", vp), ("table_budget_bytes", ctypes.c_int64), ("memoize", ctypes.c_int32),
                 ("virtual_shards", ctypes.c_int32), ("layout", ctypes.c_int32), ("stream", vp),
-                ("speculate", ctypes.c_int32), ("window", ctypes.c_int32), ("pad0_", ctypes.c_int32),
+                ("speculate", ctypes.c_int32), ("window", ctypes.c_int32), ("slab_pipeline", ctypes.c_int32),
                 ("shard_min_rows", ctypes.c_int64)]
 
 
@@ -58,6 +58,7 @@ EXPORTS = [
     "dp_fill_device", "ptas_get_unique_id", "ptas_comm_init", "ptas_comm_destroy", "ptas_strerror", "ptas_k",
     "ptas_bounds", "ptas_classify", "ptas_probe_targets", "ptas_interval_update", "ptas_shard_range",
     "dp_configs", "dp_row_index", "hmbp_solve", "ptas_table_order", "ptas_level_shard", "dp_fill_opt", "dp_fill_alg4",
+    "ptas_slab_plan",
 ]
 
 _lib = None
@@ -101,6 +102,8 @@ def lib():
     L.ptas_interval_update.argtypes = [i64p, i64p, i64p, i32p, ctypes.c_int32]
     L.ptas_shard_range.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, i64p, i64p]
     L.ptas_level_shard.argtypes = [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, i64p, i64p, i64p]
+    L.ptas_slab_plan.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, i64p, i64p, i64p, i64p,
+                                 i64p]
     L.dp_configs.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, i32p, ctypes.c_int64, i64p]
     L.dp_fill_opt.argtypes = [i32p, i64p, ctypes.c_int32, ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, i32p,
                               ctypes.POINTER(PtasStats)]

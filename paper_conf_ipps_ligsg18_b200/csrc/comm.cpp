@@ -29,6 +29,8 @@ struct NcclApi {
     decltype(&ncclAllReduce) allReduce = nullptr;
     decltype(&ncclBroadcast) broadcast = nullptr;
     decltype(&ncclCommDestroy) commDestroy = nullptr;
+    decltype(&ncclSend) send = nullptr;
+    decltype(&ncclRecv) recv = nullptr;
 };
 
 NcclApi *nccl()
@@ -45,6 +47,8 @@ NcclApi *nccl()
         api.allReduce = (decltype(api.allReduce))dlsym(h, "ncclAllReduce");
         api.broadcast = (decltype(api.broadcast))dlsym(h, "ncclBroadcast");
         api.commDestroy = (decltype(api.commDestroy))dlsym(h, "ncclCommDestroy");
+        api.send = (decltype(api.send))dlsym(h, "ncclSend");
+        api.recv = (decltype(api.recv))dlsym(h, "ncclRecv");
         api.ok = api.getUniqueId && api.commInitRank && api.allGather && api.allReduce && api.broadcast &&
                  api.commDestroy;
     });
@@ -130,6 +134,24 @@ int comm_broadcast(ptas_comm *c, void *d_buf, size_t bytes, int root, cudaStream
     NcclApi *a = nccl();
     if (!a->ok || !c) return PTAS_ENCCL;
     if (a->broadcast(d_buf, d_buf, bytes, ncclUint8, root, c->comm, st) != ncclSuccess) return PTAS_ENCCL;
+    return PTAS_OK;
+}
+
+// Point-to-point: `bytes` bytes to / from rank `peer` (stream-ordered; the
+// slab/halo pipeline's halo of one chunk).
+int comm_send(ptas_comm *c, const void *d_buf, size_t bytes, int peer, cudaStream_t st)
+{
+    NcclApi *a = nccl();
+    if (!a->ok || !a->send || !c) return PTAS_ENCCL;
+    if (a->send(d_buf, bytes, ncclUint8, peer, c->comm, st) != ncclSuccess) return PTAS_ENCCL;
+    return PTAS_OK;
+}
+
+int comm_recv(ptas_comm *c, void *d_buf, size_t bytes, int peer, cudaStream_t st)
+{
+    NcclApi *a = nccl();
+    if (!a->ok || !a->recv || !c) return PTAS_ENCCL;
+    if (a->recv(d_buf, bytes, ncclUint8, peer, c->comm, st) != ncclSuccess) return PTAS_ENCCL;
     return PTAS_OK;
 }
 

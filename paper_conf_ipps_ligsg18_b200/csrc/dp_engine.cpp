@@ -48,6 +48,8 @@ static double host_ms()
             std::fprintf(stderr, "[ptas] slow call %.2f ms at dp_engine.cpp:%d: %s\n", \
                          host_ms() - t0__, __LINE__, #x);                            \
         if (e__ != cudaSuccess) {                                                  \
+            std::fprintf(stderr, "[ptas] CUDA error at dp_engine.cpp:%d: %s: %s\n", __LINE__, #x, \
+                         cudaGetErrorString(e__));                                 \
             cudaGetLastError();                                                    \
             return e__ == cudaErrorMemoryAllocation ? PTAS_ENOMEM : PTAS_ECUDA;    \
         }                                                                          \
@@ -470,10 +472,47 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
             virt = true;
         }
     }
-    const bool comm_dp = sh && sh->comm && (G > 1 || sh->force);   // collectives in this DP
+    const bool comm_dp = sh && sh->comm && (G > 1 || sh->force || sh->slab_pipe);   // collectives in this DP
     auto sharded = [&](int64_t R) { return (G > 1 || comm_dp) && R >= std::max<int64_t>(sh->min_rows, 1); };
+    // ---- slab/halo pipeline: with a communicator and a
+    // windowed DP, rank g holds the contiguous slab range [pb, pe) of the first
+    // internal class plus the hin = min(hi0, pb) slabs below it (the halo), in one
+    // linear buffer (slab p0 at p0 - pbase).  The slab-0 levels (the other classes'
+    // row-levels) are cut into chunks; per chunk rank g receives the halo rows of
+    // the chunk from g - 1, fills the chunk's rows of its slabs in ascending order
+    // (slab p0 >= 1 reads only slabs p0 - s0, s0 >= 1, at the same or lower
+    // levels, D13), and sends the chunk's rows of its last min(hi0, pe) slabs to
+    // g + 1: a wavefront over (rank, chunk) with ncclSend / ncclRecv.  OPT(N)
+    // lives on the last rank and is broadcast.  Every rank takes the same
+    // decisions (same inputs), so the p2p calls pair up.
+    const bool pipe = window && sh && sh->comm && sh->slab_pipe && (int64_t)N[0] + 1 >= G;
+    int64_t pb = 0, pe = 0, pbase = 0, hin = 0, hout = 0;
+    std::vector<int> chunk_lv;   // chunk c = slab-0 levels [chunk_lv[c], chunk_lv[c + 1])
+    if (pipe) {
+        slab_plan((int64_t)N[0] + 1, hi0w, myrank, G, &pb, &pe, &pbase, &hin, &hout);
+        g.span_words = (pe - pbase) * slab_bytes / 4;
+        const int nlev = (K >= 3 ? gidx.rho_max : 0) + 1;   // slab 0's row-levels (cnt_sub[0 .. nlev))
+        const int64_t C = std::min<int64_t>(nlev, std::max<int64_t>(1, PTAS_KNOB("PTAS_PIPE_CHUNKS_PER_RANK", 4) * G));
+        const int64_t target = (rows_idx + C - 1) / C;
+        chunk_lv.push_back(0);
+        int64_t acc_rows = 0;
+        for (int L = 0; L < nlev; ++L) {
+            acc_rows += cnt_sub[L];
+            if (acc_rows >= target && L + 1 < nlev) {
+                chunk_lv.push_back(L + 1);
+                acc_rows = 0;
+            }
+        }
+        chunk_lv.push_back(nlev);
+    }
     size_t stage_bytes = 0;
-    {   // the sharded units: row-levels, or (window) slab 0's levels and whole slabs
+    if (pipe) {   // the halo rows of the largest chunk (chunk_lv covers slab 0's levels only)
+        for (size_t c = 0; c + 1 < chunk_lv.size(); ++c) {
+            int64_t nr = 0;
+            for (int L = chunk_lv[c]; L < chunk_lv[c + 1]; ++L) nr += cnt_sub[L];
+            stage_bytes = std::max(stage_bytes, (size_t)(std::max(hin, hout) * nr * g.Wp * e));
+        }
+    } else {   // the sharded units: row-levels, or (window) slab 0's levels and whole slabs
         std::vector<int64_t> units = window ? cnt_sub : cnt;
         if (window) units.push_back(rows_idx);
         for (int64_t R : units) {
@@ -488,7 +527,15 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // agrees on the outcome over all ranks (min of the status words) before any
     // collective, so no rank returns while its peers wait in an all-gather
     int adm = PTAS_OK;
-    if (window) {
+    if (pipe) {
+        const int64_t need = (pe - pbase) * slab_bytes + rows_idx * 8 * (1 + (g.nwords <= 1 ? 1 : 2)) + (int64_t)stage_bytes;
+        if (rq.budget > 0 || (size_t)((pe - pbase) * slab_bytes) > table_.cap) {
+            const int64_t budget = rq.budget > 0 ? rq.budget : free_budget();
+            if (need > budget) adm = PTAS_ETOOBIG;
+        }
+        if (!adm && table_.ensure((size_t)((pe - pbase) * slab_bytes)) != cudaSuccess) adm = PTAS_ENOMEM;
+        o.dev_bytes = need;
+    } else if (window) {
         const int64_t need = Rw * slab_bytes + rows_idx * 8 * (1 + (g.nwords <= 1 ? 1 : 2));
         const int64_t budget = rq.budget > 0 ? rq.budget : free_budget() + (int64_t)ring_.phys;
         if (need > budget) adm = PTAS_ETOOBIG;
@@ -524,10 +571,15 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     int64_t idxN = N[K - 1];
     for (int i = 0; i < K - 1; ++i) idxN += (int64_t)N[i] * stride[i];
     // window: ring position of slab p0 is Rw + (p0 mod Rw) (slabs), relative to the ring
+    // (pipeline: slab p0 at p0 - pbase of the rank's linear buffer)
     auto slab_ptr = [&](int64_t p0) {
+        if (pipe) return (void *)((unsigned char *)table_.p + (p0 - pbase) * slab_bytes);
         return (void *)((unsigned char *)(uintptr_t)ring_.va + (Rw + p0 % Rw) * slab_bytes);
     };
-    if (window) {
+    if (pipe) {
+        table = table_.p;
+        idxN = ((int64_t)N[0] - pbase) * stride[0] + (idxN - (int64_t)N[0] * stride[0]);   // (last rank only)
+    } else if (window) {
         table = slab_ptr(0);
         idxN = (Rw + N[0] % Rw) * stride[0] + (idxN - (int64_t)N[0] * stride[0]);   // relative to the ring
     }
@@ -885,7 +937,55 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
         ++o.launches;
         return PTAS_OK;
     };
-    if (window) {
+    if (pipe) {
+        if (trace)
+            std::fprintf(stderr, "[ptas] slab pipeline: rank %d/%d slabs [%lld, %lld) base %lld hin %lld hout %lld, %zu chunks, "
+                                 "slab %lld B (rows %lld, pitch %lld, e %d), buffer %p cap %zu\n",
+                         myrank, G, (long long)pb, (long long)pe, (long long)pbase, (long long)hin, (long long)hout,
+                         chunk_lv.size() - 1, (long long)slab_bytes, (long long)rows_idx, (long long)g.Wp, e, table_.p,
+                         table_.cap);
+        unsigned char *stg = (unsigned char *)stage_.p;
+        const int64_t rowB = g.Wp * e;
+        for (size_t c = 0; c + 1 < chunk_lv.size(); ++c) {
+            const int La = chunk_lv[c], Lb = chunk_lv[c + 1];
+            const int64_t i0 = lstart[La], nr = lstart[Lb] - i0;
+            if (nr <= 0) continue;
+            if (myrank > 0 && hin > 0) {   // the chunk's rows of slabs pb - hin .. pb - 1 from rank g - 1
+                const int crc = comm_recv(sh->comm, stg, (size_t)(hin * nr * rowB), myrank - 1, st);
+                if (crc) return crc;
+                for (int64_t j = 0; j < hin; ++j) {
+                    PT_CK(launch_row_scatter(e, slab_ptr(pb - hin + j), g, d_rb + i0, nr, stg + j * nr * rowB,
+                                             sm_count_, st));
+                    ++o.launches;
+                }
+                prev_fill = false;
+            }
+            for (int64_t p0 = pb; p0 < pe; ++p0) {
+                if (p0 == 0) {   // slab 0: the other classes' DP, level by level
+                    for (int rho = La; rho < Lb; ++rho) {
+                        if (cntU[rho] <= 0) continue;
+                        PT_CK(fill(slab_ptr(0), g, J0, lstart[rho], 0, cntU[rho], nullptr));
+                        ++o.fill_launches;
+                    }
+                } else {         // the chunk's rows of slab p0: one launch (no dependency inside)
+                    RowGeom gs = g;
+                    gs.pw_or[g.word[0]] |= (uint64_t)p0 << g.shift[0];
+                    PT_CK(fill(slab_ptr(p0), gs, J0, i0, 0, nr, nullptr));
+                    ++o.fill_launches;
+                }
+            }
+            if (myrank + 1 < G && hout > 0) {   // the chunk's rows of slabs pe - hout .. pe - 1 to rank g + 1
+                for (int64_t j = 0; j < hout; ++j) {
+                    PT_CK(launch_row_gather(e, slab_ptr(pe - hout + j), g, d_rb + i0, nr, stg + j * nr * rowB,
+                                            sm_count_, st));
+                    ++o.launches;
+                }
+                const int crc = comm_send(sh->comm, stg, (size_t)(hout * nr * rowB), myrank + 1, st);
+                if (crc) return crc;
+                prev_fill = false;
+            }
+        }
+    } else if (window) {
         // slab 0: the DP of the other classes, level by level (its rows dominate only
         // prefixes with s0 = 0); then slabs 1 .. N0, one unit each over all rows
         // (sharded over the ranks of a communicator: SURVEY.md §8(f)-2ii)
@@ -981,8 +1081,19 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     (void)ld;
 
     // ---- a-6 readout
-    PT_CK(launch_read_opt(e, window ? (void *)(uintptr_t)ring_.va : table, idxN, d_meta_, st));
-    ++o.launches;
+    if (pipe) {   // OPT(N) is in the last rank's slab N0: read there, broadcast to every rank
+        if (myrank == G - 1) {
+            PT_CK(launch_read_opt(e, table, idxN, d_meta_, st));
+            ++o.launches;
+        }
+        if (G > 1) {
+            const int crc = comm_broadcast(sh->comm, &((DpMeta *)d_meta_)->opt, sizeof(int32_t), G - 1, st);
+            if (crc) return crc;
+        }
+    } else {
+        PT_CK(launch_read_opt(e, window ? (void *)(uintptr_t)ring_.va : table, idxN, d_meta_, st));
+        ++o.launches;
+    }
     if (rq.ext_table && !in_place) {
         PT_CK(launch_compact_rows(e, table, rq.ext_table, rows, g.W, g.Wp, st));
         ++o.launches;

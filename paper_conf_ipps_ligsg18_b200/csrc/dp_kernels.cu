@@ -579,6 +579,22 @@ row_scatter_kernel(E *__restrict__ table, const RowGeom g, const int64_t *__rest
     }
 }
 
+// §8(f)-2ii: the inverse -- rows of the table (row bases rb) into compact
+// slot-major rows (pitch Wp), the halo of one chunk before ncclSend.
+template <typename E>
+__global__ void __launch_bounds__(256)
+row_gather_kernel(const E *__restrict__ table, const RowGeom g, const int64_t *__restrict__ rb, int64_t slot_count,
+                  E *__restrict__ compact)
+{
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t slot = gw; slot < slot_count; slot += nw) {
+        const int64_t rowbase = rb[slot];
+        for (int64_t x = lane; x < g.Wp; x += 32) compact[slot * g.Wp + x] = table[rowbase + x];
+    }
+}
+
 template <typename E>
 __global__ void read_opt_kernel(const E *__restrict__ table, int64_t idx, DpMeta *meta)
 {
@@ -1018,6 +1034,20 @@ cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64
         row_scatter_kernel<uint8_t><<<(unsigned)blocks, 256, 0, st>>>((uint8_t *)table, g, rb, slot_count, (const uint8_t *)compact);
     else
         row_scatter_kernel<uint16_t><<<(unsigned)blocks, 256, 0, st>>>((uint16_t *)table, g, rb, slot_count, (const uint16_t *)compact);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_row_gather(int e, const void *table, const RowGeom &g, const int64_t *rb, int64_t slot_count,
+                              void *compact, int sm_count, cudaStream_t st)
+{
+    if (slot_count <= 0) return cudaSuccess;
+    int64_t blocks = (slot_count + 7) / 8;
+    const int64_t cap = (int64_t)sm_count * 8;
+    if (blocks > cap) blocks = cap;
+    if (e == 1)
+        row_gather_kernel<uint8_t><<<(unsigned)blocks, 256, 0, st>>>((const uint8_t *)table, g, rb, slot_count, (uint8_t *)compact);
+    else
+        row_gather_kernel<uint16_t><<<(unsigned)blocks, 256, 0, st>>>((const uint16_t *)table, g, rb, slot_count, (uint16_t *)compact);
     return cudaGetLastError();
 }
 

@@ -20,6 +20,7 @@ struct ShardCtx {
     int virtual_shards = 1;     // >1: logical shards on this GPU (testing)
     int64_t min_rows = 0;       // row-levels with fewer rows are computed redundantly
     bool force = false;         // shard (slice, all-gather, scatter) also at world size 1
+    bool slab_pipe = false;     // windowed DPs: slab/halo pipeline with send/recv
 };
 
 struct DpRequest {
@@ -205,5 +206,7 @@ int comm_allgather(ptas_comm *c, const void *send, void *recv, size_t bytes_per_
                    cudaStream_t st);
 int comm_allreduce_min_i32(ptas_comm *c, int32_t *d_buf, size_t count, cudaStream_t st);
 int comm_broadcast(ptas_comm *c, void *d_buf, size_t bytes, int root, cudaStream_t st);
+int comm_send(ptas_comm *c, const void *d_buf, size_t bytes, int peer, cudaStream_t st);
+int comm_recv(ptas_comm *c, void *d_buf, size_t bytes, int peer, cudaStream_t st);
 
 }  // namespace ptas

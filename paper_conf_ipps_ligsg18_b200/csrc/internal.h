@@ -173,6 +173,20 @@ constexpr int64_t NP_CAP = 1000;
 // calling DP slot's thread; -1 = use the bound they are given).
 extern thread_local int64_t tl_np_hint;
 
+// Slab/halo pipeline plan: S slabs of the first
+// internal class over `world` ranks; rank `rank` owns [pb, pe), holds [pbase, pe)
+// (hin = pb - pbase halo slabs received from rank - 1 per chunk) and sends its
+// last hout slabs to rank + 1.  hin of rank g equals hout of rank g - 1.
+inline void slab_plan(int64_t S, int64_t hi0, int rank, int world, int64_t *pb, int64_t *pe, int64_t *pbase,
+                      int64_t *hin, int64_t *hout)
+{
+    *pb = S * rank / world;
+    *pe = S * (rank + 1) / world;
+    *pbase = *pb - hi0 > 0 ? *pb - hi0 : 0;
+    *hin = *pb - *pbase;
+    *hout = hi0 < *pe ? hi0 : *pe;
+}
+
 // ---------------------------------------------------------------- launchers
 // All launchers enqueue on `st` and return cudaGetLastError().
 // pass 1 writes nothing when the total |C| (offsets[nprefix]) exceeds cap
@@ -265,6 +279,8 @@ cudaError_t launch_compact_rows(int e, const void *src, void *dst, int64_t rows,
                                 int64_t Wp, cudaStream_t st);
 cudaError_t launch_row_scatter(int e, void *table, const RowGeom &g, const int64_t *rb,
                                int64_t slot_count, const void *compact, int sm_count, cudaStream_t st);
+cudaError_t launch_row_gather(int e, const void *table, const RowGeom &g, const int64_t *rb, int64_t slot_count,
+                              void *compact, int sm_count, cudaStream_t st);
 cudaError_t launch_read_opt(int e, const void *table, int64_t idx, DpMeta *d_meta,
                             cudaStream_t st);
 cudaError_t launch_traceback(int e, const void *table, int K, const int32_t *d_N,

@@ -337,6 +337,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         sh.virtual_shards = opt.comm ? 1 : std::max(1, opt.virtual_shards);
         sh.min_rows = opt.comm ? (opt.shard_min_rows >= 0 ? opt.shard_min_rows : 2048) : 0;
         sh.force = opt.comm && opt.shard_min_rows == 0;
+        sh.slab_pipe = opt.comm && opt.slab_pipeline == 1;
         shp = &sh;
     }
 
@@ -997,6 +998,15 @@ int ptas_table_order(const int32_t *counts, const int64_t *sizes, int32_t K, int
                                             std::vector<int64_t>(sizes, sizes + K), layout);
     for (size_t i = 0; i < o.size(); ++i) order_out[i] = o[i];
     *K_out = (int32_t)o.size();
+    return PTAS_OK;
+}
+
+int ptas_slab_plan(int64_t S, int64_t hi0, int32_t rank, int32_t world, int64_t *pb, int64_t *pe, int64_t *pbase,
+                   int64_t *hin, int64_t *hout)
+{
+    if (world < 1 || rank < 0 || rank >= world || S < world || hi0 < 0 || !pb || !pe || !pbase || !hin || !hout)
+        return PTAS_EINVAL;
+    slab_plan(S, hi0, rank, world, pb, pe, pbase, hin, hout);
     return PTAS_OK;
 }
 

@@ -127,3 +127,49 @@ def test_multisection_protocol_gloo():
 def test_level_shard_gather_scatter_gloo():
     res = _run(sharding_rank, 2)
     assert res == [True, True]
+
+
+# ---- slab/halo pipeline (ptas_options.slab_pipeline): the
+# engine's schedule with the library's own plan (ptas_slab_plan).  Per chunk,
+# rank g receives the halo slabs from g - 1 (gloo send/recv in place of
+# ncclSend/ncclRecv, carrying the slab ids), "fills" its slabs in ascending
+# order -- asserting that every slab a row reads (p0 - s0, 1 <= s0 <= hi0, at the
+# same or an earlier chunk) is present -- and forwards its last hout slabs.
+def _pipeline_protocol(rank, world):
+    import paper_conf_ipps_ligsg18_b200 as P
+    out = []
+    for S, hi0, C in [(251, 2, 8), (31, 4, 5), (7, 3, 3), (world, 5, 2), (120, 0, 4)]:
+        pb, pe, pbase, hin, hout = P.ptas_slab_plan(S, hi0, rank, world)
+        have = set()
+        for c in range(C):
+            if rank > 0 and hin > 0:
+                t = torch.zeros(hin, dtype=torch.int64)
+                dist.recv(t, src=rank - 1)
+                got = sorted(int(x) for x in t)
+                assert got == list(range(pb - hin, pb)), (S, hi0, rank, c, got)
+                have.update((s, c) for s in got)
+            for p0 in range(pb, pe):
+                for s0 in range(1, hi0 + 1):
+                    if p0 - s0 >= 0:
+                        assert p0 - s0 >= pbase, (S, hi0, rank, p0, s0)
+                        assert all((p0 - s0, cc) in have for cc in range(c + 1)), (S, hi0, rank, p0, s0, c)
+                have.add((p0, c))
+            if rank + 1 < world and hout > 0:
+                ids = list(range(pe - hout, pe))
+                assert all((s, c) in have for s in ids)
+                dist.send(torch.tensor(ids, dtype=torch.int64), dst=rank + 1)
+        out.append((pb, pe, pbase, hin, hout))
+    return out
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_slab_pipeline_protocol(world):
+    res = _run(_pipeline_protocol, world)
+    for k, (S, hi0) in enumerate([(251, 2), (31, 4), (7, 3), (world, 5), (120, 0)]):
+        plans = [r[k] for r in res]
+        # contiguous, disjoint, covering ranges; the last rank owns slab S - 1 (OPT(N))
+        assert plans[0][0] == 0 and plans[-1][1] == S
+        for g in range(1, world):
+            assert plans[g][0] == plans[g - 1][1]
+            assert plans[g][3] == plans[g - 1][4]          # hin(g) == hout(g - 1)
+        assert all(p[1] > p[0] for p in plans)

@@ -109,3 +109,29 @@ def test_window_slabs_sharded_nccl_vs_golden(comm, name):
     got = P.ptas_solve(w.p(), w.m, w.eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c, shard_min_rows=0, window=1)
     _cmp(got, g)
     assert got["stats"]["window_dps"] > 0
+
+
+@pytest.mark.parametrize("name", ["M2s", "M5s-0.3", "M3s"])
+def test_slab_pipeline_nccl_vs_golden(comm, name):
+    """Slab/halo pipeline (ptas_options.slab_pipeline): every
+    probe DP is filled in chunks of the other classes' levels, slab by slab, in the
+    rank's linear slab buffer (at world size 1 the rank owns every slab and there is
+    no halo to send); OPT(N) is read on the last rank and broadcast.  The probe log,
+    T*, makespan and assignment equal the oracle's."""
+    P, c = comm
+    w = WORKLOADS[name]
+    g = json.load(open(os.path.join(GOLD, f"solve_{name}_P1.json")))
+    got = P.ptas_solve(w.p(), w.m, w.eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c, window=1, slab_pipeline=1)
+    _cmp(got, g)
+    assert got["stats"]["window_dps"] > 0
+
+
+@pytest.mark.parametrize("chunks", ["1", "4", "64"])
+def test_slab_pipeline_random_vs_oracle(comm, monkeypatch, chunks):
+    # chunks per rank (1: the whole slab at once; 64: one level per chunk for small DPs)
+    P, c = comm
+    monkeypatch.setenv("PTAS_PIPE_CHUNKS_PER_RANK", chunks)
+    for seed, (n, m, eps) in enumerate([(60, 14, 0.3), (40, 8, 0.25), (50, 10, 0.2), (30, 9, 0.34)]):
+        p = jobs(n, 1000, seed + 11)
+        got = P.ptas_solve(p, m, eps, P=1, mode=P.MODE_LEVEL_SHARDED, comm=c, window=1, slab_pipeline=1)
+        _cmp(got, oracle.ptas(p, m, eps, 1))
