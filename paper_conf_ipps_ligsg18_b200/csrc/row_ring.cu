@@ -340,8 +340,11 @@ cudaError_t launch_ring_t(void *table, const RingArgs &ra, const PrefixEntry *d_
 {
     auto kfn = row_ring_kernel<E, CH, WIN>;
     const int64_t np = nP_bound > 1 ? nP_bound - 1 : 0;
-    const size_t smem = (((size_t)ra.R * (ra.A + ra.TB * ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + PTAS_RING_PB) * 16;
+    size_t smem = (((size_t)ra.R * (ra.A + ra.TB * ra.H) * ra.Lw * 4 + 15) & ~(size_t)15) + 4 * (size_t)(np + PTAS_RING_PB) * 16;
     if (smem > 220 * 1024) return cudaErrorNotSupported;
+    // PTAS_RING_SMEM_MIN (experiment): pad the dynamic shared memory, e.g. above half an
+    // SM's, so no two ring CTAs (of concurrent DPs) share an SM
+    smem = std::max<size_t>(smem, (size_t)std::min<int64_t>(220 * 1024, PTAS_KNOB("PTAS_RING_SMEM_MIN", 0)));
     // function attributes and the co-residency query once per (device, kernel,
     // smem, cluster size, block): they take the driver lock, and concurrent DP
     // slots issue from several host threads
