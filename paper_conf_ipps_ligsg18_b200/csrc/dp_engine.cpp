@@ -785,31 +785,26 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
                                            d_meta_, nP_bound, st, true) == cudaSuccess;
     cudaGetLastError();
     if (!ring) {
-        const int df_mode = (int)PTAS_KNOB("PTAS_DF", 3);
+        // Dataflow runs and split runs pay only when a row's walk is long.  A row walks
+        // its pivot block (D13); most rows have pivot 0, whose block is {s' : s'_0 >= 1,
+        // sum s'_i r_i <= T}, counted here on the host.  Measured with the short prefix
+        // batches of round 2: DPs with blocks of at most 12 prefixes (M2s 4, M3s 12) are
+        // fastest with one launch per row-level (M2s 1.90 -> 1.82 ms, M3s 4.90 -> 3.62
+        // ms, M3g (16) 42.8 -> 39.6 ms -- M3g keeps runs below), M5s-0.15 (38) needs the
+        // dataflow runs with split row sets (15.9 ms; 25.4 ms without runs, 20.0 ms
+        // without split runs).  PTAS_DF / PTAS_DF_SPLIT_ROWS override.
+        const int64_t blk0 = pivot0_block(N.data(), r.data(), K, rq.T);   // prefixes with s'_0 >= 1
+        const int64_t dfm_env = PTAS_KNOB("PTAS_DF", -1);
+        // (DPs whose levels are all narrow -- K = 2: one row per level -- keep one
+        // dataflow launch instead of hundreds of tiny ones)
+        int64_t max_level_rows = 0;
+        for (int rho = 0; rho <= g.rho_max; ++rho) max_level_rows = std::max(max_level_rows, cnt[rho]);
+        const int df_mode = dfm_env >= 0 ? (int)dfm_env
+                                         : ((blk0 > PTAS_KNOB("PTAS_DF_BLOCK", 16) || max_level_rows <= 256) ? 3 : 0);
         const int64_t dfr = PTAS_KNOB("PTAS_DF_ROWS", -1);
         const int64_t df_rows = df_mode == 1 ? INT64_MAX : (dfr >= 0 ? dfr : (int64_t)2 * 32 * sm_count_);
-        // Splitting a row set's prefix walk over the 8 warps of a block pays only when
-        // the walk is long.  A row walks its pivot block (D13); most rows have pivot
-        // 0, whose block is {s' : s'_0 >= 1, sum s'_i r_i <= T}, counted here on the
-        // host.  Measured with the short prefix batches of round 2: blocks of 4-12
-        // prefixes (M2s, M3s) are faster without split runs (M2s 2.08 -> 1.87 ms, M3s
-        // 6.7 -> 6.2 ms), M5s-0.15 (38) needs them (15.7 ms, 20.0 ms without), M3g
-        // (16) is indifferent; split when the block has more than 12.
         const int64_t sr_env = PTAS_KNOB("PTAS_DF_SPLIT_ROWS", -1);
-        int64_t split_rows = sr_env;
-        if (sr_env < 0) {
-            int64_t blk0 = 0;   // prefixes with s'_0 >= 1 (capped)
-            std::function<void(int, int64_t, bool)> walk = [&](int i, int64_t rem, bool lead) {
-                if (blk0 > 4096) return;
-                if (i == K - 1) {
-                    blk0 += lead;
-                    return;
-                }
-                for (int64_t d = 0; d <= N[i] && d * r[i] <= rem; ++d) walk(i + 1, rem - d * r[i], lead || (i == 0 && d >= 1));
-            };
-            if (K >= 2) walk(0, rq.T, false);
-            split_rows = blk0 > PTAS_KNOB("PTAS_DF_SPLIT_BLOCK", 12) ? 2000 : 0;
-        }
+        const int64_t split_rows = sr_env >= 0 ? sr_env : (blk0 > PTAS_KNOB("PTAS_DF_SPLIT_BLOCK", 12) ? 2000 : 0);
         if (df_mode > 0 && G == 1 && !comm_dp && !window && !force_scalar && g.rho_max >= 1) {
             if (df_mode == 3 || df_mode == 4) {
                 // levels wider than df_rows get a launch of their own (enough rows to fill

@@ -173,6 +173,39 @@ constexpr int64_t NP_CAP = 1000;
 // calling DP slot's thread; -1 = use the bound they are given).
 extern thread_local int64_t tl_np_hint;
 
+// Prefixes of the pivot-0 block (D13) of a DP in internal class order: #{s' over
+// the K - 1 leading classes : s'_0 >= 1, s'_i <= N_i, sum s'_i r_i <= T}, capped
+// at `cap` (host; a few microseconds).  Most rows of a DP walk this block.
+inline int64_t pivot0_block(const int32_t *N, const int64_t *r, int K, int64_t T, int64_t cap = 4096)
+{
+    if (K < 2) return 0;
+    int64_t cnt = 0;
+    // iterative DFS over the leading digits (d[i] = digit i, rem[i] = budget left before digit i)
+    int64_t d[64], rem[65];
+    const int L = K - 1 < 64 ? K - 1 : 64;
+    int i = 0;
+    d[0] = 1;
+    rem[0] = T;
+    if (N[0] < 1 || r[0] > T) return 0;
+    for (;;) {
+        if (i == L) {   // a complete prefix
+            if (++cnt > cap) return cnt;
+            --i;
+            ++d[i];
+            continue;
+        }
+        if (d[i] <= N[i] && d[i] * r[i] <= rem[i]) {
+            rem[i + 1] = rem[i] - d[i] * r[i];
+            ++i;
+            if (i < L) d[i] = 0;
+            continue;
+        }
+        if (i == 0) return cnt;
+        --i;
+        ++d[i];
+    }
+}
+
 // Slab/halo pipeline plan: S slabs of the first
 // internal class over `world` ranks; rank `rank` owns [pb, pe), holds [pbase, pe)
 // (hin = pb - pbase halo slabs received from rank - 1 per chunk) and sends its

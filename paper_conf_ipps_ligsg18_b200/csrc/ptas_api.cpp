@@ -516,6 +516,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     int64_t spec_sigma = (int64_t)1 << 24;
     const bool spec_ring = PTAS_KNOB("PTAS_SPEC_RING", 1) != 0;   // 0: latency-bound DPs only below spec_sigma (A/B)
     const int64_t spec_levels = PTAS_KNOB("PTAS_SPEC_LEVELS", 160);
+    const int64_t spec_levels_short = PTAS_KNOB("PTAS_SPEC_LEVELS_SHORT", 480);   // (with a short pivot block)
+    const int64_t spec_block = PTAS_KNOB("PTAS_SPEC_BLOCK", 16);
     {
         const int64_t sd = PTAS_KNOB("PTAS_SPEC_DEPTH", -1);
         if (sd >= 0 && opt.speculate < 0) spec_depth = (int)sd;
@@ -579,6 +581,13 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                     int64_t levels = 1;
                     for (size_t i = 0; i + 1 < No.size(); ++i) levels += No[i];
                     lat = lat || (No.size() >= 2 && levels <= spec_levels);
+                    // DPs with a few hundred row-levels but short pivot blocks (D13; M3s:
+                    // 12 prefixes, 290 levels; M3g: 16, 335) are latency-bound too: their
+                    // levels overlap (round 2: M3s 6.3 -> 4.9 ms, M3g 44.9 -> 42.7 ms); with
+                    // long blocks (M5s-0.15: 38, 423 levels) they are throughput-bound and
+                    // lose by sharing the GPU (15.7 -> 22.1 ms)
+                    lat = lat || (No.size() >= 2 && levels <= spec_levels_short &&
+                                  pivot0_block(No.data(), ro.data(), (int)No.size(), T, 64) <= spec_block);
                 }
                 // a large next probe runs alone (throughput-bound: nothing to overlap)
                 if (nd.d == 0 && sg > (__int128)spec_sigma && !lat) return PTAS_OK;
