@@ -453,10 +453,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 rcs[b] = probe_dp(sl[b], cls_v[j0 + b], T_v[j0 + b], nullptr,
                                   b == 0 ? (cudaStream_t)opt.stream : nullptr, gdiv[b], &outs_all[j0 + b]);
             };
-            std::vector<std::thread> th;
-            for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
-            work(0);
-            for (auto &t : th) t.join();
+            eng->pool().run(nb, work);
             for (int b = 0; b < nb; ++b) {
                 if (rcs[b]) return rcs[b];
                 slot_key[b] = outs_all[j0 + b].windowed ? std::vector<int64_t>() : key_v[j0 + b];
@@ -486,10 +483,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
                 rcs[b] = probe_dp(sl[b], cls_v[j0 + b], T_v[j0 + b], nullptr,
                                   b == 0 ? (cudaStream_t)opt.stream : nullptr, 1, &outs[b]);
             };
-            std::vector<std::thread> th;
-            for (int b = 1; b < nb; ++b) th.emplace_back(work, b);
-            work(0);
-            for (auto &t : th) t.join();
+            eng->pool().run(nb, work);
             for (int b = 0; b < nb; ++b) {
                 if (rcs[b]) return rcs[b];
                 acc.add(outs[b]);
