@@ -1,6 +1,7 @@
 // engine.h — per-device DP engine (host orchestration of the kernels).
 #pragma once
 #include <algorithm>
+#include <atomic>
 #include <condition_variable>
 #include <cstdint>
 #include <functional>
@@ -171,12 +172,14 @@ class WorkerPool {
             job_ = &fn;
             next_ = 1;
             total_ = n;
-            remaining_ = n - 1;
+            remaining_.store(n - 1, std::memory_order_release);
         }
         cv_.notify_all();
         fn(0);
-        std::unique_lock<std::mutex> lk(m_);
-        done_.wait(lk, [&] { return remaining_ == 0; });
+        // the caller's own DP is usually not the last: spin for the others (a
+        // condition-variable wake-up costs tens of microseconds on the critical path)
+        while (remaining_.load(std::memory_order_acquire) != 0) std::this_thread::yield();
+        std::lock_guard<std::mutex> lk(m_);
         job_ = nullptr;
         next_ = total_ = 0;
     }
@@ -191,15 +194,16 @@ class WorkerPool {
             const std::function<void(int)> *f = job_;
             lk.unlock();
             (*f)(i);
+            remaining_.fetch_sub(1, std::memory_order_acq_rel);
             lk.lock();
-            if (--remaining_ == 0) done_.notify_all();
         }
     }
     std::mutex m_;
-    std::condition_variable cv_, done_;
+    std::condition_variable cv_;
     std::vector<int> th_;   // one entry per started worker
     const std::function<void(int)> *job_ = nullptr;
-    int next_ = 0, total_ = 0, remaining_ = 0;
+    int next_ = 0, total_ = 0;
+    std::atomic<int> remaining_{0};
 };
 
 // Per-device engine: a lock serialising API calls on the device and up to
