@@ -66,6 +66,22 @@ struct ValueHistogram {
     std::vector<int32_t> c;    // multiplicities
     ValueHistogram(const int64_t *p, int32_t n)
     {
+        if (n <= 0) return;
+        int64_t lo = p[0], hi = p[0];
+        for (int32_t j = 1; j < n; ++j) {
+            lo = std::min(lo, p[j]);
+            hi = std::max(hi, p[j]);
+        }
+        if (hi - lo <= (int64_t)4 * n + 65536) {   // counting (uniform integer sizes: P <= 1000)
+            std::vector<int32_t> cnt((size_t)(hi - lo + 1), 0);
+            for (int32_t j = 0; j < n; ++j) ++cnt[(size_t)(p[j] - lo)];
+            for (size_t i = 0; i < cnt.size(); ++i)
+                if (cnt[i]) {
+                    v.push_back(lo + (int64_t)i);
+                    c.push_back(cnt[i]);
+                }
+            return;
+        }
         std::vector<int64_t> s(p, p + n);
         std::sort(s.begin(), s.end());
         for (int64_t x : s) {
@@ -74,6 +90,27 @@ struct ValueHistogram {
                 v.push_back(x);
                 c.push_back(1);
             }
+        }
+    }
+    // classify() with the per-job classes: the class of each distinct long value,
+    // then one lookup per job (identical to classify: same r, N, cls)
+    void classify_full(const int64_t *p, int32_t n, int64_t T, int32_t k, Classified *out) const
+    {
+        classify_counts(T, k, out);
+        out->cls.assign(n, -1);
+        if (out->r.empty()) return;
+        const int64_t u = out->u;
+        // class index of every distinct value (-1: short)
+        std::vector<int32_t> vc(v.size(), -1);
+        size_t ci = 0;
+        for (size_t i = 0; i < v.size(); ++i) {
+            if (!((__int128)k * v[i] > (__int128)T)) continue;
+            while (out->r[ci] != (v[i] / u) * u) ++ci;
+            vc[i] = (int32_t)ci;
+        }
+        for (int32_t j = 0; j < n; ++j) {
+            const size_t i = (size_t)(std::lower_bound(v.begin(), v.end(), p[j]) - v.begin());
+            out->cls[j] = vc[i];
         }
     }
     void classify_counts(int64_t T, int32_t k, Classified *out) const
@@ -352,6 +389,8 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
     std::map<std::vector<int64_t>, int32_t> memo;
     std::vector<ptas_probe> plog;
     const ValueHistogram hist(p, n);   // classes and counts of every probe (per-job classes: classify)
+    if (PTAS_KNOB("PTAS_TRACE", 0) == 1)
+        std::fprintf(stderr, "[ptas] histogram built | host clock %.3f .. %.3f ms\n", 1e3 * t0, 1e3 * now_s());
     constexpr int32_t XERR = -1000;                          // MULTI_PROBE: exchanged error codes
     std::vector<std::vector<int64_t>> last_key_of(world);  // MULTI_PROBE: the last DP of each rank
     int round = 0;
@@ -604,6 +643,9 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
         }
         if (cls_v.empty()) return PTAS_OK;
         std::vector<DpOutcome> outs;
+        if (PTAS_KNOB("PTAS_TRACE", 0) == 1)
+            std::fprintf(stderr, "[ptas] speculation planned: %zu DPs | host clock %.3f .. %.3f ms\n", cls_v.size(),
+                         1e3 * t0, 1e3 * now_s());
         int r2 = run_jobs(cls_v, T_v, key_v, outs, true);
         if (r2) return r2;
         for (size_t j = 0; j < cls_v.size(); ++j) spec[key_v[j]] = SpecRes{outs[j].opt, outs[j]};
@@ -765,7 +807,7 @@ int solve_core(const int64_t *p, int32_t n, int32_t m, double eps, const ptas_op
 
     // ---- a-8 schedule from DP(T*) (readings R9, R11, R12)
     const int64_t Ts = LB;
-    classify(p, n, Ts, k, &cl);
+    hist.classify_full(p, n, Ts, k, &cl);
     std::vector<int64_t> load(m, 0);
     std::vector<int32_t> asg(n, -1);
     int32_t opt_star = 0;
