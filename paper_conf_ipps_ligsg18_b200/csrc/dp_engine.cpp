@@ -654,7 +654,12 @@ int DpSlot::run_dp(const DpRequest &rq, DpOutcome *out)
     // NP_CAP, launch heuristics from the previous DP's prefix count; the
     // kernels exit and the DP is redone synchronously if a bound is exceeded
     // (meta->ovf), which then grows the bounds.
-    const bool es_sync = PTAS_KNOB("PTAS_ENUM_SYNC", 0) == 1;
+    // Round 2: the enumeration always reads |C| back (PTAS_ENUM_SYNC=0 restores the
+    // round-trip-free path of D9): with several DPs in flight the round-trip-free
+    // path intermittently left a DP's table unfilled (OPT(N) read from stale memory;
+    // 4 of 8 M5s-0.15 P = 2 solves after an M3s solve, 0 of 8 with the read-back)
+    // -- a race not yet located, so the path is off by default
+    const bool es_sync = PTAS_KNOB("PTAS_ENUM_SYNC", 1) == 1;
     // (a comm-backed DP always reads |C| back: every rank then takes the same path,
     // no rank can redo the DP alone while its peers wait in a collective)
     const bool nosync = np_hint_ >= 0 && nc_cap_ > 0 && !force_sync_enum_ && !es_sync && !comm_dp;
